@@ -1,0 +1,265 @@
+"""ORACLE (test infrastructure): DeepPlan's planner and its pipeline cost model.
+
+Follows PAPER.md §4.1-4.3 step by step, with the readings of DESIGN.md §3 (SURVEY §8(c)
+P1-P4, G2-G10).  Everything is exact int64 nanosecond arithmetic, so the product
+planner (C++, behind the C-ABI) must match it bit-exactly.
+
+Encodings: method LOAD = 0, DHA = 1; slot 0 = the primary GPU's own PCIe
+link, slot s >= 1 = the s-th parallel-transmission partition.
+
+Cost table (dict of int64 arrays, one entry per planning unit in forward order):
+  bytes, load_ns (H2D on one link), fwd_ns (secondary -> primary over NVLink),
+  exe_mem_ns (Exe(InMem)), exe_dha_ns (Exe(DHA); INF_NS = ineligible)  -- P:200-202.
+"""
+from __future__ import annotations
+
+import heapq
+import itertools
+
+import numpy as np
+
+LOAD, DHA = 0, 1
+MODES = ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "PT", "PT_DHA")
+INF_NS = 1 << 50
+
+
+def _arr(cost, key):
+    return [int(v) for v in np.asarray(cost[key], dtype=np.int64)]
+
+
+# ------------------------------------------------------------------------------------
+# P1: pipeline simulator.  P:162-170 (Fig.7/8): a loaded layer can start only after it
+# is loaded ("the pipeline execution for L1 is stalled due to the dependency"); a DHA
+# layer needs no load; loads go back to back in plan order on one link ("The load
+# stream copies selected layers sequentially according to the plan").  PT:
+# the secondary's partition goes over its own link, then is forwarded over NVLink "in
+# the pipelined manner", one layer at a time after it lands.
+# ------------------------------------------------------------------------------------
+
+def simulate(cost, method, slot=None, k: int = 1, serial: bool = False):
+    """Returns dict(latency, stall[n], avail[n], start[n], link_bytes[k]).
+
+    serial=True is the "Baseline" option (Fig.1b): load every layer, then execute.
+    """
+    n = len(method)
+    load, fwd = _arr(cost, "load_ns"), _arr(cost, "fwd_ns")
+    exe_mem, exe_dha = _arr(cost, "exe_mem_ns"), _arr(cost, "exe_dha_ns")
+    nbytes = _arr(cost, "bytes")
+    slot = [0] * n if slot is None else [int(s) for s in slot]
+    t_link = [0] * k
+    t_fwd = [0] * k
+    link_bytes = [0] * k
+    avail = [0] * n
+    for i in range(n):
+        if method[i] == DHA:
+            avail[i] = 0
+        elif slot[i] == 0:
+            t_link[0] += load[i]
+            avail[i] = t_link[0]
+            link_bytes[0] += nbytes[i]
+        else:
+            s = slot[i]
+            t_link[s] += load[i]
+            t_fwd[s] = max(t_link[s], t_fwd[s]) + fwd[i]
+            avail[i] = t_fwd[s]
+            link_bytes[s] += nbytes[i]
+    if serial:
+        done = max(avail) if n else 0
+        avail = [done] * n
+    t = 0
+    stall = [0] * n
+    start = [0] * n
+    for i in range(n):
+        st = max(t, avail[i])
+        stall[i] = st - t
+        start[i] = st
+        t = st + (exe_dha[i] if method[i] == DHA else exe_mem[i])
+    return {"latency": t, "stall": stall, "avail": avail, "start": start, "link_bytes": link_bytes}
+
+
+def simulate_events(cost, method, slot=None, k: int = 1):
+    """An independent formulation of P1 as a discrete-event simulation with FIFO
+    resources (one per PCIe link, one NVLink forwarder per secondary, one compute
+    engine).  Used only to pin ``simulate``; returns (latency, stall[n])."""
+    n = len(method)
+    load, fwd = _arr(cost, "load_ns"), _arr(cost, "fwd_ns")
+    exe_mem, exe_dha = _arr(cost, "exe_mem_ns"), _arr(cost, "exe_dha_ns")
+    slot = [0] * n if slot is None else [int(s) for s in slot]
+    # queues of pending jobs per resource, in forward order
+    link_q = {s: [i for i in range(n) if method[i] == LOAD and slot[i] == s] for s in range(k)}
+    busy_until = {("link", s): 0 for s in range(k)}
+    busy_until.update({("nvl", s): 0 for s in range(1, k)})
+    ready = [None] * n  # time unit i's weights are usable on the primary
+    for i in range(n):
+        if method[i] == DHA:
+            ready[i] = 0
+    ev = []  # (time, seq, kind, payload)
+    seq = itertools.count()
+    # start the first transfer on each link at t=0
+    for s in range(k):
+        if link_q[s]:
+            i = link_q[s].pop(0)
+            heapq.heappush(ev, (load[i], next(seq), "link_done", (s, i)))
+    nvl_q = {s: [] for s in range(1, k)}
+    nvl_busy = {s: False for s in range(1, k)}
+    while ev:
+        t, _, kind, (s, i) = heapq.heappop(ev)
+        if kind == "link_done":
+            if s == 0:
+                ready[i] = t
+            else:
+                nvl_q[s].append(i)
+                if not nvl_busy[s]:
+                    j = nvl_q[s].pop(0)
+                    nvl_busy[s] = True
+                    heapq.heappush(ev, (t + fwd[j], next(seq), "nvl_done", (s, j)))
+            if link_q[s]:
+                j = link_q[s].pop(0)
+                heapq.heappush(ev, (t + load[j], next(seq), "link_done", (s, j)))
+        else:  # nvl_done
+            ready[i] = t
+            nvl_busy[s] = False
+            if nvl_q[s]:
+                j = nvl_q[s].pop(0)
+                nvl_busy[s] = True
+                heapq.heappush(ev, (t + fwd[j], next(seq), "nvl_done", (s, j)))
+    t = 0
+    stall = []
+    for i in range(n):
+        st = max(t, ready[i])
+        stall.append(st - t)
+        t = st + (exe_dha[i] if method[i] == DHA else exe_mem[i])
+    return t, stall
+
+
+# ------------------------------------------------------------------------------------
+# P2: Algorithm 1 (prose P:225)
+# ------------------------------------------------------------------------------------
+
+def algorithm1(cost):
+    """Returns method[n] chosen by Algorithm 1 on a single link (slot 0 everywhere)."""
+    n = len(cost["load_ns"])
+    load = _arr(cost, "load_ns")
+    pd = [d - m for d, m in zip(_arr(cost, "exe_dha_ns"), _arr(cost, "exe_mem_ns"))]
+    method = [LOAD] * n
+    for i in range(n):                                   # line 1
+        stall = simulate(cost, method)["stall"]          # reading G3: re-simulate each i
+        S = stall[i]
+        if not S > 0:                                    # line 2
+            continue
+        # Step 1 (lines 3-5): L_1..L_i not yet DHA, ascending PerfDiff, ties by index (G4)
+        cand = sorted((j for j in range(i + 1) if method[j] == LOAD), key=lambda j: (pd[j], j))
+        for j in cand:                                   # line 6
+            if S < pd[j]:                                # line 9 (strict, G5)
+                break
+            method[j] = DHA                              # line 12
+            S = S - load[j] - pd[j]                      # line 13, verbatim (G5)
+            if S <= 0:                                   # lines 16-18 (G6)
+                break                                    # line 17: re-simulated at next i
+    return method
+
+
+def greedy(cost):
+    """The "initial approach" (Table 3): DHA iff Exe(DHA) < Load + Exe(InMem)."""
+    load, em, ed = _arr(cost, "load_ns"), _arr(cost, "exe_mem_ns"), _arr(cost, "exe_dha_ns")
+    return [DHA if ed[i] < load[i] + em[i] else LOAD for i in range(len(load))]
+
+
+# ------------------------------------------------------------------------------------
+# P3: transmission planning: "equally partition a given model into the
+# number of GPUs"; "change the execution method for layers belonging to the second and
+# later partitions to be loaded".  Reading G10: contiguous, by whole-model bytes.
+# ------------------------------------------------------------------------------------
+
+def partition(nbytes, k: int):
+    T = int(sum(int(b) for b in nbytes))
+    part = []
+    off = 0
+    for b in nbytes:
+        part.append(0 if T == 0 else min(k - 1, (k * off) // T))
+        off += int(b)
+    return part
+
+
+def plan(cost, mode: str, k: int = 1):
+    """Returns (method[n], slot[n], serial flag) for one of the five engine options
+     plus the greedy comparison."""
+    n = len(cost["load_ns"])
+    if mode == "BASELINE":
+        return [LOAD] * n, [0] * n, True
+    if mode == "PIPESWITCH":
+        return [LOAD] * n, [0] * n, False
+    if mode == "GREEDY":
+        return greedy(cost), [0] * n, False
+    if mode == "DHA":
+        return algorithm1(cost), [0] * n, False
+    if mode in ("PT", "PT_DHA"):
+        method = algorithm1(cost) if mode == "PT_DHA" else [LOAD] * n
+        part = partition(cost["bytes"], k)
+        slot = [0] * n
+        for i in range(n):
+            if part[i] >= 1:
+                slot[i] = part[i]
+                method[i] = LOAD
+        return method, slot, False
+    raise ValueError(mode)
+
+
+# ------------------------------------------------------------------------------------
+# P4: exhaustive search over method vectors (partition fixed), vectorised.
+# Ties -> lexicographically smallest method vector (LOAD=0 < DHA=1).
+# ------------------------------------------------------------------------------------
+
+def simulate_batch(cost, methods: np.ndarray, slot=None, k: int = 1) -> np.ndarray:
+    """Vectorised P1 latency over P method vectors (methods: [P, n] of 0/1)."""
+    P, n = methods.shape
+    load = np.asarray(cost["load_ns"], dtype=np.int64)
+    fwd = np.asarray(cost["fwd_ns"], dtype=np.int64)
+    em = np.asarray(cost["exe_mem_ns"], dtype=np.int64)
+    ed = np.asarray(cost["exe_dha_ns"], dtype=np.int64)
+    slot = np.zeros(n, dtype=np.int64) if slot is None else np.asarray(slot, dtype=np.int64)
+    t_link = np.zeros((k, P), dtype=np.int64)
+    t_fwd = np.zeros((k, P), dtype=np.int64)
+    t = np.zeros(P, dtype=np.int64)
+    for i in range(n):
+        is_dha = methods[:, i] == DHA
+        s = int(slot[i])
+        t_link[s] = np.where(is_dha, t_link[s], t_link[s] + load[i])
+        if s == 0:
+            avail = np.where(is_dha, 0, t_link[0])
+        else:
+            t_fwd[s] = np.where(is_dha, t_fwd[s], np.maximum(t_link[s], t_fwd[s]) + fwd[i])
+            avail = np.where(is_dha, 0, t_fwd[s])
+        t = np.maximum(t, avail) + np.where(is_dha, ed[i], em[i])
+    return t
+
+
+def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 18):
+    """Optimal method vector under P1 with the P3 partition fixed (units with part >= 1
+    are LOAD on their slot).  ``free``: indices allowed to vary (default: all part-0
+    units); others keep ``base_method``.  Returns (latency, method, slot)."""
+    n = len(cost["load_ns"])
+    part = partition(cost["bytes"], k) if k > 1 else [0] * n
+    slot = list(part)
+    if free is None:
+        free = [i for i in range(n) if part[i] == 0]
+    base = np.array([LOAD] * n if base_method is None else base_method, dtype=np.int8)
+    for i in range(n):
+        if part[i] >= 1:
+            base[i] = LOAD
+    m = len(free)
+    best_lat, best_idx = None, None
+    total = 1 << m
+    for lo in range(0, total, chunk):
+        idx = np.arange(lo, min(total, lo + chunk), dtype=np.int64)
+        methods = np.repeat(base[None, :], len(idx), axis=0)
+        for b, u in enumerate(free):  # free[0] is the most significant bit -> lexicographic
+            methods[:, u] = (idx >> (m - 1 - b)) & 1
+        lat = simulate_batch(cost, methods, slot, k)
+        j = int(np.argmin(lat))  # first minimum = lexicographically smallest
+        if best_lat is None or lat[j] < best_lat:
+            best_lat, best_idx = int(lat[j]), int(idx[j])
+    method = base.copy()
+    for b, u in enumerate(free):
+        method[u] = (best_idx >> (m - 1 - b)) & 1
+    return best_lat, [int(x) for x in method], slot
