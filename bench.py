@@ -1,0 +1,380 @@
+#!/usr/bin/env python
+"""Cold-start benchmark (BASELINE.json metric: cold-start BERT-Base/Large inference latency ms
+at 1/2/4/8 GPUs).
+
+One step = one cold-start inference of the whole hot path: the model's weights start in the
+library's pinned host arena and are NOT resident on the GPU; the step runs the DeepPlan
+plan (Algorithm 1 DHA selection; PT over the other ranks' PCIe links when N > 1) through
+dp_infer_cold -- DMA + NCCL gather + event-gated kernels -- and ends when last_hidden_state
+and the pooler output are in HBM.  Between steps the model is evicted (outside the timed
+region) and L2 is flushed (a 256 MiB write).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--model bert_base] [--seq 128]
+  python bench.py --impl reference ...   # the fp64 CPU oracle, timed on the host cores
+
+Multi-GPU: one process per GPU under torch.distributed.run; rank 0 is the primary.  The
+timed region is bracketed by a barrier + cuda synchronize on both sides; the value is the
+max over ranks of the device-timed mean step latency.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "cold-start BERT-Base/Large inference latency ms at 1/2/4/8 GPUs; p99 serving"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--model", default="bert_base")
+    ap.add_argument("--seq", type=int, default=128)
+    ap.add_argument("--batch", type=int, default=1)
+    ap.add_argument("--mode", default=None, help="plan mode (default DHA at N=1, PT_DHA at N>1)")
+    ap.add_argument("--chunk-mb", type=float, default=4.0)
+    ap.add_argument("--h2d-streams", type=int, default=1)
+    ap.add_argument("--profile-iters", type=int, default=10)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        out, _ = self.proc.communicate(timeout=10)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[3:7]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        return json.load(open(p)), "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+def cpu_oracle_ms(m, w, ids, dtype, budget_s=15.0, max_runs=10):
+    """The oracle (fp64 numpy) timed on this host's cores, on a bounded sample."""
+    from oracle import forward as F
+    t0 = time.perf_counter()
+    F.forward(m, w, ids, dtype)  # warm-up (also the first sample if it is slow)
+    first = time.perf_counter() - t0
+    runs = max(1, min(max_runs, int(budget_s / max(first, 1e-3))))
+    ts = []
+    for _ in range(runs):
+        t = time.perf_counter()
+        F.forward(m, w, ids, dtype)
+        ts.append(time.perf_counter() - t)
+    return float(np.median(ts) * 1e3), runs
+
+
+def run_reference(a):
+    """--impl reference: the CPU oracle on the host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import synth
+    m = synth.SHAPES[a.model]
+    w = synth.make_weights(m, seed=0, dtype="fp16")
+    ids = synth.make_ids(m, a.batch, a.seq, seed=1)
+    from oracle import forward as F
+    for _ in range(max(1, min(a.warmup, 2))):
+        F.forward(m, w, ids, "fp16")
+    ts = []
+    steps = max(1, min(a.steps, 10))
+    for _ in range(steps):
+        t = time.perf_counter()
+        F.forward(m, w, ids, "fp16")
+        ts.append((time.perf_counter() - t) * 1e3)
+    v = float(np.mean(ts))
+    cores = os.cpu_count()
+    line = {"metric": METRIC, "value": round(v, 4), "unit": "ms", "n_gpus": a.gpus, "steps": steps,
+            "warmup": a.warmup, "ms_per_step": round(v, 4), "higher_is_better": False, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded random-init weights, paper recipe)",
+            "impl": "reference",
+            "config": {"workload": f"{a.model} fp16-rounded weights, batch {a.batch}, seq {a.seq}, full forward "
+                                   f"on the host CPU (no transfer: weights already in host DRAM)"},
+            "cpu_baseline": {"value": round(v, 4), "unit": "ms", "cores": cores, "kind": "oracle",
+                             "sample": f"{steps} full forwards (fp64 numpy, BLAS threads = {cores})"},
+            "e2e": {"value": round(v, 4), "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+        return
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_eurosys_jeongba23_b200 as dp
+    import synth
+    from oracle import units as OU  # noqa: F401  (byte accounting cross-check only)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world == a.gpus, f"--gpus {a.gpus} but WORLD_SIZE {world}"
+    torch.cuda.set_device(local)
+    dist_on = world > 1
+    if dist_on:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    m = synth.SHAPES[a.model]
+    dtype = "fp16"
+    w = synth.make_weights(m, seed=0, dtype=dtype)
+    ids_np = synth.make_ids(m, a.batch, a.seq, seed=1)
+    ctx = dp.Context([local])
+    ctx.set_opts(chunk_bytes=int(a.chunk_mb * (1 << 20)), n_h2d_streams=a.h2d_streams)
+    model = dp.Model(ctx, m, w, dtype)
+    if dist_on:
+        uid = dp.peer_unique_id() if rank == 0 else None
+        box = [uid]
+        dist.broadcast_object_list(box, src=0)
+        ctx.peer_init(box[0], rank, world)
+
+    # profile on the primary, plan, share the plan (the plan never names GPUs)
+    mode = a.mode or ("PT_DHA" if world > 1 else "DHA")
+    if rank == 0:
+        cost = model.profile(local, a.batch, a.seq, a.profile_iters)
+    else:
+        cost = None
+    if dist_on:
+        box = [cost]
+        dist.broadcast_object_list(box, src=0)
+        cost = box[0]
+    plan = dp.plan_generate(cost, mode, world)
+    pred_ns, _, link = dp.plan_simulate(cost, plan)
+
+    T = a.batch * a.seq
+    H = m.hidden
+    stream = torch.cuda.Stream()
+    ids = torch.from_numpy(ids_np).cuda()
+    out = torch.empty(T, H, dtype=torch.float16, device="cuda")
+    pooled = torch.empty(a.batch, H, dtype=torch.float16, device="cuda") if m.family != "gpt2" else None
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(a.steps)]
+    ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(a.steps)]
+
+    def step(i=None, timed=False):
+        model.evict(local) if model.is_resident(local) else None
+        flush.fill_(i or 0)  # L2 flush (outside the timed region)
+        torch.cuda.synchronize()
+        with torch.cuda.stream(stream):
+            if timed:
+                ev0[i].record(stream)
+            if rank == 0:
+                st = model.infer_cold(plan, 0, ids, out, pooled, stream=stream)
+            else:
+                st = model.infer_cold_raw(plan, 0, None, a.batch, a.seq, None, None, stream.cuda_stream)
+            if timed:
+                ev1[i].record(stream)
+        return st
+
+    def sync_all():
+        torch.cuda.synchronize()
+        if dist_on:
+            dist.barrier()
+            torch.cuda.synchronize()
+
+    for _ in range(max(3, a.warmup)):
+        step()
+        sync_all()
+    # timed region
+    clocks = ClockSampler(local)
+    clocks.start()
+    sync_all()
+    stats = None
+    for i in range(a.steps):
+        stats = step(i, timed=True)
+        # secondaries must finish before the next eviction; the primary waits on its stream
+        torch.cuda.synchronize()
+        if dist_on:
+            dist.barrier()
+    sync_all()
+    ck = clocks.stop()
+    lat = [ev0[i].elapsed_time(ev1[i]) for i in range(a.steps)]
+    my_ms = float(np.mean(lat))
+    t = torch.tensor([my_ms], dtype=torch.float64, device="cuda")
+    if dist_on:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+
+    # ---- e2e: host buffers through the public API (H2D ids + D2H outputs inside) ----
+    e2e_ms = None
+    h2d_b = ids_np.nbytes
+    d2h_b = out.numel() * 2 + (pooled.numel() * 2 if pooled is not None else 0)
+    if rank == 0 or dist_on:
+        ids_h = torch.from_numpy(ids_np).pin_memory()
+        out_h = torch.empty(out.shape, dtype=out.dtype).pin_memory()
+        pool_h = torch.empty(pooled.shape, dtype=pooled.dtype).pin_memory() if pooled is not None else None
+        e2e = []
+        for i in range(min(a.steps, 10)):
+            model.evict(local) if model.is_resident(local) else None
+            flush.fill_(1)
+            sync_all()
+            s0 = torch.cuda.Event(enable_timing=True)
+            s1 = torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(stream):
+                s0.record(stream)
+                if rank == 0:
+                    ids.copy_(ids_h, non_blocking=True)
+                    model.infer_cold(plan, 0, ids, out, pooled, stream=stream)
+                    out_h.copy_(out, non_blocking=True)
+                    if pool_h is not None:
+                        pool_h.copy_(pooled, non_blocking=True)
+                else:
+                    model.infer_cold_raw(plan, 0, None, a.batch, a.seq, None, None, stream.cuda_stream)
+                s1.record(stream)
+            stream.synchronize()
+            e2e.append(s0.elapsed_time(s1))
+            if dist_on:
+                dist.barrier()
+        t = torch.tensor([float(np.mean(e2e))], dtype=torch.float64, device="cuda")
+        if dist_on:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_ms = float(t.item())
+
+    # ---- roofline of the path: PCIe host link (the copy engine + DHA reads) ----
+    peak_h2d = None
+    if rank == 0:
+        hb = torch.empty(256 << 20, dtype=torch.uint8).pin_memory()
+        db = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+        best = 1e9
+        for _ in range(3):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            db.copy_(hb, non_blocking=True)
+            e1.record()
+            torch.cuda.synchronize()
+            best = min(best, e0.elapsed_time(e1))
+        peak_h2d = hb.numel() / (best * 1e-3) / 1e9
+        del hb, db
+
+    if rank != 0:
+        if dist_on:
+            dist.destroy_process_group()
+        return
+
+    # warm latency (the compute-only term of the north-star roofline)
+    model.evict(local) if model.is_resident(local) else None
+    model.infer_cold(plan, 0, ids, out, pooled, stream=stream)
+    torch.cuda.synchronize()
+    wl = []
+    for i in range(10):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            e0.record(stream)
+            wst = model.infer_warm(local, ids, out, pooled, stream=stream)
+            e1.record(stream)
+        torch.cuda.synchronize()
+        wl.append(e0.elapsed_time(e1))
+    warm_ms = float(np.median(wl))
+    model.evict(local)
+
+    h2d_bytes = int(sum(stats["h2d_bytes"]))
+    dha_bytes = int(stats["dha_weight_bytes"])
+    link_bytes = h2d_bytes + dha_bytes  # bytes the path must move over host links per step
+    per_link = max(stats["h2d_bytes"][:world]) + dha_bytes
+    achieved = link_bytes / (ms * 1e-3) / 1e9
+    total_w = model.nbytes
+    R_lit = total_w / (peak_h2d * world * 1e9) * 1e3  # all weight bytes / aggregate H2D
+    R_alg = per_link / (peak_h2d * 1e9) * 1e3          # busiest link's algorithmic bytes
+    peaks, peaks_src = measured_peaks()
+
+    cpu = None
+    if not a.no_cpu_baseline:
+        cms, runs = cpu_oracle_ms(m, w, ids_np, dtype)
+        cpu = {"value": round(cms, 3), "unit": "ms", "cores": os.cpu_count(), "kind": "oracle",
+               "sample": f"{runs} full {a.model} forwards (batch {a.batch}, seq {a.seq}), fp64 numpy; "
+                         f"weights already in host DRAM (no transfer)"}
+
+    line = {
+        "metric": METRIC, "value": round(ms, 4), "unit": "ms", "n_gpus": world, "steps": a.steps,
+        "warmup": max(3, a.warmup), "ms_per_step": round(ms, 4), "higher_is_better": False, "scaling": "strong",
+        "vs_baseline": None, "dtype": "fp16", "data": "synthetic (seeded random-init weights of the HF shapes)",
+        "config": {"workload": f"{a.model} fp16 batch {a.batch} seq {a.seq} cold start from pinned host memory, "
+                               f"plan {mode} k={world}",
+                   "model": a.model, "global_batch": a.batch, "seq_len": a.seq, "parallelism": f"pt{world}",
+                   "plan_mode": mode, "dha_units": int(plan.method.sum()), "units": int(len(plan.method)),
+                   "chunk_bytes": int(a.chunk_mb * (1 << 20)), "h2d_streams": a.h2d_streams,
+                   "l2": "flushed between steps (256 MiB write)"},
+        "roofline": {"bound": "pcie", "achieved": round(achieved, 2), "peak": round(peak_h2d, 2), "unit": "GB/s",
+                     "frac": round(achieved / (peak_h2d * world), 4), "traffic": None,
+                     "bytes_per_step": link_bytes, "peak_source": "pinned 256 MiB H2D measured in this run",
+                     "note": "dominant component is the host-link transfer (copy engine + DHA reads); "
+                             "ncu cannot see copy-engine traffic"},
+        "path_roofline": {"R_literal_ms": round(R_lit, 4), "R_algorithmic_ms": round(R_alg, 4),
+                          "T_warm_ms": round(warm_ms, 4), "bound_ms": round(max(R_lit, warm_ms), 4),
+                          "value_over_R_literal": round(ms / max(R_lit, warm_ms), 4),
+                          "value_over_R_algorithmic": round(ms / max(R_alg, warm_ms), 4),
+                          "predicted_ms": round(pred_ns / 1e6, 4)},
+        "clocks": ck,
+        "e2e": {"value": round(e2e_ms, 4) if e2e_ms else None, "unit": "ms", "h2d_bytes_per_step": int(h2d_b),
+                "d2h_bytes_per_step": int(d2h_b)},
+        "gpu_launches": int(stats["n_kernels"]) * a.steps,
+        "stats": {"h2d_bytes": h2d_bytes, "dha_weight_bytes": dha_bytes, "copies": stats["n_copies"],
+                  "events": stats["n_events"], "kernels_per_step": stats["n_kernels"],
+                  "enqueue_us": round(stats["wall_enqueue_us"], 1), "step_ms_min": round(min(lat), 4),
+                  "step_ms_max": round(max(lat), 4), "warm_kernels": wst["n_kernels"]},
+        "peaks": {"source": peaks_src, "hbm_gbs": peaks.get("hbm_gbs"),
+                  "bf16_tflops_sustained": peaks.get("bf16_tflops_sustained")},
+        "cpu_baseline": cpu,
+    }
+    print(json.dumps(line), flush=True)
+    model.close()
+    ctx.close()
+    if dist_on:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

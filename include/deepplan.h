@@ -1,0 +1,343 @@
+/*
+ * deepplan.h -- C-ABI of the B200-native DeepPlan cold-start hot path.
+ *
+ * Paper: Jeong, Baek, Ahn, "Fast and Efficient Model Serving Using Multi-GPUs with
+ * Direct-Host-Access", EuroSys '23.  Citations "P:<n>" are lines of PAPER.md.
+ *
+ * DeepPlan "takes a pre-trained DL model as an input", profiles each layer (P:198,
+ * §4.3.1), generates an execution plan (Algorithm 1, transmission
+ * planning P:227-229) and deploys it to an engine with five execution options --
+ * Baseline, PipeSwitch, DHA, PT, PT+DHA -- whose load / migration / execution
+ * streams are coordinated by per-layer CUDA events (§4.3.4).  This header
+ * exposes exactly those steps.
+ *
+ * Conventions
+ *  - Every function returns dp_status: DP_OK (0) or a negative error code.  On error,
+ *    dp_last_error() returns a thread-local message.  No C++ exception crosses the ABI.
+ *  - "Device pointer": memory of the named CUDA device (allocated by the caller, e.g.
+ *    torch).  "Host pointer": ordinary host memory, read synchronously during the call.
+ *  - Streams are passed as void* (a cudaStream_t; NULL = legacy default stream).
+ *  - All int64 times are nanoseconds.  Method encoding: DP_LOAD = 0, DP_DHA = 1.
+ *  - Thread safety: a dp_context and the models registered with it must be used from one
+ *    host thread at a time (the serving harness runs its own worker threads internally).
+ */
+#ifndef DEEPPLAN_H_
+#define DEEPPLAN_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+#if defined(__GNUC__)
+#pragma GCC visibility push(default) /* the library builds with -fvisibility=hidden */
+#endif
+
+typedef int32_t dp_status;
+#define DP_OK 0
+#define DP_ERR_INVALID (-1)     /* bad argument / shape mismatch */
+#define DP_ERR_CUDA (-2)        /* a CUDA runtime/driver call failed */
+#define DP_ERR_NCCL (-3)        /* an NCCL call failed */
+#define DP_ERR_OOM (-4)         /* host (pinned) or device allocation failed */
+#define DP_ERR_UNSUPPORTED (-5) /* valid request this build does not implement */
+#define DP_ERR_STATE (-6)       /* call not valid in the object's current state */
+
+#define DP_LOAD 0 /* "O": load-then-execute (Table 3 caption) */
+#define DP_DHA 1  /* "X": direct-host-access */
+#define DP_INF_NS ((int64_t)1 << 50) /* exe_dha_ns of a DHA-ineligible unit */
+#define DP_MAX_DEVICES 8
+
+/* Model families of the paper's transformer workloads. */
+enum { DP_FAMILY_BERT = 0, DP_FAMILY_ROBERTA = 1, DP_FAMILY_GPT2 = 2 };
+/* Weight storage dtypes (the paper never states one; fp16 is the default). */
+enum { DP_FP16 = 0, DP_BF16 = 1 };
+/* Planning-unit kinds (Table 3: Emb, LN, FC). */
+enum { DP_UNIT_EMB = 0, DP_UNIT_LN = 1, DP_UNIT_LINEAR = 2 };
+/* Engine options + the "initial approach" of P:41 (GREEDY). */
+enum {
+  DP_MODE_BASELINE = 0,   /* load every layer, then execute (Fig.1b) */
+  DP_MODE_PIPESWITCH = 1, /* per-layer load/execute pipelining, all LOAD (Fig.1c, [6]) */
+  DP_MODE_GREEDY = 2,     /* DHA iff Exe(DHA) < Load + Exe(InMem), layer by layer */
+  DP_MODE_DHA = 3,        /* Algorithm 1 */
+  DP_MODE_PT = 4,         /* parallel transmission, all LOAD (§4.2) */
+  DP_MODE_PT_DHA = 5      /* Algorithm 1 on partition 0 + PT for the rest */
+};
+
+/* ---------------------------------------------------------------------------------
+ * Errors
+ * --------------------------------------------------------------------------------- */
+const char* dp_last_error(void);
+int32_t dp_abi_version(void); /* 1 */
+
+/* ---------------------------------------------------------------------------------
+ * Planner (pure host code, deterministic, no GPU).  §4.3.2-4.3.3, SURVEY §8(c) P1-P4.
+ * --------------------------------------------------------------------------------- */
+
+/* Per-unit performance table ("performance table"; Fig.10).
+ * All arrays have n entries, caller-owned.  fwd_ns = secondary->primary NVLink time
+ * (our addition for PT).  exe_dha_ns = DP_INF_NS marks DHA-ineligible units. */
+typedef struct {
+  int32_t n;
+  const int64_t* bytes;
+  const int64_t* load_ns;
+  const int64_t* fwd_ns;
+  const int64_t* exe_mem_ns;
+  const int64_t* exe_dha_ns;
+} dp_cost_table;
+
+/* Execution plan: per unit a method (DP_LOAD/DP_DHA) and a slot (0 = the primary GPU's
+ * own PCIe link; s >= 1 = PT partition s, forwarded over NVLink).  The plan
+ * never names GPUs ("we do not statically assign the GPU"). `serial` = 1 only for
+ * DP_MODE_BASELINE (no overlap).  method/slot are caller-owned arrays of n entries. */
+typedef struct {
+  int32_t n;
+  int32_t mode;
+  int32_t k; /* number of GPUs whose links carry the model (1 = no PT) */
+  int32_t serial;
+  int8_t* method;
+  int8_t* slot;
+} dp_plan;
+
+/* Generate a plan (fills out->method/slot/serial/mode/k; out->n must equal cost->n).
+ * DP_ERR_INVALID on n mismatch, k < 1 or k > DP_MAX_DEVICES, unknown mode. */
+dp_status dp_plan_generate(const dp_cost_table* cost, int32_t mode, int32_t k, dp_plan* out);
+
+/* Pipeline cost model: latency, per-unit stall (n entries, nullable) and
+ * bytes carried by each link (k entries, nullable). */
+dp_status dp_plan_simulate(const dp_cost_table* cost, const dp_plan* plan, int64_t* latency_ns,
+                           int64_t* stall_ns, int64_t* link_bytes);
+
+/* Equal-size contiguous partition ("equally partition ... in terms of size"):
+ * part[i] = min(k-1, (k * offset_i) / total_bytes).  part: n int8, caller-owned. */
+dp_status dp_plan_partition(const int64_t* bytes, int32_t n, int32_t k, int8_t* part);
+
+/* Exhaustive search (optimal under the cost model) over the methods of the `nfree` units
+ * listed in free_idx (<= 30), all other units keep base->method; PT partition fixed as in
+ * DP_MODE_PT_DHA when base->k > 1.  Ties -> lexicographically smallest method vector.
+ * out gets the best plan, *latency_ns its latency. */
+dp_status dp_plan_exhaustive(const dp_cost_table* cost, const dp_plan* base, const int32_t* free_idx,
+                             int32_t nfree, dp_plan* out, int64_t* latency_ns);
+
+/* ---------------------------------------------------------------------------------
+ * Context (devices, streams, events, workspaces, peer transport)
+ * --------------------------------------------------------------------------------- */
+typedef struct dp_context dp_context;
+
+/* devs: CUDA device ordinals usable by this context (1..8).  Creates per device: an
+ * execution stream role (the caller's stream is used), `n_h2d` load streams (P:231
+ * "load stream"), a migration stream, an event pool. */
+dp_status dp_context_create(const int32_t* devs, int32_t ndev, dp_context** out);
+dp_status dp_context_destroy(dp_context* ctx);
+
+/* Engine tunables (defaults in brackets).  chunk_bytes: adjacent LOAD units are
+ * coalesced into one DMA of up to this many bytes [4 MiB] (one completion event per
+ * chunk); n_h2d_streams: load streams per GPU used round-robin [1]; use_graph: capture
+ * the cold-start into a CUDA graph per (model, plan, shape, buffers) [0]. */
+typedef struct {
+  int64_t chunk_bytes;
+  int32_t n_h2d_streams;
+  int32_t use_graph;
+  int32_t gemm_bn;        /* 0 = auto */
+  int32_t debug_delay_us; /* fault injection: stall every load/migration stream this long
+                             before each transfer (tests event gating) [0] */
+  int32_t debug_poison;   /* 1 = fill HBM slots with 0xFF (NaN) on eviction [0] */
+  int32_t reserved[5];
+} dp_engine_opts;
+dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* opts);
+dp_status dp_context_get_opts(dp_context* ctx, dp_engine_opts* out);
+
+/* Multi-process PT (one process per GPU, P:182 migration over NVLink): every rank
+ * calls dp_peer_init with the same 128-byte NCCL unique id (rank 0 creates it with
+ * dp_peer_unique_id and the caller distributes it, e.g. via torch.distributed).  The
+ * gather uses ncclSend/ncclRecv only.  DP_ERR_NCCL on failure. */
+dp_status dp_peer_unique_id(void* out128);
+dp_status dp_peer_init(dp_context* ctx, const void* uid128, int32_t rank, int32_t nranks);
+
+/* ---------------------------------------------------------------------------------
+ * Model registration: host weight arena ("we allocate the pinned memory for the
+ * layers ... through cudaHostAlloc")
+ * --------------------------------------------------------------------------------- */
+typedef struct {
+  int32_t family;     /* DP_FAMILY_* */
+  int32_t vocab, max_pos, type_vocab, hidden, heads, ffn, layers;
+  int32_t dtype;      /* DP_FP16 | DP_BF16 */
+  int32_t pad_idx;    /* RoBERTa: position ids start at pad_idx + 1 */
+  double ln_eps;
+} dp_model_config;
+
+typedef struct dp_model dp_model;
+
+typedef struct {
+  int32_t kind;          /* DP_UNIT_* */
+  int32_t nparams;       /* 1 (embedding) or 2 (weight+bias / gamma+beta) */
+  int32_t first_param;   /* index into the parameter list (dp_model_param_info) */
+  int32_t reserved;
+  int64_t bytes;         /* payload bytes (what a load moves) */
+  int64_t arena_offset;  /* byte offset in the arena (256 B aligned) */
+  char name[32];         /* e.g. "word", "L3.fc1", "ln_f" */
+} dp_unit_info;
+
+typedef struct {
+  char hf_name[96];      /* HF state-dict key, e.g. "encoder.layer.0.attention.self.query.weight" */
+  int32_t ndim;          /* 1 or 2 */
+  int32_t unit;          /* owning unit */
+  int64_t shape[2];      /* as the caller supplies it (HF layout; GPT-2 Conv1D is [in,out]) */
+  int64_t bytes;
+} dp_param_info;
+
+/* Parameter list for a config, BEFORE creating a model (so the caller can marshal by
+ * name).  *count gets the number of params; infos (nullable) gets min(cap,count). */
+dp_status dp_config_params(const dp_model_config* cfg, dp_param_info* infos, int32_t cap, int32_t* count);
+
+/* Register a model: host_params[i] is a host pointer to parameter i (dp_config_params
+ * order) in the storage dtype, row-major, HF layout.  The library COPIES them into its
+ * own pinned, mapped, portable arena (GPT-2 Conv1D weights are transposed to [out,in]
+ * there) and owns that arena.  DP_ERR_INVALID on bad config; DP_ERR_OOM if pinning fails. */
+dp_status dp_model_create(dp_context* ctx, const dp_model_config* cfg, const void* const* host_params,
+                          int32_t nparams, dp_model** out);
+dp_status dp_model_destroy(dp_context* ctx, dp_model* m);
+int32_t dp_model_num_units(const dp_model* m);
+dp_status dp_model_unit_info(const dp_model* m, int32_t i, dp_unit_info* out);
+int64_t dp_model_bytes(const dp_model* m);
+/* Host (mapped) address of the arena, for tests that read it back. */
+dp_status dp_model_arena(const dp_model* m, const void** ptr, int64_t* bytes);
+
+/* ---------------------------------------------------------------------------------
+ * Profiling (§4.3.1; Table 5).  Per unit, median over `iters`
+ * (after 3 warm-ups) of: load_ns (H2D of the unit alone on dev's link), fwd_ns (a peer
+ * copy of the unit's bytes; on a 1-GPU context a device-to-device copy), exe_mem_ns /
+ * exe_dha_ns (the unit's kernels with its weights in HBM / host-mapped, L2 flushed).
+ * out arrays: n entries each (caller-owned; out->n must equal the unit count).
+ * --------------------------------------------------------------------------------- */
+dp_status dp_profile(dp_context* ctx, dp_model* m, int32_t dev, int32_t batch, int32_t seq, int32_t iters,
+                     dp_cost_table* out);
+
+/* ---------------------------------------------------------------------------------
+ * Inference (§4.3.4, Fig.9)
+ * --------------------------------------------------------------------------------- */
+#define DP_STATS_MAX_UNITS 512
+typedef struct {
+  int64_t h2d_bytes[DP_MAX_DEVICES];    /* bytes DMA'd host->device over each slot's link */
+  int64_t nvlink_bytes[DP_MAX_DEVICES]; /* bytes gathered from slot s into the primary */
+  int64_t dha_weight_bytes;             /* weight bytes DHA kernels must read (algorithmic) */
+  int32_t n_copies;                     /* DMA operations issued */
+  int32_t n_events;                     /* completion events recorded */
+  int32_t n_kernels;                    /* kernels launched on the execution stream */
+  int32_t n_units;
+  float wall_enqueue_us;                /* host time spent enqueuing */
+  float reserved[3];
+} dp_run_stats;
+
+/* Cold start: the model is NOT resident on `primary`.  Weights are read from the host
+ * arena per `plan`: DHA units in place by the DHA kernels; slot-0 LOAD units DMA'd over
+ * the primary's link on load streams; slot-s LOAD units via PT over secondaries[s-1]
+ * (device ordinals in a single-process context, or NCCL ranks after dp_peer_init; a
+ * secondary equal to the primary means loopback: staged and forwarded on one GPU).
+ * Execution is enqueued on `stream` (the execution stream); every non-DHA unit's first
+ * kernel waits on its load event.  d_ids: int32 [batch*seq] on the primary;
+ * d_out: [batch*seq*hidden] storage dtype; d_pooled: [batch*hidden] or NULL (BERT/
+ * RoBERTa pooler).  On return the work is enqueued (asynchronous); the model is then
+ * resident on the primary with the plan's DHA units left in host memory.
+ * On a secondary rank (after dp_peer_init) only that rank's transfers are enqueued and
+ * d_ids/d_out may be NULL.  DP_ERR_STATE if already resident on the primary. */
+dp_status dp_infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int32_t primary,
+                        const int32_t* secondaries, int32_t nsec, const int32_t* d_ids, int32_t batch,
+                        int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats);
+
+/* Warm inference: the model is resident on dev (DP_ERR_STATE otherwise). */
+dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, const int32_t* d_ids, int32_t batch,
+                        int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats);
+
+/* Residency: make the model non-resident on dev (its HBM slots return to the pool).
+ * Synchronises the device's streams first. */
+dp_status dp_model_evict(dp_context* ctx, dp_model* m, int32_t dev);
+int32_t dp_model_is_resident(const dp_model* m, int32_t dev);
+
+/* ---------------------------------------------------------------------------------
+ * Kernel entry points (parity-test hooks; same kernels the executor launches).
+ * Pointers may be device memory or host memory from dp_host_alloc (mapped) -- the
+ * kernels read host memory in place over PCIe (direct-host-access).
+ * --------------------------------------------------------------------------------- */
+/* Pinned, mapped, portable host memory (cudaHostAlloc) and its release. */
+dp_status dp_host_alloc(int64_t bytes, void** out);
+dp_status dp_host_free(void* p);
+
+/* Embedding: x[t,:] = LN(word[ids[t]] + pos[p(t)] + type[0]) for BERT/
+ * RoBERTa (ln_g/ln_b non-NULL), or wte[ids[t]] + wpe[p(t)] for GPT-2 (type, ln NULL).
+ * p(t) = pos_offset + (t mod seq).  Every table pointer may be host-mapped (DHA). */
+dp_status dp_embed(const int32_t* d_ids, int32_t ntok, int32_t seq, int32_t pos_offset, const void* word,
+                   const void* pos, const void* type, const void* ln_g, const void* ln_b, int32_t hidden,
+                   double eps, int32_t dtype, void* d_out, void* stream);
+
+/* Linear: y[M,N] = act(x[M,K] w[N,K]^T + b) + residual, row strides ldx/ldy/ldr in
+ * elements.  act: 0 none, 1 gelu_erf, 2 gelu_tanh, 3 tanh.  path: 0 = resident tcgen05/
+ * TMA GEMM (w must be device memory, N % 128 == 0, K % 64 == 0), 1 = DHA skinny linear
+ * (w may be host-mapped; reads every weight byte once). */
+dp_status dp_linear(const void* x, int32_t ldx, const void* w, const void* b, const void* residual, int32_t ldr,
+                    void* y, int32_t ldy, int32_t M, int32_t N, int32_t K, int32_t act, int32_t path, int32_t dtype,
+                    void* stream);
+
+/* LayerNorm over rows of width n: y = LN(x (+ r)) * g + b.  g/b may be host-mapped. */
+dp_status dp_layernorm(const void* x, const void* r, const void* g, const void* b, void* y, int32_t rows,
+                       int32_t n, double eps, int32_t dtype, void* stream);
+
+/* Attention core: qkv [ntok, 3H] (q | k | v column blocks, row stride ldqkv), heads of
+ * d = H/heads (d == 64), softmax(q k^T / sqrt(d) [+ causal mask]) v -> ctx [ntok, H].
+ * Sequences are contiguous blocks of `seq` tokens. */
+dp_status dp_attention(const void* qkv, int32_t ldqkv, void* ctx_out, int32_t batch, int32_t seq, int32_t hidden,
+                       int32_t heads, int32_t causal, int32_t dtype, void* stream);
+
+/* ---------------------------------------------------------------------------------
+ * Serving harness (§5.3): one inference per GPU at a time (Clockwork-like),
+ * on-demand cold starts, LRU eviction under a per-GPU byte budget, PT over <= k GPUs.
+ * --------------------------------------------------------------------------------- */
+typedef struct {
+  int64_t arrival_ns; /* offset from trace start */
+  int32_t instance;   /* which model instance the request targets */
+  int32_t reserved;
+} dp_trace_event;
+
+typedef struct {
+  int32_t plan_mode;             /* DP_MODE_PIPESWITCH | DP_MODE_DHA | DP_MODE_PT_DHA ... */
+  int32_t k_max;                 /* max GPUs per cold start (2 on p3.8xlarge) */
+  int32_t ngpu;                  /* GPUs served (dry-run: any; live: <= context devices) */
+  int32_t dry_run;               /* 1 = replay with the latency table below, no GPU */
+  int64_t per_gpu_budget_bytes;  /* HBM budget for resident instances per GPU */
+  int64_t slo_ns;                /* goodput threshold (100 ms) */
+  /* dry-run latency table, per MODEL index: cold / warm ns, resident bytes */
+  int32_t nmodels;
+  int32_t reserved0;
+  const int64_t* cold_ns;
+  const int64_t* warm_ns;
+  const int64_t* resident_bytes;
+  const int32_t* model_of_instance; /* [ninstances] */
+  int32_t ninstances;
+  int32_t batch, seq;
+  int32_t reserved1;
+  /* live mode: models[i] is instance i's dp_model (nmodels == ninstances) and plans[i]
+   * its cold-start plan; a plan with k > 1 uses the next k-1 GPUs of the context as
+   * secondaries (their PCIe links and copy engines, not their compute) */
+  const dp_plan* const* plans;
+} dp_serve_opts;
+
+typedef struct {
+  int64_t start_ns;    /* when the request began executing */
+  int64_t finish_ns;   /* completion time */
+  int32_t gpu;         /* GPU that ran it */
+  int32_t cold;        /* 1 = cold start */
+  int32_t nevicted;    /* instances evicted to make room */
+  int32_t reserved;
+} dp_serve_result;
+
+/* Replay (dry_run=1) or run live (dry_run=0: models[] are real dp_models, one per
+ * instance, requests are issued at their arrival times on a wall clock).  out: nreq. */
+dp_status dp_serve_run(dp_context* ctx, dp_model* const* models, int32_t nmodels, const dp_trace_event* trace,
+                       int32_t nreq, const dp_serve_opts* opts, dp_serve_result* out);
+
+#if defined(__GNUC__)
+#pragma GCC visibility pop
+#endif
+#ifdef __cplusplus
+}
+#endif
+#endif /* DEEPPLAN_H_ */

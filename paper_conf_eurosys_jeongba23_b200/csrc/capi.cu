@@ -1,0 +1,78 @@
+// C-ABI kernel entry points (parity-test hooks) and pinned host allocation.
+// They launch exactly the kernels the executor launches.
+#include <cuda_runtime.h>
+
+#include "common.h"
+#include "kernels.h"
+
+using namespace dp;
+
+extern "C" dp_status dp_host_alloc(int64_t bytes, void** out) {
+  return guard([&] {
+    DP_CHECK(out && bytes > 0, DP_ERR_INVALID, "bad arguments");
+    cudaError_t e = cudaHostAlloc(out, bytes, cudaHostAllocPortable | cudaHostAllocMapped);
+    if (e != cudaSuccess) fail(DP_ERR_OOM, std::string("cudaHostAlloc failed: ") + cudaGetErrorString(e));
+  });
+}
+
+extern "C" dp_status dp_host_free(void* p) {
+  return guard([&] {
+    if (p) DP_CUDA(cudaFreeHost(p));
+  });
+}
+
+static void check_dtype(int32_t dtype) {
+  DP_CHECK(dtype == DP_FP16 || dtype == DP_BF16, DP_ERR_UNSUPPORTED, "dtype must be DP_FP16 or DP_BF16");
+}
+
+extern "C" dp_status dp_embed(const int32_t* d_ids, int32_t ntok, int32_t seq, int32_t pos_offset, const void* word,
+                              const void* pos, const void* type, const void* ln_g, const void* ln_b, int32_t hidden,
+                              double eps, int32_t dtype, void* d_out, void* stream) {
+  return guard([&] {
+    check_dtype(dtype);
+    DP_CHECK(d_ids && word && pos && d_out, DP_ERR_INVALID, "NULL pointer");
+    DP_CHECK((ln_g == nullptr) == (ln_b == nullptr), DP_ERR_INVALID, "ln_g and ln_b must both be set or NULL");
+    launch_embed(dtype, d_ids, ntok, seq, pos_offset, word, pos, type, ln_g, ln_b, hidden, (float)eps, d_out,
+                 (cudaStream_t)stream);
+  });
+}
+
+extern "C" dp_status dp_linear(const void* x, int32_t ldx, const void* w, const void* b, const void* residual,
+                               int32_t ldr, void* y, int32_t ldy, int32_t M, int32_t N, int32_t K, int32_t act,
+                               int32_t path, int32_t dtype, void* stream) {
+  return guard([&] {
+    check_dtype(dtype);
+    DP_CHECK(x && w && y, DP_ERR_INVALID, "NULL pointer");
+    DP_CHECK(M >= 0 && N > 0 && K > 0 && ldx >= K && ldy >= N && (!residual || ldr >= N), DP_ERR_INVALID,
+             "bad shapes / strides");
+    DP_CHECK(act >= 0 && act <= 3, DP_ERR_INVALID, "act must be 0..3");
+    if (path == 0) {
+      cudaPointerAttributes at;
+      DP_CUDA(cudaPointerGetAttributes(&at, w));
+      DP_CHECK(at.type == cudaMemoryTypeDevice, DP_ERR_INVALID, "the tcgen05 path needs W in device memory");
+      launch_gemm_tc(dtype, x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act, 0, (cudaStream_t)stream);
+    } else if (path == 1) {
+      launch_skinny_linear(dtype, x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act, (cudaStream_t)stream);
+    } else {
+      fail(DP_ERR_INVALID, "path must be 0 (tcgen05) or 1 (skinny/DHA)");
+    }
+  });
+}
+
+extern "C" dp_status dp_layernorm(const void* x, const void* r, const void* g, const void* b, void* y, int32_t rows,
+                                  int32_t n, double eps, int32_t dtype, void* stream) {
+  return guard([&] {
+    check_dtype(dtype);
+    DP_CHECK(x && g && b && y && rows >= 0, DP_ERR_INVALID, "bad arguments");
+    launch_layernorm(dtype, x, r, g, b, y, rows, n, (float)eps, (cudaStream_t)stream);
+  });
+}
+
+extern "C" dp_status dp_attention(const void* qkv, int32_t ldqkv, void* ctx_out, int32_t batch, int32_t seq,
+                                  int32_t hidden, int32_t heads, int32_t causal, int32_t dtype, void* stream) {
+  return guard([&] {
+    check_dtype(dtype);
+    DP_CHECK(qkv && ctx_out && ldqkv >= 3 * hidden, DP_ERR_INVALID, "bad arguments");
+    launch_attention(dtype, qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal != 0, (cudaStream_t)stream);
+  });
+}

@@ -1,0 +1,88 @@
+// fp16 / bf16 <-> fp32 helpers on 16-byte vectors (8 elements).
+#pragma once
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+#include <cstdint>
+
+#include "kernels.h"
+
+namespace dp {
+
+template <class T>
+struct Cvt;
+
+template <>
+struct Cvt<__half> {
+  static __device__ __forceinline__ float2 to2(uint32_t v) {
+    __half2 h = *reinterpret_cast<__half2*>(&v);
+    return __half22float2(h);
+  }
+  static __device__ __forceinline__ uint32_t from2(float a, float b) {
+    __half2 h = __floats2half2_rn(a, b);
+    return *reinterpret_cast<uint32_t*>(&h);
+  }
+  static __device__ __forceinline__ float to1(__half v) { return __half2float(v); }
+  static __device__ __forceinline__ __half from1(float v) { return __float2half_rn(v); }
+};
+
+template <>
+struct Cvt<__nv_bfloat16> {
+  static __device__ __forceinline__ float2 to2(uint32_t v) {
+    __nv_bfloat162 h = *reinterpret_cast<__nv_bfloat162*>(&v);
+    return __bfloat1622float2(h);
+  }
+  static __device__ __forceinline__ uint32_t from2(float a, float b) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+    return *reinterpret_cast<uint32_t*>(&h);
+  }
+  static __device__ __forceinline__ float to1(__nv_bfloat16 v) { return __bfloat162float(v); }
+  static __device__ __forceinline__ __nv_bfloat16 from1(float v) { return __float2bfloat16_rn(v); }
+};
+
+template <class T>
+__device__ __forceinline__ void unpack8(const uint4& u, float* f) {
+  float2 a = Cvt<T>::to2(u.x), b = Cvt<T>::to2(u.y), c = Cvt<T>::to2(u.z), d = Cvt<T>::to2(u.w);
+  f[0] = a.x; f[1] = a.y; f[2] = b.x; f[3] = b.y; f[4] = c.x; f[5] = c.y; f[6] = d.x; f[7] = d.y;
+}
+
+template <class T>
+__device__ __forceinline__ uint4 pack8(const float* f) {
+  uint4 u;
+  u.x = Cvt<T>::from2(f[0], f[1]);
+  u.y = Cvt<T>::from2(f[2], f[3]);
+  u.z = Cvt<T>::from2(f[4], f[5]);
+  u.w = Cvt<T>::from2(f[6], f[7]);
+  return u;
+}
+
+// 16-byte read-only load; works on HBM and on host-mapped (zero-copy) addresses.
+__device__ __forceinline__ uint4 ldg16(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+__device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * (1.0f + erff(x * 0.70710678118654752f)); }
+__device__ __forceinline__ float gelu_tanh(float x) {
+  const float c = 0.7978845608028654f;  // sqrt(2/pi)
+  return 0.5f * x * (1.0f + tanhf(c * (x + 0.044715f * x * x * x)));
+}
+
+__device__ __forceinline__ float apply_act(float v, int act) {
+  switch (act) {
+    case ACT_GELU_ERF: return gelu_erf(v);
+    case ACT_GELU_TANH: return gelu_tanh(v);
+    case ACT_TANH: return tanhf(v);
+    default: return v;
+  }
+}
+
+}  // namespace dp

@@ -1,0 +1,81 @@
+// Execution engine internals: context, per-device resources, forward program.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <functional>
+#include <map>
+#include <vector>
+
+#include "model.h"
+
+namespace dp {
+
+struct EventPool {
+  int dev = -1;
+  std::vector<cudaEvent_t> ev;
+  size_t used = 0;
+  cudaEvent_t get();
+  void reset() { used = 0; }
+  void destroy();
+};
+
+// Resources of one PT slot served by device `dev`: its load stream, its migration stream
+// ("an additional migration stream on each secondary GPU") and the staging ring
+// ("we reserve a small amount of memory for storing layers temporarily").
+struct SlotRes {
+  int dev = -1;
+  cudaStream_t h2d = nullptr, mig = nullptr;
+  void* ring = nullptr;
+  int64_t ring_bytes = 0;
+};
+
+// A contiguous byte range of the arena moved by one DMA (and one forward for PT): the
+// whole units first_unit..last_unit (all selected by the plan for the same link).
+struct Piece {
+  int64_t off = 0, bytes = 0;
+  int first_unit = -1, last_unit = -1;
+};
+
+struct DevCtx {
+  int ord = -1;
+  bool ready = false;
+  std::vector<cudaStream_t> h2d;  // load streams ("load stream")
+  EventPool events;
+  void* flush = nullptr;  // L2 flush buffer (profiling)
+  int64_t flush_bytes = 0;
+};
+
+struct ForwardArgs {
+  dp_model* m = nullptr;
+  int dev = 0;
+  const int8_t* method = nullptr;  // per unit DP_LOAD / DP_DHA (where the weights are read from)
+  const int32_t* ids = nullptr;
+  int batch = 0, seq = 0;
+  void* out = nullptr;
+  void* pooled = nullptr;
+  cudaStream_t stream = nullptr;
+  std::function<void(int)> before_unit;  // called before the first kernel using a unit
+  int kernels = 0;
+  int bn_hint = 0;
+};
+
+void ensure_workspace(dp_model* m, int dev, int64_t tokens);
+void run_forward(ForwardArgs& a);
+
+// Execute one unit's ops in isolation (profiling): inputs are the workspace buffers.
+void run_unit(dp_model* m, int dev, int unit, bool dha, const int32_t* ids, int batch, int seq, cudaStream_t s,
+              int bn_hint);
+
+}  // namespace dp
+
+struct dp_context {
+  std::vector<int> devs;
+  dp::DevCtx dc[DP_MAX_DEVICES];
+  dp_engine_opts opts{};
+  std::map<std::pair<int, int>, dp::SlotRes> slots;  // (slot, device) -> resources
+  // multi-process PT (NCCL)
+  void* comm = nullptr;
+  int rank = -1, nranks = 0;
+  cudaStream_t comm_stream = nullptr;
+  dp::DevCtx& on(int dev);
+};

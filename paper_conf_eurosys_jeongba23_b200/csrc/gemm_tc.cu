@@ -1,0 +1,304 @@
+// K2: resident-weight GEMM on the 5th-generation tensor cores (tcgen05 + TMEM + TMA).
+//
+//   Y[M, N] = act(X[M, K] . W[N, K]^T + bias[N]) (+ R[M, N])
+//
+// Used only for layers whose weights are already in HBM: loaded layers
+// are true dense contractions.  Shapes on the hot path are skinny in M (tokens: 32..1024)
+// and wide in N (768..4096), so the kernel is "swap-AB": the MMA's M axis (128 lanes of
+// TMEM) runs over W's rows (N) and the MMA's N axis over tokens (BN = 32..256 columns).
+//
+// Per CTA (128 threads, one 128 x BN output tile, full K):
+//   warp 0 / lane 0  : TMA producer -- W tile [128 x 64] and X tile [BN x 64] per stage,
+//                      both K-major with the 128-byte swizzle, into a STAGES-deep ring;
+//   warp 1 / lane 0  : MMA issuer  -- 4 x tcgen05.mma (K = 16 each) per stage, fp32
+//                      accumulator in TMEM; tcgen05.commit releases the smem stage;
+//   warp 1           : TMEM allocate / free (BN columns);
+//   all 4 warps      : epilogue -- tcgen05.ld 32 lanes x 16 columns, + bias, activation,
+//                      + residual, store (warp w owns TMEM lanes 32w..32w+31).
+// Descriptor encodings follow the sm_100 UMMA descriptor layout (start>>4, LBO, SBO = 1024 B
+// for 8-row swizzle atoms, version 1, layout SWIZZLE_128B = 2).
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+
+#include "common.h"
+#include "dtype.cuh"
+#include "kernels.h"
+
+namespace dp {
+
+namespace {
+
+constexpr int BM = 128;  // W rows per tile (MMA M)
+constexpr int BK = 64;   // K per stage: 64 x 2 B = one 128-byte swizzle row
+constexpr int STAGES = 4;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  const uint32_t a = smem_u32(bar);
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra WAIT_%=;\n"
+      "}\n" ::"r"(a),
+      "r"(phase)
+      : "memory");
+}
+
+__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ uint64_t sw128_desc(const void* smem_tile) {
+  const uint64_t addr = smem_u32(smem_tile);
+  uint64_t d = 0;
+  d |= (addr & 0x3FFFFull) >> 4;  // start address
+  d |= uint64_t(1) << 16;          // LBO (unused for swizzled K-major)
+  d |= uint64_t(1024 >> 4) << 32;  // SBO: 8 rows x 128 B
+  d |= uint64_t(1) << 46;          // descriptor version (sm_100)
+  d |= uint64_t(2) << 61;          // SWIZZLE_128B
+  return d;
+}
+
+__device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+        "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+template <class T>
+struct FmtBits;
+template <>
+struct FmtBits<__half> {
+  static constexpr uint32_t v = 0;
+};
+template <>
+struct FmtBits<__nv_bfloat16> {
+  static constexpr uint32_t v = 1;
+};
+
+template <class T, int BN>
+__global__ void __launch_bounds__(128, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmX,
+                   const T* __restrict__ bias, const T* res, int ldr, T* Y, int ldy, int M,
+                   int N, int K, int act) {
+  constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
+  constexpr uint32_t B_BYTES = BN * BK * 2;
+  constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
+  constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
+  // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
+  constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
+                             (uint32_t(BM >> 4) << 24);
+
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], done_bar;
+  __shared__ uint32_t tmem_base_sh;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * BM, m0 = blockIdx.y * BN;
+  const int num_kb = K / BK;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full_bar[s], 1);
+      mbar_init(&empty_bar[s], 1);
+    }
+    mbar_init(&done_bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base_sh)),
+                 "r"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem_d = tmem_base_sh;
+
+  if (warp == 0 && lane == 0) {
+    // TMA producer
+    for (int kb = 0; kb < num_kb; ++kb) {
+      const int s = kb % STAGES;
+      if (kb >= STAGES) mbar_wait(&empty_bar[s], ((kb / STAGES) - 1) & 1);
+      uint8_t* a = smem + s * STAGE_BYTES;
+      uint8_t* b = a + A_BYTES;
+      mbar_expect_tx(&full_bar[s], STAGE_BYTES);
+      tma_load_2d(&tmW, &full_bar[s], a, kb * BK, n0);
+      tma_load_2d(&tmX, &full_bar[s], b, kb * BK, m0);
+    }
+  } else if (warp == 1 && lane == 0) {
+    // MMA issuer
+    for (int kb = 0; kb < num_kb; ++kb) {
+      const int s = kb % STAGES;
+      mbar_wait(&full_bar[s], (kb / STAGES) & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      const uint8_t* a = smem + s * STAGE_BYTES;
+      const uint8_t* b = a + A_BYTES;
+      const uint64_t da = sw128_desc(a), db = sw128_desc(b);
+#pragma unroll
+      for (int kk = 0; kk < BK / 16; ++kk)  // advance 16 elements = 32 B = 2 in descriptor units
+        umma_f16(tmem_d, da + 2 * kk, db + 2 * kk, IDESC, (kb | kk) != 0);
+      umma_commit(&empty_bar[s]);
+    }
+    umma_commit(&done_bar);
+  }
+  __syncwarp();
+
+  // Epilogue (all 4 warps)
+  mbar_wait(&done_bar, 0);
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const int n = n0 + warp * 32 + lane;
+  const float bv = (bias != nullptr && n < N) ? Cvt<T>::to1(bias[n]) : 0.f;
+#pragma unroll
+  for (int c0 = 0; c0 < BN; c0 += 16) {
+    uint32_t v[16];
+    tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
+    if (n < N) {
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        const int m = m0 + c0 + j;
+        if (m < M) {
+          float val = apply_act(__uint_as_float(v[j]) + bv, act);
+          if (res) val += Cvt<T>::to1(res[(size_t)m * ldr + n]);
+          Y[(size_t)m * ldy + n] = Cvt<T>::from1(val);
+        }
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_d), "r"(TMEM_COLS));
+  }
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  DP_CHECK(fn != nullptr, DP_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  return fn;
+}
+
+// 2D K-major tile map: rows x K elements with row stride ld (elements), box {64, box_rows}.
+CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int box_rows) {
+  CUtensorMap m;
+  std::memset(&m, 0, sizeof(m));
+  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
+  cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = get_encode()(&m, dtype == DP_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16,
+                            2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  DP_CHECK(r == CUDA_SUCCESS, DP_ERR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+  return m;
+}
+
+template <class T, int BN>
+void run(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy, int M,
+         int N, int K, int act, cudaStream_t s) {
+  constexpr size_t smem = size_t(STAGES) * (BM * BK * 2 + BN * BK * 2) + 1024;
+  static bool attr = false;
+  if (!attr) {
+    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = true;
+  }
+  const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
+  CUtensorMap mw = make_map(w, dtype, N, K, K, BM);
+  CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
+  dim3 grid(N / BM, (M + BN - 1) / BN);
+  gemm_tc_kernel<T, BN><<<grid, 128, smem, s>>>(mw, mx, (const T*)bias, (const T*)res, ldr, (T*)y, ldy, M, N, K, act);
+  DP_CUDA(cudaGetLastError());
+}
+
+template <class T>
+void dispatch(int bn, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
+              int ldy, int M, int N, int K, int act, cudaStream_t s) {
+  switch (bn) {
+    case 32: run<T, 32>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
+    case 64: run<T, 64>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
+    case 128: run<T, 128>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
+    case 256: run<T, 256>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
+    default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
+  }
+}
+
+}  // namespace
+
+bool gemm_tc_supported(int N, int K) { return N > 0 && K > 0 && N % BM == 0 && K % BK == 0; }
+
+// Tile width over tokens: the widest BN that still gives >= one CTA per SM, else 32.
+static int pick_bn(int M, int N) {
+  const int ntile = N / BM;
+  for (int bn : {256, 128, 64}) {
+    if (M >= bn && ntile * ((M + bn - 1) / bn) >= 148) return bn;
+  }
+  return 32;
+}
+
+void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
+                    void* y, int ldy, int M, int N, int K, int act, int bn_hint, cudaStream_t s) {
+  DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
+  DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0 && ((uintptr_t)w % 16) == 0, DP_ERR_INVALID,
+           "GEMM operands must be 16-byte aligned");
+  if (M <= 0) return;
+  const int bn = bn_hint > 0 ? bn_hint : pick_bn(M, N);
+  if (dtype == DP_BF16)
+    dispatch<__nv_bfloat16>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s);
+  else
+    dispatch<__half>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s);
+}
+
+}  // namespace dp

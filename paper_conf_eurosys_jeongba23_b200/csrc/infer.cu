@@ -1,0 +1,592 @@
+// Context, cold-start / warm inference, eviction and the per-layer profiler.
+//
+// Cold start = §4.3.4 + Fig.9:
+//   * slot-0 LOAD units: H2D over the primary's own PCIe link on the load stream(s), one
+//     completion event per coalesced chunk;
+//   * slot-s LOAD units (PT): H2D over the link of the slot's GPU into a staging
+//     ring, then forwarded into the primary's HBM slot by that GPU's migration stream
+//     (cudaMemcpyPeerAsync over NVLink; a D2D copy in loopback; NCCL send/recv across
+//     processes -- peer.cpp), one event per forwarded piece;
+//   * DHA units: no transfer; their kernels read the arena in place ("we can skip
+//     the dependency check");
+//   * the execution stream (the caller's) waits on a unit's event right before the first
+//     kernel that reads it.
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <numeric>
+#include <vector>
+
+#include "engine.h"
+#include "kernels.h"
+#include "peer.h"
+
+namespace dp {
+
+static thread_local std::string g_last_error;
+void set_last_error(const std::string& msg) { g_last_error = msg; }
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) {
+    cudaGetDevice(&prev);
+    DP_CUDA(cudaSetDevice(d));
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace dp
+
+using namespace dp;
+
+dp::DevCtx& dp_context::on(int dev) {
+  DP_CHECK(dev >= 0 && dev < DP_MAX_DEVICES, DP_ERR_INVALID, "device ordinal out of range");
+  DevCtx& d = dc[dev];
+  DP_CHECK(d.ready, DP_ERR_INVALID, "device " + std::to_string(dev) + " is not part of this context");
+  return d;
+}
+
+static void init_device(dp_context* ctx, int dev) {
+  DevCtx& d = ctx->dc[dev];
+  if (d.ready) return;
+  DeviceGuard g(dev);
+  d.ord = dev;
+  d.events.dev = dev;
+  d.ready = true;
+}
+
+static void ensure_h2d_streams(dp_context* ctx, int dev) {
+  DevCtx& d = ctx->on(dev);
+  const int want = std::max(1, ctx->opts.n_h2d_streams);
+  if ((int)d.h2d.size() >= want) return;
+  DeviceGuard g(dev);
+  while ((int)d.h2d.size() < want) {
+    cudaStream_t s;
+    DP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    d.h2d.push_back(s);
+  }
+}
+
+static SlotRes& slot_res(dp_context* ctx, int slot, int dev, int64_t ring_bytes) {
+  auto& r = ctx->slots[{slot, dev}];
+  DeviceGuard g(dev);
+  if (!r.h2d) {
+    r.dev = dev;
+    DP_CUDA(cudaStreamCreateWithFlags(&r.h2d, cudaStreamNonBlocking));
+    DP_CUDA(cudaStreamCreateWithFlags(&r.mig, cudaStreamNonBlocking));
+  }
+  if (r.ring_bytes < ring_bytes) {
+    if (r.ring) DP_CUDA(cudaFree(r.ring));
+    r.ring = nullptr;
+    if (cudaMalloc(&r.ring, ring_bytes) != cudaSuccess) fail(DP_ERR_OOM, "staging ring cudaMalloc failed");
+    r.ring_bytes = ring_bytes;
+  }
+  return r;
+}
+
+static void ensure_slots(dp_model* m, int dev) {
+  DevState& ds = m->dev[dev];
+  if (ds.dbase) return;
+  DeviceGuard g(dev);
+  if (cudaMalloc(&ds.dbase, m->arena_bytes) != cudaSuccess) {
+    ds.dbase = nullptr;
+    fail(DP_ERR_OOM, "HBM slot allocation for the model failed");
+  }
+}
+
+extern "C" const char* dp_last_error(void) { return g_last_error.c_str(); }
+extern "C" int32_t dp_abi_version(void) { return 1; }
+
+extern "C" dp_status dp_context_create(const int32_t* devs, int32_t ndev, dp_context** out) {
+  dp_context* ctx = nullptr;
+  dp_status st = guard([&] {
+    DP_CHECK(out && devs && ndev >= 1 && ndev <= DP_MAX_DEVICES, DP_ERR_INVALID, "bad device list");
+    int count = 0;
+    DP_CUDA(cudaGetDeviceCount(&count));
+    ctx = new dp_context();
+    ctx->opts.chunk_bytes = 4 << 20;
+    ctx->opts.n_h2d_streams = 1;
+    ctx->opts.use_graph = 0;
+    ctx->opts.gemm_bn = 0;
+    for (int i = 0; i < ndev; ++i) {
+      DP_CHECK(devs[i] >= 0 && devs[i] < count && devs[i] < DP_MAX_DEVICES, DP_ERR_INVALID,
+               "device " + std::to_string(devs[i]) + " does not exist");
+      ctx->devs.push_back(devs[i]);
+      init_device(ctx, devs[i]);
+    }
+    *out = ctx;
+  });
+  if (st != DP_OK) delete ctx;
+  return st;
+}
+
+extern "C" dp_status dp_context_destroy(dp_context* ctx) {
+  return guard([&] {
+    if (!ctx) return;
+    for (int d : ctx->devs) {
+      DeviceGuard g(d);
+      cudaDeviceSynchronize();
+      DevCtx& dc = ctx->dc[d];
+      for (auto s : dc.h2d) cudaStreamDestroy(s);
+      dc.events.destroy();
+      if (dc.flush) cudaFree(dc.flush);
+    }
+    for (auto& kv : ctx->slots) {
+      DeviceGuard g(kv.second.dev);
+      if (kv.second.h2d) cudaStreamDestroy(kv.second.h2d);
+      if (kv.second.mig) cudaStreamDestroy(kv.second.mig);
+      if (kv.second.ring) cudaFree(kv.second.ring);
+    }
+    peer_destroy(ctx);
+    delete ctx;
+  });
+}
+
+extern "C" dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* o) {
+  return guard([&] {
+    DP_CHECK(ctx && o, DP_ERR_INVALID, "NULL argument");
+    DP_CHECK(o->chunk_bytes >= 4096, DP_ERR_INVALID, "chunk_bytes must be >= 4096");
+    DP_CHECK(o->n_h2d_streams >= 1 && o->n_h2d_streams <= 8, DP_ERR_INVALID, "n_h2d_streams must be 1..8");
+    DP_CHECK(o->gemm_bn == 0 || o->gemm_bn == 32 || o->gemm_bn == 64 || o->gemm_bn == 128 || o->gemm_bn == 256,
+             DP_ERR_INVALID, "gemm_bn must be 0/32/64/128/256");
+    ctx->opts = *o;
+  });
+}
+
+extern "C" dp_status dp_context_get_opts(dp_context* ctx, dp_engine_opts* out) {
+  return guard([&] {
+    DP_CHECK(ctx && out, DP_ERR_INVALID, "NULL argument");
+    *out = ctx->opts;
+  });
+}
+
+// ---------------------------------------------------------------------------------------
+// Cold start
+// ---------------------------------------------------------------------------------------
+
+namespace dp {
+
+// Coalesce runs of units (forward order) selected by `pick` that are contiguous in the
+// arena into pieces of at most `cap` bytes.  A unit is never split: one bigger than cap
+// is a piece of its own (one DMA per unit is cheapest; its event covers the whole unit).
+template <class Pick>
+std::vector<Piece> make_pieces(const dp_model* m, Pick pick, int64_t cap) {
+  std::vector<Piece> out;
+  const int n = (int)m->units.size();
+  Piece cur;
+  auto flush = [&] {
+    if (cur.bytes > 0) out.push_back(cur);
+    cur = Piece();
+  };
+  for (int u = 0; u < n; ++u) {
+    if (!pick(u)) {
+      flush();
+      continue;
+    }
+    const auto& un = m->units[u];
+    if (un.bytes == 0) continue;
+    if (cur.bytes > 0 && (cur.off + cur.bytes != un.off || cur.bytes + un.bytes > cap)) flush();
+    if (cur.bytes == 0) {
+      cur.off = un.off;
+      cur.first_unit = u;
+    }
+    cur.bytes += un.bytes;
+    cur.last_unit = u;
+  }
+  flush();
+  return out;
+}
+
+std::vector<Piece> slot_pieces(const dp_model* m, const dp_plan* plan, int slot, int64_t cap) {
+  return make_pieces(m, [&](int u) { return plan->method[u] == DP_LOAD && plan->slot[u] == slot; }, cap);
+}
+
+void bind_units(std::vector<cudaEvent_t>& unit_ev, const Piece& p, cudaEvent_t e) {
+  for (int u = p.first_unit; u <= p.last_unit; ++u) unit_ev[u] = e;
+}
+
+static void validate_plan(const dp_model* m, const dp_plan* p) {
+  DP_CHECK(p && p->method && p->slot, DP_ERR_INVALID, "plan is NULL");
+  DP_CHECK(p->n == (int)m->units.size(), DP_ERR_INVALID, "plan.n does not match the model's unit count");
+  DP_CHECK(p->k >= 1 && p->k <= DP_MAX_DEVICES, DP_ERR_INVALID, "plan.k out of range");
+  for (int i = 0; i < p->n; ++i) {
+    DP_CHECK(p->method[i] == DP_LOAD || p->method[i] == DP_DHA, DP_ERR_INVALID, "bad method value");
+    DP_CHECK(p->slot[i] >= 0 && p->slot[i] < p->k, DP_ERR_INVALID, "slot out of range");
+    DP_CHECK(!(p->slot[i] > 0 && p->method[i] == DP_DHA), DP_ERR_INVALID, "a PT unit (slot > 0) must be LOAD");
+  }
+}
+
+static int64_t dha_bytes(const dp_model* m, const int8_t* method, int T, int seq) {
+  int64_t s = 0;
+  const int64_t row = int64_t(m->cfg.hidden) * 2;
+  for (size_t u = 0; u < m->units.size(); ++u) {
+    if (method[u] != DP_DHA) continue;
+    const auto& un = m->units[u];
+    switch (un.role) {
+      case R_WORD: case R_WTE: s += int64_t(T) * row; break;  // one row per token
+      case R_POS: case R_WPE: s += int64_t(std::min<int64_t>(seq, m->cfg.max_pos)) * row; break;
+      case R_TYPE: s += row; break;
+      default: s += un.bytes; break;  // LN gamma/beta, linear weights: every byte once
+    }
+  }
+  return s;
+}
+
+// `primary` is the serving device ordinal; `prim_rank` its rank when the PT gather runs over
+// NCCL between processes (then secondaries are ranks, see peer.cpp).
+void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, int prim_rank,
+                const int32_t* secondaries, int nsec, const int32_t* ids, int batch, int seq, void* out, void* pooled,
+                cudaStream_t stream, dp_run_stats* stats) {
+  auto t0 = std::chrono::steady_clock::now();
+  validate_plan(m, plan);
+  DevCtx& pd = ctx->on(primary);
+  DevState& ds = m->dev[primary];
+  DP_CHECK(!ds.resident, DP_ERR_STATE, "model already resident on the primary; evict it first");
+  DP_CHECK(ctx->comm || nsec >= plan->k - 1, DP_ERR_INVALID, "need k-1 secondaries for the plan");
+  DP_CHECK(batch > 0 && seq > 0 && ids && out, DP_ERR_INVALID, "bad inference arguments");
+  DP_CHECK(seq + (m->cfg.family == DP_FAMILY_ROBERTA ? m->cfg.pad_idx + 1 : 0) <= m->cfg.max_pos, DP_ERR_INVALID,
+           "sequence longer than the position table");
+  DeviceGuard g(primary);
+  ensure_slots(m, primary);
+  ensure_h2d_streams(ctx, primary);
+  ensure_workspace(m, primary, int64_t(batch) * seq);
+  pd.events.reset();
+  const int n = (int)m->units.size();
+  const int8_t* method = plan->method;
+  dp_run_stats st;
+  std::memset(&st, 0, sizeof(st));
+  st.n_units = n;
+  std::vector<cudaEvent_t> unit_ev(n, nullptr);
+
+  // fork: side streams start when the execution stream reaches this call
+  cudaEvent_t fork = pd.events.get();
+  DP_CUDA(cudaEventRecord(fork, stream));
+  ++st.n_events;
+
+  // (1) slot-0 loads on the primary's link
+  const int64_t cap = std::max<int64_t>(ctx->opts.chunk_bytes, 4096);
+  auto pieces0 = make_pieces(m, [&](int u) { return method[u] == DP_LOAD && plan->slot[u] == 0; }, cap);
+  const int nh = (int)pd.h2d.size();
+  for (int i = 0; i < nh; ++i) DP_CUDA(cudaStreamWaitEvent(pd.h2d[i], fork, 0));
+  for (size_t c = 0; c < pieces0.size(); ++c) {
+    const Piece& p = pieces0[c];
+    cudaStream_t hs = pd.h2d[c % nh];
+    if (ctx->opts.debug_delay_us > 0) launch_spin((long long)ctx->opts.debug_delay_us * 2000, hs);
+    DP_CUDA(cudaMemcpyAsync(static_cast<uint8_t*>(ds.dbase) + p.off, static_cast<const uint8_t*>(m->arena) + p.off,
+                            p.bytes, cudaMemcpyHostToDevice, hs));
+    ++st.n_copies;
+    st.h2d_bytes[0] += p.bytes;
+    cudaEvent_t e = pd.events.get();
+    DP_CUDA(cudaEventRecord(e, hs));
+    ++st.n_events;
+    bind_units(unit_ev, p, e);  // every unit inside this piece completes with it
+  }
+
+  // (2) PT slots
+  if (!ctx->comm)
+    for (int s = 1; s < plan->k; ++s) {
+      const int sdev = secondaries[s - 1];
+      DP_CHECK(sdev >= 0 && sdev < DP_MAX_DEVICES && ctx->dc[sdev].ready, DP_ERR_INVALID,
+               "secondary device not in the context");
+      if (sdev != primary) ctx->dc[sdev].events.reset();
+    }
+  if (ctx->comm && plan->k > 1) peer_recv_all(ctx, m, plan, prim_rank, primary, fork, unit_ev, st);
+  for (int s = 1; s < plan->k && !ctx->comm; ++s) {
+    auto pcs = slot_pieces(m, plan, s, cap);
+    if (pcs.empty()) continue;
+    const int sdev = secondaries[s - 1];
+    const int64_t ring_slots = 3;
+    int64_t slot_bytes = 0;
+    for (const auto& p : pcs) slot_bytes = std::max(slot_bytes, p.bytes);
+    SlotRes& r = slot_res(ctx, s, sdev, ring_slots * slot_bytes);
+    DevCtx& sd = ctx->dc[sdev];
+    {
+      DeviceGuard gs(sdev);
+      DP_CUDA(cudaStreamWaitEvent(r.h2d, fork, 0));
+    }
+    std::vector<cudaEvent_t> fwd_done(pcs.size(), nullptr);
+    for (size_t c = 0; c < pcs.size(); ++c) {
+      const Piece& p = pcs[c];
+      uint8_t* stage = static_cast<uint8_t*>(r.ring) + (c % ring_slots) * slot_bytes;
+      DeviceGuard gs(sdev);
+      if (c >= (size_t)ring_slots) DP_CUDA(cudaStreamWaitEvent(r.h2d, fwd_done[c - ring_slots], 0));
+      if (ctx->opts.debug_delay_us > 0) launch_spin((long long)ctx->opts.debug_delay_us * 2000, r.h2d);
+      DP_CUDA(cudaMemcpyAsync(stage, static_cast<const uint8_t*>(m->arena) + p.off, p.bytes, cudaMemcpyHostToDevice,
+                              r.h2d));
+      ++st.n_copies;
+      st.h2d_bytes[s] += p.bytes;
+      cudaEvent_t landed = sd.events.get();
+      DP_CUDA(cudaEventRecord(landed, r.h2d));
+      DP_CUDA(cudaStreamWaitEvent(r.mig, landed, 0));
+      if (ctx->opts.debug_delay_us > 0) launch_spin((long long)ctx->opts.debug_delay_us * 2000, r.mig);
+      uint8_t* dst = static_cast<uint8_t*>(ds.dbase) + p.off;
+      if (sdev == primary)
+        DP_CUDA(cudaMemcpyAsync(dst, stage, p.bytes, cudaMemcpyDeviceToDevice, r.mig));
+      else
+        DP_CUDA(cudaMemcpyPeerAsync(dst, primary, stage, sdev, p.bytes, r.mig));
+      st.nvlink_bytes[s] += p.bytes;
+      cudaEvent_t done = sd.events.get();
+      DP_CUDA(cudaEventRecord(done, r.mig));
+      st.n_events += 2;
+      fwd_done[c] = done;
+      bind_units(unit_ev, p, done);
+    }
+  }
+
+  // (3) execution stream: wait per unit, then its kernels
+  std::vector<char> waited_ev;
+  cudaEvent_t last_waited = nullptr;
+  ForwardArgs a;
+  a.m = m;
+  a.dev = primary;
+  a.method = method;
+  a.ids = ids;
+  a.batch = batch;
+  a.seq = seq;
+  a.out = out;
+  a.pooled = pooled;
+  a.stream = stream;
+  a.bn_hint = ctx->opts.gemm_bn;
+  a.before_unit = [&](int u) {
+    if (method[u] == DP_DHA) return;  // DHA layers skip the dependency check
+    cudaEvent_t e = unit_ev[u];
+    DP_CHECK(e != nullptr, DP_ERR_STATE, "internal: loaded unit has no completion event");
+    if (e == last_waited) return;
+    DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
+    last_waited = e;
+  };
+  run_forward(a);
+  // join every side stream (units never read, e.g. an unused pooler, still finish loading)
+  for (int i = 0; i < nh; ++i) {
+    cudaEvent_t e = pd.events.get();
+    DP_CUDA(cudaEventRecord(e, pd.h2d[i]));
+    DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
+    ++st.n_events;
+  }
+  for (int s = 1; s < plan->k && !ctx->comm; ++s) {
+    auto it = ctx->slots.find({s, secondaries[s - 1]});
+    if (it == ctx->slots.end()) continue;
+    DeviceGuard gs(it->second.dev);
+    cudaEvent_t e = ctx->dc[it->second.dev].events.get();
+    DP_CUDA(cudaEventRecord(e, it->second.mig));
+    DeviceGuard gp(primary);
+    DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
+  }
+  if (ctx->comm) peer_join(ctx, stream);
+  ds.resident = true;
+  ds.method.assign(method, method + n);
+  st.n_kernels = a.kernels;
+  st.dha_weight_bytes = dha_bytes(m, method, batch * seq, seq);
+  st.wall_enqueue_us =
+      std::chrono::duration<float, std::micro>(std::chrono::steady_clock::now() - t0).count();
+  if (stats) *stats = st;
+}
+
+}  // namespace dp
+
+extern "C" dp_status dp_infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int32_t primary,
+                                   const int32_t* secondaries, int32_t nsec, const int32_t* d_ids, int32_t batch,
+                                   int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats) {
+  return guard([&] {
+    DP_CHECK(ctx && m, DP_ERR_INVALID, "NULL context/model");
+    if (ctx->comm) {  // multi-process PT: `primary` is a rank, each process has one device
+      validate_plan(m, plan);
+      if (ctx->rank != primary) {  // secondary rank: only its transfers
+        peer_send_rank(ctx, m, plan, primary, stats);
+        return;
+      }
+      infer_cold(ctx, m, plan, ctx->devs[0], primary, nullptr, 0, d_ids, batch, seq, d_out, d_pooled,
+                 (cudaStream_t)stream, stats);
+      return;
+    }
+    infer_cold(ctx, m, plan, primary, -1, secondaries, nsec, d_ids, batch, seq, d_out, d_pooled, (cudaStream_t)stream,
+               stats);
+  });
+}
+
+extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, const int32_t* d_ids, int32_t batch,
+                                   int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats) {
+  return guard([&] {
+    DP_CHECK(ctx && m, DP_ERR_INVALID, "NULL context/model");
+    ctx->on(dev);
+    DevState& ds = m->dev[dev];
+    DP_CHECK(ds.resident, DP_ERR_STATE, "model is not resident on this device");
+    DP_CHECK(batch > 0 && seq > 0 && d_ids && d_out, DP_ERR_INVALID, "bad inference arguments");
+    DeviceGuard g(dev);
+    auto t0 = std::chrono::steady_clock::now();
+    ForwardArgs a;
+    a.m = m;
+    a.dev = dev;
+    a.method = ds.method.data();
+    a.ids = d_ids;
+    a.batch = batch;
+    a.seq = seq;
+    a.out = d_out;
+    a.pooled = d_pooled;
+    a.stream = (cudaStream_t)stream;
+    a.bn_hint = ctx->opts.gemm_bn;
+    run_forward(a);
+    if (stats) {
+      std::memset(stats, 0, sizeof(*stats));
+      stats->n_kernels = a.kernels;
+      stats->n_units = (int)m->units.size();
+      stats->dha_weight_bytes = dha_bytes(m, ds.method.data(), batch * seq, seq);
+      stats->wall_enqueue_us =
+          std::chrono::duration<float, std::micro>(std::chrono::steady_clock::now() - t0).count();
+    }
+  });
+}
+
+extern "C" dp_status dp_model_evict(dp_context* ctx, dp_model* m, int32_t dev) {
+  return guard([&] {
+    DP_CHECK(ctx && m, DP_ERR_INVALID, "NULL context/model");
+    ctx->on(dev);
+    DeviceGuard g(dev);
+    DP_CUDA(cudaDeviceSynchronize());
+    if (ctx->opts.debug_poison && m->dev[dev].dbase) {
+      DP_CUDA(cudaMemset(m->dev[dev].dbase, 0xFF, m->arena_bytes));
+      DP_CUDA(cudaDeviceSynchronize());
+    }
+    m->dev[dev].resident = false;
+  });
+}
+
+extern "C" int32_t dp_model_is_resident(const dp_model* m, int32_t dev) {
+  if (!m || dev < 0 || dev >= DP_MAX_DEVICES) return 0;
+  return m->dev[dev].resident ? 1 : 0;
+}
+
+extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
+  return guard([&] {
+    if (!m) return;
+    for (int d = 0; d < DP_MAX_DEVICES; ++d) {
+      DevState& ds = m->dev[d];
+      if (ds.dbase || ds.ws.base) {
+        DeviceGuard g(d);
+        cudaDeviceSynchronize();
+        if (ds.dbase) cudaFree(ds.dbase);
+        if (ds.ws.base) cudaFree(ds.ws.base);
+      }
+    }
+    if (m->arena) cudaFreeHost(m->arena);
+    delete m;
+  });
+}
+
+// ---------------------------------------------------------------------------------------
+// Profiler (§4.3.1; 10 iterations per Table 5)
+// ---------------------------------------------------------------------------------------
+
+namespace dp {
+
+static int64_t median_ns(std::vector<float>& ms) {
+  std::sort(ms.begin(), ms.end());
+  const size_t k = ms.size();
+  const double med = k % 2 ? ms[k / 2] : 0.5 * (ms[k / 2 - 1] + ms[k / 2]);
+  return (int64_t)llround(med * 1e6);
+}
+
+struct CostOut {  // the caller-owned output arrays of a dp_cost_table
+  int64_t *bytes, *load_ns, *fwd_ns, *exe_mem_ns, *exe_dha_ns;
+};
+
+void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iters, dp_cost_table* table) {
+  DP_CHECK(table && table->n == (int)m->units.size(), DP_ERR_INVALID, "cost table size mismatch");
+  DP_CHECK(table->bytes && table->load_ns && table->fwd_ns && table->exe_mem_ns && table->exe_dha_ns, DP_ERR_INVALID,
+           "cost table arrays are NULL");
+  CostOut o{const_cast<int64_t*>(table->bytes), const_cast<int64_t*>(table->load_ns),
+            const_cast<int64_t*>(table->fwd_ns), const_cast<int64_t*>(table->exe_mem_ns),
+            const_cast<int64_t*>(table->exe_dha_ns)};
+  CostOut* out = &o;
+  DP_CHECK(iters >= 1 && batch > 0 && seq > 0, DP_ERR_INVALID, "bad profiling arguments");
+  DevCtx& d = ctx->on(dev);
+  DevState& ds = m->dev[dev];
+  DP_CHECK(!ds.resident, DP_ERR_STATE, "evict the model before profiling");
+  DeviceGuard g(dev);
+  ensure_slots(m, dev);
+  const int T = batch * seq;
+  ensure_workspace(m, dev, T);
+  if (!d.flush) {
+    d.flush_bytes = 256ll << 20;  // > 126 MB L2
+    DP_CUDA(cudaMalloc(&d.flush, d.flush_bytes));
+  }
+  cudaStream_t s;
+  DP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  int32_t* ids = nullptr;
+  DP_CUDA(cudaMalloc(&ids, sizeof(int32_t) * T));
+  {
+    std::vector<int32_t> h(T);
+    const int lo = m->cfg.family == DP_FAMILY_ROBERTA ? 3 : 0;
+    for (int t = 0; t < T; ++t) h[t] = lo + int((uint64_t(t) * 2654435761ull) % uint64_t(m->cfg.vocab - lo));
+    DP_CUDA(cudaMemcpy(ids, h.data(), sizeof(int32_t) * T, cudaMemcpyHostToDevice));
+  }
+  DP_CUDA(cudaMemset(m->dev[dev].ws.base, 0, 1));
+  // all weights resident for the in-memory runs
+  DP_CUDA(cudaMemcpy(ds.dbase, m->arena, m->arena_bytes, cudaMemcpyHostToDevice));
+  cudaEvent_t e0, e1;
+  DP_CUDA(cudaEventCreate(&e0));
+  DP_CUDA(cudaEventCreate(&e1));
+  const int warm = 3;
+  const int n = (int)m->units.size();
+  auto timed = [&](auto&& body, bool flush) {
+    std::vector<float> v;
+    for (int it = 0; it < warm + iters; ++it) {
+      if (flush) launch_l2_flush(d.flush, d.flush_bytes, s);
+      DP_CUDA(cudaEventRecord(e0, s));
+      body();
+      DP_CUDA(cudaEventRecord(e1, s));
+      DP_CUDA(cudaEventSynchronize(e1));
+      float ms = 0;
+      DP_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+      if (it >= warm) v.push_back(ms);
+    }
+    return median_ns(v);
+  };
+  // embedding units share one fused kernel: attribute T(all HBM) evenly, and each unit's
+  // DHA cost as the marginal time of reading that table from host (DESIGN.md §3 R8)
+  std::vector<int> emb;
+  for (int u = 0; u < n; ++u)
+    if (m->units[u].role == R_WORD || m->units[u].role == R_POS || m->units[u].role == R_TYPE ||
+        m->units[u].role == R_EMB_LN || m->units[u].role == R_WTE || m->units[u].role == R_WPE)
+      emb.push_back(u);
+  int64_t emb_all_mem = 0;
+  if (!emb.empty())
+    emb_all_mem = timed([&] { run_unit(m, dev, emb[0], false, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
+  for (int u = 0; u < n; ++u) {
+    const auto& un = m->units[u];
+    out->bytes[u] = un.bytes;
+    uint8_t* dst = static_cast<uint8_t*>(ds.dbase) + un.off;
+    const uint8_t* src = static_cast<const uint8_t*>(m->arena) + un.off;
+    out->load_ns[u] = timed([&] { DP_CUDA(cudaMemcpyAsync(dst, src, un.bytes, cudaMemcpyHostToDevice, s)); }, false);
+    uint8_t* scratch = static_cast<uint8_t*>(d.flush);
+    const int64_t fb = std::min<int64_t>(un.bytes, d.flush_bytes / 2);
+    out->fwd_ns[u] = timed([&] { DP_CUDA(cudaMemcpyAsync(scratch, dst, fb, cudaMemcpyDeviceToDevice, s)); }, false);
+    const bool is_emb = std::find(emb.begin(), emb.end(), u) != emb.end();
+    if (is_emb) {
+      const int64_t share = emb_all_mem / (int64_t)emb.size();
+      const int64_t with_host = timed([&] { run_unit(m, dev, u, true, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
+      out->exe_mem_ns[u] = share;
+      out->exe_dha_ns[u] = share + std::max<int64_t>(0, with_host - emb_all_mem);
+    } else {
+      out->exe_mem_ns[u] = timed([&] { run_unit(m, dev, u, false, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
+      out->exe_dha_ns[u] = timed([&] { run_unit(m, dev, u, true, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
+    }
+  }
+  DP_CUDA(cudaStreamSynchronize(s));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaFree(ids);
+  cudaStreamDestroy(s);
+}
+
+}  // namespace dp
+
+extern "C" dp_status dp_profile(dp_context* ctx, dp_model* m, int32_t dev, int32_t batch, int32_t seq, int32_t iters,
+                                dp_cost_table* out) {
+  return guard([&] {
+    DP_CHECK(ctx && m, DP_ERR_INVALID, "NULL context/model");
+    profile(ctx, m, dev, batch, seq, iters, out);
+  });
+}

@@ -1,0 +1,39 @@
+// Internal kernel launchers (host side).  All take a cudaStream_t and return after enqueue.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace dp {
+
+// Epilogue activations (dp_linear's `act`).
+enum Act { ACT_NONE = 0, ACT_GELU_ERF = 1, ACT_GELU_TANH = 2, ACT_TANH = 3 };
+
+// K1: fused embedding gather (+ LayerNorm) -- SURVEY §8(a) a10.  Table pointers may be
+// host-mapped (direct-host-access).  ln_g == nullptr -> no LN (GPT-2).
+void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
+                  const void* type, const void* ln_g, const void* ln_b, int H, float eps, void* out,
+                  cudaStream_t s);
+
+// K4: y = LN(x (+ r)) * g + b; g/b may be host-mapped.
+void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
+                      int n, float eps, cudaStream_t s);
+
+// K3: skinny linear reading W exactly once (W may be host-mapped) -- a11.
+void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
+                          int ldr, void* y, int ldy, int M, int N, int K, int act, cudaStream_t s);
+
+// K5: attention core (mma.sync flash attention, d = 64).
+void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
+                      bool causal, cudaStream_t s);
+
+// K2: resident tcgen05/TMA GEMM -- a12.  W must be device memory.
+struct GemmPlan;  // cached tensor map for a weight
+bool gemm_tc_supported(int N, int K);
+void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
+                    void* y, int ldy, int M, int N, int K, int act, int bn_hint, cudaStream_t s);
+
+// Scratch kernels
+void launch_l2_flush(void* buf, size_t bytes, cudaStream_t s);
+void launch_spin(long long cycles, cudaStream_t s);
+
+}  // namespace dp

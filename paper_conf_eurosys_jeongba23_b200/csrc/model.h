@@ -1,0 +1,74 @@
+// Model registration: parameter list, planning units, pinned host arena, per-device state.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <map>
+#include <string>
+#include <vector>
+
+#include "common.h"
+
+namespace dp {
+
+enum Role {
+  R_WORD, R_POS, R_TYPE, R_EMB_LN,                                 // BERT/RoBERTa embeddings
+  R_Q, R_K, R_V, R_ATTN_OUT, R_LN1, R_FC1, R_FC2, R_LN2, R_POOLER,  // BERT/RoBERTa layer + pooler
+  R_WTE, R_WPE,                                                    // GPT-2 embeddings
+  R_LN_1, R_C_ATTN, R_C_PROJ, R_LN_2, R_C_FC, R_MLP_PROJ, R_LN_F   // GPT-2 block + final LN
+};
+
+struct ParamDesc {
+  std::string hf;
+  int ndim = 1;
+  int64_t shape[2] = {0, 0};
+  int unit = -1;
+  int64_t bytes = 0;
+  bool transpose = false;  // GPT-2 Conv1D [in,out] -> stored [out,in]
+  int64_t off = 0;         // arena offset
+};
+
+struct UnitDesc {
+  std::string name;
+  int kind = DP_UNIT_LINEAR;
+  int role = 0;
+  int layer = -1;
+  int first_param = 0, nparams = 0;
+  int64_t off = 0, bytes = 0;
+  int64_t N = 0, K = 0;  // linear: W [N, K] at off, bias [N] at off + N*K*2
+};
+
+// Activation workspace on one device for T tokens.
+struct Workspace {
+  int64_t tokens = 0;
+  void* x = nullptr;    // [T, H]
+  void* qkv = nullptr;  // [T, 3H]
+  void* ctx = nullptr;  // [T, H]
+  void* tmp = nullptr;  // [T, H]
+  void* x1 = nullptr;   // [T, H]
+  void* h = nullptr;    // [T, F]
+  void* base = nullptr;
+};
+
+struct DevState {
+  void* dbase = nullptr;  // HBM copy of the arena layout (slots for loaded units)
+  bool resident = false;
+  std::vector<int8_t> method;  // per unit, fixed when the model became resident
+  Workspace ws;
+};
+
+std::vector<ParamDesc> config_params(const dp_model_config& c);
+void validate_config(const dp_model_config& c);
+
+}  // namespace dp
+
+struct dp_model {
+  dp_model_config cfg{};
+  std::vector<dp::ParamDesc> params;
+  std::vector<dp::UnitDesc> units;
+  void* arena = nullptr;  // cudaHostAlloc(Portable | Mapped)
+  int64_t arena_bytes = 0;
+  dp::DevState dev[DP_MAX_DEVICES];
+
+  const uint8_t* host(int u) const { return static_cast<const uint8_t*>(arena) + units[u].off; }
+  uint8_t* device(int d, int u) const { return static_cast<uint8_t*>(dev[d].dbase) + units[u].off; }
+};

@@ -1,0 +1,26 @@
+// Multi-process parallel transmission (one process per GPU): the NCCL send/recv gather.
+#pragma once
+#include <vector>
+
+#include "engine.h"
+
+namespace dp {
+
+// Slot s of a plan is served by rank (primary + s) % nranks.
+int peer_rank_of_slot(const dp_context* ctx, int primary, int slot);
+
+// Primary: post the receives of every PT slot into the model's HBM slots, one NCCL group
+// per round (piece r of every secondary), one event per round bound to its units.
+void peer_recv_all(dp_context* ctx, dp_model* m, const dp_plan* plan, int prim_rank, int dev, cudaEvent_t fork,
+                   std::vector<cudaEvent_t>& unit_ev, dp_run_stats& st);
+// Primary: make `exec` wait for every posted receive.
+void peer_join(dp_context* ctx, cudaStream_t exec);
+// Secondary rank: H2D its slot's pieces into the staging ring and send them to the primary.
+void peer_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, dp_run_stats* stats);
+void peer_destroy(dp_context* ctx);
+
+// The piece list of one slot (shared by sender and receiver so both sides agree).
+std::vector<Piece> slot_pieces(const dp_model* m, const dp_plan* plan, int slot, int64_t cap);
+void bind_units(std::vector<cudaEvent_t>& unit_ev, const Piece& p, cudaEvent_t e);
+
+}  // namespace dp

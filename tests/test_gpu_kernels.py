@@ -1,0 +1,214 @@
+"""GPU parity of each hot-path kernel against the fp64 oracle, through the C-ABI.
+
+Tolerances: both sides see the same storage-rounded inputs; the kernel
+accumulates in fp32 and rounds its output once to fp16/bf16, so an element may differ
+from the fp64 value by half an output ulp plus the fp32 accumulation error:
+  |y - ref| <= 2^-10 |ref| + K * 2^-22 * max|x w|  (fp16)   /  2^-7 |ref| + ...  (bf16).
+Direct-host-access changes only WHERE the weights are read from, so the same kernel on a
+host-mapped pointer and on a device pointer must give bit-identical results.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import forward as F
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+DT = {"fp16": torch.float16, "bf16": torch.bfloat16}
+EPS_OUT = {"fp16": 2.0 ** -10, "bf16": 2.0 ** -7}
+
+
+def dp():
+    import paper_conf_eurosys_jeongba23_b200 as m
+    return m
+
+
+def to_t(a, dtype, dev="cuda"):
+    if dtype == "bf16":
+        t = torch.from_numpy(a.view(np.int16).copy()).view(torch.bfloat16)
+    else:
+        t = torch.from_numpy(np.ascontiguousarray(a))
+    return t.to(dev)
+
+
+def f64(t):
+    return t.float().cpu().numpy().astype(np.float64)
+
+
+class HostBuf:
+    """Pinned + mapped host memory from the library (a DHA weight location)."""
+
+    def __init__(self, arr: np.ndarray):
+        self.nbytes = arr.nbytes
+        self.ptr = dp().host_alloc(self.nbytes)
+        np.ctypeslib.as_array((np.ctypeslib.ctypes.c_uint8 * self.nbytes).from_address(self.ptr))[:] = \
+            np.frombuffer(np.ascontiguousarray(arr).tobytes(), dtype=np.uint8)
+
+    def free(self):
+        dp().host_free(self.ptr)
+
+
+def close(y, ref, dtype, K=1, scale=1.0):
+    tol = EPS_OUT[dtype] * np.abs(ref) + K * 2.0 ** -22 * scale + 1e-6
+    err = np.abs(y - ref)
+    assert np.all(err <= tol), f"max err {err.max():.3e}, worst tol {tol.flat[np.argmax(err - tol)]:.3e}"
+
+
+# ---------------------------------------------------------------------------------------
+# K1 embedding
+# ---------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("name,B,S", [("tiny_bert", 2, 33), ("bert_base", 1, 128), ("tiny_roberta", 1, 100),
+                                      ("tiny_gpt2", 3, 17), ("bert_large", 1, 384)])
+@pytest.mark.parametrize("dtype", ["fp16", "bf16"])
+def test_embed_parity_and_dha_bit_identity(name, B, S, dtype):
+    m = synth.SHAPES[name]
+    w = synth.make_weights(m, seed=1, dtype=dtype, recipe="scaled")
+    ids = synth.make_ids(m, B, S, seed=2)
+    ref = F.embed(m, w, ids, dtype).reshape(B * S, m.hidden)
+    gpt = m.family == "gpt2"
+    names = (["wte.weight", "wpe.weight"] if gpt else
+             ["embeddings.word_embeddings.weight", "embeddings.position_embeddings.weight",
+              "embeddings.token_type_embeddings.weight", "embeddings.LayerNorm.weight",
+              "embeddings.LayerNorm.bias"])
+    dev_t = {n: to_t(w[n], dtype) for n in names}
+    host_b = {n: HostBuf(w[n]) for n in names}
+    ids_t = torch.from_numpy(ids.reshape(-1)).cuda()
+    pos_off = m.pad_idx + 1 if m.family == "roberta" else 0
+    outs = []
+    for where in ("device", "host"):
+        P = (lambda n: dev_t[n].data_ptr()) if where == "device" else (lambda n: host_b[n].ptr)
+        out = torch.empty(B * S, m.hidden, dtype=DT[dtype], device="cuda")
+        if gpt:
+            dp().embed(ids_t, S, P(names[0]), P(names[1]), None, None, None, m.hidden, 0.0, out, dtype)
+        else:
+            dp().embed(ids_t, S, P(names[0]), P(names[1]), P(names[2]), P(names[3]), P(names[4]), m.hidden,
+                       m.ln_eps, out, dtype, pos_offset=pos_off)
+        torch.cuda.synchronize()
+        outs.append(out)
+    assert torch.equal(outs[0].view(torch.int16), outs[1].view(torch.int16))
+    y = f64(outs[0])
+    # LN output: fp32 statistics + one output rounding
+    tol = EPS_OUT[dtype] * np.abs(ref) + 2e-4 * (1 if gpt else np.abs(ref).max())
+    assert np.all(np.abs(y - ref) <= tol), np.abs(y - ref).max()
+    for b in host_b.values():
+        b.free()
+
+
+# ---------------------------------------------------------------------------------------
+# K2 / K3 linear
+# ---------------------------------------------------------------------------------------
+
+SHAPES_LIN = [(1, 128, 64), (7, 256, 128), (32, 768, 768), (100, 384, 128), (128, 768, 768), (128, 3072, 768),
+              (128, 768, 3072), (200, 1024, 1024), (384, 4096, 1024), (1024, 1024, 4096), (333, 2304, 768)]
+
+
+@pytest.mark.parametrize("M,N,K", SHAPES_LIN)
+@pytest.mark.parametrize("dtype", ["fp16", "bf16"])
+def test_linear_tcgen05_parity(M, N, K, dtype):
+    rng = np.random.default_rng(M * 7 + N + K)
+    x = synth.round_to(rng.standard_normal((M, K)).astype(np.float32), dtype)
+    wt = synth.round_to((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32), dtype)
+    b = synth.round_to((0.1 * rng.standard_normal(N)).astype(np.float32), dtype)
+    r = synth.round_to(rng.standard_normal((M, N)).astype(np.float32), dtype)
+    X, W, Bt, R = (to_t(a, dtype) for a in (x, wt, b, r))
+    x64, w64, b64, r64 = (synth.storage_to_f64(a, dtype) for a in (x, wt, b, r))
+    for act, res in (("none", False), ("gelu_erf", False), ("none", True), ("gelu_tanh", True)):
+        Y = torch.empty(M, N, dtype=DT[dtype], device="cuda")
+        dp().linear(X, K, W, Bt, R if res else None, N, Y, N, M, N, K, act=act, path=0, dtype=dtype)
+        torch.cuda.synchronize()
+        ref = F.linear(x64, w64, b64, act, r64 if res else None)
+        close(f64(Y), ref, dtype, K=K, scale=np.abs(x64).max() * np.abs(w64).max() * 4)
+
+
+@pytest.mark.parametrize("M,N,K", [(1, 768, 768), (5, 128, 64), (128, 768, 768), (128, 3072, 768),
+                                   (128, 768, 3072), (384, 1024, 4096), (17, 2304, 768)])
+@pytest.mark.parametrize("dtype", ["fp16", "bf16"])
+def test_linear_skinny_dha_parity_and_bit_identity(M, N, K, dtype):
+    rng = np.random.default_rng(M + 3 * N + K)
+    x = synth.round_to(rng.standard_normal((M, K)).astype(np.float32), dtype)
+    wt = synth.round_to((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32), dtype)
+    b = synth.round_to((0.1 * rng.standard_normal(N)).astype(np.float32), dtype)
+    X, W, Bt = (to_t(a, dtype) for a in (x, wt, b))
+    hw, hb = HostBuf(wt), HostBuf(b)
+    Y0 = torch.empty(M, N, dtype=DT[dtype], device="cuda")
+    Y1 = torch.empty_like(Y0)
+    dp().linear(X, K, W, Bt, None, 0, Y0, N, M, N, K, act="tanh", path=1, dtype=dtype)
+    dp().linear(X, K, hw.ptr, hb.ptr, None, 0, Y1, N, M, N, K, act="tanh", path=1, dtype=dtype)
+    torch.cuda.synchronize()
+    assert torch.equal(Y0.view(torch.int16), Y1.view(torch.int16))
+    ref = F.linear(*(synth.storage_to_f64(a, dtype) for a in (x, wt, b)), act="tanh")
+    close(f64(Y0), ref, dtype, K=K, scale=4 * np.abs(synth.storage_to_f64(x, dtype)).max())
+    hw.free()
+    hb.free()
+
+
+def test_linear_strided_output_and_input():
+    """q/k/v write into column blocks of the [T, 3H] buffer; the pooler reads every S-th row."""
+    dtype = "fp16"
+    rng = np.random.default_rng(5)
+    T, H = 96, 256
+    x = synth.round_to(rng.standard_normal((T, H)).astype(np.float32), dtype)
+    wt = synth.round_to((rng.standard_normal((H, H)) / 16).astype(np.float32), dtype)
+    X, W = to_t(x, dtype), to_t(wt, dtype)
+    qkv = torch.zeros(T, 3 * H, dtype=torch.float16, device="cuda")
+    dp().linear(X, H, W, None, None, 0, qkv[:, H:].data_ptr(), 3 * H, T, H, H, path=0, dtype=dtype)
+    torch.cuda.synchronize()
+    ref = F.linear(x.astype(np.float64), wt.astype(np.float64))
+    close(f64(qkv[:, H:2 * H]), ref, dtype, K=H, scale=16)
+    assert torch.count_nonzero(qkv[:, :H]) == 0 and torch.count_nonzero(qkv[:, 2 * H:]) == 0
+    # strided input (every 32nd row) through the skinny kernel
+    Y = torch.empty(3, H, dtype=torch.float16, device="cuda")
+    dp().linear(X, 32 * H, W, None, None, 0, Y, H, 3, H, H, path=1, dtype=dtype)
+    torch.cuda.synchronize()
+    close(f64(Y), ref[::32], dtype, K=H, scale=16)
+
+
+# ---------------------------------------------------------------------------------------
+# K4 LayerNorm, K5 attention
+# ---------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("rows,n", [(1, 128), (37, 768), (128, 1024), (1000, 768)])
+def test_layernorm_parity_and_dha(rows, n):
+    dtype = "fp16"
+    rng = np.random.default_rng(rows + n)
+    x = synth.round_to((3 * rng.standard_normal((rows, n)) + 1).astype(np.float32), dtype)
+    r = synth.round_to(rng.standard_normal((rows, n)).astype(np.float32), dtype)
+    g = synth.round_to((1 + 0.1 * rng.standard_normal(n)).astype(np.float32), dtype)
+    b = synth.round_to((0.1 * rng.standard_normal(n)).astype(np.float32), dtype)
+    X, R, G, Bt = (to_t(a, dtype) for a in (x, r, g, b))
+    hg, hb = HostBuf(g), HostBuf(b)
+    Y0 = torch.empty(rows, n, dtype=torch.float16, device="cuda")
+    Y1 = torch.empty_like(Y0)
+    dp().layernorm(X, R, G, Bt, Y0, rows, n, 1e-5)
+    dp().layernorm(X, R, hg.ptr, hb.ptr, Y1, rows, n, 1e-5)
+    torch.cuda.synchronize()
+    assert torch.equal(Y0, Y1)
+    ref = F.layer_norm(x.astype(np.float64) + r.astype(np.float64), g.astype(np.float64), b.astype(np.float64),
+                       1e-5)
+    close(f64(Y0), ref, dtype, K=n, scale=8)
+    hg.free()
+    hb.free()
+
+
+@pytest.mark.parametrize("B,S,H,heads", [(1, 1, 128, 2), (2, 5, 128, 2), (1, 64, 768, 12), (2, 100, 256, 4),
+                                         (1, 128, 768, 12), (1, 384, 1024, 16), (1, 1024, 1024, 16)])
+@pytest.mark.parametrize("causal", [False, True])
+@pytest.mark.parametrize("dtype", ["fp16", "bf16"])
+def test_attention_parity(B, S, H, heads, causal, dtype):
+    rng = np.random.default_rng(B * 1000 + S + H)
+    qkv = synth.round_to((1.5 * rng.standard_normal((B * S, 3 * H))).astype(np.float32), dtype)
+    Q = to_t(qkv, dtype)
+    O = torch.empty(B * S, H, dtype=DT[dtype], device="cuda")
+    dp().attention(Q, 3 * H, O, B, S, H, heads, causal, dtype)
+    torch.cuda.synchronize()
+    q64 = synth.storage_to_f64(qkv, dtype).reshape(B, S, 3 * H)
+    ref = F.attention(q64[..., :H], q64[..., H:2 * H], q64[..., 2 * H:], heads, causal).reshape(B * S, H)
+    # P is rounded to fp16/bf16 before the P.V product (flash attention), hence the looser bound
+    tol = (4 if dtype == "fp16" else 8) * EPS_OUT[dtype] * (np.abs(ref) + np.abs(q64).max())
+    err = np.abs(f64(O) - ref)
+    assert np.all(err <= tol), err.max()

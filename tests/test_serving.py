@@ -1,0 +1,61 @@
+"""Serving harness (C++, dry-run replay through dp_serve_run) against the independent
+event-driven oracle replay: identical GPU assignment, cold/warm decisions, eviction counts
+and start/finish times on seeded Poisson traces.  Also pins the oracle on
+hand-checkable cases (P:322 one request per GPU, P:338 LRU)."""
+import numpy as np
+import pytest
+
+import synth
+import paper_conf_eurosys_jeongba23_b200 as dp
+from oracle import serving as OS
+
+
+def _table(nmodels, rng):
+    cold = rng.integers(5_000_000, 60_000_000, nmodels)
+    warm = rng.integers(500_000, 5_000_000, nmodels)
+    rb = rng.integers(100 << 20, 700 << 20, nmodels)
+    return cold, warm, rb
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_dry_run_matches_oracle(seed):
+    rng = np.random.default_rng(seed)
+    ninst = int(rng.integers(5, 300))
+    ngpu = int(rng.integers(1, 9))
+    nmodels = 3
+    cold, warm, rb = _table(nmodels, rng)
+    moi = synth.instance_models(ninst, (4, 4, 1))
+    arr, inst = synth.make_poisson_trace(int(rng.integers(50, 1500)), float(rng.integers(20, 400)), ninst, seed)
+    budget = int(rb.max() * rng.integers(1, 30))
+    kw = dict(ngpu=ngpu, per_gpu_budget_bytes=budget, cold_ns=cold, warm_ns=warm, resident_bytes=rb,
+              model_of_instance=moi)
+    got = dp.serve_run(arr, inst, dry_run=True, **kw)
+    ref = OS.replay(arr, inst, **kw)
+    for k in ref:
+        assert np.array_equal(got[k], ref[k]), k
+
+
+def test_oracle_hand_cases():
+    # one GPU, two instances, budget for one: A cold, A warm, B cold (evicts A), A cold again
+    arr = [0, 10, 20, 30]
+    inst = [0, 0, 1, 0]
+    r = OS.replay(arr, inst, ngpu=1, per_gpu_budget_bytes=100, cold_ns=[50], warm_ns=[5], resident_bytes=[100],
+                  model_of_instance=[0, 0])
+    assert list(r["cold"]) == [1, 0, 1, 1]
+    assert list(r["nevicted"]) == [0, 0, 1, 1]
+    assert list(r["start_ns"]) == [0, 50, 55, 105]  # one request at a time
+    assert list(r["finish_ns"]) == [50, 55, 105, 155]
+    # two GPUs: a cold request goes to the GPU that frees up first
+    r = OS.replay([0, 1, 2], [0, 1, 2], ngpu=2, per_gpu_budget_bytes=1000, cold_ns=[50], warm_ns=[5],
+                  resident_bytes=[10], model_of_instance=[0, 0, 0])
+    assert list(r["gpu"]) == [0, 1, 0] and list(r["start_ns"]) == [0, 1, 50]
+    # LRU: with budget 2, touching A makes B the victim
+    r = OS.replay([0, 100, 200, 300, 400], [0, 1, 0, 2, 1], ngpu=1, per_gpu_budget_bytes=20, cold_ns=[10],
+                  warm_ns=[1], resident_bytes=[10], model_of_instance=[0, 0, 0])
+    assert list(r["cold"]) == [1, 1, 0, 1, 1]  # C evicts B (LRU), B must reload
+
+
+def test_metrics():
+    r = {"finish_ns": np.array([10, 30, 200]), "cold": np.array([1, 0, 1])}
+    m = OS.metrics([0, 0, 0], r, slo_ns=100)
+    assert m["goodput"] == pytest.approx(2 / 3) and m["cold_rate"] == pytest.approx(2 / 3)
