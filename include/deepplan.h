@@ -202,6 +202,14 @@ int64_t dp_model_bytes(const dp_model* m);
 /* Host (mapped) address of the arena, for tests that read it back. */
 dp_status dp_model_arena(const dp_model* m, const void** ptr, int64_t* bytes);
 
+/* Transfer schedule of one plan slot (host-only, no GPU): the contiguous pieces (whole
+ * units, forward order, <= chunk_bytes unless one unit is larger) that the slot's link
+ * carries -- what dp_infer_cold DMAs on slot 0 and what secondary s sends / the primary
+ * receives for slot s >= 1.  Arrays of `cap` entries (nullable); *count = #pieces. */
+dp_status dp_transfer_schedule(const dp_model_config* cfg, const dp_plan* plan, int32_t slot, int64_t chunk_bytes,
+                               int64_t* piece_off, int64_t* piece_bytes, int32_t* first_unit, int32_t* last_unit,
+                               int32_t cap, int32_t* count);
+
 /* ---------------------------------------------------------------------------------
  * Profiling (§4.3.1; Table 5).  Per unit, median over `iters`
  * (after 3 warm-ups) of: load_ns (H2D of the unit alone on dev's link), fwd_ns (a peer
@@ -264,22 +272,25 @@ dp_status dp_host_free(void* p);
 
 /* Embedding: x[t,:] = LN(word[ids[t]] + pos[p(t)] + type[0]) for BERT/
  * RoBERTa (ln_g/ln_b non-NULL), or wte[ids[t]] + wpe[p(t)] for GPT-2 (type, ln NULL).
- * p(t) = pos_offset + (t mod seq).  Every table pointer may be host-mapped (DHA). */
+ * p(t) = pos_offset + (t mod seq).  Every table pointer may be host-mapped (DHA).
+ * out_f32 = 1 writes fp32 (the GPT-2 residual stream), else the storage dtype. */
 dp_status dp_embed(const int32_t* d_ids, int32_t ntok, int32_t seq, int32_t pos_offset, const void* word,
                    const void* pos, const void* type, const void* ln_g, const void* ln_b, int32_t hidden,
-                   double eps, int32_t dtype, void* d_out, void* stream);
+                   double eps, int32_t dtype, int32_t out_f32, void* d_out, void* stream);
 
 /* Linear: y[M,N] = act(x[M,K] w[N,K]^T + b) + residual, row strides ldx/ldy/ldr in
  * elements.  act: 0 none, 1 gelu_erf, 2 gelu_tanh, 3 tanh.  path: 0 = resident tcgen05/
  * TMA GEMM (w must be device memory, N % 128 == 0, K % 64 == 0), 1 = DHA skinny linear
- * (w may be host-mapped; reads every weight byte once). */
+ * (w may be host-mapped; reads every weight byte once).  io: bit0 = residual is fp32,
+ * bit1 = y is fp32 (otherwise the storage dtype). */
 dp_status dp_linear(const void* x, int32_t ldx, const void* w, const void* b, const void* residual, int32_t ldr,
                     void* y, int32_t ldy, int32_t M, int32_t N, int32_t K, int32_t act, int32_t path, int32_t dtype,
-                    void* stream);
+                    int32_t io, void* stream);
 
-/* LayerNorm over rows of width n: y = LN(x (+ r)) * g + b.  g/b may be host-mapped. */
+/* LayerNorm over rows of width n: y = LN(x (+ r)) * g + b.  g/b may be host-mapped.
+ * x_f32 = 1: x and r are fp32; y is always the storage dtype. */
 dp_status dp_layernorm(const void* x, const void* r, const void* g, const void* b, void* y, int32_t rows,
-                       int32_t n, double eps, int32_t dtype, void* stream);
+                       int32_t n, double eps, int32_t dtype, int32_t x_f32, void* stream);
 
 /* Attention core: qkv [ntok, 3H] (q | k | v column blocks, row stride ldqkv), heads of
  * d = H/heads (d == 64), softmax(q k^T / sqrt(d) [+ causal mask]) v -> ctx [ntok, H].

@@ -26,7 +26,7 @@ class DeepPlanError(RuntimeError):
 
 if not os.path.exists(_LIB_PATH):
     raise ImportError(
-        f"{_LIB_PATH} is missing: build it with `python -m paper_conf_eurosys_jeongba23_b200.build` "
+        f"{_LIB_PATH} is missing: build it with `python paper_conf_eurosys_jeongba23_b200/build.py` "
         "(there is no CPU fallback)")
 
 lib = C.CDLL(_LIB_PATH)
@@ -121,7 +121,9 @@ _sig("dp_model_num_units", [vp])
 _sig("dp_model_unit_info", [vp, C.c_int32, C.POINTER(UnitInfo)])
 _sig("dp_model_bytes", [vp], C.c_int64)
 _sig("dp_model_arena", [vp, C.POINTER(vp), i64p])
-_sig("dp_profile", [vp, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.POINTER(CostTable)])
+_sig("dp_transfer_schedule", [C.POINTER(ModelConfig), C.POINTER(Plan), C.c_int32, C.c_int64, i64p, i64p, i32p,
+                              i32p, C.c_int32, i32p])
+_sig("dp_profile",[vp, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.POINTER(CostTable)])
 _sig("dp_infer_cold", [vp, vp, C.POINTER(Plan), C.c_int32, i32p, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp, vp,
                        C.POINTER(RunStats)])
 _sig("dp_infer_warm", [vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp, vp, C.POINTER(RunStats)])
@@ -129,11 +131,11 @@ _sig("dp_model_evict", [vp, vp, C.c_int32])
 _sig("dp_model_is_resident", [vp, C.c_int32])
 _sig("dp_host_alloc", [C.c_int64, C.POINTER(vp)])
 _sig("dp_host_free", [vp])
-_sig("dp_embed", [vp, C.c_int32, C.c_int32, C.c_int32, vp, vp, vp, vp, vp, C.c_int32, C.c_double, C.c_int32, vp,
-                  vp])
+_sig("dp_embed", [vp, C.c_int32, C.c_int32, C.c_int32, vp, vp, vp, vp, vp, C.c_int32, C.c_double, C.c_int32,
+                  C.c_int32, vp, vp])
 _sig("dp_linear", [vp, C.c_int32, vp, vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
-                   C.c_int32, C.c_int32, C.c_int32, vp])
-_sig("dp_layernorm", [vp, vp, vp, vp, vp, C.c_int32, C.c_int32, C.c_double, C.c_int32, vp])
+                   C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
+_sig("dp_layernorm", [vp, vp, vp, vp, vp, C.c_int32, C.c_int32, C.c_double, C.c_int32, C.c_int32, vp])
 _sig("dp_attention", [vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
 _sig("dp_serve_run", [vp, C.POINTER(vp), C.c_int32, C.POINTER(TraceEvent), C.c_int32, C.POINTER(ServeOpts),
                       C.POINTER(ServeResult)])
@@ -307,6 +309,30 @@ def config_params(shape, dtype: str = "fp16"):
             for p in infos]
 
 
+def transfer_schedule(shape, plan: "PlanArrays", slot: int, chunk_bytes: int, dtype: str = "fp16"):
+    """Pieces (offset, bytes, first_unit, last_unit) carried by one plan slot's link."""
+    cfg = model_config(shape, dtype)
+    cnt = C.c_int32()
+    _check(lib.dp_transfer_schedule(C.byref(cfg), C.byref(plan.s), int(slot), int(chunk_bytes), None, None, None,
+                                    None, 0, C.byref(cnt)))
+    n = cnt.value
+    off, nb = np.zeros(n, np.int64), np.zeros(n, np.int64)
+    fu, lu = np.zeros(n, np.int32), np.zeros(n, np.int32)
+    _check(lib.dp_transfer_schedule(C.byref(cfg), C.byref(plan.s), int(slot), int(chunk_bytes), _ptr(off, i64p),
+                                    _ptr(nb, i64p), _ptr(fu, i32p), _ptr(lu, i32p), n, C.byref(cnt)))
+    return off, nb, fu, lu
+
+
+def config_units(shape, dtype: str = "fp16"):
+    """Unit names / byte counts of a config without registering a model (host-only)."""
+    ps = config_params(shape, dtype)
+    nunits = max(p["unit"] for p in ps) + 1
+    nb = np.zeros(nunits, np.int64)
+    for p in ps:
+        nb[p["unit"]] += p["bytes"]
+    return nb
+
+
 class Model:
     """A model registered in the library's pinned arena.  ``weights`` maps HF state-dict
     names to host arrays in the storage dtype (fp16 / bf16 bit patterns)."""
@@ -416,22 +442,23 @@ def host_free(p: int):
     _check(lib.dp_host_free(p))
 
 
-def embed(ids, seq, word, pos, type_, ln_g, ln_b, hidden, eps, out, dtype="fp16", pos_offset=0, stream=None):
+def embed(ids, seq, word, pos, type_, ln_g, ln_b, hidden, eps, out, dtype="fp16", pos_offset=0, out_f32=False,
+          stream=None):
     ntok = ids.numel() if hasattr(ids, "numel") else int(np.prod(ids.shape))
     _check(lib.dp_embed(_dptr(ids), ntok, int(seq), int(pos_offset), _dptr(word), _dptr(pos), _dptr(type_),
-                        _dptr(ln_g), _dptr(ln_b), int(hidden), float(eps), DTYPES[dtype], _dptr(out),
-                        _stream_ptr(stream)))
+                        _dptr(ln_g), _dptr(ln_b), int(hidden), float(eps), DTYPES[dtype], int(bool(out_f32)),
+                        _dptr(out), _stream_ptr(stream)))
 
 
-def linear(x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act="none", path=0, dtype="fp16", stream=None):
+def linear(x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act="none", path=0, dtype="fp16", io=0, stream=None):
     _check(lib.dp_linear(_dptr(x), int(ldx), _dptr(w), _dptr(b), _dptr(residual), int(ldr), _dptr(y), int(ldy),
                          int(M), int(N), int(K), ACTS[act] if isinstance(act, str) else int(act), int(path),
-                         DTYPES[dtype], _stream_ptr(stream)))
+                         DTYPES[dtype], int(io), _stream_ptr(stream)))
 
 
-def layernorm(x, r, g, b, y, rows, n, eps, dtype="fp16", stream=None):
+def layernorm(x, r, g, b, y, rows, n, eps, dtype="fp16", x_f32=False, stream=None):
     _check(lib.dp_layernorm(_dptr(x), _dptr(r), _dptr(g), _dptr(b), _dptr(y), int(rows), int(n), float(eps),
-                            DTYPES[dtype], _stream_ptr(stream)))
+                            DTYPES[dtype], int(bool(x_f32)), _stream_ptr(stream)))
 
 
 def attention(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp16", stream=None):

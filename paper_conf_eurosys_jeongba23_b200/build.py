@@ -1,5 +1,5 @@
 """Build libdeepplan.so (sm_100a) in-tree with nvcc.  Incremental: a translation unit is
-recompiled when it or any csrc header changed.  Usage: python -m paper_conf_eurosys_jeongba23_b200.build"""
+recompiled when it or any csrc header changed.  Usage: python paper_conf_eurosys_jeongba23_b200/build.py  (run by path: importing the package needs the library)"""
 from __future__ import annotations
 
 import glob

@@ -27,19 +27,19 @@ static void check_dtype(int32_t dtype) {
 
 extern "C" dp_status dp_embed(const int32_t* d_ids, int32_t ntok, int32_t seq, int32_t pos_offset, const void* word,
                               const void* pos, const void* type, const void* ln_g, const void* ln_b, int32_t hidden,
-                              double eps, int32_t dtype, void* d_out, void* stream) {
+                              double eps, int32_t dtype, int32_t out_f32, void* d_out, void* stream) {
   return guard([&] {
     check_dtype(dtype);
     DP_CHECK(d_ids && word && pos && d_out, DP_ERR_INVALID, "NULL pointer");
     DP_CHECK((ln_g == nullptr) == (ln_b == nullptr), DP_ERR_INVALID, "ln_g and ln_b must both be set or NULL");
     launch_embed(dtype, d_ids, ntok, seq, pos_offset, word, pos, type, ln_g, ln_b, hidden, (float)eps, d_out,
-                 (cudaStream_t)stream);
+                 out_f32 != 0, (cudaStream_t)stream);
   });
 }
 
 extern "C" dp_status dp_linear(const void* x, int32_t ldx, const void* w, const void* b, const void* residual,
                                int32_t ldr, void* y, int32_t ldy, int32_t M, int32_t N, int32_t K, int32_t act,
-                               int32_t path, int32_t dtype, void* stream) {
+                               int32_t path, int32_t dtype, int32_t io, void* stream) {
   return guard([&] {
     check_dtype(dtype);
     DP_CHECK(x && w && y, DP_ERR_INVALID, "NULL pointer");
@@ -50,9 +50,9 @@ extern "C" dp_status dp_linear(const void* x, int32_t ldx, const void* w, const 
       cudaPointerAttributes at;
       DP_CUDA(cudaPointerGetAttributes(&at, w));
       DP_CHECK(at.type == cudaMemoryTypeDevice, DP_ERR_INVALID, "the tcgen05 path needs W in device memory");
-      launch_gemm_tc(dtype, x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act, 0, (cudaStream_t)stream);
+      launch_gemm_tc(dtype, x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act, io, 0, (cudaStream_t)stream);
     } else if (path == 1) {
-      launch_skinny_linear(dtype, x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act, (cudaStream_t)stream);
+      launch_skinny_linear(dtype, x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act, io, (cudaStream_t)stream);
     } else {
       fail(DP_ERR_INVALID, "path must be 0 (tcgen05) or 1 (skinny/DHA)");
     }
@@ -60,11 +60,11 @@ extern "C" dp_status dp_linear(const void* x, int32_t ldx, const void* w, const 
 }
 
 extern "C" dp_status dp_layernorm(const void* x, const void* r, const void* g, const void* b, void* y, int32_t rows,
-                                  int32_t n, double eps, int32_t dtype, void* stream) {
+                                  int32_t n, double eps, int32_t dtype, int32_t x_f32, void* stream) {
   return guard([&] {
     check_dtype(dtype);
     DP_CHECK(x && g && b && y && rows >= 0, DP_ERR_INVALID, "bad arguments");
-    launch_layernorm(dtype, x, r, g, b, y, rows, n, (float)eps, (cudaStream_t)stream);
+    launch_layernorm(dtype, x, r, g, b, y, rows, n, (float)eps, x_f32 != 0, (cudaStream_t)stream);
   });
 }
 

@@ -64,6 +64,42 @@ __device__ __forceinline__ uint4 ldg16(const void* p) {
   return r;
 }
 
+// 8 consecutive elements at element index i of a T or fp32 array (f32 selects).
+template <class T>
+__device__ __forceinline__ void load8(const void* base, size_t i, float* f, int f32) {
+  if (f32) {
+    const float4* p = reinterpret_cast<const float4*>(static_cast<const float*>(base) + i);
+    const float4 a = p[0], b = p[1];
+    f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w; f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
+  } else {
+    unpack8<T>(ldg16(static_cast<const T*>(base) + i), f);
+  }
+}
+
+template <class T>
+__device__ __forceinline__ void store8(void* base, size_t i, const float* f, int f32) {
+  if (f32) {
+    float4* p = reinterpret_cast<float4*>(static_cast<float*>(base) + i);
+    p[0] = make_float4(f[0], f[1], f[2], f[3]);
+    p[1] = make_float4(f[4], f[5], f[6], f[7]);
+  } else {
+    *reinterpret_cast<uint4*>(static_cast<T*>(base) + i) = pack8<T>(f);
+  }
+}
+
+template <class T>
+__device__ __forceinline__ float load1(const void* base, size_t i, int f32) {
+  return f32 ? static_cast<const float*>(base)[i] : Cvt<T>::to1(static_cast<const T*>(base)[i]);
+}
+
+template <class T>
+__device__ __forceinline__ void store1(void* base, size_t i, float v, int f32) {
+  if (f32)
+    static_cast<float*>(base)[i] = v;
+  else
+    static_cast<T*>(base)[i] = Cvt<T>::from1(v);
+}
+
 __device__ __forceinline__ float warp_sum(float v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);

@@ -120,8 +120,8 @@ struct FmtBits<__nv_bfloat16> {
 template <class T, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmX,
-                   const T* __restrict__ bias, const T* res, int ldr, T* Y, int ldy, int M,
-                   int N, int K, int act) {
+                   const T* __restrict__ bias, const void* res, int ldr, void* Y, int ldy, int M,
+                   int N, int K, int act, int io) {
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
@@ -203,8 +203,8 @@ __global__ void __launch_bounds__(128, 1)
         const int m = m0 + c0 + j;
         if (m < M) {
           float val = apply_act(__uint_as_float(v[j]) + bv, act);
-          if (res) val += Cvt<T>::to1(res[(size_t)m * ldr + n]);
-          Y[(size_t)m * ldy + n] = Cvt<T>::from1(val);
+          if (res) val += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
+          store1<T>(Y, (size_t)m * ldy + n, val, io & IO_OUT_F32);
         }
       }
     }
@@ -248,7 +248,7 @@ CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int b
 
 template <class T, int BN>
 void run(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy, int M,
-         int N, int K, int act, cudaStream_t s) {
+         int N, int K, int act, int io, cudaStream_t s) {
   constexpr size_t smem = size_t(STAGES) * (BM * BK * 2 + BN * BK * 2) + 1024;
   static bool attr = false;
   if (!attr) {
@@ -259,18 +259,18 @@ void run(const void* x, int ldx, const void* w, const void* bias, const void* re
   CUtensorMap mw = make_map(w, dtype, N, K, K, BM);
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
   dim3 grid(N / BM, (M + BN - 1) / BN);
-  gemm_tc_kernel<T, BN><<<grid, 128, smem, s>>>(mw, mx, (const T*)bias, (const T*)res, ldr, (T*)y, ldy, M, N, K, act);
+  gemm_tc_kernel<T, BN><<<grid, 128, smem, s>>>(mw, mx, (const T*)bias, res, ldr, y, ldy, M, N, K, act, io);
   DP_CUDA(cudaGetLastError());
 }
 
 template <class T>
 void dispatch(int bn, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
-              int ldy, int M, int N, int K, int act, cudaStream_t s) {
+              int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   switch (bn) {
-    case 32: run<T, 32>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
-    case 64: run<T, 64>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
-    case 128: run<T, 128>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
-    case 256: run<T, 256>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s); break;
+    case 32: run<T, 32>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 64: run<T, 64>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 128: run<T, 128>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 256: run<T, 256>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
     default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
   }
 }
@@ -289,16 +289,16 @@ static int pick_bn(int M, int N) {
 }
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
-                    void* y, int ldy, int M, int N, int K, int act, int bn_hint, cudaStream_t s) {
+                    void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
   DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
   DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0 && ((uintptr_t)w % 16) == 0, DP_ERR_INVALID,
            "GEMM operands must be 16-byte aligned");
   if (M <= 0) return;
   const int bn = bn_hint > 0 ? bn_hint : pick_bn(M, N);
   if (dtype == DP_BF16)
-    dispatch<__nv_bfloat16>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s);
+    dispatch<__nv_bfloat16>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
   else
-    dispatch<__half>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s);
+    dispatch<__half>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
 }
 
 }  // namespace dp

@@ -203,6 +203,32 @@ std::vector<Piece> slot_pieces(const dp_model* m, const dp_plan* plan, int slot,
   return make_pieces(m, [&](int u) { return plan->method[u] == DP_LOAD && plan->slot[u] == slot; }, cap);
 }
 
+}  // namespace dp
+
+extern "C" dp_status dp_transfer_schedule(const dp_model_config* cfg, const dp_plan* plan, int32_t slot,
+                                          int64_t chunk_bytes, int64_t* piece_off, int64_t* piece_bytes,
+                                          int32_t* first_unit, int32_t* last_unit, int32_t cap, int32_t* count) {
+  return dp::guard([&] {
+    DP_CHECK(cfg && plan && count, DP_ERR_INVALID, "NULL argument");
+    dp_model tmp;
+    tmp.cfg = *cfg;
+    tmp.params = dp::config_params(*cfg);
+    dp::build_units(&tmp);
+    DP_CHECK(plan->n == (int)tmp.units.size() && plan->method && plan->slot, DP_ERR_INVALID, "plan/model mismatch");
+    DP_CHECK(slot >= 0 && slot < plan->k, DP_ERR_INVALID, "slot out of range");
+    auto pcs = dp::slot_pieces(&tmp, plan, slot, std::max<int64_t>(chunk_bytes, 4096));
+    *count = (int32_t)pcs.size();
+    for (int i = 0; i < (int)pcs.size() && i < cap; ++i) {
+      if (piece_off) piece_off[i] = pcs[i].off;
+      if (piece_bytes) piece_bytes[i] = pcs[i].bytes;
+      if (first_unit) first_unit[i] = pcs[i].first_unit;
+      if (last_unit) last_unit[i] = pcs[i].last_unit;
+    }
+  });
+}
+
+namespace dp {
+
 void bind_units(std::vector<cudaEvent_t>& unit_ev, const Piece& p, cudaEvent_t e) {
   for (int u = p.first_unit; u <= p.last_unit; ++u) unit_ev[u] = e;
 }
@@ -268,7 +294,7 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   // (1) slot-0 loads on the primary's link
   const int64_t cap = std::max<int64_t>(ctx->opts.chunk_bytes, 4096);
   auto pieces0 = make_pieces(m, [&](int u) { return method[u] == DP_LOAD && plan->slot[u] == 0; }, cap);
-  const int nh = (int)pd.h2d.size();
+  const int nh = std::min((int)pd.h2d.size(), std::max(1, ctx->opts.n_h2d_streams));
   for (int i = 0; i < nh; ++i) DP_CUDA(cudaStreamWaitEvent(pd.h2d[i], fork, 0));
   for (size_t c = 0; c < pieces0.size(); ++c) {
     const Piece& p = pieces0[c];
@@ -534,6 +560,9 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
     std::vector<float> v;
     for (int it = 0; it < warm + iters; ++it) {
       if (flush) launch_l2_flush(d.flush, d.flush_bytes, s);
+      // keep the stream busy while the host enqueues the measured work, so the interval
+      // e0..e1 holds device time only (not the host's launch latency)
+      launch_spin(60000, s);
       DP_CUDA(cudaEventRecord(e0, s));
       body();
       DP_CUDA(cudaEventRecord(e1, s));

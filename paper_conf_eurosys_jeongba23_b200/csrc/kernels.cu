@@ -24,7 +24,8 @@ namespace dp {
 template <class T, int VPL>
 __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ ids, int ntok, int seq, int pos_off,
                                                     const T* word, const T* pos, const T* type, const T* g,
-                                                    const T* b, int H, float eps, T* __restrict__ out) {
+                                                    const T* b, int H, float eps, void* __restrict__ out_,
+                                                    int out_f32) {
   extern __shared__ uint4 sm[];  // [type0 | gamma | beta] as 16-byte vectors
   const int nv = H / 8;
   const bool has_type = type != nullptr, has_ln = g != nullptr;
@@ -70,12 +71,11 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
       for (int e = 0; e < 8; ++e) sum += x[v][e];
     }
   }
-  T* o = out + (size_t)t * H;
   if (!has_ln) {
 #pragma unroll
     for (int v = 0; v < VPL; ++v) {
       const int c = lane + 32 * v;
-      if (c < nv) reinterpret_cast<uint4*>(o)[c] = pack8<T>(x[v]);
+      if (c < nv) store8<T>(out_, (size_t)t * H + 8 * c, x[v], out_f32);
     }
     return;
   }
@@ -102,21 +102,22 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
       unpack8<T>(sm[2 * nv + c], bb);
 #pragma unroll
       for (int e = 0; e < 8; ++e) y[e] = (x[v][e] - mean) * rstd * gg[e] + bb[e];
-      reinterpret_cast<uint4*>(o)[c] = pack8<T>(y);
+      store8<T>(out_, (size_t)t * H + 8 * c, y, out_f32);
     }
   }
 }
 
 template <class T>
 static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
-                    const void* type, const void* g, const void* b, int H, float eps, void* out, cudaStream_t s) {
+                    const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
+                    cudaStream_t s) {
   const int warps = 8;
   dim3 grid((ntok + warps - 1) / warps);
   const size_t sm = size_t(3) * (H / 8) * 16;
   const int vpl = (H / 8 + 31) / 32;
 #define DP_EMB(V)                                                                                      \
   embed_kernel<T, V><<<grid, warps * 32, sm, s>>>(ids, ntok, seq, pos_off, (const T*)word, (const T*)pos, \
-                                                  (const T*)type, (const T*)g, (const T*)b, H, eps, (T*)out)
+                                                  (const T*)type, (const T*)g, (const T*)b, H, eps, out, out_f32)
   switch (vpl) {
     case 1: DP_EMB(1); break;
     case 2: DP_EMB(2); break;
@@ -131,23 +132,24 @@ static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const vo
 }
 
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
-                  const void* type, const void* g, const void* b, int H, float eps, void* out, cudaStream_t s) {
+                  const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
+                  cudaStream_t s) {
   DP_CHECK(H % 8 == 0 && H > 0, DP_ERR_INVALID, "hidden must be a multiple of 8");
   DP_CHECK(seq > 0 && ntok >= 0, DP_ERR_INVALID, "bad token counts");
   if (ntok == 0) return;
   if (dtype == DP_BF16)
-    embed_t<__nv_bfloat16>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, s);
+    embed_t<__nv_bfloat16>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, s);
   else
-    embed_t<__half>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, s);
+    embed_t<__half>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, s);
 }
 
 // -------------------------------------------------------------------------------------
 // K4: LayerNorm (+ residual).  gamma/beta staged once per CTA (they may be host-mapped).
 // -------------------------------------------------------------------------------------
 template <class T, int VPL>
-__global__ void __launch_bounds__(256) layernorm_kernel(const T* __restrict__ x, const T* __restrict__ r,
+__global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__ x, const void* __restrict__ r,
                                                         const T* g, const T* b, T* __restrict__ y, int rows,
-                                                        int n, float eps) {
+                                                        int n, float eps, int in_f32) {
   extern __shared__ uint4 sm[];  // [gamma | beta]
   const int nv = n / 8;
   for (int i = threadIdx.x; i < 2 * nv; i += blockDim.x) sm[i] = ldg16(i < nv ? g + 8 * i : b + 8 * (i - nv));
@@ -161,10 +163,10 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const T* __restrict__ x,
     for (int k = 0; k < VPL; ++k) {
       const int c = lane + 32 * k;
       if (c < nv) {
-        unpack8<T>(ldg16(x + (size_t)row * n + 8 * c), v[k]);
+        load8<T>(x, (size_t)row * n + 8 * c, v[k], in_f32);
         if (r) {
           float a[8];
-          unpack8<T>(ldg16(r + (size_t)row * n + 8 * c), a);
+          load8<T>(r, (size_t)row * n + 8 * c, a, in_f32);
 #pragma unroll
           for (int e = 0; e < 8; ++e) v[k][e] += a[e];
         }
@@ -203,15 +205,15 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const T* __restrict__ x,
 
 template <class T>
 static void layernorm_t(const void* x, const void* r, const void* g, const void* b, void* y, int rows, int n,
-                        float eps, cudaStream_t s) {
+                        float eps, bool in_f32, cudaStream_t s) {
   const int warps = 8;
   int grid = (rows + 4 * warps - 1) / (4 * warps);  // ~4 rows per warp: few CTAs -> few host reads of g/b
   if (grid < 1) grid = 1;
   const size_t sm = size_t(2) * (n / 8) * 16;
   const int vpl = (n / 8 + 31) / 32;
 #define DP_LN(V)                                                                                       \
-  layernorm_kernel<T, V><<<grid, warps * 32, sm, s>>>((const T*)x, (const T*)r, (const T*)g, (const T*)b, \
-                                                      (T*)y, rows, n, eps)
+  layernorm_kernel<T, V><<<grid, warps * 32, sm, s>>>(x, r, (const T*)g, (const T*)b, (T*)y, rows, n, eps, \
+                                                      in_f32)
   switch (vpl) {
     case 1: DP_LN(1); break;
     case 2: DP_LN(2); break;
@@ -226,13 +228,13 @@ static void layernorm_t(const void* x, const void* r, const void* g, const void*
 }
 
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
-                      int n, float eps, cudaStream_t s) {
+                      int n, float eps, bool in_f32, cudaStream_t s) {
   DP_CHECK(n % 8 == 0 && n > 0, DP_ERR_INVALID, "LN width must be a multiple of 8");
   if (rows <= 0) return;
   if (dtype == DP_BF16)
-    layernorm_t<__nv_bfloat16>(x, r, g, b, y, rows, n, eps, s);
+    layernorm_t<__nv_bfloat16>(x, r, g, b, y, rows, n, eps, in_f32, s);
   else
-    layernorm_t<__half>(x, r, g, b, y, rows, n, eps, s);
+    layernorm_t<__half>(x, r, g, b, y, rows, n, eps, in_f32, s);
 }
 
 // -------------------------------------------------------------------------------------
@@ -245,9 +247,9 @@ void launch_layernorm(int dtype, const void* x, const void* r, const void* g, co
 // -------------------------------------------------------------------------------------
 template <class T, int R>
 __global__ void __launch_bounds__(256) skinny_linear_kernel(const T* __restrict__ X, int ldx, const T* W,
-                                                            const T* bias, const T* res, int ldr,
-                                                            T* Y, int ldy, int M, int N, int K,
-                                                            int act) {
+                                                            const T* bias, const void* res, int ldr,
+                                                            void* Y, int ldy, int M, int N, int K,
+                                                            int act, int io) {
   extern __shared__ uint4 sw[];  // R*K/8 vectors (+ R bias values)
   const int kv = K / 8;
   const int n0 = blockIdx.x * R;
@@ -296,15 +298,15 @@ __global__ void __launch_bounds__(256) skinny_linear_kernel(const T* __restrict_
     if (lane < rows) {
       const int n = n0 + lane;
       float v = apply_act(mine + sbias[lane], act);
-      if (res) v += Cvt<T>::to1(res[(size_t)m * ldr + n]);
-      Y[(size_t)m * ldy + n] = Cvt<T>::from1(v);
+      if (res) v += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
+      store1<T>(Y, (size_t)m * ldy + n, v, io & IO_OUT_F32);
     }
   }
 }
 
 template <class T>
 static void skinny_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
-                     int ldy, int M, int N, int K, int act, cudaStream_t s) {
+                     int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   constexpr int R = 8;
   const size_t sm = size_t(R) * K * sizeof(T);
   static bool attr_set = false;  // one per template instantiation
@@ -313,19 +315,19 @@ static void skinny_t(const void* x, int ldx, const void* w, const void* bias, co
     attr_set = true;
   }
   skinny_linear_kernel<T, R><<<(N + R - 1) / R, 256, sm, s>>>((const T*)x, ldx, (const T*)w, (const T*)bias,
-                                                               (const T*)res, ldr, (T*)y, ldy, M, N, K, act);
+                                                               res, ldr, y, ldy, M, N, K, act, io);
   DP_CUDA(cudaGetLastError());
 }
 
 void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
-                          int ldr, void* y, int ldy, int M, int N, int K, int act, cudaStream_t s) {
+                          int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   DP_CHECK(K % 8 == 0 && K > 0 && N > 0, DP_ERR_INVALID, "skinny linear needs K % 8 == 0");
   DP_CHECK(size_t(8) * K * 2 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
   if (M <= 0) return;
   if (dtype == DP_BF16)
-    skinny_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s);
+    skinny_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
   else
-    skinny_t<__half>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s);
+    skinny_t<__half>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
 }
 
 // -------------------------------------------------------------------------------------

@@ -7,20 +7,22 @@ namespace dp {
 
 // Epilogue activations (dp_linear's `act`).
 enum Act { ACT_NONE = 0, ACT_GELU_ERF = 1, ACT_GELU_TANH = 2, ACT_TANH = 3 };
+// Linear epilogue I/O precision (the pre-LN GPT-2 residual stream is kept in fp32).
+enum Io { IO_RES_F32 = 1, IO_OUT_F32 = 2 };
 
 // K1: fused embedding gather (+ LayerNorm) -- SURVEY §8(a) a10.  Table pointers may be
 // host-mapped (direct-host-access).  ln_g == nullptr -> no LN (GPT-2).
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
-                  const void* type, const void* ln_g, const void* ln_b, int H, float eps, void* out,
+                  const void* type, const void* ln_g, const void* ln_b, int H, float eps, void* out, bool out_f32,
                   cudaStream_t s);
 
 // K4: y = LN(x (+ r)) * g + b; g/b may be host-mapped.
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
-                      int n, float eps, cudaStream_t s);
+                      int n, float eps, bool in_f32, cudaStream_t s);
 
 // K3: skinny linear reading W exactly once (W may be host-mapped) -- a11.
 void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
-                          int ldr, void* y, int ldy, int M, int N, int K, int act, cudaStream_t s);
+                          int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s);
 
 // K5: attention core (mma.sync flash attention, d = 64).
 void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
@@ -30,7 +32,7 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
 struct GemmPlan;  // cached tensor map for a weight
 bool gemm_tc_supported(int N, int K);
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
-                    void* y, int ldy, int M, int N, int K, int act, int bn_hint, cudaStream_t s);
+                    void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);
 
 // Scratch kernels
 void launch_l2_flush(void* buf, size_t bytes, cudaStream_t s);

@@ -88,7 +88,7 @@ std::vector<ParamDesc> config_params(const dp_model_config& c) {
   return ps;
 }
 
-static void build_units(dp_model* m) {
+void build_units(dp_model* m) {
   const auto& c = m->cfg;
   auto& U = m->units;
   int pi = 0;

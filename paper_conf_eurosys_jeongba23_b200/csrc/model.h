@@ -61,6 +61,12 @@ void validate_config(const dp_model_config& c);
 
 }  // namespace dp
 
+struct dp_model;
+namespace dp {
+// Units + arena layout for m->cfg / m->params (host-only; no allocation).
+void build_units(dp_model* m);
+}  // namespace dp
+
 struct dp_model {
   dp_model_config cfg{};
   std::vector<dp::ParamDesc> params;

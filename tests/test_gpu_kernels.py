@@ -212,3 +212,29 @@ def test_attention_parity(B, S, H, heads, causal, dtype):
     tol = (4 if dtype == "fp16" else 8) * EPS_OUT[dtype] * (np.abs(ref) + np.abs(q64).max())
     err = np.abs(f64(O) - ref)
     assert np.all(err <= tol), err.max()
+
+
+def test_fp32_residual_stream_io():
+    """GPT-2's pre-LN residual stream stays fp32: linear with fp32 residual+output (io=3),
+    LayerNorm reading fp32, embedding writing fp32."""
+    rng = np.random.default_rng(77)
+    M, N, K = 130, 256, 512
+    x = synth.round_to(rng.standard_normal((M, K)).astype(np.float32), "fp16")
+    wt = synth.round_to((rng.standard_normal((N, K)) / 22).astype(np.float32), "fp16")
+    r = (rng.standard_normal((M, N)) * 3).astype(np.float32)
+    X, W = to_t(x, "fp16"), to_t(wt, "fp16")
+    for path in (0, 1):
+        R = torch.from_numpy(r.copy()).cuda()
+        dp().linear(X, K, W, None, R, N, R, N, M, N, K, path=path, io=3)  # in place, fp32
+        torch.cuda.synchronize()
+        ref = F.linear(x.astype(np.float64), wt.astype(np.float64), None, "none", r.astype(np.float64))
+        err = np.abs(R.cpu().numpy().astype(np.float64) - ref)
+        assert err.max() <= 1e-4 * (1 + np.abs(ref).max()), err.max()
+    g = synth.round_to((1 + 0.1 * rng.standard_normal(N)).astype(np.float32), "fp16")
+    b = synth.round_to((0.1 * rng.standard_normal(N)).astype(np.float32), "fp16")
+    Rt = torch.from_numpy(r).cuda()
+    Y = torch.empty(M, N, dtype=torch.float16, device="cuda")
+    dp().layernorm(Rt, None, to_t(g, "fp16"), to_t(b, "fp16"), Y, M, N, 1e-5, x_f32=True)
+    torch.cuda.synchronize()
+    ref = F.layer_norm(r.astype(np.float64), g.astype(np.float64), b.astype(np.float64), 1e-5)
+    close(f64(Y), ref, "fp16", K=N, scale=8)
