@@ -196,6 +196,10 @@ dp_status dp_config_params(const dp_model_config* cfg, dp_param_info* infos, int
 dp_status dp_model_create(dp_context* ctx, const dp_model_config* cfg, const void* const* host_params,
                           int32_t nparams, dp_model** out);
 dp_status dp_model_destroy(dp_context* ctx, dp_model* m);
+/* Another instance of the same model (serving, "each instance mimics a model
+ * corresponding to a different user"): shares src's pinned arena read-only (freed with the
+ * last instance), has its own residency and device state. */
+dp_status dp_model_clone(dp_context* ctx, const dp_model* src, dp_model** out);
 int32_t dp_model_num_units(const dp_model* m);
 dp_status dp_model_unit_info(const dp_model* m, int32_t i, dp_unit_info* out);
 int64_t dp_model_bytes(const dp_model* m);

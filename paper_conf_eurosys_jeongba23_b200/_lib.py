@@ -117,6 +117,7 @@ _sig("dp_peer_init", [vp, vp, C.c_int32, C.c_int32])
 _sig("dp_config_params", [C.POINTER(ModelConfig), C.POINTER(ParamInfo), C.c_int32, i32p])
 _sig("dp_model_create", [vp, C.POINTER(ModelConfig), C.POINTER(vp), C.c_int32, C.POINTER(vp)])
 _sig("dp_model_destroy", [vp, vp])
+_sig("dp_model_clone", [vp, vp, C.POINTER(vp)])
 _sig("dp_model_num_units", [vp])
 _sig("dp_model_unit_info", [vp, C.c_int32, C.POINTER(UnitInfo)])
 _sig("dp_model_bytes", [vp], C.c_int64)
@@ -355,6 +356,14 @@ class Model:
         _check(lib.dp_model_create(ctx.h, C.byref(self.cfg), ptrs, len(params), C.byref(h)))
         self.h = h
         self.n = lib.dp_model_num_units(h)
+
+    def clone(self) -> "Model":
+        m = Model.__new__(Model)
+        m.ctx, m.shape, m.dtype, m.cfg, m.n = self.ctx, self.shape, self.dtype, self.cfg, self.n
+        h = vp()
+        _check(lib.dp_model_clone(self.ctx.h, self.h, C.byref(h)))
+        m.h = h
+        return m
 
     def units(self):
         out = []

@@ -262,12 +262,61 @@ static int64_t dha_bytes(const dp_model* m, const int8_t* method, int T, int seq
 
 // `primary` is the serving device ordinal; `prim_rank` its rank when the PT gather runs over
 // NCCL between processes (then secondaries are ranks, see peer.cpp).
+static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, int prim_rank,
+                                 const int32_t* secondaries, const int32_t* ids, int batch, int seq, void* out,
+                                 void* pooled, cudaStream_t stream);
+
+// Key of a captured cold-start / warm graph: everything the enqueued work depends on.
+static std::string graph_key(const dp_context* ctx, const dp_plan* plan, const int32_t* secondaries, const void* ids,
+                             int batch, int seq, const void* out, const void* pooled) {
+  std::string k;
+  if (plan) {
+    k.append(reinterpret_cast<const char*>(plan->method), plan->n);
+    k.append(reinterpret_cast<const char*>(plan->slot), plan->n);
+    k += "|" + std::to_string(plan->k);
+    for (int s = 1; s < plan->k; ++s) k += "," + std::to_string(secondaries[s - 1]);
+  }
+  k += "|" + std::to_string((uintptr_t)ids) + "|" + std::to_string((uintptr_t)out) + "|" +
+       std::to_string((uintptr_t)pooled) + "|" + std::to_string(batch) + "x" + std::to_string(seq) + "|" +
+       std::to_string(ctx->opts.chunk_bytes) + "," + std::to_string(ctx->opts.n_h2d_streams) + "," +
+       std::to_string(ctx->opts.gemm_bn) + "," + std::to_string(ctx->opts.debug_delay_us);
+  return k;
+}
+
+// Capture `body` (which enqueues on `stream` and joins every side stream back into it) into
+// a CUDA graph once per key; afterwards replay it.  Replay removes the host enqueue cost and
+// turns the per-piece events into graph edges.
+template <class Body>
+static dp_run_stats run_graph(DevState& ds, const std::string& key, cudaStream_t stream, Body body) {
+  auto it = ds.graphs.find(key);
+  if (it == ds.graphs.end()) {
+    cudaGraph_t gph = nullptr;
+    DP_CUDA(cudaStreamBeginCapture(stream, cudaStreamCaptureModeRelaxed));
+    dp_run_stats st;
+    try {
+      st = body();
+    } catch (...) {
+      cudaStreamEndCapture(stream, &gph);
+      if (gph) cudaGraphDestroy(gph);
+      throw;
+    }
+    DP_CUDA(cudaStreamEndCapture(stream, &gph));
+    cudaGraphExec_t ex = nullptr;
+    cudaError_t e = cudaGraphInstantiate(&ex, gph, 0);
+    cudaGraphDestroy(gph);
+    DP_CUDA(e);
+    it = ds.graphs.emplace(key, GraphEntry{ex, st}).first;
+  }
+  DP_CUDA(cudaGraphLaunch(it->second.exec, stream));
+  return it->second.stats;
+}
+
 void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, int prim_rank,
                 const int32_t* secondaries, int nsec, const int32_t* ids, int batch, int seq, void* out, void* pooled,
                 cudaStream_t stream, dp_run_stats* stats) {
   auto t0 = std::chrono::steady_clock::now();
   validate_plan(m, plan);
-  DevCtx& pd = ctx->on(primary);
+  ctx->on(primary);
   DevState& ds = m->dev[primary];
   DP_CHECK(!ds.resident, DP_ERR_STATE, "model already resident on the primary; evict it first");
   DP_CHECK(ctx->comm || nsec >= plan->k - 1, DP_ERR_INVALID, "need k-1 secondaries for the plan");
@@ -278,6 +327,28 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   ensure_slots(m, primary);
   ensure_h2d_streams(ctx, primary);
   ensure_workspace(m, primary, int64_t(batch) * seq);
+  bool graph = ctx->opts.use_graph != 0 && !ctx->comm;
+  for (int s = 1; s < plan->k && graph; ++s) graph = secondaries[s - 1] == primary;  // single-device graphs only
+  dp_run_stats st;
+  if (graph) {
+    st = run_graph(ds, graph_key(ctx, plan, secondaries, ids, batch, seq, out, pooled), stream, [&] {
+      return enqueue_cold(ctx, m, plan, primary, prim_rank, secondaries, ids, batch, seq, out, pooled, stream);
+    });
+  } else {
+    st = enqueue_cold(ctx, m, plan, primary, prim_rank, secondaries, ids, batch, seq, out, pooled, stream);
+  }
+  ds.resident = true;
+  ds.method.assign(plan->method, plan->method + plan->n);
+  st.wall_enqueue_us =
+      std::chrono::duration<float, std::micro>(std::chrono::steady_clock::now() - t0).count();
+  if (stats) *stats = st;
+}
+
+static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, int prim_rank,
+                                 const int32_t* secondaries, const int32_t* ids, int batch, int seq, void* out,
+                                 void* pooled, cudaStream_t stream) {
+  DevCtx& pd = ctx->on(primary);
+  DevState& ds = m->dev[primary];
   pd.events.reset();
   const int n = (int)m->units.size();
   const int8_t* method = plan->method;
@@ -401,13 +472,9 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
     DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
   }
   if (ctx->comm) peer_join(ctx, stream);
-  ds.resident = true;
-  ds.method.assign(method, method + n);
   st.n_kernels = a.kernels;
   st.dha_weight_bytes = dha_bytes(m, method, batch * seq, seq);
-  st.wall_enqueue_us =
-      std::chrono::duration<float, std::micro>(std::chrono::steady_clock::now() - t0).count();
-  if (stats) *stats = st;
+  return st;
 }
 
 }  // namespace dp
@@ -453,7 +520,19 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.pooled = d_pooled;
     a.stream = (cudaStream_t)stream;
     a.bn_hint = ctx->opts.gemm_bn;
-    run_forward(a);
+    if (ctx->opts.use_graph) {
+      std::string key = "warm|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
+                        graph_key(ctx, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);
+      dp_run_stats gs = run_graph(ds, key, (cudaStream_t)stream, [&] {
+        run_forward(a);
+        dp_run_stats s{};
+        s.n_kernels = a.kernels;
+        return s;
+      });
+      a.kernels = gs.n_kernels;
+    } else {
+      run_forward(a);
+    }
     if (stats) {
       std::memset(stats, 0, sizeof(*stats));
       stats->n_kernels = a.kernels;
@@ -492,12 +571,13 @@ extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
       if (ds.dbase || ds.ws.base) {
         DeviceGuard g(d);
         cudaDeviceSynchronize();
+        for (auto& kv : ds.graphs) cudaGraphExecDestroy(kv.second.exec);
+        ds.graphs.clear();
         if (ds.dbase) cudaFree(ds.dbase);
         if (ds.ws.base) cudaFree(ds.ws.base);
       }
     }
-    if (m->arena) cudaFreeHost(m->arena);
-    delete m;
+    delete m;  // the last instance sharing the arena frees it
   });
 }
 

@@ -256,16 +256,15 @@ __global__ void __launch_bounds__(256) skinny_linear_kernel(const T* __restrict_
   const int rows = min(R, N - n0);
   const int total = rows * kv;
   const uint4* src = reinterpret_cast<const uint4*>(W + (size_t)n0 * K);
-  {
-    int i = threadIdx.x;
-    for (; i + 3 * 256 < total; i += 4 * 256) {  // 4 independent 16 B loads in flight per thread
-      uint4 a = ldg16(src + i), b = ldg16(src + i + 256), c = ldg16(src + i + 512), d = ldg16(src + i + 768);
-      sw[i] = a;
-      sw[i + 256] = b;
-      sw[i + 512] = c;
-      sw[i + 768] = d;
-    }
-    for (; i < total; i += 256) sw[i] = ldg16(src + i);
+  // up to 8 independent 16-byte loads in flight per thread before the first store
+  for (int base = threadIdx.x; base < total; base += 8 * 256) {
+    uint4 r[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if (base + j * 256 < total) r[j] = ldg16(src + base + j * 256);
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if (base + j * 256 < total) sw[base + j * 256] = r[j];
   }
   __shared__ float sbias[R];
   if (threadIdx.x < rows) sbias[threadIdx.x] = bias ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;

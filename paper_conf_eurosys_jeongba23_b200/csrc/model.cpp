@@ -197,6 +197,7 @@ extern "C" dp_status dp_model_create(dp_context* ctx, const dp_model_config* cfg
       m->arena = nullptr;
       fail(DP_ERR_OOM, std::string("cudaHostAlloc of the weight arena failed: ") + cudaGetErrorString(e));
     }
+    m->arena_owner = std::shared_ptr<void>(m->arena, [](void* p) { cudaFreeHost(p); });
     std::memset(m->arena, 0, m->arena_bytes);
     uint8_t* base = static_cast<uint8_t*>(m->arena);
     for (size_t i = 0; i < m->params.size(); ++i) {
@@ -214,11 +215,22 @@ extern "C" dp_status dp_model_create(dp_context* ctx, const dp_model_config* cfg
     }
     *out = m;
   });
-  if (st != DP_OK && m) {
-    if (m->arena) cudaFreeHost(m->arena);
-    delete m;
-  }
+  if (st != DP_OK && m) delete m;  // the arena owner frees the pinned memory
   return st;
+}
+
+extern "C" dp_status dp_model_clone(dp_context* ctx, const dp_model* src, dp_model** out) {
+  return guard([&] {
+    DP_CHECK(src && out, DP_ERR_INVALID, "NULL argument");
+    dp_model* m = new dp_model();
+    m->cfg = src->cfg;
+    m->params = src->params;
+    m->units = src->units;
+    m->arena = src->arena;
+    m->arena_bytes = src->arena_bytes;
+    m->arena_owner = src->arena_owner;
+    *out = m;
+  });
 }
 
 extern "C" int32_t dp_model_num_units(const dp_model* m) { return m ? (int32_t)m->units.size() : 0; }

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <map>
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -49,11 +50,17 @@ struct Workspace {
   void* base = nullptr;
 };
 
+struct GraphEntry {
+  cudaGraphExec_t exec = nullptr;
+  dp_run_stats stats{};
+};
+
 struct DevState {
   void* dbase = nullptr;  // HBM copy of the arena layout (slots for loaded units)
   bool resident = false;
   std::vector<int8_t> method;  // per unit, fixed when the model became resident
   Workspace ws;
+  std::map<std::string, GraphEntry> graphs;  // captured cold / warm runs (opts.use_graph)
 };
 
 std::vector<ParamDesc> config_params(const dp_model_config& c);
@@ -72,6 +79,7 @@ struct dp_model {
   std::vector<dp::ParamDesc> params;
   std::vector<dp::UnitDesc> units;
   void* arena = nullptr;  // cudaHostAlloc(Portable | Mapped)
+  std::shared_ptr<void> arena_owner;  // shared by dp_model_clone instances
   int64_t arena_bytes = 0;
   dp::DevState dev[DP_MAX_DEVICES];
 

@@ -226,3 +226,36 @@ def test_gpt2_medium_causal_prefix_full_size():
     model.evict(0)
     assert np.abs(f64(out[:48]) - ref.reshape(48, -1)).max() <= 1e-2
     model.close()
+
+
+@pytest.mark.parametrize("name,mode,k", [("tiny_bert", "DHA", 1), ("tiny_gpt2", "PT_DHA", 2),
+                                         ("bert_base", "DHA", 1)])
+def test_graph_replay_matches_eager(name, mode, k):
+    """opts.use_graph captures the cold start (DMAs, events as edges, kernels) once and
+    replays it: outputs must equal the eager run bit for bit, across repeated replays."""
+    m = synth.SHAPES[name]
+    dtype = "fp16"
+    w = synth.make_weights(m, seed=14, dtype=dtype)
+    ids = synth.make_ids(m, 1, 64, seed=15)
+    c = dp().Context([0])
+    model = dp().Model(c, m, w, dtype)
+    plan = dp().plan_generate(fake_cost(m, dtype), mode, k)
+    eager, pe, st0 = run_cold(model, plan, ids, dtype, secondaries=[0] * (k - 1))
+    eager = eager.clone()
+    model.evict(0)
+    c.set_opts(use_graph=1, debug_poison=1)
+    ids_t = torch.from_numpy(ids).cuda()
+    out = torch.empty_like(eager)
+    pool = torch.empty_like(pe) if pe is not None else None
+    for _ in range(3):
+        st = model.infer_cold(plan, 0, ids_t, out, pool, secondaries=[0] * (k - 1))
+        torch.cuda.synchronize()
+        assert torch.equal(out, eager)
+        assert st["h2d_bytes"] == st0["h2d_bytes"]
+        w_out = torch.empty_like(out)
+        model.infer_warm(0, ids_t, w_out, pool)
+        torch.cuda.synchronize()
+        assert torch.equal(w_out, eager)
+        model.evict(0)
+    model.close()
+    c.close()

@@ -1,0 +1,87 @@
+"""Per-kernel device timings through the C-ABI hooks (CUDA events around back-to-back
+launches on one stream, after warm-up).  Used with ncu too:
+  ncu --set full -k regex:gemm_tc -c 3 python tools/kbench.py gemm
+python tools/kbench.py [all|gemm|ln|attn|skinny|embed] [reps]"""
+import json
+import math
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import paper_conf_eurosys_jeongba23_b200 as dp
+
+which = sys.argv[1] if len(sys.argv) > 1 else "all"
+reps = int(sys.argv[2]) if len(sys.argv) > 2 else 50
+torch.manual_seed(0)
+res = {}
+
+
+def timeit(fn, n=reps):
+    for _ in range(3):
+        fn()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(n):
+        fn()
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) * 1e3 / n  # us per launch
+
+
+if which in ("all", "gemm"):
+    for (M, N, K) in [(128, 768, 768), (128, 3072, 768), (128, 768, 3072), (384, 1024, 1024), (384, 4096, 1024),
+                      (384, 1024, 4096), (1024, 3072, 1024), (1024, 4096, 1024), (1024, 1024, 4096)]:
+        x = torch.randn(M, K, device="cuda").half()
+        w = (torch.randn(N, K, device="cuda") / math.sqrt(K)).half()
+        b = torch.randn(N, device="cuda").half()
+        y = torch.empty(M, N, device="cuda").half()
+        for bn in (0,):
+            us = timeit(lambda: dp.linear(x, K, w, b, None, 0, y, N, M, N, K, path=0))
+            flops = 2 * M * N * K
+            byts = 2 * (N * K + M * K + M * N)
+            res[f"gemm_tc M{M} N{N} K{K}"] = {"us": round(us, 2), "tflops": round(flops / us / 1e6, 1),
+                                             "gbs": round(byts / us / 1e3, 1)}
+        ref_us = timeit(lambda: torch.nn.functional.linear(x, w, b))
+        res[f"torch(cuBLAS) M{M} N{N} K{K}"] = {"us": round(ref_us, 2)}
+if which in ("all", "ln"):
+    for rows, n in [(128, 768), (384, 1024), (1024, 1024)]:
+        x = torch.randn(rows, n, device="cuda").half()
+        g = torch.ones(n, device="cuda").half()
+        bb = torch.zeros(n, device="cuda").half()
+        y = torch.empty_like(x)
+        us = timeit(lambda: dp.layernorm(x, None, g, bb, y, rows, n, 1e-5))
+        res[f"layernorm {rows}x{n}"] = {"us": round(us, 2), "gbs": round(4 * rows * n / us / 1e3, 1)}
+if which in ("all", "attn"):
+    for B, S, H, heads, causal in [(1, 128, 768, 12, 0), (1, 384, 1024, 16, 0), (1, 1024, 1024, 16, 1)]:
+        qkv = torch.randn(B * S, 3 * H, device="cuda").half()
+        o = torch.empty(B * S, H, device="cuda").half()
+        us = timeit(lambda: dp.attention(qkv, 3 * H, o, B, S, H, heads, causal))
+        fl = 4 * S * S * H * B * (0.5 if causal else 1)
+        res[f"attention S{S} H{H} causal{causal}"] = {"us": round(us, 2), "tflops": round(fl / us / 1e6, 2)}
+if which in ("all", "skinny"):
+    for (M, N, K) in [(128, 768, 768), (128, 3072, 768), (128, 768, 3072), (1, 768, 768)]:
+        x = torch.randn(M, K, device="cuda").half()
+        wh = dp.host_alloc(N * K * 2)
+        wd = torch.randn(N, K, device="cuda").half()
+        y = torch.empty(M, N, device="cuda").half()
+        us_h = timeit(lambda: dp.linear(x, K, wh, None, None, 0, y, N, M, N, K, path=1), n=20)
+        us_d = timeit(lambda: dp.linear(x, K, wd, None, None, 0, y, N, M, N, K, path=1), n=20)
+        res[f"skinny M{M} N{N} K{K}"] = {"us_host": round(us_h, 2), "pcie_gbs": round(N * K * 2 / us_h / 1e3, 1),
+                                        "us_hbm": round(us_d, 2)}
+        dp.host_free(wh)
+if which in ("all", "embed"):
+    V, P, H, S = 30522, 512, 768, 128
+    word = dp.host_alloc(V * H * 2)
+    pos = dp.host_alloc(P * H * 2)
+    typ = dp.host_alloc(2 * H * 2)
+    g = dp.host_alloc(H * 2)
+    bb = dp.host_alloc(H * 2)
+    ids = torch.randint(0, V, (S,), device="cuda", dtype=torch.int32)
+    out = torch.empty(S, H, device="cuda").half()
+    us = timeit(lambda: dp.embed(ids, S, word, pos, typ, g, bb, H, 1e-12, out), n=20)
+    res["embed DHA S128 H768"] = {"us": round(us, 2), "pcie_gbs": round((2 * S + 3) * H * 2 / us / 1e3, 1)}
+print(json.dumps(res, indent=1))
