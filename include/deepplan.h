@@ -141,7 +141,9 @@ typedef struct {
   int32_t debug_delay_us; /* fault injection: stall every load/migration stream this long
                              before each transfer (tests event gating) [0] */
   int32_t debug_poison;   /* 1 = fill HBM slots with 0xFF (NaN) on eviction [0] */
-  int32_t reserved[5];
+  int32_t use_pdl;        /* chain consecutive kernels with programmatic dependent launch:
+                             a kernel's weight prefetch overlaps its predecessor [1] */
+  int32_t reserved[4];
 } dp_engine_opts;
 dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* opts);
 dp_status dp_context_get_opts(dp_context* ctx, dp_engine_opts* out);

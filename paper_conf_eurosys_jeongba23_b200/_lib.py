@@ -49,7 +49,7 @@ class Plan(C.Structure):
 class EngineOpts(C.Structure):
     _fields_ = [("chunk_bytes", C.c_int64), ("n_h2d_streams", C.c_int32), ("use_graph", C.c_int32),
                 ("gemm_bn", C.c_int32), ("debug_delay_us", C.c_int32), ("debug_poison", C.c_int32),
-                ("reserved", C.c_int32 * 5)]
+                ("use_pdl", C.c_int32), ("reserved", C.c_int32 * 4)]
 
 
 class ModelConfig(C.Structure):
@@ -266,7 +266,7 @@ class Context:
         self.devs = list(devs)
 
     def set_opts(self, chunk_bytes=None, n_h2d_streams=None, use_graph=None, gemm_bn=None, debug_delay_us=None,
-                 debug_poison=None):
+                 debug_poison=None, use_pdl=None):
         o = EngineOpts()
         _check(lib.dp_context_get_opts(self.h, C.byref(o)))
         if chunk_bytes is not None:
@@ -281,6 +281,8 @@ class Context:
             o.debug_delay_us = int(debug_delay_us)
         if debug_poison is not None:
             o.debug_poison = int(debug_poison)
+        if use_pdl is not None:
+            o.use_pdl = int(use_pdl)
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))
 
     def peer_init(self, uid: bytes, rank: int, nranks: int):

@@ -57,6 +57,7 @@ struct ForwardArgs {
   std::function<void(int)> before_unit;  // called before the first kernel using a unit
   int kernels = 0;
   int bn_hint = 0;
+  bool pdl = false;  // chain kernels with programmatic dependent launch (opts.use_pdl)
 };
 
 void ensure_workspace(dp_model* m, int dev, int64_t tokens);

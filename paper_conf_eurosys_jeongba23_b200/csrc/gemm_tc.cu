@@ -28,6 +28,7 @@
 #include "common.h"
 #include "dtype.cuh"
 #include "kernels.h"
+#include "launch.cuh"
 
 namespace dp {
 
@@ -35,7 +36,6 @@ namespace {
 
 constexpr int BM = 128;  // W rows per tile (MMA M)
 constexpr int BK = 64;   // K per stage: 64 x 2 B = one 128-byte swizzle row
-constexpr int STAGES = 4;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -117,11 +117,21 @@ struct FmtBits<__nv_bfloat16> {
   static constexpr uint32_t v = 1;
 };
 
+// Ring depth per tile width: as many stages as ~224 KB of shared memory holds (<= 12), so a
+// K = 768 layer (12 k-blocks) has its whole weight slice in flight at once.
+template <int BN>
+__host__ __device__ constexpr int stages_for() {
+  constexpr int bytes = BM * BK * 2 + BN * BK * 2;
+  constexpr int s = (224 * 1024) / bytes;
+  return s > 12 ? 12 : s;
+}
+
 template <class T, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmX,
                    const T* __restrict__ bias, const void* res, int ldr, void* Y, int ldy, int M,
                    int N, int K, int act, int io) {
+  constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
@@ -158,16 +168,31 @@ __global__ void __launch_bounds__(128, 1)
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem_d = tmem_base_sh;
+  pdl_trigger();
+
+  // Weights never depend on the previous kernel: the producer puts the first ring's worth
+  // of W tiles in flight BEFORE the grid-dependency wait (PDL), so their HBM latency
+  // overlaps the predecessor's tail.  Activations (X, residual) and every store come after.
+  const int pre = num_kb < STAGES ? num_kb : STAGES;
+  if (warp == 0 && lane == 0) {
+    for (int kb = 0; kb < pre; ++kb) {
+      mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
+      tma_load_2d(&tmW, &full_bar[kb], smem + kb * STAGE_BYTES, kb * BK, n0);
+    }
+  }
+  pdl_wait();
 
   if (warp == 0 && lane == 0) {
     // TMA producer
     for (int kb = 0; kb < num_kb; ++kb) {
       const int s = kb % STAGES;
-      if (kb >= STAGES) mbar_wait(&empty_bar[s], ((kb / STAGES) - 1) & 1);
       uint8_t* a = smem + s * STAGE_BYTES;
       uint8_t* b = a + A_BYTES;
-      mbar_expect_tx(&full_bar[s], STAGE_BYTES);
-      tma_load_2d(&tmW, &full_bar[s], a, kb * BK, n0);
+      if (kb >= pre) {
+        mbar_wait(&empty_bar[s], ((kb / STAGES) - 1) & 1);
+        mbar_expect_tx(&full_bar[s], STAGE_BYTES);
+        tma_load_2d(&tmW, &full_bar[s], a, kb * BK, n0);
+      }
       tma_load_2d(&tmX, &full_bar[s], b, kb * BK, m0);
     }
   } else if (warp == 1 && lane == 0) {
@@ -249,7 +274,7 @@ CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int b
 template <class T, int BN>
 void run(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy, int M,
          int N, int K, int act, int io, cudaStream_t s) {
-  constexpr size_t smem = size_t(STAGES) * (BM * BK * 2 + BN * BK * 2) + 1024;
+  constexpr size_t smem = size_t(stages_for<BN>()) * (BM * BK * 2 + BN * BK * 2) + 1024;
   static bool attr = false;
   if (!attr) {
     DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -259,8 +284,8 @@ void run(const void* x, int ldx, const void* w, const void* bias, const void* re
   CUtensorMap mw = make_map(w, dtype, N, K, K, BM);
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
   dim3 grid(N / BM, (M + BN - 1) / BN);
-  gemm_tc_kernel<T, BN><<<grid, 128, smem, s>>>(mw, mx, (const T*)bias, res, ldr, y, ldy, M, N, K, act, io);
-  DP_CUDA(cudaGetLastError());
+  launch_kernel(gemm_tc_kernel<T, BN>, grid, dim3(128), smem, s, mw, mx, (const T*)bias, res, ldr, y, ldy, M, N, K,
+                act, io);
 }
 
 template <class T>

@@ -19,6 +19,7 @@
 
 #include "engine.h"
 #include "kernels.h"
+#include "launch.cuh"
 #include "peer.h"
 
 namespace dp {
@@ -110,6 +111,7 @@ extern "C" dp_status dp_context_create(const int32_t* devs, int32_t ndev, dp_con
     ctx->opts.n_h2d_streams = 1;
     ctx->opts.use_graph = 0;
     ctx->opts.gemm_bn = 0;
+    ctx->opts.use_pdl = 1;
     for (int i = 0; i < ndev; ++i) {
       DP_CHECK(devs[i] >= 0 && devs[i] < count && devs[i] < DP_MAX_DEVICES, DP_ERR_INVALID,
                "device " + std::to_string(devs[i]) + " does not exist");
@@ -279,28 +281,33 @@ static std::string graph_key(const dp_context* ctx, const dp_plan* plan, const i
   k += "|" + std::to_string((uintptr_t)ids) + "|" + std::to_string((uintptr_t)out) + "|" +
        std::to_string((uintptr_t)pooled) + "|" + std::to_string(batch) + "x" + std::to_string(seq) + "|" +
        std::to_string(ctx->opts.chunk_bytes) + "," + std::to_string(ctx->opts.n_h2d_streams) + "," +
-       std::to_string(ctx->opts.gemm_bn) + "," + std::to_string(ctx->opts.debug_delay_us);
+       std::to_string(ctx->opts.gemm_bn) + "," + std::to_string(ctx->opts.debug_delay_us) + "," +
+       std::to_string(ctx->opts.use_pdl);
   return k;
 }
 
 // Capture `body` (which enqueues on `stream` and joins every side stream back into it) into
 // a CUDA graph once per key; afterwards replay it.  Replay removes the host enqueue cost and
 // turns the per-piece events into graph edges.
+// Capture happens on a private stream (the caller's may be the legacy stream, which cannot
+// be captured); the executable graph is then launched on the caller's stream.
 template <class Body>
 static dp_run_stats run_graph(DevState& ds, const std::string& key, cudaStream_t stream, Body body) {
   auto it = ds.graphs.find(key);
   if (it == ds.graphs.end()) {
+    if (!ds.capture) DP_CUDA(cudaStreamCreateWithFlags(&ds.capture, cudaStreamNonBlocking));
+    cudaStream_t cs = ds.capture;
     cudaGraph_t gph = nullptr;
-    DP_CUDA(cudaStreamBeginCapture(stream, cudaStreamCaptureModeRelaxed));
+    DP_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeRelaxed));
     dp_run_stats st;
     try {
-      st = body();
+      st = body(cs);
     } catch (...) {
-      cudaStreamEndCapture(stream, &gph);
+      cudaStreamEndCapture(cs, &gph);
       if (gph) cudaGraphDestroy(gph);
       throw;
     }
-    DP_CUDA(cudaStreamEndCapture(stream, &gph));
+    DP_CUDA(cudaStreamEndCapture(cs, &gph));
     cudaGraphExec_t ex = nullptr;
     cudaError_t e = cudaGraphInstantiate(&ex, gph, 0);
     cudaGraphDestroy(gph);
@@ -331,8 +338,8 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   for (int s = 1; s < plan->k && graph; ++s) graph = secondaries[s - 1] == primary;  // single-device graphs only
   dp_run_stats st;
   if (graph) {
-    st = run_graph(ds, graph_key(ctx, plan, secondaries, ids, batch, seq, out, pooled), stream, [&] {
-      return enqueue_cold(ctx, m, plan, primary, prim_rank, secondaries, ids, batch, seq, out, pooled, stream);
+    st = run_graph(ds, graph_key(ctx, plan, secondaries, ids, batch, seq, out, pooled), stream, [&](cudaStream_t cs) {
+      return enqueue_cold(ctx, m, plan, primary, prim_rank, secondaries, ids, batch, seq, out, pooled, cs);
     });
   } else {
     st = enqueue_cold(ctx, m, plan, primary, prim_rank, secondaries, ids, batch, seq, out, pooled, stream);
@@ -452,8 +459,10 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     DP_CHECK(e != nullptr, DP_ERR_STATE, "internal: loaded unit has no completion event");
     if (e == last_waited) return;
     DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
+    pdl_state().block_next = true;  // the next kernel must see the landed weights: no PDL overlap
     last_waited = e;
   };
+  a.pdl = ctx->opts.use_pdl != 0;
   run_forward(a);
   // join every side stream (units never read, e.g. an unused pooler, still finish loading)
   for (int i = 0; i < nh; ++i) {
@@ -520,10 +529,12 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.pooled = d_pooled;
     a.stream = (cudaStream_t)stream;
     a.bn_hint = ctx->opts.gemm_bn;
+    a.pdl = ctx->opts.use_pdl != 0;
     if (ctx->opts.use_graph) {
       std::string key = "warm|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
                         graph_key(ctx, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);
-      dp_run_stats gs = run_graph(ds, key, (cudaStream_t)stream, [&] {
+      dp_run_stats gs = run_graph(ds, key, (cudaStream_t)stream, [&](cudaStream_t cs) {
+        a.stream = cs;
         run_forward(a);
         dp_run_stats s{};
         s.n_kernels = a.kernels;
@@ -573,6 +584,7 @@ extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
         cudaDeviceSynchronize();
         for (auto& kv : ds.graphs) cudaGraphExecDestroy(kv.second.exec);
         ds.graphs.clear();
+        if (ds.capture) cudaStreamDestroy(ds.capture);
         if (ds.dbase) cudaFree(ds.dbase);
         if (ds.ws.base) cudaFree(ds.ws.base);
       }

@@ -15,8 +15,14 @@
 #include "common.h"
 #include "dtype.cuh"
 #include "kernels.h"
+#include "launch.cuh"
 
 namespace dp {
+
+PdlState& pdl_state() {
+  static thread_local PdlState s;
+  return s;
+}
 
 // -------------------------------------------------------------------------------------
 // K1: embedding gather + LayerNorm.  One warp per token; VPL 16-byte vectors per lane.
@@ -27,13 +33,15 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
                                                     const T* b, int H, float eps, void* __restrict__ out_,
                                                     int out_f32) {
   extern __shared__ uint4 sm[];  // [type0 | gamma | beta] as 16-byte vectors
+  pdl_trigger();
   const int nv = H / 8;
   const bool has_type = type != nullptr, has_ln = g != nullptr;
-  for (int i = threadIdx.x; i < 3 * nv; i += blockDim.x) {
+  for (int i = threadIdx.x; i < 3 * nv; i += blockDim.x) {  // weights: no dependency on the previous kernel
     const int which = i / nv, c = i - which * nv;
     const T* src = which == 0 ? type : (which == 1 ? g : b);
     if (src) sm[i] = ldg16(src + 8 * c);
   }
+  pdl_wait();
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const int t = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -116,8 +124,8 @@ static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const vo
   const size_t sm = size_t(3) * (H / 8) * 16;
   const int vpl = (H / 8 + 31) / 32;
 #define DP_EMB(V)                                                                                      \
-  embed_kernel<T, V><<<grid, warps * 32, sm, s>>>(ids, ntok, seq, pos_off, (const T*)word, (const T*)pos, \
-                                                  (const T*)type, (const T*)g, (const T*)b, H, eps, out, out_f32)
+  launch_kernel(embed_kernel<T, V>, grid, dim3(warps * 32), sm, s, ids, ntok, seq, pos_off, (const T*)word, \
+                (const T*)pos, (const T*)type, (const T*)g, (const T*)b, H, eps, out, (int)out_f32)
   switch (vpl) {
     case 1: DP_EMB(1); break;
     case 2: DP_EMB(2); break;
@@ -151,8 +159,10 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__
                                                         const T* g, const T* b, T* __restrict__ y, int rows,
                                                         int n, float eps, int in_f32) {
   extern __shared__ uint4 sm[];  // [gamma | beta]
+  pdl_trigger();
   const int nv = n / 8;
   for (int i = threadIdx.x; i < 2 * nv; i += blockDim.x) sm[i] = ldg16(i < nv ? g + 8 * i : b + 8 * (i - nv));
+  pdl_wait();
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
@@ -206,14 +216,17 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__
 template <class T>
 static void layernorm_t(const void* x, const void* r, const void* g, const void* b, void* y, int rows, int n,
                         float eps, bool in_f32, cudaStream_t s) {
+  // one row per warp (latency: every row's loads in flight at once); gamma/beta are read
+  // once per CTA, so a DHA LayerNorm costs rows/8 x 4H bytes of host reads
   const int warps = 8;
-  int grid = (rows + 4 * warps - 1) / (4 * warps);  // ~4 rows per warp: few CTAs -> few host reads of g/b
+  int grid = (rows + warps - 1) / warps;
+  if (grid > 148 * 8) grid = 148 * 8;
   if (grid < 1) grid = 1;
   const size_t sm = size_t(2) * (n / 8) * 16;
   const int vpl = (n / 8 + 31) / 32;
 #define DP_LN(V)                                                                                       \
-  layernorm_kernel<T, V><<<grid, warps * 32, sm, s>>>(x, r, (const T*)g, (const T*)b, (T*)y, rows, n, eps, \
-                                                      in_f32)
+  launch_kernel(layernorm_kernel<T, V>, dim3(grid), dim3(warps * 32), sm, s, x, r, (const T*)g, (const T*)b, (T*)y, \
+                rows, n, eps, (int)in_f32)
   switch (vpl) {
     case 1: DP_LN(1); break;
     case 2: DP_LN(2); break;
@@ -250,13 +263,15 @@ __global__ void __launch_bounds__(256) skinny_linear_kernel(const T* __restrict_
                                                             const T* bias, const void* res, int ldr,
                                                             void* Y, int ldy, int M, int N, int K,
                                                             int act, int io) {
-  extern __shared__ uint4 sw[];  // R*K/8 vectors (+ R bias values)
+  extern __shared__ float4 swf[];  // R rows x K as fp32 (converted once), 2 float4 per 8 elements
+  pdl_trigger();
   const int kv = K / 8;
   const int n0 = blockIdx.x * R;
   const int rows = min(R, N - n0);
   const int total = rows * kv;
   const uint4* src = reinterpret_cast<const uint4*>(W + (size_t)n0 * K);
-  // up to 8 independent 16-byte loads in flight per thread before the first store
+  // weights never depend on the previous kernel: stream them (host or HBM) before the
+  // grid-dependency wait, up to 8 independent 16-byte loads in flight per thread
   for (int base = threadIdx.x; base < total; base += 8 * 256) {
     uint4 r[8];
 #pragma unroll
@@ -264,41 +279,57 @@ __global__ void __launch_bounds__(256) skinny_linear_kernel(const T* __restrict_
       if (base + j * 256 < total) r[j] = ldg16(src + base + j * 256);
 #pragma unroll
     for (int j = 0; j < 8; ++j)
-      if (base + j * 256 < total) sw[base + j * 256] = r[j];
+      if (base + j * 256 < total) {
+        float f[8];
+        unpack8<T>(r[j], f);
+        swf[2 * (base + j * 256)] = make_float4(f[0], f[1], f[2], f[3]);
+        swf[2 * (base + j * 256) + 1] = make_float4(f[4], f[5], f[6], f[7]);
+      }
   }
   __shared__ float sbias[R];
   if (threadIdx.x < rows) sbias[threadIdx.x] = bias ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
+  pdl_wait();
   __syncthreads();
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (int m = warp; m < M; m += 8) {
-    float acc[R];
+  // two tokens per warp iteration: every staged weight read feeds two FMAs
+  for (int m = 2 * warp; m < M; m += 16) {
+    const bool two = m + 1 < M;
+    float acc[2][R];
 #pragma unroll
-    for (int r = 0; r < R; ++r) acc[r] = 0.f;
-    const T* xr = X + (size_t)m * ldx;
+    for (int r = 0; r < R; ++r) acc[0][r] = acc[1][r] = 0.f;
+    const T* x0 = X + (size_t)m * ldx;
+    const T* x1 = two ? x0 + ldx : x0;
     for (int c = lane; c < kv; c += 32) {
-      float xf[8];
-      unpack8<T>(*reinterpret_cast<const uint4*>(xr + 8 * c), xf);
+      float a[8], b[8];
+      unpack8<T>(*reinterpret_cast<const uint4*>(x0 + 8 * c), a);
+      unpack8<T>(*reinterpret_cast<const uint4*>(x1 + 8 * c), b);
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         if (r < rows) {
-          float wf[8];
-          unpack8<T>(sw[r * kv + c], wf);
+          const float4 w0 = swf[2 * (r * kv + c)], w1 = swf[2 * (r * kv + c) + 1];
+          const float wf[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
 #pragma unroll
-          for (int e = 0; e < 8; ++e) acc[r] = fmaf(xf[e], wf[e], acc[r]);
+          for (int e = 0; e < 8; ++e) {
+            acc[0][r] = fmaf(a[e], wf[e], acc[0][r]);
+            acc[1][r] = fmaf(b[e], wf[e], acc[1][r]);
+          }
         }
       }
     }
 #pragma unroll
-    for (int r = 0; r < R; ++r) acc[r] = warp_sum(acc[r]);
-    float mine = 0.f;
+    for (int t = 0; t < 2; ++t) {
 #pragma unroll
-    for (int r = 0; r < R; ++r)
-      if (lane == r) mine = acc[r];
-    if (lane < rows) {
-      const int n = n0 + lane;
-      float v = apply_act(mine + sbias[lane], act);
-      if (res) v += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
-      store1<T>(Y, (size_t)m * ldy + n, v, io & IO_OUT_F32);
+      for (int r = 0; r < R; ++r) acc[t][r] = warp_sum(acc[t][r]);
+      float mine = 0.f;
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+        if (lane == r) mine = acc[t][r];
+      if (lane < rows && (t == 0 || two)) {
+        const int n = n0 + lane, mm = m + t;
+        float v = apply_act(mine + sbias[lane], act);
+        if (res) v += load1<T>(res, (size_t)mm * ldr + n, io & IO_RES_F32);
+        store1<T>(Y, (size_t)mm * ldy + n, v, io & IO_OUT_F32);
+      }
     }
   }
 }
@@ -307,21 +338,20 @@ template <class T>
 static void skinny_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
                      int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   constexpr int R = 8;
-  const size_t sm = size_t(R) * K * sizeof(T);
+  const size_t sm = size_t(R) * K * sizeof(float);
   static bool attr_set = false;  // one per template instantiation
   if (!attr_set) {
     DP_CUDA(cudaFuncSetAttribute(skinny_linear_kernel<T, R>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
     attr_set = true;
   }
-  skinny_linear_kernel<T, R><<<(N + R - 1) / R, 256, sm, s>>>((const T*)x, ldx, (const T*)w, (const T*)bias,
-                                                               res, ldr, y, ldy, M, N, K, act, io);
-  DP_CUDA(cudaGetLastError());
+  launch_kernel(skinny_linear_kernel<T, R>, dim3((N + R - 1) / R), dim3(256), sm, s, (const T*)x, ldx, (const T*)w,
+                (const T*)bias, res, ldr, y, ldy, M, N, K, act, io);
 }
 
 void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
                           int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   DP_CHECK(K % 8 == 0 && K > 0 && N > 0, DP_ERR_INVALID, "skinny linear needs K % 8 == 0");
-  DP_CHECK(size_t(8) * K * 2 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
+  DP_CHECK(size_t(8) * K * 4 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
   if (M <= 0) return;
   if (dtype == DP_BF16)
     skinny_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
@@ -378,6 +408,8 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
   __shared__ __align__(16) T sq[ATT_BQ * ATT_LD];
   __shared__ __align__(16) T sk[ATT_BK * ATT_LD];
   __shared__ __align__(16) T sv[ATT_BK * ATT_LD];
+  pdl_trigger();
+  pdl_wait();  // q, k, v come from the previous kernels
   const int qt = blockIdx.x, head = blockIdx.y, bidx = blockIdx.z;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const size_t tok0 = (size_t)bidx * seq;
@@ -522,12 +554,11 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   dim3 grid((seq + ATT_BQ - 1) / ATT_BQ, heads, batch);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)ATT_D);
   if (dtype == DP_BF16)
-    attention_kernel<__nv_bfloat16><<<grid, 128, 0, s>>>((const __nv_bfloat16*)qkv, ldqkv, (__nv_bfloat16*)ctx, seq,
-                                                         H, causal ? 1 : 0, scale_log2);
+    launch_kernel(attention_kernel<__nv_bfloat16>, grid, dim3(128), 0, s, (const __nv_bfloat16*)qkv, ldqkv,
+                  (__nv_bfloat16*)ctx, seq, H, causal ? 1 : 0, scale_log2);
   else
-    attention_kernel<__half><<<grid, 128, 0, s>>>((const __half*)qkv, ldqkv, (__half*)ctx, seq, H, causal ? 1 : 0,
-                                                  scale_log2);
-  DP_CUDA(cudaGetLastError());
+    launch_kernel(attention_kernel<__half>, grid, dim3(128), 0, s, (const __half*)qkv, ldqkv, (__half*)ctx, seq, H,
+                  causal ? 1 : 0, scale_log2);
 }
 
 // -------------------------------------------------------------------------------------

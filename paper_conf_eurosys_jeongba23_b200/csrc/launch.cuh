@@ -1,0 +1,51 @@
+// Kernel launch with optional programmatic dependent launch (PDL).
+//
+// Inside a forward pass consecutive kernels on the execution stream are chained with PDL:
+// a kernel starts its prologue (barrier init, TMEM alloc, and -- for weights, which never
+// depend on the previous kernel -- its first weight tiles) while its predecessor drains,
+// then `griddepcontrol.wait`s before touching activations.  Right after an event wait
+// (a layer that just landed) the next launch is a plain stream-ordered one.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "common.h"
+
+namespace dp {
+
+// Engine-controlled state (thread-local: one host thread drives a context at a time).
+struct PdlState {
+  bool enabled = false;     // inside run_forward with PDL allowed
+  bool block_next = true;   // the next launch must not overlap its predecessor
+};
+PdlState& pdl_state();
+
+inline bool take_pdl() {
+  PdlState& s = pdl_state();
+  const bool r = s.enabled && !s.block_next;
+  s.block_next = false;
+  return r;
+}
+
+template <class... KArgs, class... Args>
+inline void launch_kernel(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                          Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  if (take_pdl()) {
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+  }
+  DP_CUDA(cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...));
+}
+
+// Device side: no-ops when the grid was not launched with PDL.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+}  // namespace dp

@@ -61,6 +61,7 @@ struct DevState {
   std::vector<int8_t> method;  // per unit, fixed when the model became resident
   Workspace ws;
   std::map<std::string, GraphEntry> graphs;  // captured cold / warm runs (opts.use_graph)
+  cudaStream_t capture = nullptr;            // private stream the graphs are captured on
 };
 
 std::vector<ParamDesc> config_params(const dp_model_config& c);

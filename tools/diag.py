@@ -16,6 +16,7 @@ S = int(sys.argv[2]) if len(sys.argv) > 2 else 128
 m = synth.SHAPES[name]
 w = synth.make_weights(m, seed=0)
 ctx = dp.Context([0])
+ctx.set_opts(use_graph=int(os.environ.get("DP_GRAPH", "1")), use_pdl=int(os.environ.get("DP_PDL", "1")))
 model = dp.Model(ctx, m, w)
 cost = model.profile(0, 1, S, 10)
 units = model.units()

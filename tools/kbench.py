@@ -20,10 +20,13 @@ res = {}
 
 
 def timeit(fn, n=reps):
+    """Device time per launch: a sleep kernel holds the stream while the host enqueues the
+    n launches, so the interval between the events contains no host launch latency."""
     for _ in range(3):
         fn()
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda._sleep(int(2e6 + n * 40000))
     e0.record()
     for _ in range(n):
         fn()
