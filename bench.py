@@ -44,8 +44,11 @@ def parse():
     ap.add_argument("--seq", type=int, default=128)
     ap.add_argument("--batch", type=int, default=1)
     ap.add_argument("--mode", default=None, help="plan mode (default DHA at N=1, PT_DHA at N>1)")
-    ap.add_argument("--chunk-mb", type=float, default=4.0)
+    ap.add_argument("--chunk-mb", type=float, default=32.0)
+    ap.add_argument("--tail-mb", type=float, default=2.0)
     ap.add_argument("--h2d-streams", type=int, default=1)
+    ap.add_argument("--no-graph", action="store_true", help="eager enqueue instead of CUDA-graph replay")
+    ap.add_argument("--no-pdl", action="store_true")
     ap.add_argument("--profile-iters", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     return ap.parse_args()
@@ -173,7 +176,9 @@ def main():
     w = synth.make_weights(m, seed=0, dtype=dtype)
     ids_np = synth.make_ids(m, a.batch, a.seq, seed=1)
     ctx = dp.Context([local])
-    ctx.set_opts(chunk_bytes=int(a.chunk_mb * (1 << 20)), n_h2d_streams=a.h2d_streams)
+    ctx.set_opts(chunk_bytes=int(a.chunk_mb * (1 << 20)), n_h2d_streams=a.h2d_streams,
+                 tail_bytes=int(a.tail_mb * (1 << 20)), use_graph=0 if (a.no_graph or world > 1) else 1,
+                 use_pdl=0 if a.no_pdl else 1)
     model = dp.Model(ctx, m, w, dtype)
     if dist_on:
         uid = dp.peer_unique_id() if rank == 0 else None

@@ -143,7 +143,11 @@ typedef struct {
   int32_t debug_poison;   /* 1 = fill HBM slots with 0xFF (NaN) on eviction [0] */
   int32_t use_pdl;        /* chain consecutive kernels with programmatic dependent launch:
                              a kernel's weight prefetch overlaps its predecessor [1] */
-  int32_t reserved[4];
+  int32_t reserved0;
+  int64_t tail_bytes;     /* the last DMA piece of a link carries at most this many bytes
+                             (a unit suffix), so little compute remains after the last byte
+                             lands [2 MiB]; 0 = off */
+  int32_t reserved[2];
 } dp_engine_opts;
 dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* opts);
 dp_status dp_context_get_opts(dp_context* ctx, dp_engine_opts* out);
@@ -209,12 +213,13 @@ int64_t dp_model_bytes(const dp_model* m);
 dp_status dp_model_arena(const dp_model* m, const void** ptr, int64_t* bytes);
 
 /* Transfer schedule of one plan slot (host-only, no GPU): the contiguous pieces (whole
- * units, forward order, <= chunk_bytes unless one unit is larger) that the slot's link
- * carries -- what dp_infer_cold DMAs on slot 0 and what secondary s sends / the primary
- * receives for slot s >= 1.  Arrays of `cap` entries (nullable); *count = #pieces. */
+ * units, forward order, <= chunk_bytes unless one unit is larger; the last piece cut down
+ * to the longest unit suffix <= tail_bytes) that the slot's link carries -- what
+ * dp_infer_cold DMAs on slot 0 and what secondary s sends / the primary receives for
+ * slot s >= 1.  Arrays of `cap` entries (nullable); *count = #pieces. */
 dp_status dp_transfer_schedule(const dp_model_config* cfg, const dp_plan* plan, int32_t slot, int64_t chunk_bytes,
-                               int64_t* piece_off, int64_t* piece_bytes, int32_t* first_unit, int32_t* last_unit,
-                               int32_t cap, int32_t* count);
+                               int64_t tail_bytes, int64_t* piece_off, int64_t* piece_bytes, int32_t* first_unit,
+                               int32_t* last_unit, int32_t cap, int32_t* count);
 
 /* ---------------------------------------------------------------------------------
  * Profiling (§4.3.1; Table 5).  Per unit, median over `iters`

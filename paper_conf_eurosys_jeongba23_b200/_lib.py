@@ -49,7 +49,8 @@ class Plan(C.Structure):
 class EngineOpts(C.Structure):
     _fields_ = [("chunk_bytes", C.c_int64), ("n_h2d_streams", C.c_int32), ("use_graph", C.c_int32),
                 ("gemm_bn", C.c_int32), ("debug_delay_us", C.c_int32), ("debug_poison", C.c_int32),
-                ("use_pdl", C.c_int32), ("reserved", C.c_int32 * 4)]
+                ("use_pdl", C.c_int32), ("reserved0", C.c_int32), ("tail_bytes", C.c_int64),
+                ("reserved", C.c_int32 * 2)]
 
 
 class ModelConfig(C.Structure):
@@ -122,8 +123,8 @@ _sig("dp_model_num_units", [vp])
 _sig("dp_model_unit_info", [vp, C.c_int32, C.POINTER(UnitInfo)])
 _sig("dp_model_bytes", [vp], C.c_int64)
 _sig("dp_model_arena", [vp, C.POINTER(vp), i64p])
-_sig("dp_transfer_schedule", [C.POINTER(ModelConfig), C.POINTER(Plan), C.c_int32, C.c_int64, i64p, i64p, i32p,
-                              i32p, C.c_int32, i32p])
+_sig("dp_transfer_schedule", [C.POINTER(ModelConfig), C.POINTER(Plan), C.c_int32, C.c_int64, C.c_int64, i64p, i64p,
+                              i32p, i32p, C.c_int32, i32p])
 _sig("dp_profile",[vp, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.POINTER(CostTable)])
 _sig("dp_infer_cold", [vp, vp, C.POINTER(Plan), C.c_int32, i32p, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp, vp,
                        C.POINTER(RunStats)])
@@ -266,7 +267,7 @@ class Context:
         self.devs = list(devs)
 
     def set_opts(self, chunk_bytes=None, n_h2d_streams=None, use_graph=None, gemm_bn=None, debug_delay_us=None,
-                 debug_poison=None, use_pdl=None):
+                 debug_poison=None, use_pdl=None, tail_bytes=None):
         o = EngineOpts()
         _check(lib.dp_context_get_opts(self.h, C.byref(o)))
         if chunk_bytes is not None:
@@ -283,6 +284,8 @@ class Context:
             o.debug_poison = int(debug_poison)
         if use_pdl is not None:
             o.use_pdl = int(use_pdl)
+        if tail_bytes is not None:
+            o.tail_bytes = int(tail_bytes)
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))
 
     def peer_init(self, uid: bytes, rank: int, nranks: int):
@@ -312,17 +315,19 @@ def config_params(shape, dtype: str = "fp16"):
             for p in infos]
 
 
-def transfer_schedule(shape, plan: "PlanArrays", slot: int, chunk_bytes: int, dtype: str = "fp16"):
+def transfer_schedule(shape, plan: "PlanArrays", slot: int, chunk_bytes: int, tail_bytes: int = 2 << 20,
+                      dtype: str = "fp16"):
     """Pieces (offset, bytes, first_unit, last_unit) carried by one plan slot's link."""
     cfg = model_config(shape, dtype)
     cnt = C.c_int32()
-    _check(lib.dp_transfer_schedule(C.byref(cfg), C.byref(plan.s), int(slot), int(chunk_bytes), None, None, None,
-                                    None, 0, C.byref(cnt)))
+    _check(lib.dp_transfer_schedule(C.byref(cfg), C.byref(plan.s), int(slot), int(chunk_bytes), int(tail_bytes),
+                                    None, None, None, None, 0, C.byref(cnt)))
     n = cnt.value
     off, nb = np.zeros(n, np.int64), np.zeros(n, np.int64)
     fu, lu = np.zeros(n, np.int32), np.zeros(n, np.int32)
-    _check(lib.dp_transfer_schedule(C.byref(cfg), C.byref(plan.s), int(slot), int(chunk_bytes), _ptr(off, i64p),
-                                    _ptr(nb, i64p), _ptr(fu, i32p), _ptr(lu, i32p), n, C.byref(cnt)))
+    _check(lib.dp_transfer_schedule(C.byref(cfg), C.byref(plan.s), int(slot), int(chunk_bytes), int(tail_bytes),
+                                    _ptr(off, i64p), _ptr(nb, i64p), _ptr(fu, i32p), _ptr(lu, i32p), n,
+                                    C.byref(cnt)))
     return off, nb, fu, lu
 
 

@@ -112,6 +112,8 @@ extern "C" dp_status dp_context_create(const int32_t* devs, int32_t ndev, dp_con
     ctx->opts.use_graph = 0;
     ctx->opts.gemm_bn = 0;
     ctx->opts.use_pdl = 1;
+    ctx->opts.tail_bytes = 2 << 20;
+    ctx->opts.chunk_bytes = 32 << 20;
     for (int i = 0; i < ndev; ++i) {
       DP_CHECK(devs[i] >= 0 && devs[i] < count && devs[i] < DP_MAX_DEVICES, DP_ERR_INVALID,
                "device " + std::to_string(devs[i]) + " does not exist");
@@ -201,14 +203,39 @@ std::vector<Piece> make_pieces(const dp_model* m, Pick pick, int64_t cap) {
   return out;
 }
 
-std::vector<Piece> slot_pieces(const dp_model* m, const dp_plan* plan, int slot, int64_t cap) {
-  return make_pieces(m, [&](int u) { return plan->method[u] == DP_LOAD && plan->slot[u] == slot; }, cap);
+std::vector<Piece> slot_pieces(const dp_model* m, const dp_plan* plan, int slot, int64_t cap, int64_t tail) {
+  auto p = make_pieces(m, [&](int u) { return plan->method[u] == DP_LOAD && plan->slot[u] == slot; }, cap);
+  // Cold-start latency = (last byte lands) + (compute of what it carried): the link never
+  // waits for compute, so only the LAST piece's size matters for the pipeline tail.  Peel
+  // trailing units off the last piece until it holds <= `tail` bytes (or one unit).
+  if (tail > 0 && !p.empty() && p.back().bytes > tail) {
+    Piece& b = p.back();
+    int64_t acc = 0;
+    int first = b.last_unit + 1;
+    for (int u = b.last_unit; u > b.first_unit; --u) {  // longest suffix <= tail, b keeps >= 1 unit
+      if (acc + m->units[u].bytes > tail) break;
+      acc += m->units[u].bytes;
+      first = u;
+    }
+    if (first <= b.last_unit) {
+      Piece q;
+      q.first_unit = first;
+      q.last_unit = b.last_unit;
+      q.off = m->units[first].off;
+      q.bytes = b.off + b.bytes - q.off;
+      b.bytes = q.off - b.off;
+      b.last_unit = first - 1;
+      p.push_back(q);
+    }
+  }
+  return p;
 }
 
 }  // namespace dp
 
 extern "C" dp_status dp_transfer_schedule(const dp_model_config* cfg, const dp_plan* plan, int32_t slot,
-                                          int64_t chunk_bytes, int64_t* piece_off, int64_t* piece_bytes,
+                                          int64_t chunk_bytes, int64_t tail_bytes, int64_t* piece_off,
+                                          int64_t* piece_bytes,
                                           int32_t* first_unit, int32_t* last_unit, int32_t cap, int32_t* count) {
   return dp::guard([&] {
     DP_CHECK(cfg && plan && count, DP_ERR_INVALID, "NULL argument");
@@ -218,7 +245,7 @@ extern "C" dp_status dp_transfer_schedule(const dp_model_config* cfg, const dp_p
     dp::build_units(&tmp);
     DP_CHECK(plan->n == (int)tmp.units.size() && plan->method && plan->slot, DP_ERR_INVALID, "plan/model mismatch");
     DP_CHECK(slot >= 0 && slot < plan->k, DP_ERR_INVALID, "slot out of range");
-    auto pcs = dp::slot_pieces(&tmp, plan, slot, std::max<int64_t>(chunk_bytes, 4096));
+    auto pcs = dp::slot_pieces(&tmp, plan, slot, std::max<int64_t>(chunk_bytes, 4096), tail_bytes);
     *count = (int32_t)pcs.size();
     for (int i = 0; i < (int)pcs.size() && i < cap; ++i) {
       if (piece_off) piece_off[i] = pcs[i].off;
@@ -371,7 +398,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
 
   // (1) slot-0 loads on the primary's link
   const int64_t cap = std::max<int64_t>(ctx->opts.chunk_bytes, 4096);
-  auto pieces0 = make_pieces(m, [&](int u) { return method[u] == DP_LOAD && plan->slot[u] == 0; }, cap);
+  auto pieces0 = slot_pieces(m, plan, 0, cap, opt_tail(ctx));
   const int nh = std::min((int)pd.h2d.size(), std::max(1, ctx->opts.n_h2d_streams));
   for (int i = 0; i < nh; ++i) DP_CUDA(cudaStreamWaitEvent(pd.h2d[i], fork, 0));
   for (size_t c = 0; c < pieces0.size(); ++c) {
@@ -398,7 +425,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     }
   if (ctx->comm && plan->k > 1) peer_recv_all(ctx, m, plan, prim_rank, primary, fork, unit_ev, st);
   for (int s = 1; s < plan->k && !ctx->comm; ++s) {
-    auto pcs = slot_pieces(m, plan, s, cap);
+    auto pcs = slot_pieces(m, plan, s, cap, opt_tail(ctx));
     if (pcs.empty()) continue;
     const int sdev = secondaries[s - 1];
     const int64_t ring_slots = 3;

@@ -100,7 +100,7 @@ void peer_recv_all(dp_context* ctx, dp_model* m, const dp_plan* plan, int primar
   std::vector<std::vector<Piece>> pcs(plan->k);
   size_t rounds = 0;
   for (int s = 1; s < plan->k; ++s) {
-    pcs[s] = slot_pieces(m, plan, s, cap);
+    pcs[s] = slot_pieces(m, plan, s, cap, opt_tail(ctx));
     rounds = std::max(rounds, pcs[s].size());
   }
   DP_CUDA(cudaStreamWaitEvent(ctx->comm_stream, fork, 0));
@@ -144,7 +144,7 @@ void peer_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int prima
     return;
   }
   const int64_t cap = std::max<int64_t>(ctx->opts.chunk_bytes, 4096);
-  auto pcs = slot_pieces(m, plan, slot, cap);
+  auto pcs = slot_pieces(m, plan, slot, cap, opt_tail(ctx));
   int64_t big = 0;
   for (auto& pc : pcs) big = std::max(big, pc.bytes);
   if (!p.h2d) DP_CUDA(cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking));

@@ -20,7 +20,9 @@ void peer_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int prima
 void peer_destroy(dp_context* ctx);
 
 // The piece list of one slot (shared by sender and receiver so both sides agree).
-std::vector<Piece> slot_pieces(const dp_model* m, const dp_plan* plan, int slot, int64_t cap);
+std::vector<Piece> slot_pieces(const dp_model* m, const dp_plan* plan, int slot, int64_t cap, int64_t tail);
+inline int64_t opt_cap(const dp_context* ctx) { return ctx->opts.chunk_bytes < 4096 ? 4096 : ctx->opts.chunk_bytes; }
+inline int64_t opt_tail(const dp_context* ctx) { return ctx->opts.tail_bytes; }
 void bind_units(std::vector<cudaEvent_t>& unit_ev, const Piece& p, cudaEvent_t e);
 
 }  // namespace dp
