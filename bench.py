@@ -103,6 +103,12 @@ def measured_peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
 
 
+def measure_h2d_peak(dp, torch, nbytes=256 << 20, reps=5):
+    """Best-of-reps pinned host->device copy rate (GB/s), measured by the library on
+    memory allocated exactly like its weight arena (dp_measure_h2d)."""
+    return dp.measure_h2d(torch.cuda.current_device(), nbytes, reps)
+
+
 def cpu_oracle_ms(m, w, ids, dtype, budget_s=15.0, max_runs=10):
     """The oracle (fp64 numpy) timed on this host's cores, on a bounded sample."""
     from oracle import forward as F
@@ -186,6 +192,10 @@ def main():
         dist.broadcast_object_list(box, src=0)
         ctx.peer_init(box[0], rank, world)
 
+    # roofline denominator: pinned H2D bandwidth of this GPU's link, measured now with the
+    # library's own pinned+mapped allocation (256 MiB, best of 5, CUDA events)
+    peak_h2d = measure_h2d_peak(dp, torch)
+
     # profile on the primary, plan, share the plan (the plan never names GPUs)
     mode = a.mode or ("PT_DHA" if world > 1 else "DHA")
     if rank == 0:
@@ -230,14 +240,18 @@ def main():
             dist.barrier()
             torch.cuda.synchronize()
 
+    # clocks are sampled (100 ms period) from before the warm-up to the end of the timed
+    # region; the region itself is short, so it is padded to >= 1 s of repeated steps
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
     for _ in range(max(3, a.warmup)):
         step()
         sync_all()
     # timed region
-    clocks = ClockSampler(local)
-    clocks.start()
     sync_all()
     stats = None
+    t_start = time.perf_counter()
     for i in range(a.steps):
         stats = step(i, timed=True)
         # secondaries must finish before the next eviction; the primary waits on its stream
@@ -245,6 +259,9 @@ def main():
         if dist_on:
             dist.barrier()
     sync_all()
+    while time.perf_counter() - t_start < 1.0:  # keep the GPU busy for the clock samples
+        step()
+        sync_all()
     ck = clocks.stop()
     lat = [ev0[i].elapsed_time(ev1[i]) for i in range(a.steps)]
     my_ms = float(np.mean(lat))
@@ -287,22 +304,6 @@ def main():
         if dist_on:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
-
-    # ---- roofline of the path: PCIe host link (the copy engine + DHA reads) ----
-    peak_h2d = None
-    if rank == 0:
-        hb = torch.empty(256 << 20, dtype=torch.uint8).pin_memory()
-        db = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
-        best = 1e9
-        for _ in range(3):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            db.copy_(hb, non_blocking=True)
-            e1.record()
-            torch.cuda.synchronize()
-            best = min(best, e0.elapsed_time(e1))
-        peak_h2d = hb.numel() / (best * 1e-3) / 1e9
-        del hb, db
 
     if rank != 0:
         if dist_on:

@@ -231,6 +231,10 @@ dp_status dp_transfer_schedule(const dp_model_config* cfg, const dp_plan* plan, 
 dp_status dp_profile(dp_context* ctx, dp_model* m, int32_t dev, int32_t batch, int32_t seq, int32_t iters,
                      dp_cost_table* out);
 
+/* Link roofline denominator: best of `reps` H2D copies of `bytes` from memory allocated
+ * like the weight arena (pinned, mapped, portable) to device `dev`, in GB/s (1e9 B/s). */
+dp_status dp_measure_h2d(int32_t dev, int64_t bytes, int32_t reps, double* gbs);
+
 /* ---------------------------------------------------------------------------------
  * Inference (§4.3.4, Fig.9)
  * --------------------------------------------------------------------------------- */

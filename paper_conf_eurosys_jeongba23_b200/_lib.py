@@ -125,6 +125,7 @@ _sig("dp_model_bytes", [vp], C.c_int64)
 _sig("dp_model_arena", [vp, C.POINTER(vp), i64p])
 _sig("dp_transfer_schedule", [C.POINTER(ModelConfig), C.POINTER(Plan), C.c_int32, C.c_int64, C.c_int64, i64p, i64p,
                               i32p, i32p, C.c_int32, i32p])
+_sig("dp_measure_h2d", [C.c_int32, C.c_int64, C.c_int32, C.POINTER(C.c_double)])
 _sig("dp_profile",[vp, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.POINTER(CostTable)])
 _sig("dp_infer_cold", [vp, vp, C.POINTER(Plan), C.c_int32, i32p, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp, vp,
                        C.POINTER(RunStats)])
@@ -447,6 +448,13 @@ def _stats(st: RunStats) -> dict:
 # --------------------------------------------------------------------------------------
 # Pinned host memory and kernel hooks
 # --------------------------------------------------------------------------------------
+
+def measure_h2d(dev: int, nbytes: int = 256 << 20, reps: int = 5) -> float:
+    """Pinned H2D GB/s of device `dev` (the link roofline denominator)."""
+    g = C.c_double()
+    _check(lib.dp_measure_h2d(int(dev), int(nbytes), int(reps), C.byref(g)))
+    return float(g.value)
+
 
 def host_alloc(nbytes: int) -> int:
     p = vp()

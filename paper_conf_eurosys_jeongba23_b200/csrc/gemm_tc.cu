@@ -7,14 +7,21 @@
 // and wide in N (768..4096), so the kernel is "swap-AB": the MMA's M axis (128 lanes of
 // TMEM) runs over W's rows (N) and the MMA's N axis over tokens (BN = 32..256 columns).
 //
-// Per CTA (128 threads, one 128 x BN output tile, full K):
+// Per CTA (128 threads, one 128 x BN output tile, a K range):
 //   warp 0 / lane 0  : TMA producer -- W tile [128 x 64] and X tile [BN x 64] per stage,
-//                      both K-major with the 128-byte swizzle, into a STAGES-deep ring;
+//                      both K-major with the 128-byte swizzle, into a STAGES-deep ring; the
+//                      first ring of W tiles is issued BEFORE the grid-dependency wait (PDL):
+//                      weights never depend on the previous kernel;
 //   warp 1 / lane 0  : MMA issuer  -- 4 x tcgen05.mma (K = 16 each) per stage, fp32
 //                      accumulator in TMEM; tcgen05.commit releases the smem stage;
 //   warp 1           : TMEM allocate / free (BN columns);
 //   all 4 warps      : epilogue -- tcgen05.ld 32 lanes x 16 columns, + bias, activation,
 //                      + residual, store (warp w owns TMEM lanes 32w..32w+31).
+// Split-K for the latency-bound skinny layers: a thread-block cluster of SPLIT CTAs along z
+// shares one output tile, each CTA streams 1/SPLIT of K; ranks >= 1 park their fp32 partial
+// tile in shared memory and rank 0 sums them through distributed shared memory (DSMEM)
+// before the epilogue.  More SMs pull the weight slice in parallel; no extra launch, no
+// global-memory workspace.
 // Descriptor encodings follow the sm_100 UMMA descriptor layout (start>>4, LBO, SBO = 1024 B
 // for 8-row swizzle atoms, version 1, layout SWIZZLE_128B = 2).
 #include <cuda.h>
@@ -106,6 +113,27 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+__device__ __forceinline__ float4 ld_dsmem_f4(uint32_t local_addr, uint32_t rank) {
+  uint32_t remote;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(local_addr), "r"(rank));
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(remote)
+               : "memory");
+  return v;
+}
+
 template <class T>
 struct FmtBits;
 template <>
@@ -126,7 +154,7 @@ __host__ __device__ constexpr int stages_for() {
   return s > 12 ? 12 : s;
 }
 
-template <class T, int BN>
+template <class T, int BN, int SPLIT>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmX,
                    const T* __restrict__ bias, const void* res, int ldr, void* Y, int ldy, int M,
@@ -136,6 +164,7 @@ __global__ void __launch_bounds__(128, 1)
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
+  constexpr int PROW = BN + 4;  // fp32 partial row stride (16 B pad against bank conflicts)
   // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
   constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
                              (uint32_t(BM >> 4) << 24);
@@ -147,7 +176,11 @@ __global__ void __launch_bounds__(128, 1)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n0 = blockIdx.x * BM, m0 = blockIdx.y * BN;
-  const int num_kb = K / BK;
+  const int rank = SPLIT > 1 ? (int)cluster_rank() : 0;
+  const int total_kb = K / BK;
+  const int per = (total_kb + SPLIT - 1) / SPLIT;
+  const int kb0 = rank * per;
+  const int num_kb = max(0, min(total_kb, kb0 + per) - kb0);
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
@@ -177,7 +210,7 @@ __global__ void __launch_bounds__(128, 1)
   if (warp == 0 && lane == 0) {
     for (int kb = 0; kb < pre; ++kb) {
       mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
-      tma_load_2d(&tmW, &full_bar[kb], smem + kb * STAGE_BYTES, kb * BK, n0);
+      tma_load_2d(&tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb0 + kb) * BK, n0);
     }
   }
   pdl_wait();
@@ -191,9 +224,9 @@ __global__ void __launch_bounds__(128, 1)
       if (kb >= pre) {
         mbar_wait(&empty_bar[s], ((kb / STAGES) - 1) & 1);
         mbar_expect_tx(&full_bar[s], STAGE_BYTES);
-        tma_load_2d(&tmW, &full_bar[s], a, kb * BK, n0);
+        tma_load_2d(&tmW, &full_bar[s], a, (kb0 + kb) * BK, n0);
       }
-      tma_load_2d(&tmX, &full_bar[s], b, kb * BK, m0);
+      tma_load_2d(&tmX, &full_bar[s], b, (kb0 + kb) * BK, m0);
     }
   } else if (warp == 1 && lane == 0) {
     // MMA issuer
@@ -209,31 +242,75 @@ __global__ void __launch_bounds__(128, 1)
         umma_f16(tmem_d, da + 2 * kk, db + 2 * kk, IDESC, (kb | kk) != 0);
       umma_commit(&empty_bar[s]);
     }
-    umma_commit(&done_bar);
+    if (num_kb > 0) umma_commit(&done_bar);
   }
   __syncwarp();
 
-  // Epilogue (all 4 warps)
-  mbar_wait(&done_bar, 0);
-  asm volatile("tcgen05.fence::after_thread_sync;");
-  const int n = n0 + warp * 32 + lane;
-  const float bv = (bias != nullptr && n < N) ? Cvt<T>::to1(bias[n]) : 0.f;
+  if (num_kb > 0) {
+    mbar_wait(&done_bar, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;");
+  }
+  const int row = warp * 32 + lane;  // TMEM lane = W row within the tile
+  float* part = reinterpret_cast<float*>(smem) + row * PROW;  // the ring is free once MMAs are done
+
+  if (SPLIT > 1 && rank > 0) {
+    // park this K slice's partial tile for rank 0
 #pragma unroll
-  for (int c0 = 0; c0 < BN; c0 += 16) {
-    uint32_t v[16];
-    tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
-    if (n < N) {
+    for (int c0 = 0; c0 < BN; c0 += 16) {
+      uint32_t v[16];
+      if (num_kb > 0) tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
 #pragma unroll
-      for (int j = 0; j < 16; ++j) {
-        const int m = m0 + c0 + j;
-        if (m < M) {
-          float val = apply_act(__uint_as_float(v[j]) + bv, act);
-          if (res) val += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
-          store1<T>(Y, (size_t)m * ldy + n, val, io & IO_OUT_F32);
+      for (int j = 0; j < 16; j += 4)
+        *reinterpret_cast<float4*>(part + c0 + j) =
+            num_kb > 0 ? make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
+                                     __uint_as_float(v[j + 3]))
+                       : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+  }
+  if (SPLIT > 1) cluster_sync();  // partials visible cluster-wide
+
+  if (rank == 0) {
+    // Epilogue (all 4 warps of rank 0)
+    const int n = n0 + row;
+    const float bv = (bias != nullptr && n < N) ? Cvt<T>::to1(bias[n]) : 0.f;
+#pragma unroll
+    for (int c0 = 0; c0 < BN; c0 += 16) {
+      uint32_t v[16];
+      if (num_kb > 0) {
+        tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
+      } else {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) v[j] = 0u;
+      }
+      float acc[16];
+#pragma unroll
+      for (int j = 0; j < 16; ++j) acc[j] = __uint_as_float(v[j]);
+      if (SPLIT > 1) {
+        for (int r = 1; r < SPLIT; ++r) {
+#pragma unroll
+          for (int j = 0; j < 16; j += 4) {
+            const float4 q = ld_dsmem_f4(smem_u32(part + c0 + j), (uint32_t)r);
+            acc[j] += q.x;
+            acc[j + 1] += q.y;
+            acc[j + 2] += q.z;
+            acc[j + 3] += q.w;
+          }
+        }
+      }
+      if (n < N) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const int m = m0 + c0 + j;
+          if (m < M) {
+            float val = apply_act(acc[j] + bv, act);
+            if (res) val += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
+            store1<T>(Y, (size_t)m * ldy + n, val, io & IO_OUT_F32);
+          }
         }
       }
     }
   }
+  if (SPLIT > 1) cluster_sync();  // ranks >= 1 keep their shared memory until rank 0 has read it
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (warp == 1) {
@@ -271,31 +348,64 @@ CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int b
   return m;
 }
 
-template <class T, int BN>
+template <class T, int BN, int SPLIT>
 void run(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy, int M,
          int N, int K, int act, int io, cudaStream_t s) {
   constexpr size_t smem = size_t(stages_for<BN>()) * (BM * BK * 2 + BN * BK * 2) + 1024;
+  static_assert(size_t(BM) * (BN + 4) * 4 + 1024 <= smem, "partial tile must fit the ring");
   static bool attr = false;
   if (!attr) {
-    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN, SPLIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smem));
     attr = true;
   }
   const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
   CUtensorMap mw = make_map(w, dtype, N, K, K, BM);
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
-  dim3 grid(N / BM, (M + BN - 1) / BN);
-  launch_kernel(gemm_tc_kernel<T, BN>, grid, dim3(128), smem, s, mw, mx, (const T*)bias, res, ldr, y, ldy, M, N, K,
-                act, io);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(N / BM, (M + BN - 1) / BN, SPLIT);
+  cfg.blockDim = dim3(128);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  int na = 0;
+  if (SPLIT > 1) {
+    at[na].id = cudaLaunchAttributeClusterDimension;
+    at[na].val.clusterDim.x = 1;
+    at[na].val.clusterDim.y = 1;
+    at[na].val.clusterDim.z = SPLIT;
+    ++na;
+  }
+  if (take_pdl()) {
+    at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+  }
+  cfg.attrs = at;
+  cfg.numAttrs = na;
+  DP_CUDA(cudaLaunchKernelEx(&cfg, gemm_tc_kernel<T, BN, SPLIT>, mw, mx, (const T*)bias, res, ldr, y, ldy, M, N, K,
+                             act, io));
+}
+
+template <class T, int BN>
+void run_split(int split, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
+               int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
+  switch (split) {
+    case 1: run<T, BN, 1>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 2: run<T, BN, 2>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 4: run<T, BN, 4>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    default: fail(DP_ERR_INVALID, "gemm: split must be 1/2/4");
+  }
 }
 
 template <class T>
-void dispatch(int bn, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
-              int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
+void dispatch(int bn, int split, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
+              void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   switch (bn) {
-    case 32: run<T, 32>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 64: run<T, 64>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 128: run<T, 128>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 256: run<T, 256>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 32: run_split<T, 32>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 64: run_split<T, 64>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 128: run_split<T, 128>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 256: run_split<T, 256>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
     default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
   }
 }
@@ -313,6 +423,15 @@ static int pick_bn(int M, int N) {
   return 32;
 }
 
+// Split-K factor: enough CTAs to put the weight slice on most SMs, >= 3 k-blocks each.
+static int pick_split(int M, int N, int K, int bn) {
+  const int tiles = (N / BM) * ((M + bn - 1) / bn);
+  const int kb = K / BK;
+  int split = 1;
+  while (split < 4 && tiles * split * 2 <= 160 && kb / (split * 2) >= 3) split *= 2;
+  return split;
+}
+
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
   DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
@@ -320,10 +439,11 @@ void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void
            "GEMM operands must be 16-byte aligned");
   if (M <= 0) return;
   const int bn = bn_hint > 0 ? bn_hint : pick_bn(M, N);
+  const int split = pick_split(M, N, K, bn);
   if (dtype == DP_BF16)
-    dispatch<__nv_bfloat16>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+    dispatch<__nv_bfloat16>(bn, split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
   else
-    dispatch<__half>(bn, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+    dispatch<__half>(bn, split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
 }
 
 }  // namespace dp

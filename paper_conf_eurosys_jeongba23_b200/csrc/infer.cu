@@ -731,6 +731,46 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
 
 }  // namespace dp
 
+extern "C" dp_status dp_measure_h2d(int32_t dev, int64_t bytes, int32_t reps, double* gbs) {
+  void* h = nullptr;
+  void* d = nullptr;
+  cudaStream_t s = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  dp_status st = guard([&] {
+    DP_CHECK(gbs && bytes > 0 && reps >= 1, DP_ERR_INVALID, "bad arguments");
+    DeviceGuard g(dev);
+    if (cudaHostAlloc(&h, bytes, cudaHostAllocPortable | cudaHostAllocMapped) != cudaSuccess) {
+      h = nullptr;
+      fail(DP_ERR_OOM, "cudaHostAlloc failed");
+    }
+    std::memset(h, 1, bytes);
+    if (cudaMalloc(&d, bytes) != cudaSuccess) {
+      d = nullptr;
+      fail(DP_ERR_OOM, "cudaMalloc failed");
+    }
+    DP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    DP_CUDA(cudaEventCreate(&e0));
+    DP_CUDA(cudaEventCreate(&e1));
+    float best = 1e30f;
+    for (int r = 0; r <= reps; ++r) {  // first copy is a warm-up
+      DP_CUDA(cudaEventRecord(e0, s));
+      DP_CUDA(cudaMemcpyAsync(d, h, bytes, cudaMemcpyHostToDevice, s));
+      DP_CUDA(cudaEventRecord(e1, s));
+      DP_CUDA(cudaEventSynchronize(e1));
+      float ms = 0;
+      DP_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+      if (r > 0) best = std::min(best, ms);
+    }
+    *gbs = double(bytes) / (double(best) * 1e-3) / 1e9;
+  });
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (s) cudaStreamDestroy(s);
+  if (d) cudaFree(d);
+  if (h) cudaFreeHost(h);
+  return st;
+}
+
 extern "C" dp_status dp_profile(dp_context* ctx, dp_model* m, int32_t dev, int32_t batch, int32_t seq, int32_t iters,
                                 dp_cost_table* out) {
   return guard([&] {

@@ -36,27 +36,45 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
   pdl_trigger();
   const int nv = H / 8;
   const bool has_type = type != nullptr, has_ln = g != nullptr;
-  for (int i = threadIdx.x; i < 3 * nv; i += blockDim.x) {  // weights: no dependency on the previous kernel
-    const int which = i / nv, c = i - which * nv;
-    const T* src = which == 0 ? type : (which == 1 ? g : b);
-    if (src) sm[i] = ldg16(src + 8 * c);
+  // the shared rows (token type 0, gamma, beta) go into registers first; their host round
+  // trip overlaps the word/position gathers below (one PCIe latency per CTA, not two)
+  constexpr int SPT = 3;  // 3*nv <= 3*192 vectors over 256 threads
+  uint4 stage[SPT];
+#pragma unroll
+  for (int k = 0; k < SPT; ++k) {
+    const int i = threadIdx.x + k * 256;
+    if (i < 3 * nv) {
+      const int which = i / nv, c = i - which * nv;
+      const T* src = which == 0 ? type : (which == 1 ? g : b);
+      if (src) stage[k] = ldg16(src + 8 * c);
+    }
   }
   pdl_wait();
-  __syncthreads();
   const int lane = threadIdx.x & 31;
   const int t = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-  if (t >= ntok) return;
-  const int id = ids[t];
-  const int p = pos_off + (t % seq);
+  const bool live = t < ntok;
+  const int id = live ? ids[t] : 0;
+  const int p = pos_off + (live ? t % seq : 0);
   uint4 wv[VPL], pv[VPL];
 #pragma unroll
   for (int v = 0; v < VPL; ++v) {  // issue every host read of this row before using any
     const int c = lane + 32 * v;
-    if (c < nv) {
+    if (live && c < nv) {
       wv[v] = ldg16(word + (size_t)id * H + 8 * c);
       pv[v] = ldg16(pos + (size_t)p * H + 8 * c);
     }
   }
+#pragma unroll
+  for (int k = 0; k < SPT; ++k) {
+    const int i = threadIdx.x + k * 256;
+    if (i < 3 * nv) {
+      const int which = i / nv;
+      const T* src = which == 0 ? type : (which == 1 ? g : b);
+      if (src) sm[i] = stage[k];
+    }
+  }
+  __syncthreads();
+  if (!live) return;
   float x[VPL][8];
   float sum = 0.f;
 #pragma unroll
