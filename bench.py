@@ -109,6 +109,55 @@ def measure_h2d_peak(dp, torch, nbytes=256 << 20, reps=5):
     return dp.measure_h2d(torch.cuda.current_device(), nbytes, reps)
 
 
+def kernel_rooflines(dp, torch, m, T, peaks, peak_h2d, reps=50):
+    """Per-kernel achieved rates, measured live with CUDA events on the launching stream:
+    a sleep kernel holds the stream while the host enqueues `reps` launches, so the event
+    interval is device time only.  Algorithmic bytes / flops per launch are in DESIGN.md §5."""
+    import math
+    H, F = m.hidden, m.ffn
+    out = []
+
+    def dev_us(fn):
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda._sleep(int(2e6 + reps * 40000))
+        e0.record()
+        for _ in range(reps):
+            fn()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) * 1e3 / reps
+
+    ridge = peaks["bf16_tflops_sustained"] * 1e12 / (peaks["hbm_gbs"] * 1e9)
+    for name, N, K in (("gemm_tc fc1", F, H), ("gemm_tc q", H, H), ("gemm_tc fc2", H, F)):
+        x = torch.randn(T, K, device="cuda").half()
+        w = (torch.randn(N, K, device="cuda") / math.sqrt(K)).half()
+        b = torch.randn(N, device="cuda").half()
+        y = torch.empty(T, N, device="cuda").half()
+        us = dev_us(lambda: dp.linear(x, K, w, b, None, 0, y, N, T, N, K, path=0))
+        flops, byts = 2.0 * T * N * K, 2.0 * (N * K + T * K + T * N + N)
+        if T < ridge:  # below the ridge the weight stream bounds it
+            out.append({"kernel": f"{name} [{T}x{N}x{K}]", "bound": "hbm", "us": round(us, 2),
+                        "achieved": round(byts / us / 1e3, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                        "frac": round(byts / us / 1e3 / peaks["hbm_gbs"], 4)})
+        else:
+            out.append({"kernel": f"{name} [{T}x{N}x{K}]", "bound": "tensor", "us": round(us, 2),
+                        "achieved": round(flops / us / 1e6, 1), "peak": peaks["bf16_tflops_sustained"],
+                        "unit": "TFLOP/s", "frac": round(flops / us / 1e6 / peaks["bf16_tflops_sustained"], 4)})
+    # DHA skinny linear (weights read over PCIe exactly once)
+    x = torch.randn(T, H, device="cuda").half()
+    wh = dp.host_alloc(H * H * 2)
+    y = torch.empty(T, H, device="cuda").half()
+    us = dev_us(lambda: dp.linear(x, H, wh, None, None, 0, y, H, T, H, H, path=1))
+    out.append({"kernel": f"skinny_linear DHA [{T}x{H}x{H}]", "bound": "pcie", "us": round(us, 2),
+                "achieved": round(H * H * 2 / us / 1e3, 1), "peak": round(peak_h2d, 1), "unit": "GB/s",
+                "frac": round(H * H * 2 / us / 1e3 / peak_h2d, 4)})
+    dp.host_free(wh)
+    return out
+
+
 def cpu_oracle_ms(m, w, ids, dtype, budget_s=15.0, max_runs=10):
     """The oracle (fp64 numpy) timed on this host's cores, on a bounded sample."""
     from oracle import forward as F
@@ -335,6 +384,7 @@ def main():
     R_lit = total_w / (peak_h2d * world * 1e9) * 1e3  # all weight bytes / aggregate H2D
     R_alg = per_link / (peak_h2d * 1e9) * 1e3          # busiest link's algorithmic bytes
     peaks, peaks_src = measured_peaks()
+    krl = kernel_rooflines(dp, torch, m, T, peaks, peak_h2d)
 
     cpu = None
     if not a.no_cpu_baseline:
@@ -373,6 +423,7 @@ def main():
                   "step_ms_max": round(max(lat), 4), "warm_kernels": wst["n_kernels"]},
         "peaks": {"source": peaks_src, "hbm_gbs": peaks.get("hbm_gbs"),
                   "bf16_tflops_sustained": peaks.get("bf16_tflops_sustained")},
+        "kernel_rooflines": krl,
         "cpu_baseline": cpu,
     }
     print(json.dumps(line), flush=True)
