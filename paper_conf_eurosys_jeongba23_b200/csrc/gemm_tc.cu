@@ -123,14 +123,11 @@ __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
-__device__ __forceinline__ float4 ld_dsmem_f4(uint32_t local_addr, uint32_t rank) {
+__device__ __forceinline__ float ld_dsmem_f32(uint32_t local_addr, uint32_t rank) {
   uint32_t remote;
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(local_addr), "r"(rank));
-  float4 v;
-  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-               : "r"(remote)
-               : "memory");
+  float v;
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(remote) : "memory");
   return v;
 }
 
@@ -164,7 +161,7 @@ __global__ void __launch_bounds__(128, 1)
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
-  constexpr int PROW = BN + 4;  // fp32 partial row stride (16 B pad against bank conflicts)
+  constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free row and column access)
   // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
   constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
                              (uint32_t(BM >> 4) << 24);
@@ -250,63 +247,48 @@ __global__ void __launch_bounds__(128, 1)
     mbar_wait(&done_bar, 0);
     asm volatile("tcgen05.fence::after_thread_sync;");
   }
+  // 1) TMEM -> shared memory (the ring is free once the MMAs are done): the fp32 tile,
+  //    [128 W rows][BN tokens] with an odd row stride, so column-wise reads are conflict-free
   const int row = warp * 32 + lane;  // TMEM lane = W row within the tile
-  float* part = reinterpret_cast<float*>(smem) + row * PROW;  // the ring is free once MMAs are done
-
-  if (SPLIT > 1 && rank > 0) {
-    // park this K slice's partial tile for rank 0
+  float* tile = reinterpret_cast<float*>(smem);
+#pragma unroll 1
+  for (int c0 = 0; c0 < BN; c0 += 16) {
+    uint32_t v[16];
+    if (num_kb > 0) {
+      tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
+    } else {
 #pragma unroll
-    for (int c0 = 0; c0 < BN; c0 += 16) {
-      uint32_t v[16];
-      if (num_kb > 0) tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
-#pragma unroll
-      for (int j = 0; j < 16; j += 4)
-        *reinterpret_cast<float4*>(part + c0 + j) =
-            num_kb > 0 ? make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
-                                     __uint_as_float(v[j + 3]))
-                       : make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int j = 0; j < 16; ++j) v[j] = 0u;
     }
+#pragma unroll
+    for (int j = 0; j < 16; ++j) tile[row * PROW + c0 + j] = __uint_as_float(v[j]);
   }
-  if (SPLIT > 1) cluster_sync();  // partials visible cluster-wide
-
+  // 2) make every K slice's tile visible (cluster-wide for split-K)
+  if (SPLIT > 1)
+    cluster_sync();
+  else
+    __syncthreads();
+  // 3) rank 0: out[m][n] for all tokens; thread t owns W row n = n0 + t, so for each token
+  //    the CTA's 128 stores are contiguous; split-K partials come over DSMEM
   if (rank == 0) {
-    // Epilogue (all 4 warps of rank 0)
-    const int n = n0 + row;
-    const float bv = (bias != nullptr && n < N) ? Cvt<T>::to1(bias[n]) : 0.f;
-#pragma unroll
-    for (int c0 = 0; c0 < BN; c0 += 16) {
-      uint32_t v[16];
-      if (num_kb > 0) {
-        tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
-      } else {
-#pragma unroll
-        for (int j = 0; j < 16; ++j) v[j] = 0u;
-      }
-      float acc[16];
-#pragma unroll
-      for (int j = 0; j < 16; ++j) acc[j] = __uint_as_float(v[j]);
+    const int t = threadIdx.x;
+    const int n = n0 + t;
+    const bool nok = n < N;
+    const float bv = (bias != nullptr && nok) ? Cvt<T>::to1(bias[n]) : 0.f;
+    const int mcount = min(BN, M - m0);
+    const uint32_t base = smem_u32(tile + t * PROW);
+#pragma unroll 4
+    for (int ml = 0; ml < mcount; ++ml) {
+      float acc = tile[t * PROW + ml];
       if (SPLIT > 1) {
-        for (int r = 1; r < SPLIT; ++r) {
 #pragma unroll
-          for (int j = 0; j < 16; j += 4) {
-            const float4 q = ld_dsmem_f4(smem_u32(part + c0 + j), (uint32_t)r);
-            acc[j] += q.x;
-            acc[j + 1] += q.y;
-            acc[j + 2] += q.z;
-            acc[j + 3] += q.w;
-          }
-        }
+        for (int r = 1; r < SPLIT; ++r) acc += ld_dsmem_f32(base + ml * 4, (uint32_t)r);
       }
-      if (n < N) {
-#pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const int m = m0 + c0 + j;
-          if (m < M) {
-            float val = apply_act(acc[j] + bv, act);
-            if (res) val += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
-            store1<T>(Y, (size_t)m * ldy + n, val, io & IO_OUT_F32);
-          }
-        }
+      if (nok) {
+        const int m = m0 + ml;
+        float val = apply_act(acc + bv, act);
+        if (res) val += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
+        store1<T>(Y, (size_t)m * ldy + n, val, io & IO_OUT_F32);
       }
     }
   }
@@ -352,7 +334,7 @@ template <class T, int BN, int SPLIT>
 void run(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy, int M,
          int N, int K, int act, int io, cudaStream_t s) {
   constexpr size_t smem = size_t(stages_for<BN>()) * (BM * BK * 2 + BN * BK * 2) + 1024;
-  static_assert(size_t(BM) * (BN + 4) * 4 + 1024 <= smem, "partial tile must fit the ring");
+  static_assert(size_t(BM) * (BN + 1) * 4 + 1024 <= smem, "fp32 tile must fit the ring");
   static bool attr = false;
   if (!attr) {
     DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN, SPLIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
