@@ -30,6 +30,7 @@
 
 #include <cstdint>
 #include <cstring>
+#include <cstdlib>
 #include <mutex>
 
 #include "common.h"
@@ -420,8 +421,11 @@ void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void
   DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0 && ((uintptr_t)w % 16) == 0, DP_ERR_INVALID,
            "GEMM operands must be 16-byte aligned");
   if (M <= 0) return;
-  const int bn = bn_hint > 0 ? bn_hint : pick_bn(M, N);
-  const int split = pick_split(M, N, K, bn);
+  // tuning overrides for experiments (DP_GEMM_BN / DP_GEMM_SPLIT), read once
+  static const int env_bn = getenv("DP_GEMM_BN") ? atoi(getenv("DP_GEMM_BN")) : 0;
+  static const int env_split = getenv("DP_GEMM_SPLIT") ? atoi(getenv("DP_GEMM_SPLIT")) : 0;
+  const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : pick_bn(M, N));
+  const int split = env_split > 0 ? env_split : pick_split(M, N, K, bn);
   if (dtype == DP_BF16)
     dispatch<__nv_bfloat16>(bn, split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
   else
