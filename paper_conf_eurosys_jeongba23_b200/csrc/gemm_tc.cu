@@ -269,28 +269,41 @@ __global__ void __launch_bounds__(128, 1)
     cluster_sync();
   else
     __syncthreads();
-  // 3) rank 0: out[m][n] for all tokens; thread t owns W row n = n0 + t, so for each token
-  //    the CTA's 128 stores are contiguous; split-K partials come over DSMEM
+  // 3) rank 0 writes out[m][n0 .. n0+127] for every token m: thread t owns 8 consecutive W
+  //    rows (n = n0 + 8*(t%16) ..+7) of token m = t/16 + 8*pass -> one 16-byte store (and
+  //    one 16-byte residual load) per 8 outputs; split-K partials come over DSMEM
   if (rank == 0) {
     const int t = threadIdx.x;
-    const int n = n0 + t;
-    const bool nok = n < N;
-    const float bv = (bias != nullptr && nok) ? Cvt<T>::to1(bias[n]) : 0.f;
+    const int nl = 8 * (t & 15);
+    const int n = n0 + nl;
+    const bool nok = n < N;  // N % 128 == 0, so all 8 rows are valid together
+    float bv[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) bv[e] = (bias != nullptr && nok) ? Cvt<T>::to1(bias[n + e]) : 0.f;
     const int mcount = min(BN, M - m0);
-    const uint32_t base = smem_u32(tile + t * PROW);
-#pragma unroll 4
-    for (int ml = 0; ml < mcount; ++ml) {
-      float acc = tile[t * PROW + ml];
+    const bool res32 = io & IO_RES_F32, out32 = io & IO_OUT_F32;
+#pragma unroll 1
+    for (int ml = t >> 4; ml < mcount; ml += 8) {
+      float acc[8];
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] = tile[(nl + e) * PROW + ml];
       if (SPLIT > 1) {
 #pragma unroll
-        for (int r = 1; r < SPLIT; ++r) acc += ld_dsmem_f32(base + ml * 4, (uint32_t)r);
+        for (int r = 1; r < SPLIT; ++r)
+#pragma unroll
+          for (int e = 0; e < 8; ++e) acc[e] += ld_dsmem_f32(smem_u32(tile + (nl + e) * PROW + ml), (uint32_t)r);
       }
-      if (nok) {
-        const int m = m0 + ml;
-        float val = apply_act(acc + bv, act);
-        if (res) val += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
-        store1<T>(Y, (size_t)m * ldy + n, val, io & IO_OUT_F32);
+      if (!nok) continue;
+      const size_t m = (size_t)(m0 + ml);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] = apply_act(acc[e] + bv[e], act);
+      if (res) {
+        float r8[8];
+        load8<T>(res, m * ldr + n, r8, res32);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) acc[e] += r8[e];
       }
+      store8<T>(Y, m * ldy + n, acc, out32);
     }
   }
   if (SPLIT > 1) cluster_sync();  // ranks >= 1 keep their shared memory until rank 0 has read it
@@ -406,14 +419,10 @@ static int pick_bn(int M, int N) {
   return 32;
 }
 
-// Split-K factor: enough CTAs to put the weight slice on most SMs, >= 3 k-blocks each.
-static int pick_split(int M, int N, int K, int bn) {
-  const int tiles = (N / BM) * ((M + bn - 1) / bn);
-  const int kb = K / BK;
-  int split = 1;
-  while (split < 4 && tiles * split * 2 <= 160 && kb / (split * 2) >= 3) split *= 2;
-  return split;
-}
+// Split-K factor.  Measured on B200 (profiles/r01_gemm_sweep.txt): the cluster barrier +
+// DSMEM reduction costs more than the extra SMs gain at every hot-path shape, so the
+// default is 1; DP_GEMM_SPLIT=2|4 selects the clustered variant for experiments.
+static int pick_split(int, int, int, int) { return 1; }
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
