@@ -60,7 +60,11 @@ enum {
   DP_MODE_GREEDY = 2,     /* DHA iff Exe(DHA) < Load + Exe(InMem), layer by layer */
   DP_MODE_DHA = 3,        /* Algorithm 1 */
   DP_MODE_PT = 4,         /* parallel transmission, all LOAD (§4.2) */
-  DP_MODE_PT_DHA = 5      /* Algorithm 1 on partition 0 + PT for the rest */
+  DP_MODE_PT_DHA = 5,     /* Algorithm 1 on partition 0 + PT for the rest */
+  /* NEXT-row extension, not the paper's (R19): Algorithm 1 on a
+   * pipeline model where DHA reads occupy the primary link (cost.dha_link_ns) */
+  DP_MODE_DHA_LINK = 6,
+  DP_MODE_PT_DHA_LINK = 7
 };
 
 /* ---------------------------------------------------------------------------------
@@ -83,6 +87,9 @@ typedef struct {
   const int64_t* fwd_ns;
   const int64_t* exe_mem_ns;
   const int64_t* exe_dha_ns;
+  /* nullable; our NEXT-row extension: time the unit's DHA reads occupy
+   * the primary PCIe link (touched bytes / link bandwidth); used only by the *_LINK modes */
+  const int64_t* dha_link_ns;
 } dp_cost_table;
 
 /* Execution plan: per unit a method (DP_LOAD/DP_DHA) and a slot (0 = the primary GPU's
@@ -102,7 +109,8 @@ typedef struct {
  * DP_ERR_INVALID on n mismatch, k < 1 or k > DP_MAX_DEVICES, unknown mode. */
 dp_status dp_plan_generate(const dp_cost_table* cost, int32_t mode, int32_t k, dp_plan* out);
 
-/* Pipeline cost model: latency, per-unit stall (n entries, nullable) and
+/* Pipeline cost model (the link-aware variant for plan->mode *_LINK): latency,
+ * per-unit stall (n entries, nullable) and
  * bytes carried by each link (k entries, nullable). */
 dp_status dp_plan_simulate(const dp_cost_table* cost, const dp_plan* plan, int64_t* latency_ns,
                            int64_t* stall_ns, int64_t* link_bytes);

@@ -19,7 +19,9 @@ import itertools
 import numpy as np
 
 LOAD, DHA = 0, 1
-MODES = ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "PT", "PT_DHA")
+MODES = ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "PT", "PT_DHA")  # the paper's options
+EXT_MODES = ("DHA_LINK", "PT_DHA_LINK")  # NEXT-row extension (link-aware), R19
+LINK_AWARE = {"DHA_LINK", "PT_DHA_LINK"}
 INF_NS = 1 << 50
 
 
@@ -36,15 +38,19 @@ def _arr(cost, key):
 # the pipelined manner", one layer at a time after it lands.
 # ------------------------------------------------------------------------------------
 
-def simulate(cost, method, slot=None, k: int = 1, serial: bool = False):
+def simulate(cost, method, slot=None, k: int = 1, serial: bool = False, link_aware: bool = False):
     """Returns dict(latency, stall[n], avail[n], start[n], link_bytes[k]).
 
     serial=True is the "Baseline" option (Fig.1b): load every layer, then execute.
+    link_aware=True is our NEXT-row extension (R19): a DHA unit's
+    reads occupy the primary link for cost["dha_link_ns"][i], in forward order with the loads
+    (the paper profiles Exe(DHA) in isolation and ignores that sharing, G11).
     """
     n = len(method)
     load, fwd = _arr(cost, "load_ns"), _arr(cost, "fwd_ns")
     exe_mem, exe_dha = _arr(cost, "exe_mem_ns"), _arr(cost, "exe_dha_ns")
     nbytes = _arr(cost, "bytes")
+    dlink = _arr(cost, "dha_link_ns") if (link_aware and "dha_link_ns" in cost) else [0] * n
     slot = [0] * n if slot is None else [int(s) for s in slot]
     t_link = [0] * k
     t_fwd = [0] * k
@@ -53,6 +59,7 @@ def simulate(cost, method, slot=None, k: int = 1, serial: bool = False):
     for i in range(n):
         if method[i] == DHA:
             avail[i] = 0
+            t_link[0] += dlink[i]
         elif slot[i] == 0:
             t_link[0] += load[i]
             avail[i] = t_link[0]
@@ -77,16 +84,21 @@ def simulate(cost, method, slot=None, k: int = 1, serial: bool = False):
     return {"latency": t, "stall": stall, "avail": avail, "start": start, "link_bytes": link_bytes}
 
 
-def simulate_events(cost, method, slot=None, k: int = 1):
+def simulate_events(cost, method, slot=None, k: int = 1, link_aware: bool = False):
     """An independent formulation of P1 as a discrete-event simulation with FIFO
     resources (one per PCIe link, one NVLink forwarder per secondary, one compute
-    engine).  Used only to pin ``simulate``; returns (latency, stall[n])."""
+    engine).  Used only to pin ``simulate``; returns (latency, stall[n]).  link_aware:
+    DHA units' reads are jobs on link 0 too (forward order), gating nothing."""
     n = len(method)
     load, fwd = _arr(cost, "load_ns"), _arr(cost, "fwd_ns")
     exe_mem, exe_dha = _arr(cost, "exe_mem_ns"), _arr(cost, "exe_dha_ns")
     slot = [0] * n if slot is None else [int(s) for s in slot]
+    dlink = _arr(cost, "dha_link_ns") if (link_aware and "dha_link_ns" in cost) else None
+    if dlink is not None:
+        load = [load[i] if method[i] == LOAD else dlink[i] for i in range(n)]
     # queues of pending jobs per resource, in forward order
-    link_q = {s: [i for i in range(n) if method[i] == LOAD and slot[i] == s] for s in range(k)}
+    link_q = {s: [i for i in range(n) if (method[i] == LOAD or (dlink is not None and s == 0)) and slot[i] == s]
+              for s in range(k)}
     busy_until = {("link", s): 0 for s in range(k)}
     busy_until.update({("nvl", s): 0 for s in range(1, k)})
     ready = [None] * n  # time unit i's weights are usable on the primary
@@ -106,7 +118,8 @@ def simulate_events(cost, method, slot=None, k: int = 1):
         t, _, kind, (s, i) = heapq.heappop(ev)
         if kind == "link_done":
             if s == 0:
-                ready[i] = t
+                if method[i] == LOAD:  # a DHA read completing gates nothing
+                    ready[i] = t
             else:
                 nvl_q[s].append(i)
                 if not nvl_busy[s]:
@@ -159,6 +172,36 @@ def algorithm1(cost):
     return method
 
 
+def algorithm1_link(cost):
+    """NEXT-row extension (R19), not the paper's algorithm: the
+    same loop as Algorithm 1 run on the link-aware simulator, where switching L_j to DHA frees
+    only saved_j = Load_j - DhaLink_j of link time.  Line 9 still breaks on S < PerfDiff_j;
+    a candidate with saved_j <= 0 is skipped (no link time freed: it cannot advance any later
+    load); line 13 becomes S - saved_j - PerfDiff_j.  With DhaLink = 0 and every Load > 0
+    this is exactly algorithm1."""
+    n = len(cost["load_ns"])
+    load = _arr(cost, "load_ns")
+    dlink = _arr(cost, "dha_link_ns") if "dha_link_ns" in cost else [0] * n
+    pd = [d - m for d, m in zip(_arr(cost, "exe_dha_ns"), _arr(cost, "exe_mem_ns"))]
+    method = [LOAD] * n
+    for i in range(n):
+        S = simulate(cost, method, link_aware=True)["stall"][i]
+        if not S > 0:
+            continue
+        cand = sorted((j for j in range(i + 1) if method[j] == LOAD), key=lambda j: (pd[j], j))
+        for j in cand:
+            if S < pd[j]:
+                break
+            saved = load[j] - dlink[j]
+            if saved <= 0:
+                continue
+            method[j] = DHA
+            S = S - saved - pd[j]
+            if S <= 0:
+                break
+    return method
+
+
 def greedy(cost):
     """The "initial approach" (Table 3): DHA iff Exe(DHA) < Load + Exe(InMem)."""
     load, em, ed = _arr(cost, "load_ns"), _arr(cost, "exe_mem_ns"), _arr(cost, "exe_dha_ns")
@@ -193,8 +236,11 @@ def plan(cost, mode: str, k: int = 1):
         return greedy(cost), [0] * n, False
     if mode == "DHA":
         return algorithm1(cost), [0] * n, False
-    if mode in ("PT", "PT_DHA"):
-        method = algorithm1(cost) if mode == "PT_DHA" else [LOAD] * n
+    if mode == "DHA_LINK":
+        return algorithm1_link(cost), [0] * n, False
+    if mode in ("PT", "PT_DHA", "PT_DHA_LINK"):
+        method = (algorithm1(cost) if mode == "PT_DHA" else
+                  algorithm1_link(cost) if mode == "PT_DHA_LINK" else [LOAD] * n)
         part = partition(cost["bytes"], k)
         slot = [0] * n
         for i in range(n):
@@ -210,13 +256,15 @@ def plan(cost, mode: str, k: int = 1):
 # Ties -> lexicographically smallest method vector (LOAD=0 < DHA=1).
 # ------------------------------------------------------------------------------------
 
-def simulate_batch(cost, methods: np.ndarray, slot=None, k: int = 1) -> np.ndarray:
+def simulate_batch(cost, methods: np.ndarray, slot=None, k: int = 1, link_aware: bool = False) -> np.ndarray:
     """Vectorised P1 latency over P method vectors (methods: [P, n] of 0/1)."""
     P, n = methods.shape
     load = np.asarray(cost["load_ns"], dtype=np.int64)
     fwd = np.asarray(cost["fwd_ns"], dtype=np.int64)
     em = np.asarray(cost["exe_mem_ns"], dtype=np.int64)
     ed = np.asarray(cost["exe_dha_ns"], dtype=np.int64)
+    dl = (np.asarray(cost["dha_link_ns"], dtype=np.int64) if (link_aware and "dha_link_ns" in cost)
+          else np.zeros(n, dtype=np.int64))
     slot = np.zeros(n, dtype=np.int64) if slot is None else np.asarray(slot, dtype=np.int64)
     t_link = np.zeros((k, P), dtype=np.int64)
     t_fwd = np.zeros((k, P), dtype=np.int64)
@@ -224,7 +272,7 @@ def simulate_batch(cost, methods: np.ndarray, slot=None, k: int = 1) -> np.ndarr
     for i in range(n):
         is_dha = methods[:, i] == DHA
         s = int(slot[i])
-        t_link[s] = np.where(is_dha, t_link[s], t_link[s] + load[i])
+        t_link[s] = np.where(is_dha, t_link[s] + (dl[i] if s == 0 else 0), t_link[s] + load[i])
         if s == 0:
             avail = np.where(is_dha, 0, t_link[0])
         else:
@@ -234,7 +282,7 @@ def simulate_batch(cost, methods: np.ndarray, slot=None, k: int = 1) -> np.ndarr
     return t
 
 
-def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 18):
+def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 18, link_aware: bool = False):
     """Optimal method vector under P1 with the P3 partition fixed (units with part >= 1
     are LOAD on their slot).  ``free``: indices allowed to vary (default: all part-0
     units); others keep ``base_method``.  Returns (latency, method, slot)."""
@@ -255,7 +303,7 @@ def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 
         methods = np.repeat(base[None, :], len(idx), axis=0)
         for b, u in enumerate(free):  # free[0] is the most significant bit -> lexicographic
             methods[:, u] = (idx >> (m - 1 - b)) & 1
-        lat = simulate_batch(cost, methods, slot, k)
+        lat = simulate_batch(cost, methods, slot, k, link_aware)
         j = int(np.argmin(lat))  # first minimum = lexicographically smallest
         if best_lat is None or lat[j] < best_lat:
             best_lat, best_idx = int(lat[j]), int(idx[j])

@@ -10,7 +10,8 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "libdeepplan.so")
 
 LOAD, DHA = 0, 1
-MODES = {"BASELINE": 0, "PIPESWITCH": 1, "GREEDY": 2, "DHA": 3, "PT": 4, "PT_DHA": 5}
+MODES = {"BASELINE": 0, "PIPESWITCH": 1, "GREEDY": 2, "DHA": 3, "PT": 4, "PT_DHA": 5, "DHA_LINK": 6,
+         "PT_DHA_LINK": 7}
 UNIT_KINDS = {0: "emb", 1: "ln", 2: "linear"}
 FAMILIES = {"bert": 0, "roberta": 1, "gpt2": 2}
 DTYPES = {"fp16": 0, "bf16": 1}
@@ -38,7 +39,7 @@ i64p = C.POINTER(C.c_int64)
 
 class CostTable(C.Structure):
     _fields_ = [("n", C.c_int32), ("bytes", i64p), ("load_ns", i64p), ("fwd_ns", i64p),
-                ("exe_mem_ns", i64p), ("exe_dha_ns", i64p)]
+                ("exe_mem_ns", i64p), ("exe_dha_ns", i64p), ("dha_link_ns", i64p)]
 
 
 class Plan(C.Structure):
@@ -167,10 +168,13 @@ _COST_KEYS = ("bytes", "load_ns", "fwd_ns", "exe_mem_ns", "exe_dha_ns")
 def _cost(cost: dict):
     arrs = [_i64(cost[k]) for k in _COST_KEYS]
     n = len(arrs[0])
+    if cost.get("dha_link_ns") is not None:
+        arrs.append(_i64(cost["dha_link_ns"]))
     for a in arrs:
         if len(a) != n:
             raise ValueError("cost table arrays differ in length")
-    ct = CostTable(n, *[_ptr(a, i64p) for a in arrs])
+    ptrs = [_ptr(a, i64p) for a in arrs] + ([None] if len(arrs) == 5 else [])
+    ct = CostTable(n, *ptrs)
     return ct, arrs
 
 
@@ -396,8 +400,8 @@ class Model:
         return np.ctypeslib.as_array(C.cast(p, C.POINTER(C.c_uint8)), shape=(n.value,))
 
     def profile(self, dev: int, batch: int, seq: int, iters: int = 10) -> dict:
-        arrs = {k: np.zeros(self.n, dtype=np.int64) for k in _COST_KEYS}
-        ct = CostTable(self.n, *[_ptr(arrs[k], i64p) for k in _COST_KEYS])
+        arrs = {k: np.zeros(self.n, dtype=np.int64) for k in _COST_KEYS + ("dha_link_ns",)}
+        ct = CostTable(self.n, *[_ptr(arrs[k], i64p) for k in _COST_KEYS + ("dha_link_ns",)])
         _check(lib.dp_profile(self.ctx.h, self.h, int(dev), int(batch), int(seq), int(iters), C.byref(ct)))
         return arrs
 

@@ -410,11 +410,13 @@ void dispatch(int bn, int split, const void* x, int ldx, const void* w, const vo
 
 bool gemm_tc_supported(int N, int K) { return N > 0 && K > 0 && N % BM == 0 && K % BK == 0; }
 
-// Tile width over tokens: the widest BN that still gives >= one CTA per SM, else 32.
+// Tile width over tokens: the widest BN that still gives >= 96 CTAs (~2/3 of the SMs), else
+// 32.  Chosen from the B200 sweep in profiles/r01_gemm_sweep_v2.txt: it picks the fastest
+// measured BN at every hot-path shape (M = 128 / 384 / 1024; N, K in 768..4096).
 static int pick_bn(int M, int N) {
   const int ntile = N / BM;
   for (int bn : {256, 128, 64}) {
-    if (M >= bn && ntile * ((M + bn - 1) / bn) >= 148) return bn;
+    if (M >= bn && ntile * ((M + bn - 1) / bn) >= 96) return bn;
   }
   return 32;
 }

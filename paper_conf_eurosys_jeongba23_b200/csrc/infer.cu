@@ -273,19 +273,21 @@ static void validate_plan(const dp_model* m, const dp_plan* p) {
   }
 }
 
+// Host-link bytes a unit's DHA kernels must read (algorithmic; Table 1's closed forms).
+static int64_t unit_dha_bytes(const dp_model* m, int u, int T, int seq) {
+  const int64_t row = int64_t(m->cfg.hidden) * 2;
+  switch (m->units[u].role) {
+    case R_WORD: case R_WTE: return int64_t(T) * row;  // one row per token
+    case R_POS: case R_WPE: return int64_t(std::min<int64_t>(seq, m->cfg.max_pos)) * row;
+    case R_TYPE: return row;
+    default: return m->units[u].bytes;  // LN gamma/beta, linear weights: every byte once
+  }
+}
+
 static int64_t dha_bytes(const dp_model* m, const int8_t* method, int T, int seq) {
   int64_t s = 0;
-  const int64_t row = int64_t(m->cfg.hidden) * 2;
-  for (size_t u = 0; u < m->units.size(); ++u) {
-    if (method[u] != DP_DHA) continue;
-    const auto& un = m->units[u];
-    switch (un.role) {
-      case R_WORD: case R_WTE: s += int64_t(T) * row; break;  // one row per token
-      case R_POS: case R_WPE: s += int64_t(std::min<int64_t>(seq, m->cfg.max_pos)) * row; break;
-      case R_TYPE: s += row; break;
-      default: s += un.bytes; break;  // LN gamma/beta, linear weights: every byte once
-    }
-  }
+  for (size_t u = 0; u < m->units.size(); ++u)
+    if (method[u] == DP_DHA) s += unit_dha_bytes(m, (int)u, T, seq);
   return s;
 }
 
@@ -721,6 +723,19 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
       out->exe_mem_ns[u] = timed([&] { run_unit(m, dev, u, false, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
       out->exe_dha_ns[u] = timed([&] { run_unit(m, dev, u, true, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
     }
+  }
+  // link time of each unit's DHA reads (link-aware modes): touched bytes at the best measured
+  // load rate of the units >= 1 MiB (the link's bulk DMA rate)
+  if (table->dha_link_ns) {
+    int64_t* dl = const_cast<int64_t*>(table->dha_link_ns);
+    double ns_per_byte = 0;
+    for (int u = 0; u < n; ++u)
+      if (out->bytes[u] >= (1 << 20) && out->load_ns[u] > 0) {
+        const double r = double(out->load_ns[u]) / double(out->bytes[u]);
+        ns_per_byte = ns_per_byte == 0 ? r : std::min(ns_per_byte, r);
+      }
+    if (ns_per_byte == 0) ns_per_byte = 1.0 / 50.0;  // no large unit: assume ~50 GB/s
+    for (int u = 0; u < n; ++u) dl[u] = (int64_t)llround(unit_dha_bytes(m, u, T, seq) * ns_per_byte);
   }
   DP_CUDA(cudaStreamSynchronize(s));
   cudaEventDestroy(e0);

@@ -31,14 +31,21 @@ static void check_cost(const dp_cost_table* c) {
 // a slot-s (s >= 1) unit is forwarded over NVLink after it lands on the secondary and
 // after the previous forward from that secondary; compute runs units in order, each
 // starting when the previous one ended and its weights are available (DHA: at once).
-static Sim simulate(const dp_cost_table* c, const int8_t* method, const int8_t* slot, int k, bool serial) {
+// link_aware (our NEXT-row extension, R19): a DHA unit's reads occupy the primary
+// link for dha_link_ns[i], in forward order with the loads.
+static Sim simulate(const dp_cost_table* c, const int8_t* method, const int8_t* slot, int k, bool serial,
+                    bool link_aware = false) {
   const int n = c->n;
   Sim r;
   r.stall.assign(n, 0);
   r.link_bytes.assign(std::max(k, 1), 0);
   std::vector<int64_t> link_t(std::max(k, 1), 0), fwd_t(std::max(k, 1), 0), ready(n, 0);
+  const bool la = link_aware && c->dha_link_ns != nullptr;
   for (int i = 0; i < n; ++i) {
-    if (method[i] == DP_DHA) continue;  // in host memory: usable immediately
+    if (method[i] == DP_DHA) {  // in host memory: usable immediately
+      if (la) link_t[0] += c->dha_link_ns[i];
+      continue;
+    }
     const int s = slot ? slot[i] : 0;
     link_t[s] += c->load_ns[i];
     r.link_bytes[s] += c->bytes[i];
@@ -92,6 +99,36 @@ static void algorithm1(const dp_cost_table* c, int8_t* method) {
   }
 }
 
+// Link-aware Algorithm 1 (NEXT-row extension, not the paper's; R19): the same loop
+// on the link-aware model; switching L_j frees only saved_j = Load_j - DhaLink_j of link
+// time, so a candidate with saved_j <= 0 is skipped and line 13 deducts saved_j.
+static void algorithm1_link(const dp_cost_table* c, int8_t* method) {
+  const int n = c->n;
+  std::vector<int64_t> pd(n);
+  for (int i = 0; i < n; ++i) pd[i] = c->exe_dha_ns[i] - c->exe_mem_ns[i];
+  for (int i = 0; i < n; ++i) method[i] = DP_LOAD;
+  std::vector<int> cand;
+  cand.reserve(n);
+  for (int i = 0; i < n; ++i) {
+    int64_t S = simulate(c, method, nullptr, 1, false, true).stall[i];
+    if (S <= 0) continue;
+    cand.clear();
+    for (int j = 0; j <= i; ++j)
+      if (method[j] == DP_LOAD) cand.push_back(j);
+    std::stable_sort(cand.begin(), cand.end(), [&](int a, int b) { return pd[a] < pd[b]; });
+    for (int j : cand) {
+      if (S < pd[j]) break;
+      const int64_t saved = c->load_ns[j] - (c->dha_link_ns ? c->dha_link_ns[j] : 0);
+      if (saved <= 0) continue;
+      method[j] = DP_DHA;
+      S = S - saved - pd[j];
+      if (S <= 0) break;
+    }
+  }
+}
+
+static bool link_mode(int mode) { return mode == DP_MODE_DHA_LINK || mode == DP_MODE_PT_DHA_LINK; }
+
 static void partition(const int64_t* bytes, int n, int k, int8_t* part) {
   int64_t total = 0;
   for (int i = 0; i < n; ++i) total += bytes[i];
@@ -132,10 +169,17 @@ static void generate(const dp_cost_table* c, int mode, int k, dp_plan* out) {
       algorithm1(c, out->method);
       out->k = 1;
       return;
+    case DP_MODE_DHA_LINK:
+      algorithm1_link(c, out->method);
+      out->k = 1;
+      return;
     case DP_MODE_PT:
-    case DP_MODE_PT_DHA: {
+    case DP_MODE_PT_DHA:
+    case DP_MODE_PT_DHA_LINK: {
       if (mode == DP_MODE_PT_DHA)
         algorithm1(c, out->method);
+      else if (mode == DP_MODE_PT_DHA_LINK)
+        algorithm1_link(c, out->method);
       else
         std::memset(out->method, DP_LOAD, n);
       std::vector<int8_t> part(n);
@@ -168,7 +212,7 @@ extern "C" dp_status dp_plan_simulate(const dp_cost_table* cost, const dp_plan* 
     DP_CHECK(plan->k >= 1 && plan->k <= DP_MAX_DEVICES, DP_ERR_INVALID, "plan.k out of range");
     for (int i = 0; i < plan->n; ++i)
       DP_CHECK(plan->slot[i] >= 0 && plan->slot[i] < plan->k, DP_ERR_INVALID, "slot out of range");
-    Sim r = simulate(cost, plan->method, plan->slot, plan->k, plan->serial != 0);
+    Sim r = simulate(cost, plan->method, plan->slot, plan->k, plan->serial != 0, link_mode(plan->mode));
     if (latency_ns) *latency_ns = r.latency;
     if (stall_ns) std::copy(r.stall.begin(), r.stall.end(), stall_ns);
     if (link_bytes) std::copy(r.link_bytes.begin(), r.link_bytes.begin() + plan->k, link_bytes);
@@ -202,7 +246,7 @@ extern "C" dp_status dp_plan_exhaustive(const dp_cost_table* cost, const dp_plan
     const uint64_t total = uint64_t(1) << nfree;
     for (uint64_t v = 0; v < total; ++v) {  // free_idx[0] is the most significant bit
       for (int b = 0; b < nfree; ++b) m[free_idx[b]] = int8_t((v >> (nfree - 1 - b)) & 1);
-      int64_t lat = simulate(cost, m.data(), part.data(), k, false).latency;
+      int64_t lat = simulate(cost, m.data(), part.data(), k, false, link_mode(base->mode)).latency;
       if (lat < best) {
         best = lat;
         best_v = v;

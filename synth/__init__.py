@@ -204,8 +204,11 @@ def make_cost_table(n: int, seed: int, *, max_ns: int = 1000, p_inf: float = 0.0
     exe_dha = np.maximum(exe_dha, 0)
     if p_inf > 0:
         exe_dha = np.where(rng.random(n) < p_inf, INF_NS, exe_dha)
+    # link time of a unit's DHA reads: mostly below its load time (embedding-like), sometimes
+    # about equal or above it (linear-like: every weight byte crosses the link anyway)
+    dha_link = (load * rng.integers(0, 130, size=n) // 100).astype(np.int64)
     return {"bytes": bytes_, "load_ns": load, "fwd_ns": fwd, "exe_mem_ns": exe_mem,
-            "exe_dha_ns": exe_dha.astype(np.int64)}
+            "exe_dha_ns": exe_dha.astype(np.int64), "dha_link_ns": dha_link}
 
 
 # --------------------------------------------------------------------------------------

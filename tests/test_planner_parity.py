@@ -17,23 +17,32 @@ def _check_one(c, mode, k):
     assert list(p.slot) == osl, (mode, k)
     assert p.serial == int(oser)
     lat, stall, link = dp.plan_simulate(c, p)
-    r = P.simulate(c, om, osl, max(k, 1) if mode in ("PT", "PT_DHA") else 1, serial=oser)
+    r = P.simulate(c, om, osl, max(k, 1) if mode.startswith("PT") else 1, serial=oser,
+                   link_aware=mode in P.LINK_AWARE)
     assert lat == r["latency"]
     assert list(stall) == r["stall"]
     assert list(link) == r["link_bytes"][:len(link)]
 
 
+ALL_MODES = P.MODES + P.EXT_MODES
+
+
 @pytest.mark.parametrize("block", range(20))
 def test_random_tables_all_modes(block):
-    """10^4 random integer tables (20 blocks x 500)."""
+    """10^4 random integer tables (20 blocks x 500), the paper's modes and the link-aware
+    extension."""
     rng = np.random.default_rng(block)
     for t in range(500):
         seed = block * 1000 + t
         n = int(rng.integers(1, 40))
         c = synth.make_cost_table(n, seed, max_ns=int(rng.integers(10, 100000)), p_inf=0.05)
-        mode = P.MODES[t % len(P.MODES)]
-        k = int(rng.integers(1, 9)) if mode in ("PT", "PT_DHA") else 1
+        mode = ALL_MODES[t % len(ALL_MODES)]
+        k = int(rng.integers(1, 9)) if mode.startswith("PT") else 1
         _check_one(c, mode, k)
+        if t % 7 == 0:  # the paper's modes must not depend on dha_link_ns
+            c2 = {kk: v for kk, v in c.items() if kk != "dha_link_ns"}
+            if mode in P.MODES:
+                _check_one(c2, mode, k)
 
 
 @pytest.mark.parametrize("name", ["tiny_bert", "bert_base", "bert_large", "roberta_large", "gpt2_medium"])
@@ -47,7 +56,8 @@ def test_model_shaped_tables(name):
     c = {"bytes": nb, "load_ns": load, "fwd_ns": nb // 700, "exe_mem_ns": exe,
          "exe_dha_ns": exe + load + rng.integers(-5000, 40000, n)}
     c["exe_dha_ns"] = np.maximum(c["exe_dha_ns"], 0)
-    for mode in P.MODES:
+    c["dha_link_ns"] = load.copy()
+    for mode in ALL_MODES:
         for k in ((1, 2, 4, 8) if mode.startswith("PT") else (1,)):
             _check_one(c, mode, k)
 
