@@ -724,18 +724,16 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
       out->exe_dha_ns[u] = timed([&] { run_unit(m, dev, u, true, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
     }
   }
-  // link time of each unit's DHA reads (link-aware modes): touched bytes at the best measured
-  // load rate of the units >= 1 MiB (the link's bulk DMA rate)
+  // link time of each unit's DHA reads (link-aware modes): the unit's own measured load time
+  // scaled by the fraction of its bytes a DHA execution touches -- a linear or LayerNorm reads
+  // every byte (no link time freed), an embedding only the used rows (R19)
   if (table->dha_link_ns) {
     int64_t* dl = const_cast<int64_t*>(table->dha_link_ns);
-    double ns_per_byte = 0;
-    for (int u = 0; u < n; ++u)
-      if (out->bytes[u] >= (1 << 20) && out->load_ns[u] > 0) {
-        const double r = double(out->load_ns[u]) / double(out->bytes[u]);
-        ns_per_byte = ns_per_byte == 0 ? r : std::min(ns_per_byte, r);
-      }
-    if (ns_per_byte == 0) ns_per_byte = 1.0 / 50.0;  // no large unit: assume ~50 GB/s
-    for (int u = 0; u < n; ++u) dl[u] = (int64_t)llround(unit_dha_bytes(m, u, T, seq) * ns_per_byte);
+    for (int u = 0; u < n; ++u) {
+      const int64_t touched = std::min(unit_dha_bytes(m, u, T, seq), out->bytes[u]);
+      dl[u] = out->bytes[u] > 0 ? (int64_t)llround(double(out->load_ns[u]) * double(touched) / double(out->bytes[u]))
+                                : 0;
+    }
   }
   DP_CUDA(cudaStreamSynchronize(s));
   cudaEventDestroy(e0);
