@@ -366,11 +366,26 @@ static void skinny_t(const void* x, int ldx, const void* w, const void* bias, co
                 (const T*)bias, res, ldr, y, ldy, M, N, K, act, io);
 }
 
+template <class T>
+void skinny_mma_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy,
+                  int M, int N, int K, int act, int io, cudaStream_t s);
+
+// M <= 16 tokens (e.g. the pooler): warp-shuffle dot products; more tokens: the same one-pass
+// weight staging with the per-CTA products on mma.sync (the link stays the bound).
 void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
                           int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   DP_CHECK(K % 8 == 0 && K > 0 && N > 0, DP_ERR_INVALID, "skinny linear needs K % 8 == 0");
-  DP_CHECK(size_t(8) * K * 4 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
   if (M <= 0) return;
+  const bool mma = M > 16 && N % 16 == 0 && K % 16 == 0 && ldx % 2 == 0;
+  if (mma) {
+    DP_CHECK(size_t(16) * (K + 8) * 2 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
+    if (dtype == DP_BF16)
+      skinny_mma_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+    else
+      skinny_mma_t<__half>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+    return;
+  }
+  DP_CHECK(size_t(8) * K * 4 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
   if (dtype == DP_BF16)
     skinny_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
   else
@@ -577,6 +592,86 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   else
     launch_kernel(attention_kernel<__half>, grid, dim3(128), 0, s, (const __half*)qkv, ldqkv, (__half*)ctx, seq, H,
                   causal ? 1 : 0, scale_log2);
+}
+
+// -------------------------------------------------------------------------------------
+// K3 (M > 16 tokens): the DHA skinny linear with its products on mma.sync.  Each CTA owns
+// 16 W rows: it streams them from (host) memory once -- coalesced 16-byte loads, all issued
+// before the grid-dependency wait -- into padded shared memory (row stride K+8 elements, so
+// ldmatrix is conflict-free); then each warp takes groups of 8 tokens and runs
+// m16n8k16 MMAs (A = the 16 staged W rows via ldmatrix, B = X^T fragments straight from the
+// L2-resident activations, fp32 accumulate).  Host-link bytes = N*K*2 + N*2 exactly.
+// -------------------------------------------------------------------------------------
+template <class T>
+__global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X, int ldx, const T* W,
+                                                         const T* bias, const void* res, int ldr, void* Y, int ldy,
+                                                         int M, int N, int K, int act, int io) {
+  extern __shared__ __align__(16) uint8_t smem_sk[];
+  T* sw16 = reinterpret_cast<T*>(smem_sk);  // [16][K + 8]
+  pdl_trigger();
+  const int KP = K + 8;
+  const int kv = K / 8;
+  const int n0 = blockIdx.x * 16;
+  const uint4* src = reinterpret_cast<const uint4*>(W + (size_t)n0 * K);
+  const int total = 16 * kv;
+  for (int base = threadIdx.x; base < total; base += 8 * 256) {
+    uint4 r[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if (base + j * 256 < total) r[j] = ldg16(src + base + j * 256);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int i = base + j * 256;
+      if (i < total) *reinterpret_cast<uint4*>(&sw16[(i / kv) * KP + (i % kv) * 8]) = r[j];
+    }
+  }
+  __shared__ float sbias[16];
+  if (threadIdx.x < 16) sbias[threadIdx.x] = bias ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
+  pdl_wait();
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int g = lane >> 2, t4 = lane & 3;
+  const int groups = (M + 7) / 8;
+  const T* arow = &sw16[(lane & 15) * KP + (lane >> 4) * 8];  // ldmatrix row address (k = 0)
+  for (int grp = warp; grp < groups; grp += 8) {
+    const int tok = grp * 8 + g;
+    const bool tok_ok = tok < M;
+    const uint32_t* xr = reinterpret_cast<const uint32_t*>(X + (size_t)(tok_ok ? tok : 0) * ldx);
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll 4
+    for (int k0 = 0; k0 < K; k0 += 16) {
+      uint32_t a[4], b[2];
+      ldsm_x4(a, arow + k0);
+      b[0] = tok_ok ? __ldg(xr + (k0 >> 1) + t4) : 0u;
+      b[1] = tok_ok ? __ldg(xr + (k0 >> 1) + 4 + t4) : 0u;
+      MmaOp<T>::mma(acc, a, b);
+    }
+    // acc: c0,c1 -> W row g, tokens 2*t4, 2*t4+1; c2,c3 -> W row g+8, same tokens
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int r = g + (e >> 1) * 8;
+      const int m = grp * 8 + 2 * t4 + (e & 1);
+      if (m < M) {
+        const int n = n0 + r;
+        float v = apply_act(acc[e] + sbias[r], act);
+        if (res) v += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
+        store1<T>(Y, (size_t)m * ldy + n, v, io & IO_OUT_F32);
+      }
+    }
+  }
+}
+
+template <class T>
+void skinny_mma_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy,
+                  int M, int N, int K, int act, int io, cudaStream_t s) {
+  const size_t sm = size_t(16) * (K + 8) * sizeof(T);
+  static bool attr_set = false;  // one per template instantiation
+  if (!attr_set) {
+    DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+    attr_set = true;
+  }
+  launch_kernel(skinny_mma_kernel<T>, dim3(N / 16), dim3(256), sm, s, (const T*)x, ldx, (const T*)w, (const T*)bias,
+                res, ldr, y, ldy, M, N, K, act, io);
 }
 
 // -------------------------------------------------------------------------------------
