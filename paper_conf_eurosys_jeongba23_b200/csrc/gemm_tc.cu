@@ -15,13 +15,11 @@
 //   warp 1 / lane 0  : MMA issuer  -- 4 x tcgen05.mma (K = 16 each) per stage, fp32
 //                      accumulator in TMEM; tcgen05.commit releases the smem stage;
 //   warp 1           : TMEM allocate / free (BN columns);
-//   all 4 warps      : epilogue -- tcgen05.ld 32 lanes x 16 columns, + bias, activation,
-//                      + residual, store (warp w owns TMEM lanes 32w..32w+31).
-// Split-K for the latency-bound skinny layers: a thread-block cluster of SPLIT CTAs along z
-// shares one output tile, each CTA streams 1/SPLIT of K; ranks >= 1 park their fp32 partial
-// tile in shared memory and rank 0 sums them through distributed shared memory (DSMEM)
-// before the epilogue.  More SMs pull the weight slice in parallel; no extra launch, no
-// global-memory workspace.
+//   all 4 warps      : epilogue -- tcgen05.ld 32 lanes x 16 columns into a shared-memory
+//                      fp32 tile, then + bias, activation, + residual and 16-byte stores.
+// blockIdx.z selects one of up to 3 weight matrices sharing X (BERT q/k/v in one launch).
+// Explored and measured slower on B200 (profiles/r01_gemm_sweep_v1.txt): split-K over a
+// thread-block cluster with a DSMEM reduction (cluster-barrier waits dominated).
 // Descriptor encodings follow the sm_100 UMMA descriptor layout (start>>4, LBO, SBO = 1024 B
 // for 8-row swizzle atoms, version 1, layout SWIZZLE_128B = 2).
 #include <cuda.h>
@@ -114,23 +112,8 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-__device__ __forceinline__ uint32_t cluster_rank() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-  return r;
-}
 
-__device__ __forceinline__ void cluster_sync() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
 
-__device__ __forceinline__ float ld_dsmem_f32(uint32_t local_addr, uint32_t rank) {
-  uint32_t remote;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(local_addr), "r"(rank));
-  float v;
-  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(remote) : "memory");
-  return v;
-}
 
 template <class T>
 struct FmtBits;
@@ -152,17 +135,24 @@ __host__ __device__ constexpr int stages_for() {
   return s > 12 ? 12 : s;
 }
 
-template <class T, int BN, int SPLIT>
+// Up to 3 independent weight matrices sharing X, M, N, K (BERT's q/k/v): blockIdx.z selects
+// the weight, its bias and the output column offset, so the three projections are one launch.
+struct GemmGroup {
+  CUtensorMap w[3];
+  const void* bias[3];
+  long long ycol[3];
+};
+
+template <class T, int BN>
 __global__ void __launch_bounds__(128, 1)
-    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmX,
-                   const T* __restrict__ bias, const void* res, int ldr, void* Y, int ldy, int M,
-                   int N, int K, int act, int io) {
+    gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
+                   const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io) {
   constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
-  constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free row and column access)
+  constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free TMEM->smem writes)
   // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
   constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
                              (uint32_t(BM >> 4) << 24);
@@ -174,14 +164,13 @@ __global__ void __launch_bounds__(128, 1)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n0 = blockIdx.x * BM, m0 = blockIdx.y * BN;
-  const int rank = SPLIT > 1 ? (int)cluster_rank() : 0;
-  const int total_kb = K / BK;
-  const int per = (total_kb + SPLIT - 1) / SPLIT;
-  const int kb0 = rank * per;
-  const int num_kb = max(0, min(total_kb, kb0 + per) - kb0);
+  const CUtensorMap* tmW = &grp.w[blockIdx.z];
+  const T* bias = static_cast<const T*>(grp.bias[blockIdx.z]);
+  const long long ycol = grp.ycol[blockIdx.z];
+  const int num_kb = K / BK;
 
   if (warp == 0 && lane == 0) {
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmW)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full_bar[s], 1);
@@ -208,7 +197,7 @@ __global__ void __launch_bounds__(128, 1)
   if (warp == 0 && lane == 0) {
     for (int kb = 0; kb < pre; ++kb) {
       mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
-      tma_load_2d(&tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb0 + kb) * BK, n0);
+      tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, kb * BK, n0);
     }
   }
   pdl_wait();
@@ -222,9 +211,9 @@ __global__ void __launch_bounds__(128, 1)
       if (kb >= pre) {
         mbar_wait(&empty_bar[s], ((kb / STAGES) - 1) & 1);
         mbar_expect_tx(&full_bar[s], STAGE_BYTES);
-        tma_load_2d(&tmW, &full_bar[s], a, (kb0 + kb) * BK, n0);
+        tma_load_2d(tmW, &full_bar[s], a, kb * BK, n0);
       }
-      tma_load_2d(&tmX, &full_bar[s], b, (kb0 + kb) * BK, m0);
+      tma_load_2d(&tmX, &full_bar[s], b, kb * BK, m0);
     }
   } else if (warp == 1 && lane == 0) {
     // MMA issuer
@@ -240,39 +229,28 @@ __global__ void __launch_bounds__(128, 1)
         umma_f16(tmem_d, da + 2 * kk, db + 2 * kk, IDESC, (kb | kk) != 0);
       umma_commit(&empty_bar[s]);
     }
-    if (num_kb > 0) umma_commit(&done_bar);
+    umma_commit(&done_bar);
   }
   __syncwarp();
 
-  if (num_kb > 0) {
-    mbar_wait(&done_bar, 0);
-    asm volatile("tcgen05.fence::after_thread_sync;");
-  }
+  mbar_wait(&done_bar, 0);
+  asm volatile("tcgen05.fence::after_thread_sync;");
   // 1) TMEM -> shared memory (the ring is free once the MMAs are done): the fp32 tile,
-  //    [128 W rows][BN tokens] with an odd row stride, so column-wise reads are conflict-free
+  //    [128 W rows][BN tokens] with an odd row stride
   const int row = warp * 32 + lane;  // TMEM lane = W row within the tile
   float* tile = reinterpret_cast<float*>(smem);
 #pragma unroll 1
   for (int c0 = 0; c0 < BN; c0 += 16) {
     uint32_t v[16];
-    if (num_kb > 0) {
-      tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
-    } else {
-#pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = 0u;
-    }
+    tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
 #pragma unroll
     for (int j = 0; j < 16; ++j) tile[row * PROW + c0 + j] = __uint_as_float(v[j]);
   }
-  // 2) make every K slice's tile visible (cluster-wide for split-K)
-  if (SPLIT > 1)
-    cluster_sync();
-  else
-    __syncthreads();
-  // 3) rank 0 writes out[m][n0 .. n0+127] for every token m: thread t owns 8 consecutive W
-  //    rows (n = n0 + 8*(t%16) ..+7) of token m = t/16 + 8*pass -> one 16-byte store (and
-  //    one 16-byte residual load) per 8 outputs; split-K partials come over DSMEM
-  if (rank == 0) {
+  __syncthreads();
+  // 2) out[m][n0 .. n0+127] for every token m: thread t owns 8 consecutive W rows
+  //    (n = n0 + 8*(t%16) ..+7) of token m = t/16 + 8*pass -> one 16-byte store (and one
+  //    16-byte residual load) per 8 outputs
+  {
     const int t = threadIdx.x;
     const int nl = 8 * (t & 15);
     const int n = n0 + nl;
@@ -283,30 +261,20 @@ __global__ void __launch_bounds__(128, 1)
     const int mcount = min(BN, M - m0);
     const bool res32 = io & IO_RES_F32, out32 = io & IO_OUT_F32;
 #pragma unroll 1
-    for (int ml = t >> 4; ml < mcount; ml += 8) {
+    for (int ml = t >> 4; ml < mcount && nok; ml += 8) {
       float acc[8];
 #pragma unroll
-      for (int e = 0; e < 8; ++e) acc[e] = tile[(nl + e) * PROW + ml];
-      if (SPLIT > 1) {
-#pragma unroll
-        for (int r = 1; r < SPLIT; ++r)
-#pragma unroll
-          for (int e = 0; e < 8; ++e) acc[e] += ld_dsmem_f32(smem_u32(tile + (nl + e) * PROW + ml), (uint32_t)r);
-      }
-      if (!nok) continue;
+      for (int e = 0; e < 8; ++e) acc[e] = apply_act(tile[(nl + e) * PROW + ml] + bv[e], act);
       const size_t m = (size_t)(m0 + ml);
-#pragma unroll
-      for (int e = 0; e < 8; ++e) acc[e] = apply_act(acc[e] + bv[e], act);
       if (res) {
         float r8[8];
         load8<T>(res, m * ldr + n, r8, res32);
 #pragma unroll
         for (int e = 0; e < 8; ++e) acc[e] += r8[e];
       }
-      store8<T>(Y, m * ldy + n, acc, out32);
+      store8<T>(Y, m * ldy + n + ycol, acc, out32);
     }
   }
-  if (SPLIT > 1) cluster_sync();  // ranks >= 1 keep their shared memory until rank 0 has read it
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (warp == 1) {
@@ -344,64 +312,38 @@ CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int b
   return m;
 }
 
-template <class T, int BN, int SPLIT>
-void run(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy, int M,
-         int N, int K, int act, int io, cudaStream_t s) {
+template <class T, int BN>
+void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
+         const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   constexpr size_t smem = size_t(stages_for<BN>()) * (BM * BK * 2 + BN * BK * 2) + 1024;
   static_assert(size_t(BM) * (BN + 1) * 4 + 1024 <= smem, "fp32 tile must fit the ring");
   static bool attr = false;
   if (!attr) {
-    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN, SPLIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)smem));
+    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     attr = true;
   }
   const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
-  CUtensorMap mw = make_map(w, dtype, N, K, K, BM);
+  GemmGroup g;
+  std::memset(&g, 0, sizeof(g));
+  for (int i = 0; i < ngroups; ++i) {
+    g.w[i] = make_map(w[i], dtype, N, K, K, BM);
+    g.bias[i] = bias ? bias[i] : nullptr;
+    g.ycol[i] = ycol ? ycol[i] : 0;
+  }
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(N / BM, (M + BN - 1) / BN, SPLIT);
-  cfg.blockDim = dim3(128);
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = s;
-  cudaLaunchAttribute at[2];
-  int na = 0;
-  if (SPLIT > 1) {
-    at[na].id = cudaLaunchAttributeClusterDimension;
-    at[na].val.clusterDim.x = 1;
-    at[na].val.clusterDim.y = 1;
-    at[na].val.clusterDim.z = SPLIT;
-    ++na;
-  }
-  if (take_pdl()) {
-    at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    at[na].val.programmaticStreamSerializationAllowed = 1;
-    ++na;
-  }
-  cfg.attrs = at;
-  cfg.numAttrs = na;
-  DP_CUDA(cudaLaunchKernelEx(&cfg, gemm_tc_kernel<T, BN, SPLIT>, mw, mx, (const T*)bias, res, ldr, y, ldy, M, N, K,
-                             act, io));
-}
-
-template <class T, int BN>
-void run_split(int split, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
-               int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
-  switch (split) {
-    case 1: run<T, BN, 1>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 2: run<T, BN, 2>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 4: run<T, BN, 4>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    default: fail(DP_ERR_INVALID, "gemm: split must be 1/2/4");
-  }
+  launch_kernel(gemm_tc_kernel<T, BN>, dim3(N / BM, (M + BN - 1) / BN, ngroups), dim3(128), smem, s, g, mx, res, ldr,
+                y, ldy, M, N, K, act, io);
 }
 
 template <class T>
-void dispatch(int bn, int split, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
-              void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
+void dispatch(int bn, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
+              const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io,
+              cudaStream_t s) {
   switch (bn) {
-    case 32: run_split<T, 32>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 64: run_split<T, 64>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 128: run_split<T, 128>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 256: run_split<T, 256>(split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 32: run<T, 32>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 64: run<T, 64>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 128: run<T, 128>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 256: run<T, 256>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
     default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
   }
 }
@@ -421,26 +363,29 @@ static int pick_bn(int M, int N) {
   return 32;
 }
 
-// Split-K factor.  Measured on B200 (profiles/r01_gemm_sweep.txt): the cluster barrier +
-// DSMEM reduction costs more than the extra SMs gain at every hot-path shape, so the
-// default is 1; DP_GEMM_SPLIT=2|4 selects the clustered variant for experiments.
-static int pick_split(int, int, int, int) { return 1; }
+void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
+                          const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
+                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
+  DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
+  DP_CHECK(ngroups >= 1 && ngroups <= 3, DP_ERR_INVALID, "gemm: 1..3 weight groups");
+  DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0, DP_ERR_INVALID, "GEMM activations must be 16-byte aligned");
+  for (int i = 0; i < ngroups; ++i)
+    DP_CHECK(((uintptr_t)w[i] % 16) == 0 && (!ycol || ycol[i] % 8 == 0), DP_ERR_INVALID,
+             "GEMM weights / output columns must be 16-byte aligned");
+  DP_CHECK(ldy % 8 == 0 && (!res || ldr % 8 == 0), DP_ERR_INVALID, "GEMM output rows must be 16-byte aligned");
+  if (M <= 0) return;
+  // tuning override for experiments (DP_GEMM_BN), read once
+  static const int env_bn = getenv("DP_GEMM_BN") ? atoi(getenv("DP_GEMM_BN")) : 0;
+  const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : pick_bn(M, N * ngroups));
+  if (dtype == DP_BF16)
+    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s);
+  else
+    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s);
+}
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
-  DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
-  DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0 && ((uintptr_t)w % 16) == 0, DP_ERR_INVALID,
-           "GEMM operands must be 16-byte aligned");
-  if (M <= 0) return;
-  // tuning overrides for experiments (DP_GEMM_BN / DP_GEMM_SPLIT), read once
-  static const int env_bn = getenv("DP_GEMM_BN") ? atoi(getenv("DP_GEMM_BN")) : 0;
-  static const int env_split = getenv("DP_GEMM_SPLIT") ? atoi(getenv("DP_GEMM_SPLIT")) : 0;
-  const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : pick_bn(M, N));
-  const int split = env_split > 0 ? env_split : pick_split(M, N, K, bn);
-  if (dtype == DP_BF16)
-    dispatch<__nv_bfloat16>(bn, split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
-  else
-    dispatch<__half>(bn, split, x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+  launch_gemm_tc_group(dtype, x, ldx, 1, &w, &bias, nullptr, res, ldr, y, ldy, M, N, K, act, io, bn_hint, s);
 }
 
 }  // namespace dp

@@ -602,18 +602,6 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
 // m16n8k16 MMAs (A = the 16 staged W rows via ldmatrix, B = X^T fragments straight from the
 // L2-resident activations, fp32 accumulate).  Host-link bytes = N*K*2 + N*2 exactly.
 // -------------------------------------------------------------------------------------
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(smem))),
-               "l"(gmem)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
-constexpr int SK_CHUNKS = 4;   // K is streamed in 4 chunks: compute on chunk c overlaps chunk c+1's PCIe reads
 constexpr int SK_GMAX = 8;     // token groups (of 8) a warp keeps accumulators for at once
 
 template <class T>
@@ -624,44 +612,34 @@ __global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X
   T* sw16 = reinterpret_cast<T*>(smem_sk);  // [16][K + 8]
   pdl_trigger();
   const int KP = K + 8;
+  const int kv = K / 8;
   const int n0 = blockIdx.x * 16;
-  const T* wsrc = W + (size_t)n0 * K;
-  // every PCIe read of this CTA's 16 W rows is issued up front (cp.async, before the
-  // grid-dependency wait: weights never depend on the previous kernel), one commit group per
-  // K chunk, so the MMAs on chunk c run while chunks c+1.. are still in flight
-  const int kc = K / SK_CHUNKS;      // elements per chunk (a multiple of 16)
-  const int cv = kc / 8;             // 16-byte vectors per row per chunk
+  // every PCIe read of this CTA's 16 W rows is issued up front -- coalesced 16-byte loads,
+  // up to 8 in flight per thread, before the grid-dependency wait (weights never depend on
+  // the previous kernel).  (cp.async from mapped host memory measured 2x slower.)
+  const uint4* src = reinterpret_cast<const uint4*>(W + (size_t)n0 * K);
+  const int total = 16 * kv;
+  for (int base = threadIdx.x; base < total; base += 8 * 256) {
+    uint4 r[8];
 #pragma unroll
-  for (int c = 0; c < SK_CHUNKS; ++c) {
-    for (int i = threadIdx.x; i < 16 * cv; i += 256) {
-      const int r = i / cv, v = i - r * cv;
-      const int k = c * kc + v * 8;
-      cp_async16(&sw16[r * KP + k], wsrc + (size_t)r * K + k);
+    for (int j = 0; j < 8; ++j)
+      if (base + j * 256 < total) r[j] = ldg16(src + base + j * 256);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int i = base + j * 256;
+      if (i < total) *reinterpret_cast<uint4*>(&sw16[(i / kv) * KP + (i % kv) * 8]) = r[j];
     }
-    cp_async_commit();
   }
   __shared__ float sbias[16];
   if (threadIdx.x < 16) sbias[threadIdx.x] = bias ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
   pdl_wait();
+  __syncthreads();
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int g = lane >> 2, t4 = lane & 3;
   const int groups = (M + 7) / 8;
   const T* arow = &sw16[(lane & 15) * KP + (lane >> 4) * 8];  // ldmatrix row address (k = 0)
-  if (warp >= groups) {  // no tokens for this warp: take part in the 4 chunk barriers only
-#pragma unroll
-    for (int c = 0; c < SK_CHUNKS; ++c) {
-      switch (c) {
-        case 0: cp_async_wait<SK_CHUNKS - 1>(); break;
-        case 1: cp_async_wait<SK_CHUNKS - 2>(); break;
-        case 2: cp_async_wait<SK_CHUNKS - 3>(); break;
-        default: cp_async_wait<0>(); break;
-      }
-      __syncthreads();
-    }
-    return;
-  }
   // token groups of this warp: warp, warp+8, ...; processed SK_GMAX at a time (one ldmatrix
-  // of the W fragment feeds all of them); the first pass waits chunk by chunk
+  // of the W fragment feeds all of them, and their X loads are independent)
   for (int gb = warp; gb < groups; gb += 8 * SK_GMAX) {
     float acc[SK_GMAX][4];
     const uint32_t* xr[SK_GMAX];
@@ -673,29 +651,17 @@ __global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X
       xr[q] = reinterpret_cast<const uint32_t*>(X + (size_t)(ok[q] ? tok : 0) * ldx);
       acc[q][0] = acc[q][1] = acc[q][2] = acc[q][3] = 0.f;
     }
-#pragma unroll
-    for (int c = 0; c < SK_CHUNKS; ++c) {
-      if (gb == warp) {  // first pass: wait for chunk c (later passes find everything landed)
-        switch (c) {
-          case 0: cp_async_wait<SK_CHUNKS - 1>(); break;
-          case 1: cp_async_wait<SK_CHUNKS - 2>(); break;
-          case 2: cp_async_wait<SK_CHUNKS - 3>(); break;
-          default: cp_async_wait<0>(); break;
-        }
-        __syncthreads();
-      }
 #pragma unroll 2
-      for (int k0 = c * kc; k0 < (c + 1) * kc; k0 += 16) {
-        uint32_t a[4];
-        ldsm_x4(a, arow + k0);
+    for (int k0 = 0; k0 < K; k0 += 16) {
+      uint32_t a[4];
+      ldsm_x4(a, arow + k0);
 #pragma unroll
-        for (int q = 0; q < SK_GMAX; ++q) {
-          if (ok[q]) {
-            uint32_t b[2];
-            b[0] = __ldg(xr[q] + (k0 >> 1) + t4);
-            b[1] = __ldg(xr[q] + (k0 >> 1) + 4 + t4);
-            MmaOp<T>::mma(acc[q], a, b);
-          }
+      for (int q = 0; q < SK_GMAX; ++q) {
+        if (ok[q]) {
+          uint32_t b[2];
+          b[0] = __ldg(xr[q] + (k0 >> 1) + t4);
+          b[1] = __ldg(xr[q] + (k0 >> 1) + 4 + t4);
+          MmaOp<T>::mma(acc[q], a, b);
         }
       }
     }

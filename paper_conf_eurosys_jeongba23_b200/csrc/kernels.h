@@ -33,6 +33,10 @@ struct GemmPlan;  // cached tensor map for a weight
 bool gemm_tc_supported(int N, int K);
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);
+// ngroups (1..3) weights sharing X; group i writes y at column offset ycol[i].
+void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
+                          const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
+                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);
 
 // Scratch kernels
 void launch_l2_flush(void* buf, size_t bytes, cudaStream_t s);
