@@ -352,6 +352,7 @@ typedef struct {
    * its cold-start plan; a plan with k > 1 uses the next k-1 GPUs of the context as
    * secondaries (their PCIe links and copy engines, not their compute) */
   const dp_plan* const* plans;
+  const int32_t* seq_of_model; /* nullable: per model index sequence length (else `seq`) */
 } dp_serve_opts;
 
 typedef struct {

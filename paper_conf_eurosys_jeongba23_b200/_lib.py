@@ -88,7 +88,8 @@ class ServeOpts(C.Structure):
                 ("per_gpu_budget_bytes", C.c_int64), ("slo_ns", C.c_int64), ("nmodels", C.c_int32),
                 ("reserved0", C.c_int32), ("cold_ns", i64p), ("warm_ns", i64p), ("resident_bytes", i64p),
                 ("model_of_instance", i32p), ("ninstances", C.c_int32), ("batch", C.c_int32),
-                ("seq", C.c_int32), ("reserved1", C.c_int32), ("plans", C.POINTER(C.POINTER(Plan)))]
+                ("seq", C.c_int32), ("reserved1", C.c_int32), ("plans", C.POINTER(C.POINTER(Plan))),
+                ("seq_of_model", i32p)]
 
 
 class ServeResult(C.Structure):
@@ -500,7 +501,7 @@ def attention(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp1
 
 def serve_run(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, cold_ns, warm_ns, resident_bytes,
               model_of_instance, slo_ns=100_000_000, dry_run=True, ctx: Context | None = None, models=None,
-              plans=None, batch=1, seq=128, plan_mode="DHA", k_max=1):
+              plans=None, batch=1, seq=128, plan_mode="DHA", k_max=1, seq_of_model=None):
     arrival_ns = _i64(arrival_ns)
     instance = np.ascontiguousarray(instance, dtype=np.int32)
     n = len(arrival_ns)
@@ -527,6 +528,10 @@ def serve_run(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, cold_ns, warm
     o.ninstances = len(moi)
     o.batch = int(batch)
     o.seq = int(seq)
+    som = None
+    if seq_of_model is not None:
+        som = np.ascontiguousarray(seq_of_model, dtype=np.int32)
+        o.seq_of_model = _ptr(som, i32p)
     mh = None
     if not dry_run:
         pp = (C.POINTER(Plan) * len(plans))(*[C.pointer(p.s) for p in plans])

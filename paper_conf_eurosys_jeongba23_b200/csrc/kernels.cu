@@ -376,9 +376,9 @@ void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, cons
                           int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   DP_CHECK(K % 8 == 0 && K > 0 && N > 0, DP_ERR_INVALID, "skinny linear needs K % 8 == 0");
   if (M <= 0) return;
-  const bool mma = M > 16 && N % 16 == 0 && K % 64 == 0 && ldx % 2 == 0;  // 4 chunks of 16-multiples
+  const bool mma = M > 16 && N % 16 == 0 && K % 16 == 0 && ldx % 8 == 0 && ((uintptr_t)x % 16) == 0;
   if (mma) {
-    DP_CHECK(size_t(16) * (K + 8) * 2 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
+    DP_CHECK((size_t(16) * (K + 8) + 128 * 136) * 2 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
     if (dtype == DP_BF16)
       skinny_mma_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
     else
@@ -602,16 +602,21 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
 // m16n8k16 MMAs (A = the 16 staged W rows via ldmatrix, B = X^T fragments straight from the
 // L2-resident activations, fp32 accumulate).  Host-link bytes = N*K*2 + N*2 exactly.
 // -------------------------------------------------------------------------------------
-constexpr int SK_GMAX = 8;     // token groups (of 8) a warp keeps accumulators for at once
+constexpr int SK_TOK = 128;  // tokens per pass (16 groups of 8: two per warp)
+constexpr int SK_KCH = 128;  // K elements of X staged per chunk
 
+// X fragments for two token groups at once (ldmatrix.x4 over 16 staged X rows: tokens
+// 0-7 / 8-15 x k 0-7 / 8-15), then one m16n8k16 per group against the shared W fragment.
 template <class T>
 __global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X, int ldx, const T* W,
                                                          const T* bias, const void* res, int ldr, void* Y, int ldy,
                                                          int M, int N, int K, int act, int io) {
   extern __shared__ __align__(16) uint8_t smem_sk[];
-  T* sw16 = reinterpret_cast<T*>(smem_sk);  // [16][K + 8]
-  pdl_trigger();
   const int KP = K + 8;
+  T* sw16 = reinterpret_cast<T*>(smem_sk);        // W slice [16][K + 8]
+  T* sx = sw16 + 16 * KP;                          // X chunk [SK_TOK][SK_KCH + 8]
+  constexpr int XP = SK_KCH + 8;
+  pdl_trigger();
   const int kv = K / 8;
   const int n0 = blockIdx.x * 16;
   // every PCIe read of this CTA's 16 W rows is issued up front -- coalesced 16-byte loads,
@@ -633,47 +638,43 @@ __global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X
   __shared__ float sbias[16];
   if (threadIdx.x < 16) sbias[threadIdx.x] = bias ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
   pdl_wait();
-  __syncthreads();
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int g = lane >> 2, t4 = lane & 3;
-  const int groups = (M + 7) / 8;
-  const T* arow = &sw16[(lane & 15) * KP + (lane >> 4) * 8];  // ldmatrix row address (k = 0)
-  // token groups of this warp: warp, warp+8, ...; processed SK_GMAX at a time (one ldmatrix
-  // of the W fragment feeds all of them, and their X loads are independent)
-  for (int gb = warp; gb < groups; gb += 8 * SK_GMAX) {
-    float acc[SK_GMAX][4];
-    const uint32_t* xr[SK_GMAX];
-    bool ok[SK_GMAX];
-#pragma unroll
-    for (int q = 0; q < SK_GMAX; ++q) {
-      const int tok = (gb + 8 * q) * 8 + g;
-      ok[q] = (gb + 8 * q) < groups && tok < M;
-      xr[q] = reinterpret_cast<const uint32_t*>(X + (size_t)(ok[q] ? tok : 0) * ldx);
-      acc[q][0] = acc[q][1] = acc[q][2] = acc[q][3] = 0.f;
-    }
-#pragma unroll 2
-    for (int k0 = 0; k0 < K; k0 += 16) {
-      uint32_t a[4];
-      ldsm_x4(a, arow + k0);
-#pragma unroll
-      for (int q = 0; q < SK_GMAX; ++q) {
-        if (ok[q]) {
-          uint32_t b[2];
-          b[0] = __ldg(xr[q] + (k0 >> 1) + t4);
-          b[1] = __ldg(xr[q] + (k0 >> 1) + 4 + t4);
-          MmaOp<T>::mma(acc[q], a, b);
+  const T* arow = &sw16[(lane & 15) * KP + (lane >> 4) * 8];  // W fragment rows (k = 0)
+  // X fragment rows for this warp's two groups: tokens 16*warp + (lane&7) + 8*(lane>>4),
+  // k half (lane>>3)&1
+  const T* brow = &sx[(16 * warp + (lane & 7) + ((lane >> 4) << 3)) * XP + ((lane >> 3) & 1) * 8];
+  for (int t0 = 0; t0 < M; t0 += SK_TOK) {
+    const int nt = min(SK_TOK, M - t0);
+    float acc[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+    for (int kc = 0; kc < K; kc += SK_KCH) {
+      const int kw = min(SK_KCH, K - kc);  // K % 16 == 0, so kw is a multiple of 16
+      __syncthreads();                      // previous chunk consumed (and W staged, first time)
+      for (int i = threadIdx.x; i < SK_TOK * (SK_KCH / 8); i += 256) {
+        const int r = i / (SK_KCH / 8), c = i - r * (SK_KCH / 8);
+        uint4 v = make_uint4(0, 0, 0, 0);
+        if (r < nt && c * 8 < kw) v = *reinterpret_cast<const uint4*>(X + (size_t)(t0 + r) * ldx + kc + c * 8);
+        *reinterpret_cast<uint4*>(&sx[r * XP + c * 8]) = v;
+      }
+      __syncthreads();
+      if (16 * warp < nt) {
+#pragma unroll 4
+        for (int ks = 0; ks < kw; ks += 16) {
+          uint32_t a[4], b[4];
+          ldsm_x4(a, arow + kc + ks);
+          ldsm_x4(b, brow + ks);
+          MmaOp<T>::mma(acc[0], a, b);
+          MmaOp<T>::mma(acc[1], a, b + 2);
         }
       }
     }
-    // acc: c0,c1 -> W row g, tokens 2*t4, 2*t4+1; c2,c3 -> W row g+8, same tokens
+    // acc[q]: c0,c1 -> W row g, tokens 2*t4, 2*t4+1 of group q; c2,c3 -> W row g+8
 #pragma unroll
-    for (int q = 0; q < SK_GMAX; ++q) {
-      if (!ok[q]) continue;
-      const int grp = gb + 8 * q;
+    for (int q = 0; q < 2; ++q) {
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
         const int r = g + (e >> 1) * 8;
-        const int m = grp * 8 + 2 * t4 + (e & 1);
+        const int m = t0 + 16 * warp + 8 * q + 2 * t4 + (e & 1);
         if (m < M) {
           const int n = n0 + r;
           float v = apply_act(acc[q][e] + sbias[r], act);
@@ -688,7 +689,7 @@ __global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X
 template <class T>
 void skinny_mma_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy,
                   int M, int N, int K, int act, int io, cudaStream_t s) {
-  const size_t sm = size_t(16) * (K + 8) * sizeof(T);
+  const size_t sm = (size_t(16) * (K + 8) + size_t(SK_TOK) * (SK_KCH + 8)) * sizeof(T);
   static bool attr_set = false;  // one per template instantiation
   if (!attr_set) {
     DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));

@@ -57,7 +57,10 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
   }
   int maxH = 0;
   for (int i = 0; i < nmodels; ++i) maxH = std::max(maxH, models[i]->cfg.hidden);
-  const int T = o.batch * o.seq;
+  auto seq_of = [&](int inst) { return o.seq_of_model ? o.seq_of_model[o.model_of_instance[inst]] : o.seq; };
+  int max_seq = o.seq;
+  for (int i = 0; i < o.ninstances; ++i) max_seq = std::max(max_seq, seq_of(i));
+  const int T = o.batch * max_seq;
   std::vector<std::vector<int>> queue(G);
   for (int r = 0; r < nreq; ++r) queue[out[r].gpu].push_back(r);
   // Workers first pre-warm every instance they will serve (HBM slots, workspace, captured
@@ -97,8 +100,8 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
             for (int k = 1; k < plan->k; ++k) sec.push_back(ctx->devs[(g + k) % G]);
             std::lock_guard<std::mutex> lk(enqueue_mu);
             m->dev[dev].resident = false;
-            infer_cold(ctx, m, plan, dev, -1, sec.data(), (int)sec.size(), ids, o.batch, o.seq, y, pool, s, nullptr);
-            dp_status st = dp_infer_warm(ctx, m, dev, ids, o.batch, o.seq, y, pool, s, nullptr);
+            infer_cold(ctx, m, plan, dev, -1, sec.data(), (int)sec.size(), ids, o.batch, seq_of(inst), y, pool, s, nullptr);
+            dp_status st = dp_infer_warm(ctx, m, dev, ids, o.batch, seq_of(inst), y, pool, s, nullptr);
             DP_CHECK(st == DP_OK, st, "warm inference failed");
             DP_CUDA(cudaStreamSynchronize(s));
             m->dev[dev].resident = false;
@@ -124,10 +127,10 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
             for (int k = 1; k < plan->k; ++k) sec.push_back(ctx->devs[(g + k) % G]);
             if (m->dev[dev].resident) m->dev[dev].resident = false;  // defensive: decisions say cold
             std::lock_guard<std::mutex> lk(enqueue_mu);
-            infer_cold(ctx, m, plan, dev, -1, sec.data(), (int)sec.size(), ids, o.batch, o.seq, y, pool, s, nullptr);
+            infer_cold(ctx, m, plan, dev, -1, sec.data(), (int)sec.size(), ids, o.batch, seq_of(inst), y, pool, s, nullptr);
           } else {
             std::lock_guard<std::mutex> lk(enqueue_mu);
-            dp_status st = dp_infer_warm(ctx, m, dev, ids, o.batch, o.seq, y, pool, s, nullptr);
+            dp_status st = dp_infer_warm(ctx, m, dev, ids, o.batch, seq_of(inst), y, pool, s, nullptr);
             DP_CHECK(st == DP_OK, st, "warm inference failed");
           }
           DP_CUDA(cudaStreamSynchronize(s));

@@ -1,13 +1,15 @@
-"""Multi-instance serving on real GPUs (SURVEY §8(a) a16, config 5; PAPER.md §5.3 P:322-338).
+"""Multi-instance serving on real GPUs (SURVEY §8(a) a16, config 5; PAPER.md §5.3 P:322-350).
 
-Instances are clones of one registered model (same shapes, shared pinned arena, separate
-residency).  Each plan mode (PIPESWITCH = all loaded, DHA = Algorithm 1, PT_DHA when several
-GPUs) gets its measured cold / warm latency and resident bytes (DHA units stay in host
-memory); a seeded Poisson trace is replayed live through dp_serve_run with
-one request per GPU at a time and LRU eviction under a per-GPU budget.  Reports p99,
-goodput at the SLO and the cold-start rate, beside the dry-run replay of the same decisions.
+Instances are clones of registered base models (same shapes, shared pinned arena, separate
+residency), mixed by ratio (BERT-Base : RoBERTa-Base : GPT-2 = 4:4:1).  Each plan mode
+(PIPESWITCH = all loaded, DHA = Algorithm 1, DHA_LINK, PT_DHA* with several GPUs) gets its
+measured cold / warm latency and resident bytes per model (DHA units stay in host memory,
+P:332); a seeded Poisson trace is replayed live through dp_serve_run with one request
+per GPU at a time and LRU eviction under a per-GPU budget.  Reports p99, goodput at the SLO,
+the cold-start rate and throughput, beside the dry-run replay of the same decisions.
 
-python tools/serve_bench.py [--gpus 1] [--instances 40] [--fit 8] [--rate 400] [--requests 600]
+python tools/serve_bench.py [--gpus 1] [--mix bert_base:128:1] [--instances 40] [--fit 8]
+                            [--rate 300] [--requests 600] [--slo-ms 10] [--modes PIPESWITCH,DHA,DHA_LINK]
 """
 import argparse
 import json
@@ -22,70 +24,74 @@ import paper_conf_eurosys_jeongba23_b200 as dp
 import synth
 
 
+def dev_ms(fn, reps=6):
+    ts = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record()
+        fn()
+        e1.record()
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    return float(np.median(ts[1:]))
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--model", default="bert_base")
-    ap.add_argument("--seq", type=int, default=128)
+    ap.add_argument("--mix", default="bert_base:128:1", help="name:seq:weight,...")
     ap.add_argument("--instances", type=int, default=40)
-    ap.add_argument("--fit", type=int, default=8, help="all-loaded instances that fit one GPU's budget")
-    ap.add_argument("--rate", type=float, default=400.0, help="requests per second (Poisson)")
+    ap.add_argument("--fit", type=float, default=8, help="all-loaded instances of model 0 per GPU budget")
+    ap.add_argument("--rate", type=float, default=300.0, help="requests per second (Poisson)")
     ap.add_argument("--requests", type=int, default=600)
     ap.add_argument("--slo-ms", type=float, default=10.0)
-    ap.add_argument("--modes", default="PIPESWITCH,DHA")
+    ap.add_argument("--modes", default="PIPESWITCH,DHA,DHA_LINK")
     a = ap.parse_args()
-    m = synth.SHAPES[a.model]
-    w = synth.make_weights(m, seed=0)
+    mix = [(n, int(s), int(wt)) for n, s, wt in (x.split(":") for x in a.mix.split(","))]
     ctx = dp.Context(list(range(a.gpus)))
     ctx.set_opts(use_graph=1)
-    base = dp.Model(ctx, m, w)
-    cost = base.profile(0, 1, a.seq, 5)
-    insts = [base] + [base.clone() for _ in range(a.instances - 1)]
-    ids = torch.from_numpy(synth.make_ids(m, 1, a.seq)).cuda()
-    out = torch.empty(a.seq, m.hidden, dtype=torch.float16, device="cuda")
-    pool = torch.empty(1, m.hidden, dtype=torch.float16, device="cuda") if m.family != "gpt2" else None
-    budget = a.fit * base.nbytes
+    bases, costs, io = [], [], []
+    for name, seq, _ in mix:
+        m = synth.SHAPES[name]
+        base = dp.Model(ctx, m, synth.make_weights(m, seed=0))
+        costs.append(base.profile(0, 1, seq, 5))
+        bases.append(base)
+        ids = torch.from_numpy(synth.make_ids(m, 1, seq)).cuda()
+        out = torch.empty(seq, m.hidden, dtype=torch.float16, device="cuda")
+        pool = torch.empty(1, m.hidden, dtype=torch.float16, device="cuda") if m.family != "gpt2" else None
+        io.append((ids, out, pool))
+    moi = synth.instance_models(a.instances, tuple(w for _, _, w in mix)) if len(mix) > 1 \
+        else np.zeros(a.instances, np.int32)
+    insts = [bases[moi[i]].clone() for i in range(a.instances)]  # the bases are profiling-only
+    budget = int(a.fit * bases[0].nbytes)
     arr, inst = synth.make_poisson_trace(a.requests, a.rate, a.instances, seed=11)
-    report = {"model": a.model, "seq": a.seq, "gpus": a.gpus, "instances": a.instances, "rate_rps": a.rate,
-              "requests": a.requests, "slo_ms": a.slo_ms, "per_gpu_budget_bytes": budget, "modes": {}}
+    report = {"mix": a.mix, "gpus": a.gpus, "instances": a.instances, "rate_rps": a.rate, "requests": a.requests,
+              "slo_ms": a.slo_ms, "per_gpu_budget_bytes": budget, "modes": {}}
     for mode in a.modes.split(","):
         k = a.gpus if mode.startswith("PT") else 1
-        plan = dp.plan_generate(cost, mode, k)
-        sec = list(range(1, k))
+        plans, cold, warm, resident = [], [], [], []
+        for mi, base in enumerate(bases):
+            plan = dp.plan_generate(costs[mi], mode, k)
+            sec = list(range(1, k))
+            ids, out, pool = io[mi]
 
-        def cold():
-            if base.is_resident(0):
-                base.evict(0)
-            base.infer_cold(plan, 0, ids, out, pool, secondaries=sec)
-        times = []
-        for _ in range(6):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            if base.is_resident(0):
-                base.evict(0)
-            torch.cuda.synchronize()
-            e0.record()
-            base.infer_cold(plan, 0, ids, out, pool, secondaries=sec)
-            e1.record()
-            torch.cuda.synchronize()
-            times.append(e0.elapsed_time(e1))
-        cold_ns = int(np.median(times[1:]) * 1e6)
-        wt = []
-        for _ in range(6):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            base.infer_warm(0, ids, out, pool)
-            e1.record()
-            torch.cuda.synchronize()
-            wt.append(e0.elapsed_time(e1))
-        warm_ns = int(np.median(wt[1:]) * 1e6)
-        base.evict(0)
-        resident = int(sum(b for b, mt in zip(base.unit_bytes(), plan.method) if mt == dp.LOAD))
-        kw = dict(ngpu=a.gpus, per_gpu_budget_bytes=budget, cold_ns=[cold_ns], warm_ns=[warm_ns],
-                  resident_bytes=[resident], model_of_instance=np.zeros(a.instances, np.int32),
-                  slo_ns=int(a.slo_ms * 1e6), batch=1, seq=a.seq)
+            def cold_run():
+                if base.is_resident(0):
+                    base.evict(0)
+                base.infer_cold(plan, 0, ids, out, pool, secondaries=sec)
+            cold.append(int(dev_ms(cold_run) * 1e6))
+            warm.append(int(dev_ms(lambda: base.infer_warm(0, ids, out, pool)) * 1e6))
+            base.evict(0)
+            plans.append(plan)
+            resident.append(int(sum(b for b, mt in zip(base.unit_bytes(), plan.method) if mt == dp.LOAD)))
+        kw = dict(ngpu=a.gpus, per_gpu_budget_bytes=budget, cold_ns=cold, warm_ns=warm, resident_bytes=resident,
+                  model_of_instance=moi, slo_ns=int(a.slo_ms * 1e6), batch=1,
+                  seq=max(s for _, s, _ in mix), seq_of_model=[s for _, s, _ in mix])
         dry = dp.serve_run(arr, inst, dry_run=True, **kw)
-        live = dp.serve_run(arr, inst, dry_run=False, ctx=ctx, models=insts, plans=[plan] * a.instances, **kw)
-        for i in insts:
+        live = dp.serve_run(arr, inst, dry_run=False, ctx=ctx, models=insts,
+                            plans=[plans[moi[i]] for i in range(a.instances)], **kw)
+        for i in insts + bases:
             for g in range(a.gpus):
                 if i.is_resident(g):
                     i.evict(g)
@@ -96,9 +102,11 @@ def main():
                     "goodput": round(float(np.mean(lat <= a.slo_ms)), 4),
                     "cold_rate": round(float(np.mean(r["cold"])), 4),
                     "throughput_rps": round(len(lat) / ((r["finish_ns"].max() - arr.min()) / 1e9), 1)}
-        report["modes"][mode] = {"cold_ms": cold_ns / 1e6, "warm_ms": warm_ns / 1e6, "resident_mb": resident / 2**20,
-                                 "instances_fit_per_gpu": budget // resident, "live": summarize(live),
-                                 "replay": summarize(dry)}
+        report["modes"][mode] = {
+            "per_model": {mix[mi][0]: {"cold_ms": cold[mi] / 1e6, "warm_ms": warm[mi] / 1e6,
+                                       "resident_mb": round(resident[mi] / 2 ** 20, 1),
+                                       "dha_units": int(plans[mi].method.sum())} for mi in range(len(mix))},
+            "live": summarize(live), "replay": summarize(dry)}
     print(json.dumps(report))
 
 
