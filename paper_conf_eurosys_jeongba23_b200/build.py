@@ -16,7 +16,9 @@ LIB = os.path.join(HERE, "libdeepplan.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
-         "-I" + os.path.join(ROOT, "include"), "-DDP_BUILD"]
+         "-I" + os.path.join(ROOT, "include"), "-DDP_BUILD"] + os.environ.get("DP_NVCC_EXTRA", "").split()
+if os.environ.get("DP_NVCC_EXTRA"):  # instrumented builds (e.g. -DDP_GEMM_TRACE) keep their own objects
+    BUILD += "_" + "".join(c for c in os.environ["DP_NVCC_EXTRA"] if c.isalnum())
 
 
 def _sources():
@@ -47,7 +49,10 @@ def build(verbose: bool = False) -> str:
     srcs = _sources()
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose), srcs))
-    if os.path.exists(LIB) and os.path.getmtime(LIB) >= max(os.path.getmtime(o) for o in objs):
+    stamp = os.path.join(BUILD, "..", "flavor")
+    flavor = os.environ.get("DP_NVCC_EXTRA", "")
+    same = os.path.exists(stamp) and open(stamp).read() == flavor
+    if same and os.path.exists(LIB) and os.path.getmtime(LIB) >= max(os.path.getmtime(o) for o in objs):
         return LIB
     cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-lcudart", "-ldl", "-lpthread"]
     if verbose:
@@ -55,6 +60,8 @@ def build(verbose: bool = False) -> str:
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
+    with open(stamp, "w") as f:
+        f.write(flavor)
     return LIB
 
 

@@ -29,6 +29,7 @@
 #include <cstdint>
 #include <cstring>
 #include <cstdlib>
+#include <algorithm>
 #include <mutex>
 
 #include "common.h"
@@ -143,10 +144,36 @@ struct GemmGroup {
   long long ycol[3];
 };
 
+#ifdef DP_GEMM_TRACE
+// phase timestamps (globaltimer, ns) per CTA: entry, setup done, after grid-dependency wait,
+// first stage landed (MMA issuer), all MMAs done, partial/tile in smem, end; [7] = SM id
+__device__ unsigned long long g_gemm_trace[4096][8];
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TRACE(i)                                                                                  \
+  do {                                                                                            \
+    const int b_ = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;                \
+    if (b_ < 4096) g_gemm_trace[b_][i] = gtime();                                                 \
+  } while (0)
+#else
+#define TRACE(i) \
+  do {           \
+  } while (0)
+#endif
+
+// Split-K: blockIdx.z = group * splits + split; each split accumulates its K range in TMEM,
+// writes the fp32 tile to a workspace slot and bumps the tile's counter; the LAST split to
+// arrive sums the slots in split order 0..splits-1 (deterministic whichever CTA is last),
+// resets the counter and runs the epilogue.  Spreads a weight tile's bytes over `splits`
+// SMs: at the hot path's 128-token shapes a CTA's time is set by the bytes it ingests.
 template <class T, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
-                   const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io) {
+                   const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io, int splits,
+                   float* __restrict__ ws, int* __restrict__ cnt) {
   constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
@@ -162,12 +189,16 @@ __global__ void __launch_bounds__(128, 1)
   __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], done_bar;
   __shared__ uint32_t tmem_base_sh;
 
+  TRACE(0);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n0 = blockIdx.x * BM, m0 = blockIdx.y * BN;
-  const CUtensorMap* tmW = &grp.w[blockIdx.z];
-  const T* bias = static_cast<const T*>(grp.bias[blockIdx.z]);
-  const long long ycol = grp.ycol[blockIdx.z];
-  const int num_kb = K / BK;
+  const int grp_i = blockIdx.z / splits, sp = blockIdx.z - grp_i * splits;
+  const CUtensorMap* tmW = &grp.w[grp_i];
+  const T* bias = static_cast<const T*>(grp.bias[grp_i]);
+  const long long ycol = grp.ycol[grp_i];
+  const int kb_all = K / BK;
+  const int kb_lo = sp * kb_all / splits;
+  const int num_kb = (sp + 1) * kb_all / splits - kb_lo;  // >= 1 (splits <= kb_all)
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmW)) : "memory");
@@ -197,10 +228,12 @@ __global__ void __launch_bounds__(128, 1)
   if (warp == 0 && lane == 0) {
     for (int kb = 0; kb < pre; ++kb) {
       mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
-      tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, kb * BK, n0);
+      tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb_lo + kb) * BK, n0);
     }
   }
+  TRACE(1);
   pdl_wait();
+  TRACE(2);
 
   if (warp == 0 && lane == 0) {
     // TMA producer
@@ -211,15 +244,16 @@ __global__ void __launch_bounds__(128, 1)
       if (kb >= pre) {
         mbar_wait(&empty_bar[s], ((kb / STAGES) - 1) & 1);
         mbar_expect_tx(&full_bar[s], STAGE_BYTES);
-        tma_load_2d(tmW, &full_bar[s], a, kb * BK, n0);
+        tma_load_2d(tmW, &full_bar[s], a, (kb_lo + kb) * BK, n0);
       }
-      tma_load_2d(&tmX, &full_bar[s], b, kb * BK, m0);
+      tma_load_2d(&tmX, &full_bar[s], b, (kb_lo + kb) * BK, m0);
     }
   } else if (warp == 1 && lane == 0) {
     // MMA issuer
     for (int kb = 0; kb < num_kb; ++kb) {
       const int s = kb % STAGES;
       mbar_wait(&full_bar[s], (kb / STAGES) & 1);
+      if (kb == 0) TRACE(3);
       asm volatile("tcgen05.fence::after_thread_sync;");
       const uint8_t* a = smem + s * STAGE_BYTES;
       const uint8_t* b = a + A_BYTES;
@@ -234,6 +268,7 @@ __global__ void __launch_bounds__(128, 1)
   __syncwarp();
 
   mbar_wait(&done_bar, 0);
+  if (threadIdx.x == 0) TRACE(4);
   asm volatile("tcgen05.fence::after_thread_sync;");
   // 1) TMEM -> shared memory (the ring is free once the MMAs are done): the fp32 tile,
   //    [128 W rows][BN tokens] with an odd row stride
@@ -247,6 +282,45 @@ __global__ void __launch_bounds__(128, 1)
     for (int j = 0; j < 16; ++j) tile[row * PROW + c0 + j] = __uint_as_float(v[j]);
   }
   __syncthreads();
+  if (splits > 1) {
+    // 1b) split-K fixup (see above): publish this split's tile, count arrivals
+    __shared__ int last_sh;
+    const int tile_id = (grp_i * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
+    float* slots = ws + (size_t)tile_id * splits * (BM * BN);
+    float* mine = slots + (size_t)sp * (BM * BN);
+    for (int i = threadIdx.x; i < BM * BN / 4; i += 128) {
+      const int r = (4 * i) / BN, c = (4 * i) % BN;
+      reinterpret_cast<float4*>(mine)[i] =
+          make_float4(tile[r * PROW + c], tile[r * PROW + c + 1], tile[r * PROW + c + 2], tile[r * PROW + c + 3]);
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) last_sh = atomicAdd(&cnt[tile_id], 1) == splits - 1;
+    __syncthreads();
+    if (!last_sh) {
+      if (threadIdx.x == 0) {
+        TRACE(5);
+        TRACE(6);
+      }
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      __syncthreads();
+      if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_d), "r"(TMEM_COLS));
+      return;
+    }
+    __threadfence();
+    for (int i = threadIdx.x; i < BM * BN / 4; i += 128) {
+      float4 a = __ldcg(reinterpret_cast<const float4*>(slots) + i);
+      for (int p = 1; p < splits; ++p) {
+        const float4 b = __ldcg(reinterpret_cast<const float4*>(slots + (size_t)p * (BM * BN)) + i);
+        a.x += b.x, a.y += b.y, a.z += b.z, a.w += b.w;
+      }
+      const int r = (4 * i) / BN, c = (4 * i) % BN;
+      tile[r * PROW + c] = a.x, tile[r * PROW + c + 1] = a.y, tile[r * PROW + c + 2] = a.z, tile[r * PROW + c + 3] = a.w;
+    }
+    if (threadIdx.x == 0) cnt[tile_id] = 0;  // ready for the next launch
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) TRACE(5);
   // 2) out[m][n0 .. n0+127] for every token m: thread t owns 8 consecutive W rows
   //    (n = n0 + 8*(t%16) ..+7) of token m = t/16 + 8*pass -> one 16-byte store (and one
   //    16-byte residual load) per 8 outputs
@@ -275,6 +349,15 @@ __global__ void __launch_bounds__(128, 1)
       store8<T>(Y, m * ldy + n + ycol, acc, out32);
     }
   }
+#ifdef DP_GEMM_TRACE
+  if (threadIdx.x == 0) {
+    TRACE(6);
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    const int b_ = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
+    if (b_ < 4096) g_gemm_trace[b_][7] = smid;
+  }
+#endif
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (warp == 1) {
@@ -312,9 +395,38 @@ CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int b
   return m;
 }
 
+// Split-K workspace, one per device: fp32 tile slots + per-tile arrival counters (zeroed
+// once; the last split of every tile resets its counter).  Kernels on one device use it in
+// stream order (the engine runs a forward's kernels on one stream; PDL successors touch it
+// only after griddepcontrol.wait, i.e. after the previous GEMM completed).
+constexpr size_t SPLIT_WS_BYTES = size_t(32) << 20;
+constexpr int SPLIT_MAX_TILES = 16384;
+struct SplitWs {
+  float* ws = nullptr;
+  int* cnt = nullptr;
+};
+SplitWs& split_ws(int dev) {
+  static SplitWs w[64];
+  return w[dev];
+}
+std::mutex split_mu;
+
+SplitWs& split_ws_ready(cudaStream_t s) {
+  int dev;
+  DP_CUDA(cudaGetDevice(&dev));
+  SplitWs& w = split_ws(dev);
+  if (w.ws) return w;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  DP_CUDA(cudaStreamIsCapturing(s, &cs));
+  DP_CHECK(cs == cudaStreamCaptureStatusNone, DP_ERR_STATE, "split-K workspace must be prepared before capture");
+  gemm_prepare(dev);
+  return w;
+}
+
 template <class T, int BN>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
-         const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
+         const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
+         cudaStream_t s) {
   constexpr size_t smem = size_t(stages_for<BN>()) * (BM * BK * 2 + BN * BK * 2) + 1024;
   static_assert(size_t(BM) * (BN + 1) * 4 + 1024 <= smem, "fp32 tile must fit the ring");
   static bool attr = false;
@@ -331,24 +443,53 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
     g.ycol[i] = ycol ? ycol[i] : 0;
   }
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
-  launch_kernel(gemm_tc_kernel<T, BN>, dim3(N / BM, (M + BN - 1) / BN, ngroups), dim3(128), smem, s, g, mx, res, ldr,
-                y, ldy, M, N, K, act, io);
+  const int mt = (M + BN - 1) / BN;
+  float* ws = nullptr;
+  int* cnt = nullptr;
+  if (splits > 1) {
+    const size_t tiles = size_t(N / BM) * mt * ngroups;
+    if (tiles * splits * BM * BN * 4 > SPLIT_WS_BYTES || tiles > (size_t)SPLIT_MAX_TILES) splits = 1;
+  }
+  if (splits > 1) {
+    SplitWs& sw = split_ws_ready(s);
+    ws = sw.ws;
+    cnt = sw.cnt;
+  }
+  launch_kernel(gemm_tc_kernel<T, BN>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem, s, g, mx, res, ldr, y,
+                ldy, M, N, K, act, io, splits, ws, cnt);
 }
 
 template <class T>
 void dispatch(int bn, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
               const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io,
-              cudaStream_t s) {
+              int sp, cudaStream_t s) {
   switch (bn) {
-    case 32: run<T, 32>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 64: run<T, 64>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 128: run<T, 128>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
-    case 256: run<T, 256>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s); break;
+    case 32: run<T, 32>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
+    case 64: run<T, 64>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
+    case 128: run<T, 128>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
+    case 256: run<T, 256>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
     default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
   }
 }
 
 }  // namespace
+
+void gemm_prepare(int dev) {
+  std::lock_guard<std::mutex> lk(split_mu);
+  SplitWs& w = split_ws(dev);
+  if (w.ws) return;
+  int cur;
+  DP_CUDA(cudaGetDevice(&cur));
+  DP_CUDA(cudaSetDevice(dev));
+  void *a = nullptr, *b = nullptr;
+  if (cudaMalloc(&a, SPLIT_WS_BYTES) != cudaSuccess || cudaMalloc(&b, SPLIT_MAX_TILES * sizeof(int)) != cudaSuccess)
+    fail(DP_ERR_OOM, "split-K workspace cudaMalloc failed");
+  DP_CUDA(cudaMemset(b, 0, SPLIT_MAX_TILES * sizeof(int)));
+  DP_CUDA(cudaDeviceSynchronize());
+  w.ws = static_cast<float*>(a);
+  w.cnt = static_cast<int*>(b);
+  DP_CUDA(cudaSetDevice(cur));
+}
 
 bool gemm_tc_supported(int N, int K) { return N > 0 && K > 0 && N % BM == 0 && K % BK == 0; }
 
@@ -361,6 +502,14 @@ static int pick_bn(int M, int N) {
     if (M >= bn && ntile * ((M + bn - 1) / bn) >= 96) return bn;
   }
   return 32;
+}
+
+// Split-K factor: enough K splits to put ~one CTA on every SM, each with >= 2 k-blocks.
+static int pick_split(int M, int N, int K, int bn) {
+  const int tiles = (N / BM) * ((M + bn - 1) / bn);
+  int sp = 148 / std::max(1, tiles);
+  sp = std::min(sp, (K / BK) / 2);
+  return std::max(1, sp);
 }
 
 void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
@@ -377,10 +526,13 @@ void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const 
   // tuning override for experiments (DP_GEMM_BN), read once
   static const int env_bn = getenv("DP_GEMM_BN") ? atoi(getenv("DP_GEMM_BN")) : 0;
   const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : pick_bn(M, N * ngroups));
+  static const int env_sp = getenv("DP_GEMM_SPLIT") ? atoi(getenv("DP_GEMM_SPLIT")) : 0;
+  int sp = env_sp > 0 ? env_sp : pick_split(M, N * ngroups, K, bn);
+  sp = std::max(1, std::min(sp, K / BK));
   if (dtype == DP_BF16)
-    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s);
+    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
   else
-    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, s);
+    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
 }
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
@@ -389,3 +541,10 @@ void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void
 }
 
 }  // namespace dp
+
+#ifdef DP_GEMM_TRACE
+extern "C" __attribute__((visibility("default"))) int dp_debug_gemm_trace(void* host, int nblocks) {
+  if (nblocks > 4096) nblocks = 4096;
+  return (int)cudaMemcpyFromSymbol(host, dp::g_gemm_trace, size_t(nblocks) * 8 * sizeof(unsigned long long));
+}
+#endif

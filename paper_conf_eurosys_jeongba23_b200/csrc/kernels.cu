@@ -369,6 +369,7 @@ static void skinny_t(const void* x, int ldx, const void* w, const void* bias, co
 template <class T>
 void skinny_mma_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy,
                   int M, int N, int K, int act, int io, cudaStream_t s);
+int skinny_cluster(int K);
 
 // M <= 16 tokens (e.g. the pooler): warp-shuffle dot products; more tokens: the same one-pass
 // weight staging with the per-CTA products on mma.sync (the link stays the bound).
@@ -376,9 +377,9 @@ void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, cons
                           int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   DP_CHECK(K % 8 == 0 && K > 0 && N > 0, DP_ERR_INVALID, "skinny linear needs K % 8 == 0");
   if (M <= 0) return;
-  const bool mma = M > 16 && N % 16 == 0 && K % 16 == 0 && ldx % 8 == 0 && ((uintptr_t)x % 16) == 0;
+  const bool mma = M > 16 && N % 16 == 0 && K % 16 == 0 && ldx % 8 == 0 && ((uintptr_t)x % 16) == 0 &&
+                   skinny_cluster(K) > 0;
   if (mma) {
-    DP_CHECK((size_t(16) * (K + 8) + 128 * 136) * 2 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");
     if (dtype == DP_BF16)
       skinny_mma_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
     else
@@ -595,108 +596,198 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
 }
 
 // -------------------------------------------------------------------------------------
-// K3 (M > 16 tokens): the DHA skinny linear with its products on mma.sync.  Each CTA owns
-// 16 W rows: it streams them from (host) memory once -- coalesced 16-byte loads, all issued
-// before the grid-dependency wait -- into padded shared memory (row stride K+8 elements, so
-// ldmatrix is conflict-free); then each warp takes groups of 8 tokens and runs
-// m16n8k16 MMAs (A = the 16 staged W rows via ldmatrix, B = X^T fragments straight from the
-// L2-resident activations, fp32 accumulate).  Host-link bytes = N*K*2 + N*2 exactly.
+// K3 (M > 16 tokens): the DHA skinny linear with its products on mma.sync.
+//
+// The cost is set by the host link: one host round trip (~7 us measured on this box,
+// profiles/r01_linkprobe.json zc_gather) plus W bytes at ~51 GB/s.  Everything else must
+// hide under that.  Each CTA owns 16 W rows x a K slice KS = K / cs (cs = cluster size,
+// chosen so KS <= 768):
+//   1. its whole W slice (<= 6 x 16-byte loads per thread, coalesced) is issued into
+//      registers before the grid-dependency wait -- weights never depend on the previous
+//      kernel, so under PDL these host reads overlap the predecessor's tail;
+//   2. right after the wait, the first X chunks ([128 tokens][64 k], from L2) go into a
+//      4-stage cp.async ring, so X staging overlaps the W round trip;
+//   3. the registers land in padded shared memory ([16][KS+8], conflict-free ldmatrix);
+//   4. per chunk: ldmatrix A = W rows, B = X rows, two m16n8k16 per warp (16 tokens).
+//   5. cs > 1: the fp32 partial tiles are summed across the cluster through distributed
+//      shared memory in rank order 0..cs-1 (deterministic; each rank finishes a share of
+//      the tokens), then bias / activation / residual.
+// Host-link bytes = N*K*2 + N*2 exactly; the kernel is the same whether W lives in host or
+// device memory, so DHA and loaded execution of a layer are bit-identical.
 // -------------------------------------------------------------------------------------
-constexpr int SK_TOK = 128;  // tokens per pass (16 groups of 8: two per warp)
-constexpr int SK_KCH = 128;  // K elements of X staged per chunk
+constexpr int SK_TOK = 128;  // tokens per block (8 warps x 16)
+constexpr int SK_KCH = 64;   // K elements per X chunk
+constexpr int SK_STG = 4;    // cp.async ring depth
+constexpr int SK_XP = SK_KCH + 8;
+constexpr int SK_WREG = 6;   // W vectors per thread: 16 rows x 768 / 8 / 256
 
-// X fragments for two token groups at once (ldmatrix.x4 over 16 staged X rows: tokens
-// 0-7 / 8-15 x k 0-7 / 8-15), then one m16n8k16 per group against the shared W fragment.
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ float ld_dsmem_f32(const float* p, uint32_t rank) {
+  uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(p)), ra;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(rank));
+  float v;
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(ra) : "memory");
+  return v;
+}
+
 template <class T>
 __global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X, int ldx, const T* W,
                                                          const T* bias, const void* res, int ldr, void* Y, int ldy,
-                                                         int M, int N, int K, int act, int io) {
+                                                         int M, int N, int K, int KS, int cs, int act, int io) {
   extern __shared__ __align__(16) uint8_t smem_sk[];
-  const int KP = K + 8;
-  T* sw16 = reinterpret_cast<T*>(smem_sk);        // W slice [16][K + 8]
-  T* sx = sw16 + 16 * KP;                          // X chunk [SK_TOK][SK_KCH + 8]
-  constexpr int XP = SK_KCH + 8;
+  const int KP = KS + 8;
+  T* sw = reinterpret_cast<T*>(smem_sk);  // W slice [16][KS + 8]
+  T* sx = sw + 16 * KP;                   // X ring [SK_STG][SK_TOK][SK_XP]
+  float* red = reinterpret_cast<float*>(sx);  // cs > 1: partial tile [SK_TOK][16], aliases the ring
   pdl_trigger();
-  const int kv = K / 8;
-  const int n0 = blockIdx.x * 16;
-  // every PCIe read of this CTA's 16 W rows is issued up front -- coalesced 16-byte loads,
-  // up to 8 in flight per thread, before the grid-dependency wait (weights never depend on
-  // the previous kernel).  (cp.async from mapped host memory measured 2x slower.)
-  const uint4* src = reinterpret_cast<const uint4*>(W + (size_t)n0 * K);
-  const int total = 16 * kv;
-  for (int base = threadIdx.x; base < total; base += 8 * 256) {
-    uint4 r[8];
+  const int rank = cs > 1 ? (int)cluster_rank() : 0;
+  const int n0 = (blockIdx.x / cs) * 16;
+  const int k0 = rank * KS;
+  const int kv = KS / 8;
+  // (1) the W slice, all in flight at once
+  uint4 wr[SK_WREG];
 #pragma unroll
-    for (int j = 0; j < 8; ++j)
-      if (base + j * 256 < total) r[j] = ldg16(src + base + j * 256);
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int i = base + j * 256;
-      if (i < total) *reinterpret_cast<uint4*>(&sw16[(i / kv) * KP + (i % kv) * 8]) = r[j];
-    }
+  for (int j = 0; j < SK_WREG; ++j) {
+    const int i = threadIdx.x + j * 256;
+    if (i < 16 * kv) wr[j] = ldg16(W + (size_t)(n0 + i / kv) * K + k0 + (i % kv) * 8);
   }
+  float breg = 0.f;
+  if (bias && threadIdx.x < 16) breg = Cvt<T>::to1(bias[n0 + threadIdx.x]);
   __shared__ float sbias[16];
-  if (threadIdx.x < 16) sbias[threadIdx.x] = bias ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
   pdl_wait();
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int g = lane >> 2, t4 = lane & 3;
-  const T* arow = &sw16[(lane & 15) * KP + (lane >> 4) * 8];  // W fragment rows (k = 0)
-  // X fragment rows for this warp's two groups: tokens 16*warp + (lane&7) + 8*(lane>>4),
-  // k half (lane>>3)&1
-  const T* brow = &sx[(16 * warp + (lane & 7) + ((lane >> 4) << 3)) * XP + ((lane >> 3) & 1) * 8];
+  const int nch = KS / SK_KCH + (KS % SK_KCH ? 1 : 0);
+  auto stage = [&](int t0, int nt, int c) {  // X chunk c of token block t0 -> ring slot c % SK_STG
+    T* dst = sx + (c % SK_STG) * SK_TOK * SK_XP;
+    const int kc = k0 + c * SK_KCH, kw = min(SK_KCH, KS - c * SK_KCH);
+    for (int i = threadIdx.x; i < SK_TOK * (SK_KCH / 8); i += 256) {
+      const int r = i / (SK_KCH / 8), q = i % (SK_KCH / 8);
+      if (r < nt && q * 8 < kw) cp_async16(dst + r * SK_XP + q * 8, X + (size_t)(t0 + r) * ldx + kc + q * 8);
+    }
+  };
+  const T* arow = &sw[(lane & 15) * KP + (lane >> 4) * 8];
+  const int brow_off = (16 * warp + (lane & 7) + ((lane >> 4) << 3)) * SK_XP + ((lane >> 3) & 1) * 8;
   for (int t0 = 0; t0 < M; t0 += SK_TOK) {
     const int nt = min(SK_TOK, M - t0);
-    float acc[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
-    for (int kc = 0; kc < K; kc += SK_KCH) {
-      const int kw = min(SK_KCH, K - kc);  // K % 16 == 0, so kw is a multiple of 16
-      __syncthreads();                      // previous chunk consumed (and W staged, first time)
-      for (int i = threadIdx.x; i < SK_TOK * (SK_KCH / 8); i += 256) {
-        const int r = i / (SK_KCH / 8), c = i - r * (SK_KCH / 8);
-        uint4 v = make_uint4(0, 0, 0, 0);
-        if (r < nt && c * 8 < kw) v = *reinterpret_cast<const uint4*>(X + (size_t)(t0 + r) * ldx + kc + c * 8);
-        *reinterpret_cast<uint4*>(&sx[r * XP + c * 8]) = v;
+    // (2) prefetch the first chunks
+#pragma unroll
+    for (int c = 0; c < SK_STG - 1; ++c) {
+      if (c < nch) stage(t0, nt, c);
+      cp_async_commit();
+    }
+    if (t0 == 0) {  // (3) W registers -> shared (waits for the host round trip)
+#pragma unroll
+      for (int j = 0; j < SK_WREG; ++j) {
+        const int i = threadIdx.x + j * 256;
+        if (i < 16 * kv) *reinterpret_cast<uint4*>(&sw[(i / kv) * KP + (i % kv) * 8]) = wr[j];
       }
-      __syncthreads();
+      if (threadIdx.x < 16) sbias[threadIdx.x] = breg;
+    }
+    float acc[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+    // (4) the ring
+    for (int c = 0; c < nch; ++c) {
+      cp_async_wait<SK_STG - 2>();
+      __syncthreads();  // chunk c visible to all; slot (c-1) % SK_STG free
+      if (c + SK_STG - 1 < nch) stage(t0, nt, c + SK_STG - 1);
+      cp_async_commit();
       if (16 * warp < nt) {
-#pragma unroll 4
-        for (int ks = 0; ks < kw; ks += 16) {
-          uint32_t a[4], b[4];
-          ldsm_x4(a, arow + kc + ks);
-          ldsm_x4(b, brow + ks);
-          MmaOp<T>::mma(acc[0], a, b);
-          MmaOp<T>::mma(acc[1], a, b + 2);
+        const T* xs = sx + (c % SK_STG) * SK_TOK * SK_XP + brow_off;
+        const int kw = min(SK_KCH, KS - c * SK_KCH);
+#pragma unroll
+        for (int ks = 0; ks < SK_KCH; ks += 16) {
+          if (ks < kw) {
+            uint32_t a[4], b[4];
+            ldsm_x4(a, arow + c * SK_KCH + ks);
+            ldsm_x4(b, xs + ks);
+            MmaOp<T>::mma(acc[0], a, b);
+            MmaOp<T>::mma(acc[1], a, b + 2);
+          }
         }
       }
     }
+    cp_async_wait<0>();
+    __syncthreads();  // every warp is done with the ring (it is reused below / next block)
     // acc[q]: c0,c1 -> W row g, tokens 2*t4, 2*t4+1 of group q; c2,c3 -> W row g+8
+    if (cs == 1) {
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {
+      for (int q = 0; q < 2; ++q) {
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int r = g + (e >> 1) * 8;
-        const int m = t0 + 16 * warp + 8 * q + 2 * t4 + (e & 1);
-        if (m < M) {
-          const int n = n0 + r;
-          float v = apply_act(acc[q][e] + sbias[r], act);
-          if (res) v += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
-          store1<T>(Y, (size_t)m * ldy + n, v, io & IO_OUT_F32);
+        for (int e = 0; e < 4; ++e) {
+          const int r = g + (e >> 1) * 8;
+          const int m = t0 + 16 * warp + 8 * q + 2 * t4 + (e & 1);
+          if (m < M) {
+            const int n = n0 + r;
+            float v = apply_act(acc[q][e] + sbias[r], act);
+            if (res) v += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
+            store1<T>(Y, (size_t)m * ldy + n, v, io & IO_OUT_F32);
+          }
         }
       }
+    } else {
+      // (5) deterministic cluster reduction over distributed shared memory
+#pragma unroll
+      for (int q = 0; q < 2; ++q)
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          red[(16 * warp + 8 * q + 2 * t4 + (e & 1)) * 16 + g + (e >> 1) * 8] = acc[q][e];
+      cluster_sync_all();
+      const int per = ((SK_TOK + cs - 1) / cs) * 16;  // elements (token-major, 16 rows each) per rank
+      const int lo = rank * per, hi = min(SK_TOK * 16, lo + per);
+      for (int i = lo + threadIdx.x; i < hi; i += 256) {
+        const int tok = i >> 4, r = i & 15, m = t0 + tok;
+        if (m >= M) continue;
+        float v = 0.f;
+        for (int s = 0; s < cs; ++s) v += ld_dsmem_f32(red + i, (uint32_t)s);
+        const int n = n0 + r;
+        v = apply_act(v + sbias[r], act);
+        if (res) v += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
+        store1<T>(Y, (size_t)m * ldy + n, v, io & IO_OUT_F32);
+      }
+      cluster_sync_all();  // peers have read this CTA's partials before the ring is reused / exit
     }
   }
+}
+
+// the K-slice split: smallest cluster size with a slice of at most 768 elements
+int skinny_cluster(int K) {
+  for (int cs = 1; cs <= 8; ++cs)
+    if (K % (16 * cs) == 0 && K / cs <= 768) return cs;
+  return 0;
 }
 
 template <class T>
 void skinny_mma_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy,
                   int M, int N, int K, int act, int io, cudaStream_t s) {
-  const size_t sm = (size_t(16) * (K + 8) + size_t(SK_TOK) * (SK_KCH + 8)) * sizeof(T);
+  const int cs = skinny_cluster(K);
+  DP_CHECK(cs > 0, DP_ERR_UNSUPPORTED, "skinny linear: K must split into <= 8 slices of <= 768 (multiples of 16)");
+  const int KS = K / cs;
+  const size_t sm = (size_t(16) * (KS + 8) + size_t(SK_STG) * SK_TOK * SK_XP) * sizeof(T);
   static bool attr_set = false;  // one per template instantiation
   if (!attr_set) {
-    DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+    DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024));
+    DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     attr_set = true;
   }
-  launch_kernel(skinny_mma_kernel<T>, dim3(N / 16), dim3(256), sm, s, (const T*)x, ldx, (const T*)w, (const T*)bias,
-                res, ldr, y, ldy, M, N, K, act, io);
+  launch_kernel_cluster(skinny_mma_kernel<T>, dim3((N / 16) * cs), dim3(256), sm, cs, s, (const T*)x, ldx,
+                        (const T*)w, (const T*)bias, res, ldr, y, ldy, M, N, K, KS, cs, act, io);
 }
 
 // -------------------------------------------------------------------------------------

@@ -147,6 +147,32 @@ def test_linear_skinny_dha_parity_and_bit_identity(M, N, K, dtype):
     hb.free()
 
 
+@pytest.mark.parametrize("M,N,K", [(300, 256, 1536), (129, 64, 2304), (257, 128, 6144), (45, 32, 48)])
+def test_linear_skinny_split_k_cluster_residual(M, N, K):
+    """K split over a thread-block cluster (cs = 2, 3, 8) and one CTA (K = 48, a ragged last
+    chunk), ragged token blocks, fp32 residual read and written in place (the GPT-2 stream)."""
+    dtype = "fp16"
+    rng = np.random.default_rng(M + N + K)
+    x = synth.round_to(rng.standard_normal((M, K)).astype(np.float32), dtype)
+    wt = synth.round_to((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32), dtype)
+    b = synth.round_to((0.1 * rng.standard_normal(N)).astype(np.float32), dtype)
+    r = rng.standard_normal((M, N))
+    X, W, Bt = (to_t(a, dtype) for a in (x, wt, b))
+    hw = HostBuf(wt)
+    outs = []
+    for wptr in (W, hw.ptr):
+        Rf = torch.from_numpy(r.astype(np.float32)).cuda()
+        dp().linear(X, K, wptr, Bt, Rf, N, Rf, N, M, N, K, act="gelu_erf", path=1, dtype=dtype, io=3)
+        torch.cuda.synchronize()
+        outs.append(Rf)
+    assert torch.equal(outs[0], outs[1])
+    x64, w64, b64 = (synth.storage_to_f64(a, dtype) for a in (x, wt, b))
+    ref = F.linear(x64, w64, b64, "gelu_erf", r.astype(np.float32).astype(np.float64))
+    err = np.abs(outs[0].double().cpu().numpy() - ref).max()
+    assert err <= 1e-4 * math.sqrt(K) * (1 + np.abs(ref).max()), err
+    hw.free()
+
+
 def test_linear_strided_output_and_input():
     """q/k/v write into column blocks of the [T, 3H] buffer; the pooler reads every S-th row."""
     dtype = "fp16"

@@ -1,0 +1,39 @@
+"""Per-CTA phase timeline of the tcgen05 GEMM (needs the instrumented build:
+DP_NVCC_EXTRA=-DDP_GEMM_TRACE python paper_conf_eurosys_jeongba23_b200/build.py).
+
+Phases (globaltimer ns, relative to the earliest CTA entry): 0 entry, 1 setup done (barriers,
+TMEM), 2 after griddepcontrol.wait, 3 first stage landed, 4 all MMAs done, 5 tile ready for the
+epilogue (after the split-K fixup), 6 end.  python tools/gemm_trace.py M N K [reps]"""
+import ctypes
+import json
+import math
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import paper_conf_eurosys_jeongba23_b200 as dp
+from paper_conf_eurosys_jeongba23_b200 import _lib
+
+M, N, K = (int(v) for v in sys.argv[1:4])
+reps = int(sys.argv[4]) if len(sys.argv) > 4 else 20
+x = torch.randn(M, K, device="cuda").half()
+w = (torch.randn(N, K, device="cuda") / math.sqrt(K)).half()
+y = torch.empty(M, N, device="cuda").half()
+for _ in range(reps):
+    dp.linear(x, K, w, None, None, 0, y, N, M, N, K, path=0)
+torch.cuda.synchronize()
+buf = np.zeros((4096, 8), dtype=np.uint64)
+assert _lib.lib.dp_debug_gemm_trace(buf.ctypes.data_as(ctypes.c_void_p), 4096) == 0
+rows = buf[(buf[:, 0] > 0) & (buf[:, 6] > 0)]
+t0 = rows[:, 0].min()
+rel = (rows[:, :7].astype(np.int64) - int(t0)) / 1e3  # us
+names = ["entry", "setup", "pdl_wait", "first_stage", "mma_done", "tile_ready", "end"]
+out = {"shape": [M, N, K], "ctas": int(len(rows)), "env": {k: os.environ.get(k) for k in ("DP_GEMM_BN", "DP_GEMM_SPLIT")}}
+for i, n in enumerate(names):
+    col = rel[:, i]
+    out[n] = {"min": round(float(col.min()), 3), "med": round(float(np.median(col)), 3), "max": round(float(col.max()), 3)}
+out["per_cta_active_us_med"] = round(float(np.median(rel[:, 6] - rel[:, 0])), 3)
+print(json.dumps(out))

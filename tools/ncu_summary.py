@@ -46,7 +46,9 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "sm__throughput.avg.pct_of_peak_sustained_elapsed", "sm__warps_active.avg.pct_of_peak_sustained_active",
         "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
         "launch__shared_mem_per_block_dynamic", "launch__cluster_dim_z", "sm__cycles_elapsed.avg.per_second",
-        "smsp__average_warp_latency_issue_stalled_long_scoreboard"]
+        "smsp__average_warp_latency_issue_stalled_long_scoreboard", "pcie__read_bytes.sum.per_second",
+        "syslts__t_sectors_srcunit_tex_aperture_sysmem_op_read_lookup_miss.sum",
+        "l1tex__m_xbar2l1tex_read_bytes.sum"]
 
 
 def report(path):
@@ -64,8 +66,54 @@ def report(path):
     return out
 
 
+# algorithmic bytes / flops of the kbench shapes captured by tools/evidence.sh
+ALGO = {
+    "gemm_q": {"shape": "M128 N768 K768", "bytes": 2 * (768 * 768 + 128 * 768 + 128 * 768), "flops": 2 * 128 * 768 * 768},
+    "gemm_fc1": {"shape": "M128 N3072 K768", "bytes": 2 * (3072 * 768 + 128 * 768 + 128 * 3072),
+                 "flops": 2 * 128 * 3072 * 768},
+    "gemm_fc2": {"shape": "M128 N768 K3072", "bytes": 2 * (768 * 3072 + 128 * 3072 + 128 * 768),
+                 "flops": 2 * 128 * 768 * 3072},
+    "skinny_dha": {"shape": "M128 N768 K768, W in pinned host memory", "host_bytes": 2 * 768 * 768},
+    "embed_dha": {"shape": "S128 H768, tables in pinned host memory", "host_bytes": (2 * 128 + 3) * 768 * 2},
+    "attention": {"shape": "B1 S128 H768 12 heads", "flops": 4 * 128 * 128 * 768},
+    "layernorm": {"shape": "128 x 768", "bytes": 2 * 2 * 128 * 768},
+}
+
+
+def bundle(d, launches_csv, peaks):
+    """profiles/ summary: per-kernel ncu --set full metrics + algorithmic rooflines, and the
+    per-kernel time shares of one bench step from the launch list."""
+    out = {"kernels": {}, "bench_step_launches": launches(launches_csv, 86) if launches_csv else None}
+    for name, algo in ALGO.items():
+        path = f"{d}/full_{name}.ncu-rep"
+        try:
+            r = report(path)[0]
+        except Exception as e:  # noqa: BLE001
+            out["kernels"][name] = {"error": str(e)}
+            continue
+        us = float(r["gpu__time_duration.sum"].split()[0])
+        e = {"ncu": r, "algorithmic": algo, "duration_us": us}
+        if "bytes" in algo:
+            e["hbm_roofline"] = {"achieved_gbs": round(algo["bytes"] / us / 1e3, 1), "peak_gbs": peaks["hbm"],
+                                 "frac": round(algo["bytes"] / us / 1e3 / peaks["hbm"], 4)}
+        if "flops" in algo:
+            e["tensor_roofline"] = {"achieved_tflops": round(algo["flops"] / us / 1e6, 2), "peak_tflops": peaks["tc"],
+                                    "frac": round(algo["flops"] / us / 1e6 / peaks["tc"], 4)}
+        if "host_bytes" in algo:
+            sect = float(r["syslts__t_sectors_srcunit_tex_aperture_sysmem_op_read_lookup_miss.sum"].split()[0])
+            e["host_link"] = {"algorithmic_bytes": algo["host_bytes"], "sysmem_read_bytes": int(sect * 32),
+                              "achieved_gbs": round(algo["host_bytes"] / us / 1e3, 2), "peak_gbs": peaks["h2d"],
+                              "frac": round(algo["host_bytes"] / us / 1e3 / peaks["h2d"], 4)}
+        out["kernels"][name] = e
+    return out
+
+
 if __name__ == "__main__":
-    if sys.argv[1] == "launches":
+    if sys.argv[1] == "bundle":
+        pk = json.load(open("MEASURED_PEAKS.json"))  # driver-measured; fp16 dense peak = bf16's (same rate)
+        peaks = {"hbm": pk["hbm_gbs"], "tc": pk["bf16_tflops"], "h2d": 55.6}  # h2d: profiles/r01_linkprobe.json
+        print(json.dumps(bundle(sys.argv[2], sys.argv[3] if len(sys.argv) > 3 else None, peaks), indent=1))
+    elif sys.argv[1] == "launches":
         last = int(sys.argv[sys.argv.index("--last") + 1]) if "--last" in sys.argv else None
         print(json.dumps(launches(sys.argv[2], last), indent=1))
     else:
