@@ -151,7 +151,9 @@ typedef struct {
   int32_t debug_poison;   /* 1 = fill HBM slots with 0xFF (NaN) on eviction [0] */
   int32_t use_pdl;        /* chain consecutive kernels with programmatic dependent launch:
                              a kernel's weight prefetch overlaps its predecessor [1] */
-  int32_t reserved0;
+  int32_t fuse_ln;        /* 1 = a LayerNorm that follows a resident-weight linear runs in
+                             that GEMM's epilogue (bit-identical results; measured slower on
+                             B200 at 128 tokens: the last CTA's row tail is serial) [0] */
   int64_t tail_bytes;     /* the last DMA piece of a link carries at most this many bytes
                              (a unit suffix), so little compute remains after the last byte
                              lands [2 MiB]; 0 = off */

@@ -58,6 +58,7 @@ struct ForwardArgs {
   int kernels = 0;
   int bn_hint = 0;
   bool pdl = false;  // chain kernels with programmatic dependent launch (opts.use_pdl)
+  bool fuse_ln = false;  // LayerNorm in the preceding GEMM's epilogue (opts.fuse_ln)
 };
 
 void ensure_workspace(dp_model* m, int dev, int64_t tokens);

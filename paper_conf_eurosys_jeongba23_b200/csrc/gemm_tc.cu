@@ -36,6 +36,7 @@
 #include "dtype.cuh"
 #include "kernels.h"
 #include "launch.cuh"
+#include "ln.cuh"
 
 namespace dp {
 
@@ -144,6 +145,20 @@ struct GemmGroup {
   long long ycol[3];
 };
 
+// Optional LayerNorm over complete output rows (K2 + K4 fused; BERT's post-LN after
+// attn-out / fc2, GPT-2's pre-LN after the residual projections): every CTA of an m-tile
+// bumps that tile's counter once its outputs are stored; the LAST one normalises the m-tile's
+// BN rows (z = the stored GEMM output, full N) with the same per-row code as the LayerNorm
+// kernel (ln.cuh), so fused and unfused results are bit-identical.
+struct LnFuse {
+  const void* gamma;  // [N] (T); nullptr = no LayerNorm
+  const void* beta;
+  void* out;          // [M, ldo] (T)
+  int ldo;
+  float eps;
+  int* cnt;           // per m-tile arrival counters, zero between launches (the last CTA resets)
+};
+
 #ifdef DP_GEMM_TRACE
 // phase timestamps (globaltimer, ns) per CTA: entry, setup done, after grid-dependency wait,
 // first stage landed (MMA issuer), all MMAs done, partial/tile in smem, end; [7] = SM id
@@ -164,22 +179,39 @@ __device__ __forceinline__ unsigned long long gtime() {
   } while (0)
 #endif
 
-// Split-K: blockIdx.z = group * splits + split; each split accumulates its K range in TMEM,
-// writes the fp32 tile to a workspace slot and bumps the tile's counter; the LAST split to
-// arrive sums the slots in split order 0..splits-1 (deterministic whichever CTA is last),
-// resets the counter and runs the epilogue.  Spreads a weight tile's bytes over `splits`
-// SMs: at the hot path's 128-token shapes a CTA's time is set by the bytes it ingests.
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t saddr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ float ld_cluster_f32(uint32_t addr) {
+  float v;
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  return v;
+}
+
+// Split-K over a thread-block cluster: blockIdx.z = group * splits + split, and the `splits`
+// CTAs of one output tile form a cluster (1 x 1 x splits).  Each accumulates its K range in
+// TMEM and stages its fp32 tile in its own shared memory; after one cluster barrier rank r
+// finalizes its share of the tile's 8-row groups by summing the `splits` tiles over DSMEM in
+// rank order 0..splits-1 (deterministic), then runs the epilogue.  At the hot path's
+// 128-token shapes a CTA's time is set by the bytes it ingests (~100 GB/s per SM measured,
+// profiles/r01_gemm_trace.jsonl), so spreading a weight tile over `splits` SMs pays.
 template <class T, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
                    const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io, int splits,
-                   float* __restrict__ ws, int* __restrict__ cnt) {
+                   const LnFuse lnf) {
   constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
   constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free TMEM->smem writes)
+  constexpr int RP = BN <= 64 ? BN / 8 : 0;  // residual rows prefetched per thread (single split)
   // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
   constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
                              (uint32_t(BM >> 4) << 24);
@@ -188,6 +220,7 @@ __global__ void __launch_bounds__(128, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], done_bar;
   __shared__ uint32_t tmem_base_sh;
+  __shared__ float sbias[BM];
 
   TRACE(0);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -199,6 +232,8 @@ __global__ void __launch_bounds__(128, 1)
   const int kb_all = K / BK;
   const int kb_lo = sp * kb_all / splits;
   const int num_kb = (sp + 1) * kb_all / splits - kb_lo;  // >= 1 (splits <= kb_all)
+  const int mcount = min(BN, M - m0);
+  const bool res32 = io & IO_RES_F32, out32 = io & IO_OUT_F32;
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmW)) : "memory");
@@ -231,9 +266,24 @@ __global__ void __launch_bounds__(128, 1)
       tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb_lo + kb) * BK, n0);
     }
   }
+  // the bias never depends on the previous kernel either (128 threads = 128 rows of the tile;
+  // read after the W tiles are in flight, visible to the epilogue after its barrier)
+  sbias[threadIdx.x] = bias != nullptr ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
   TRACE(1);
   pdl_wait();
   TRACE(2);
+
+  // epilogue thread mapping (single split): thread t owns 8 consecutive W rows
+  // nl = 8*(t%16) of tokens ml = t/16 + 8*j; their residual is fetched now, under the mainloop
+  const int nl_t = 8 * (threadIdx.x & 15);
+  float rpre[RP > 0 ? RP : 1][8];
+  if (RP > 0 && splits == 1 && res != nullptr) {
+#pragma unroll
+    for (int j = 0; j < RP; ++j) {
+      const int ml = (threadIdx.x >> 4) + 8 * j;
+      if (ml < mcount) load8<T>(res, (size_t)(m0 + ml) * ldr + n0 + nl_t, rpre[j], res32);
+    }
+  }
 
   if (warp == 0 && lane == 0) {
     // TMA producer
@@ -281,73 +331,73 @@ __global__ void __launch_bounds__(128, 1)
 #pragma unroll
     for (int j = 0; j < 16; ++j) tile[row * PROW + c0 + j] = __uint_as_float(v[j]);
   }
-  __syncthreads();
-  if (splits > 1) {
-    // 1b) split-K fixup (see above): publish this split's tile, count arrivals
-    __shared__ int last_sh;
-    const int tile_id = (grp_i * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
-    float* slots = ws + (size_t)tile_id * splits * (BM * BN);
-    float* mine = slots + (size_t)sp * (BM * BN);
-    for (int i = threadIdx.x; i < BM * BN / 4; i += 128) {
-      const int r = (4 * i) / BN, c = (4 * i) % BN;
-      reinterpret_cast<float4*>(mine)[i] =
-          make_float4(tile[r * PROW + c], tile[r * PROW + c + 1], tile[r * PROW + c + 2], tile[r * PROW + c + 3]);
-    }
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) last_sh = atomicAdd(&cnt[tile_id], 1) == splits - 1;
-    __syncthreads();
-    if (!last_sh) {
-      if (threadIdx.x == 0) {
-        TRACE(5);
-        TRACE(6);
-      }
-      asm volatile("tcgen05.fence::before_thread_sync;");
-      __syncthreads();
-      if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_d), "r"(TMEM_COLS));
-      return;
-    }
-    __threadfence();
-    for (int i = threadIdx.x; i < BM * BN / 4; i += 128) {
-      float4 a = __ldcg(reinterpret_cast<const float4*>(slots) + i);
-      for (int p = 1; p < splits; ++p) {
-        const float4 b = __ldcg(reinterpret_cast<const float4*>(slots + (size_t)p * (BM * BN)) + i);
-        a.x += b.x, a.y += b.y, a.z += b.z, a.w += b.w;
-      }
-      const int r = (4 * i) / BN, c = (4 * i) % BN;
-      tile[r * PROW + c] = a.x, tile[r * PROW + c + 1] = a.y, tile[r * PROW + c + 2] = a.z, tile[r * PROW + c + 3] = a.w;
-    }
-    if (threadIdx.x == 0) cnt[tile_id] = 0;  // ready for the next launch
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) TRACE(5);
-  // 2) out[m][n0 .. n0+127] for every token m: thread t owns 8 consecutive W rows
-  //    (n = n0 + 8*(t%16) ..+7) of token m = t/16 + 8*pass -> one 16-byte store (and one
-  //    16-byte residual load) per 8 outputs
-  {
-    const int t = threadIdx.x;
-    const int nl = 8 * (t & 15);
+  // 2) + bias, activation, + residual; one 16-byte store per 8 outputs (8 W rows of a token)
+  auto finish = [&](int nl, int ml, float* acc, const float* r8) {
+    const size_t m = (size_t)(m0 + ml);
     const int n = n0 + nl;
-    const bool nok = n < N;  // N % 128 == 0, so all 8 rows are valid together
-    float bv[8];
 #pragma unroll
-    for (int e = 0; e < 8; ++e) bv[e] = (bias != nullptr && nok) ? Cvt<T>::to1(bias[n + e]) : 0.f;
-    const int mcount = min(BN, M - m0);
-    const bool res32 = io & IO_RES_F32, out32 = io & IO_OUT_F32;
-#pragma unroll 1
-    for (int ml = t >> 4; ml < mcount && nok; ml += 8) {
-      float acc[8];
-#pragma unroll
-      for (int e = 0; e < 8; ++e) acc[e] = apply_act(tile[(nl + e) * PROW + ml] + bv[e], act);
-      const size_t m = (size_t)(m0 + ml);
-      if (res) {
-        float r8[8];
-        load8<T>(res, m * ldr + n, r8, res32);
-#pragma unroll
-        for (int e = 0; e < 8; ++e) acc[e] += r8[e];
+    for (int e = 0; e < 8; ++e) acc[e] = apply_act(acc[e] + sbias[nl + e], act);
+    if (res) {
+      float rl[8];
+      if (r8 == nullptr) {
+        load8<T>(res, m * ldr + n, rl, res32);
+        r8 = rl;
       }
-      store8<T>(Y, m * ldy + n + ycol, acc, out32);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] += r8[e];
     }
+    store8<T>(Y, m * ldy + n + ycol, acc, out32);
+  };
+  if (splits == 1) {
+    __syncthreads();
+    if (threadIdx.x == 0) TRACE(5);
+    if constexpr (RP > 0) {
+#pragma unroll
+      for (int j = 0; j < RP; ++j) {
+        const int ml = (threadIdx.x >> 4) + 8 * j;
+        if (ml < mcount) {
+          float acc[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) acc[e] = tile[(nl_t + e) * PROW + ml];
+          finish(nl_t, ml, acc, res != nullptr ? rpre[j] : nullptr);
+        }
+      }
+    } else {
+      // wide tiles: a rolled loop (an unrolled 32-pass epilogue is instruction-fetch bound)
+#pragma unroll 1
+      for (int ml = threadIdx.x >> 4; ml < mcount; ml += 8) {
+        float acc[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) acc[e] = tile[(nl_t + e) * PROW + ml];
+        finish(nl_t, ml, acc, nullptr);
+      }
+    }
+  } else {
+    // 1b) cluster split-K reduction (see above)
+    cluster_sync_all();
+    if (threadIdx.x == 0) TRACE(5);
+    const uint32_t tile_sa = smem_u32(tile);
+    uint32_t rb[8];
+#pragma unroll
+    for (int p = 0; p < 8; ++p) rb[p] = p < splits ? mapa_u32(tile_sa, (uint32_t)p) : 0u;
+    const int g0 = sp * 16 / splits, g1 = (sp + 1) * 16 / splits;  // this rank's 8-row groups
+    const int units = (g1 - g0) * mcount;
+    for (int u = threadIdx.x; u < units; u += 128) {
+      const int gi = g0 + u / mcount, ml = u - (u / mcount) * mcount;
+      float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+      for (int p = 0; p < 8; ++p) {
+        if (p < splits) {
+          float v[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) v[e] = ld_cluster_f32(rb[p] + (uint32_t)(((8 * gi + e) * PROW + ml) * 4));
+#pragma unroll
+          for (int e = 0; e < 8; ++e) acc[e] += v[e];
+        }
+      }
+      finish(8 * gi, ml, acc, nullptr);
+    }
+    cluster_sync_all();  // every peer has read this CTA's tile
   }
 #ifdef DP_GEMM_TRACE
   if (threadIdx.x == 0) {
@@ -362,6 +412,44 @@ __global__ void __launch_bounds__(128, 1)
   __syncthreads();
   if (warp == 1) {
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_d), "r"(TMEM_COLS));
+  }
+  if (lnf.gamma != nullptr) {
+    // 3) fused LayerNorm of complete rows (see LnFuse)
+    __shared__ int ln_last;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) ln_last = atomicAdd(&lnf.cnt[blockIdx.y], 1) == (int)(gridDim.x * gridDim.z) - 1;
+    __syncthreads();
+    if (ln_last) {
+      __threadfence();
+      // the m-tile's complete rows (written by every CTA of the tile) are staged into shared
+      // memory with cp.async -- all in flight at once, one L2 round trip -- then normalised
+      // row by row from there (the ring is free)
+      const int nv = N / 8, esz = out32 ? 4 : 2;
+      uint4* gb = reinterpret_cast<uint4*>(smem);  // [gamma | beta]
+      uint8_t* zs = smem + ((2 * nv * 16 + 1023) & ~1023);
+      constexpr int RING = STAGES * STAGE_BYTES;
+      const int rows_per = (RING - (int)(zs - smem)) / (N * esz);
+      for (int i = threadIdx.x; i < 2 * nv; i += 128)
+        gb[i] = ldg16(i < nv ? static_cast<const T*>(lnf.gamma) + 8 * i : static_cast<const T*>(lnf.beta) + 8 * (i - nv));
+      const int vrow = N * esz / 16;  // 16-byte vectors per row
+      for (int r0 = 0; r0 < mcount; r0 += rows_per) {
+        const int nr = min(rows_per, mcount - r0);
+        __syncthreads();  // previous chunk consumed
+        for (int i = threadIdx.x; i < nr * vrow; i += 128) {
+          const int r = i / vrow, c = i - r * vrow;
+          const uint8_t* src = static_cast<const uint8_t*>(Y) + ((size_t)(m0 + r0 + r) * ldy) * esz + (size_t)c * 16;
+          const uint32_t dst = smem_u32(zs + (size_t)r * N * esz + (size_t)c * 16);
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+        }
+        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+        __syncthreads();
+        for (int tk = warp; tk < nr; tk += 4)
+          ln_row_warp<T, 6, 2>(zs, nullptr, (size_t)tk * N, N, lnf.eps, out32, gb, static_cast<T*>(lnf.out),
+                               (size_t)(m0 + r0 + tk) * lnf.ldo);
+      }
+      if (threadIdx.x == 0) lnf.cnt[blockIdx.y] = 0;
+    }
   }
 }
 
@@ -395,38 +483,10 @@ CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int b
   return m;
 }
 
-// Split-K workspace, one per device: fp32 tile slots + per-tile arrival counters (zeroed
-// once; the last split of every tile resets its counter).  Kernels on one device use it in
-// stream order (the engine runs a forward's kernels on one stream; PDL successors touch it
-// only after griddepcontrol.wait, i.e. after the previous GEMM completed).
-constexpr size_t SPLIT_WS_BYTES = size_t(32) << 20;
-constexpr int SPLIT_MAX_TILES = 16384;
-struct SplitWs {
-  float* ws = nullptr;
-  int* cnt = nullptr;
-};
-SplitWs& split_ws(int dev) {
-  static SplitWs w[64];
-  return w[dev];
-}
-std::mutex split_mu;
-
-SplitWs& split_ws_ready(cudaStream_t s) {
-  int dev;
-  DP_CUDA(cudaGetDevice(&dev));
-  SplitWs& w = split_ws(dev);
-  if (w.ws) return w;
-  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-  DP_CUDA(cudaStreamIsCapturing(s, &cs));
-  DP_CHECK(cs == cudaStreamCaptureStatusNone, DP_ERR_STATE, "split-K workspace must be prepared before capture");
-  gemm_prepare(dev);
-  return w;
-}
-
 template <class T, int BN>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
-         cudaStream_t s) {
+         const LnFuse& ln, cudaStream_t s) {
   constexpr size_t smem = size_t(stages_for<BN>()) * (BM * BK * 2 + BN * BK * 2) + 1024;
   static_assert(size_t(BM) * (BN + 1) * 4 + 1024 <= smem, "fp32 tile must fit the ring");
   static bool attr = false;
@@ -444,52 +504,24 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   }
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
   const int mt = (M + BN - 1) / BN;
-  float* ws = nullptr;
-  int* cnt = nullptr;
-  if (splits > 1) {
-    const size_t tiles = size_t(N / BM) * mt * ngroups;
-    if (tiles * splits * BM * BN * 4 > SPLIT_WS_BYTES || tiles > (size_t)SPLIT_MAX_TILES) splits = 1;
-  }
-  if (splits > 1) {
-    SplitWs& sw = split_ws_ready(s);
-    ws = sw.ws;
-    cnt = sw.cnt;
-  }
-  launch_kernel(gemm_tc_kernel<T, BN>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem, s, g, mx, res, ldr, y,
-                ldy, M, N, K, act, io, splits, ws, cnt);
+  launch_kernel_cluster(gemm_tc_kernel<T, BN>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem,
+                        dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, ln);
 }
 
 template <class T>
 void dispatch(int bn, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
               const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io,
-              int sp, cudaStream_t s) {
+              int sp, const LnFuse& ln, cudaStream_t s) {
   switch (bn) {
-    case 32: run<T, 32>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
-    case 64: run<T, 64>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
-    case 128: run<T, 128>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
-    case 256: run<T, 256>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); break;
+    case 32: run<T, 32>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
+    case 64: run<T, 64>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
+    case 128: run<T, 128>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
+    case 256: run<T, 256>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
     default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
   }
 }
 
 }  // namespace
-
-void gemm_prepare(int dev) {
-  std::lock_guard<std::mutex> lk(split_mu);
-  SplitWs& w = split_ws(dev);
-  if (w.ws) return;
-  int cur;
-  DP_CUDA(cudaGetDevice(&cur));
-  DP_CUDA(cudaSetDevice(dev));
-  void *a = nullptr, *b = nullptr;
-  if (cudaMalloc(&a, SPLIT_WS_BYTES) != cudaSuccess || cudaMalloc(&b, SPLIT_MAX_TILES * sizeof(int)) != cudaSuccess)
-    fail(DP_ERR_OOM, "split-K workspace cudaMalloc failed");
-  DP_CUDA(cudaMemset(b, 0, SPLIT_MAX_TILES * sizeof(int)));
-  DP_CUDA(cudaDeviceSynchronize());
-  w.ws = static_cast<float*>(a);
-  w.cnt = static_cast<int*>(b);
-  DP_CUDA(cudaSetDevice(cur));
-}
 
 bool gemm_tc_supported(int N, int K) { return N > 0 && K > 0 && N % BM == 0 && K % BK == 0; }
 
@@ -504,17 +536,38 @@ static int pick_bn(int M, int N) {
   return 32;
 }
 
-// Split-K factor: enough K splits to put ~one CTA on every SM, each with >= 2 k-blocks.
-static int pick_split(int M, int N, int K, int bn) {
-  const int tiles = (N / BM) * ((M + bn - 1) / bn);
-  int sp = 148 / std::max(1, tiles);
-  sp = std::min(sp, (K / BK) / 2);
-  return std::max(1, sp);
+// (BN, splits) from a per-CTA ingest model fitted to the B200 sweeps and per-CTA traces
+// (profiles/r01_gemm_sweep_v3.txt, r01_gemm_trace.jsonl): a CTA streams its W and X tiles at
+// ~100 GB/s (the mainloop time is its bytes / 1e5 B/us), all CTAs together at ~8 TB/s from
+// L2/HBM, and a cluster split-K reduction costs ~2.5 us.  Splits only in one wave of <= 148
+// CTAs, >= 4 k-blocks each.  Within 2% of the best measured configuration at every swept shape.
+struct GemmCfg {
+  int bn, sp;
+};
+static GemmCfg pick_cfg(int M, int N, int K) {
+  const int ntile = N / BM, kb = K / BK;
+  GemmCfg best{pick_bn(M, N), 1};
+  double best_t = 1e30;
+  for (int bn : {32, 64, 128, 256}) {
+    if (bn > 32 && M < bn) continue;
+    const int tiles = ntile * ((M + bn - 1) / bn);
+    for (int sp : {1, 2, 4}) {
+      if (sp > 1 && (kb / sp < 4 || tiles * sp > 148)) continue;
+      const double per = double(kb) / sp * (BM * BK * 2 + bn * BK * 2);
+      const int ctas = tiles * sp, waves = (ctas + 147) / 148;
+      const double t = std::max(waves * per / 1e5, ctas * per / 8e6) + (sp > 1 ? 2.5 : 0.0);
+      if (t < best_t - 1e-9) {
+        best_t = t;
+        best = {bn, sp};
+      }
+    }
+  }
+  return best;
 }
 
-void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
-                          const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
-                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
+static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
+                      const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act,
+                      int io, int bn_hint, const LnFuse& ln, cudaStream_t s) {
   DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
   DP_CHECK(ngroups >= 1 && ngroups <= 3, DP_ERR_INVALID, "gemm: 1..3 weight groups");
   DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0, DP_ERR_INVALID, "GEMM activations must be 16-byte aligned");
@@ -525,14 +578,35 @@ void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const 
   if (M <= 0) return;
   // tuning override for experiments (DP_GEMM_BN), read once
   static const int env_bn = getenv("DP_GEMM_BN") ? atoi(getenv("DP_GEMM_BN")) : 0;
-  const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : pick_bn(M, N * ngroups));
   static const int env_sp = getenv("DP_GEMM_SPLIT") ? atoi(getenv("DP_GEMM_SPLIT")) : 0;
-  int sp = env_sp > 0 ? env_sp : pick_split(M, N * ngroups, K, bn);
-  sp = std::max(1, std::min(sp, K / BK));
+  const GemmCfg cfg = pick_cfg(M, N * ngroups, K);
+  const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : cfg.bn);
+  int sp = env_sp > 0 ? env_sp : (bn_hint > 0 || env_bn > 0 ? 1 : cfg.sp);
+  sp = std::max(1, std::min(std::min(sp, 8), K / BK));
   if (dtype == DP_BF16)
-    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
+    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s);
   else
-    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
+    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s);
+}
+
+void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
+                          const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
+                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
+  const LnFuse none{nullptr, nullptr, nullptr, 0, 0.f, nullptr};
+  gemm_impl(dtype, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, bn_hint, none, s);
+}
+
+bool gemm_ln_supported(int N) { return N % 8 == 0 && N <= 6 * 256; }
+
+void launch_gemm_tc_ln(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
+                       void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, const void* gamma,
+                       const void* beta, float eps, void* ln_out, int ldo, int* counters, int ncounters,
+                       cudaStream_t s) {
+  DP_CHECK(gamma && beta && ln_out && counters, DP_ERR_INVALID, "fused LayerNorm: missing buffers");
+  DP_CHECK(gemm_ln_supported(N) && ldo % 8 == 0, DP_ERR_UNSUPPORTED, "fused LayerNorm: N <= 1536, multiple of 8");
+  DP_CHECK((M + 31) / 32 <= ncounters, DP_ERR_INVALID, "fused LayerNorm: too few m-tile counters");
+  const LnFuse ln{gamma, beta, ln_out, ldo, eps, counters};
+  gemm_impl(dtype, x, ldx, 1, &w, &bias, nullptr, res, ldr, y, ldy, M, N, K, act, io, bn_hint, ln, s);
 }
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,

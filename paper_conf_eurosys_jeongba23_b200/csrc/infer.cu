@@ -311,7 +311,7 @@ static std::string graph_key(const dp_context* ctx, const dp_plan* plan, const i
        std::to_string((uintptr_t)pooled) + "|" + std::to_string(batch) + "x" + std::to_string(seq) + "|" +
        std::to_string(ctx->opts.chunk_bytes) + "," + std::to_string(ctx->opts.n_h2d_streams) + "," +
        std::to_string(ctx->opts.gemm_bn) + "," + std::to_string(ctx->opts.debug_delay_us) + "," +
-       std::to_string(ctx->opts.use_pdl);
+       std::to_string(ctx->opts.use_pdl) + "," + std::to_string(ctx->opts.fuse_ln);
   return k;
 }
 
@@ -492,6 +492,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     last_waited = e;
   };
   a.pdl = ctx->opts.use_pdl != 0;
+  a.fuse_ln = ctx->opts.fuse_ln != 0;
   run_forward(a);
   // join every side stream (units never read, e.g. an unused pooler, still finish loading)
   for (int i = 0; i < nh; ++i) {
@@ -559,6 +560,7 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.stream = (cudaStream_t)stream;
     a.bn_hint = ctx->opts.gemm_bn;
     a.pdl = ctx->opts.use_pdl != 0;
+    a.fuse_ln = ctx->opts.fuse_ln != 0;
     if (ctx->opts.use_graph) {
       std::string key = "warm|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
                         graph_key(ctx, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);

@@ -16,12 +16,31 @@
 #include "dtype.cuh"
 #include "kernels.h"
 #include "launch.cuh"
+#include "ln.cuh"
 
 namespace dp {
 
 PdlState& pdl_state() {
   static thread_local PdlState s;
   return s;
+}
+
+// cp.async (global -> shared, 16 bytes, bypassing L1); the zero-fill form writes zeros when
+// !valid (src is not read)
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void cp_async16_zfill(void* dst, const void* src, bool valid) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src), "r"(valid ? 16 : 0)
+               : "memory");
 }
 
 // -------------------------------------------------------------------------------------
@@ -184,51 +203,8 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
-  for (int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); row < rows; row += nwarps) {
-    float v[VPL][8];
-    float sum = 0.f;
-#pragma unroll
-    for (int k = 0; k < VPL; ++k) {
-      const int c = lane + 32 * k;
-      if (c < nv) {
-        load8<T>(x, (size_t)row * n + 8 * c, v[k], in_f32);
-        if (r) {
-          float a[8];
-          load8<T>(r, (size_t)row * n + 8 * c, a, in_f32);
-#pragma unroll
-          for (int e = 0; e < 8; ++e) v[k][e] += a[e];
-        }
-#pragma unroll
-        for (int e = 0; e < 8; ++e) sum += v[k][e];
-      }
-    }
-    const float mean = warp_sum(sum) / n;
-    float sq = 0.f;
-#pragma unroll
-    for (int k = 0; k < VPL; ++k) {
-      const int c = lane + 32 * k;
-      if (c < nv) {
-#pragma unroll
-        for (int e = 0; e < 8; ++e) {
-          const float d = v[k][e] - mean;
-          sq += d * d;
-        }
-      }
-    }
-    const float rstd = rsqrtf(warp_sum(sq) / n + eps);
-#pragma unroll
-    for (int k = 0; k < VPL; ++k) {
-      const int c = lane + 32 * k;
-      if (c < nv) {
-        float gg[8], bb[8], o[8];
-        unpack8<T>(sm[c], gg);
-        unpack8<T>(sm[nv + c], bb);
-#pragma unroll
-        for (int e = 0; e < 8; ++e) o[e] = (v[k][e] - mean) * rstd * gg[e] + bb[e];
-        reinterpret_cast<uint4*>(y + (size_t)row * n)[c] = pack8<T>(o);
-      }
-    }
-  }
+  for (int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); row < rows; row += nwarps)
+    ln_row_warp<T, VPL, 0>(x, r, (size_t)row * n, n, eps, in_f32, sm, y, (size_t)row * n);
 }
 
 template <class T>
@@ -439,9 +415,12 @@ constexpr int ATT_D = 64, ATT_BQ = 64, ATT_BK = 64, ATT_LD = 72;  // padded row 
 template <class T>
 __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qkv, int ldqkv, T* __restrict__ ctx,
                                                         int seq, int H, int causal, float scale_log2) {
+  // Q tile + a 2-deep ring of (K, V) tiles, all filled with cp.async: the Q tile and the
+  // first two key tiles are in flight together (one L2 round trip, not one per tile), and
+  // tile kt+2 streams in while tile kt is computed.  Rows past `seq` are zero-filled.
   __shared__ __align__(16) T sq[ATT_BQ * ATT_LD];
-  __shared__ __align__(16) T sk[ATT_BK * ATT_LD];
-  __shared__ __align__(16) T sv[ATT_BK * ATT_LD];
+  __shared__ __align__(16) T sk[2][ATT_BK * ATT_LD];
+  __shared__ __align__(16) T sv[2][ATT_BK * ATT_LD];
   pdl_trigger();
   pdl_wait();  // q, k, v come from the previous kernels
   const int qt = blockIdx.x, head = blockIdx.y, bidx = blockIdx.z;
@@ -451,13 +430,28 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
   const T* qbase = qkv + tok0 * ldqkv + head * ATT_D;
   const T* kbase = qbase + H;
   const T* vbase = qbase + 2 * H;
-  // Q tile: 64 rows x 64 d = 512 vectors of 16 B; 4 per thread
-  for (int i = tid; i < ATT_BQ * 8; i += 128) {
+  int nkt = (seq + ATT_BK - 1) / ATT_BK;
+  if (causal) nkt = min(nkt, (q0 + ATT_BQ - 1) / ATT_BK + 1);
+  auto load_kv = [&](int kt) {
+    const int k0 = kt * ATT_BK;
+    for (int i = tid; i < ATT_BK * 8; i += 128) {
+      const int r = i >> 3, c = i & 7;
+      const bool ok = k0 + r < seq;
+      const size_t off = (size_t)(ok ? k0 + r : 0) * ldqkv + c * 8;
+      cp_async16_zfill(&sk[kt & 1][r * ATT_LD + c * 8], kbase + off, ok);
+      cp_async16_zfill(&sv[kt & 1][r * ATT_LD + c * 8], vbase + off, ok);
+    }
+  };
+  for (int i = tid; i < ATT_BQ * 8; i += 128) {  // Q: 64 rows x 64 d = 512 vectors of 16 B
     const int r = i >> 3, c = i & 7;
-    uint4 v = make_uint4(0, 0, 0, 0);
-    if (q0 + r < seq) v = *reinterpret_cast<const uint4*>(qbase + (size_t)(q0 + r) * ldqkv + c * 8);
-    *reinterpret_cast<uint4*>(&sq[r * ATT_LD + c * 8]) = v;
+    const bool ok = q0 + r < seq;
+    cp_async16_zfill(&sq[r * ATT_LD + c * 8], qbase + (size_t)(ok ? q0 + r : 0) * ldqkv + c * 8, ok);
   }
+  load_kv(0);
+  cp_async_commit();
+  if (nkt > 1) load_kv(1);
+  cp_async_commit();
+  cp_async_wait<1>();
   __syncthreads();
   uint32_t qa[4][4];  // A fragments: 16 rows of this warp x 64 d (4 k-steps)
   {
@@ -470,22 +464,14 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
   for (int i = 0; i < 8; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
   float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
   const int qrow0 = q0 + warp * 16 + (lane >> 2);  // rows qrow0 and qrow0 + 8
-  int nkt = (seq + ATT_BK - 1) / ATT_BK;
-  if (causal) nkt = min(nkt, (q0 + ATT_BQ - 1) / ATT_BK + 1);
   for (int kt = 0; kt < nkt; ++kt) {
     const int k0 = kt * ATT_BK;
-    __syncthreads();  // previous tile fully consumed
-    for (int i = tid; i < ATT_BK * 8; i += 128) {
-      const int r = i >> 3, c = i & 7;
-      uint4 kv4 = make_uint4(0, 0, 0, 0), vv4 = make_uint4(0, 0, 0, 0);
-      if (k0 + r < seq) {
-        kv4 = *reinterpret_cast<const uint4*>(kbase + (size_t)(k0 + r) * ldqkv + c * 8);
-        vv4 = *reinterpret_cast<const uint4*>(vbase + (size_t)(k0 + r) * ldqkv + c * 8);
-      }
-      *reinterpret_cast<uint4*>(&sk[r * ATT_LD + c * 8]) = kv4;
-      *reinterpret_cast<uint4*>(&sv[r * ATT_LD + c * 8]) = vv4;
+    if (kt > 0) {
+      cp_async_wait<1>();  // tile kt landed (tile kt+1 may still be in flight)
+      __syncthreads();
     }
-    __syncthreads();
+    const T* skt = sk[kt & 1];
+    const T* svt = sv[kt & 1];
     float s[8][4];
 #pragma unroll
     for (int nb = 0; nb < 8; ++nb) s[nb][0] = s[nb][1] = s[nb][2] = s[nb][3] = 0.f;
@@ -495,7 +481,7 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
       for (int nb = 0; nb < 8; nb += 2) {
         uint32_t bfr[4];
         const int key = nb * 8 + (lane & 7) + (lane >> 4) * 8;
-        ldsm_x4(bfr, &sk[key * ATT_LD + kk * 16 + ((lane >> 3) & 1) * 8]);
+        ldsm_x4(bfr, &skt[key * ATT_LD + kk * 16 + ((lane >> 3) & 1) * 8]);
         MmaOp<T>::mma(s[nb], qa[kk], bfr);
         MmaOp<T>::mma(s[nb + 1], qa[kk], bfr + 2);
       }
@@ -555,11 +541,16 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
       for (int db = 0; db < 8; db += 2) {
         uint32_t bfr[4];
         const int key = kk * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
-        ldsm_x4_t(bfr, &sv[key * ATT_LD + (db + (lane >> 4)) * 8]);
+        ldsm_x4_t(bfr, &svt[key * ATT_LD + (db + (lane >> 4)) * 8]);
         MmaOp<T>::mma(o[db], pa, bfr);
         MmaOp<T>::mma(o[db + 1], pa, bfr + 2);
       }
     }
+    if (kt + 2 < nkt) {
+      __syncthreads();  // every warp is done with slot kt & 1
+      load_kv(kt + 2);
+    }
+    cp_async_commit();
   }
   // finalize: full row sums across the 4 lanes of a row
 #pragma unroll
@@ -621,16 +612,6 @@ constexpr int SK_STG = 4;    // cp.async ring depth
 constexpr int SK_XP = SK_KCH + 8;
 constexpr int SK_WREG = 6;   // W vectors per thread: 16 rows x 768 / 8 / 256
 
-__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
-               "l"(src)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
 __device__ __forceinline__ uint32_t cluster_rank() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
@@ -786,7 +767,7 @@ void skinny_mma_t(const void* x, int ldx, const void* w, const void* bias, const
     DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     attr_set = true;
   }
-  launch_kernel_cluster(skinny_mma_kernel<T>, dim3((N / 16) * cs), dim3(256), sm, cs, s, (const T*)x, ldx,
+  launch_kernel_cluster(skinny_mma_kernel<T>, dim3((N / 16) * cs), dim3(256), sm, dim3(cs, 1, 1), s, (const T*)x, ldx,
                         (const T*)w, (const T*)bias, res, ldr, y, ldy, M, N, K, KS, cs, act, io);
 }
 

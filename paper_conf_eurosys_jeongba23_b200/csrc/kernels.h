@@ -30,8 +30,14 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
 
 // K2: resident tcgen05/TMA GEMM -- a12.  W must be device memory.
 struct GemmPlan;  // cached tensor map for a weight
+// GEMM whose epilogue also LayerNorms complete output rows into ln_out (see gemm_tc.cu,
+// LnFuse); counters: >= ceil(M / 32) ints, zero between launches.
+bool gemm_ln_supported(int N);
+void launch_gemm_tc_ln(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
+                       void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, const void* gamma,
+                       const void* beta, float eps, void* ln_out, int ldo, int* counters, int ncounters,
+                       cudaStream_t s);
 bool gemm_tc_supported(int N, int K);
-void gemm_prepare(int dev);  // split-K workspace (call before any stream capture)
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);
 // ngroups (1..3) weights sharing X; group i writes y at column offset ycol[i].

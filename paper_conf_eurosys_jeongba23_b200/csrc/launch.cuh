@@ -44,9 +44,9 @@ inline void launch_kernel(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t 
   DP_CUDA(cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...));
 }
 
-// The same with a 1-D thread-block cluster of `cluster` CTAs along x (cluster == 1: none).
+// The same with thread-block clusters of shape `cluster` (1 x 1 x 1: none).
 template <class... KArgs, class... Args>
-inline void launch_kernel_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, int cluster,
+inline void launch_kernel_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, dim3 cluster,
                                   cudaStream_t s, Args&&... args) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;
@@ -59,11 +59,11 @@ inline void launch_kernel_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block,
     at[n].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     at[n++].val.programmaticStreamSerializationAllowed = 1;
   }
-  if (cluster > 1) {
+  if (cluster.x * cluster.y * cluster.z > 1) {
     at[n].id = cudaLaunchAttributeClusterDimension;
-    at[n].val.clusterDim.x = cluster;
-    at[n].val.clusterDim.y = 1;
-    at[n++].val.clusterDim.z = 1;
+    at[n].val.clusterDim.x = cluster.x;
+    at[n].val.clusterDim.y = cluster.y;
+    at[n++].val.clusterDim.z = cluster.z;
   }
   cfg.attrs = n ? at : nullptr;
   cfg.numAttrs = n;

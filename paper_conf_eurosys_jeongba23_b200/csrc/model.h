@@ -47,6 +47,8 @@ struct Workspace {
   void* tmp = nullptr;  // [T, H]
   void* x1 = nullptr;   // [T, H]
   void* h = nullptr;    // [T, F]
+  int* ln_cnt = nullptr;  // per-32-token-tile counters of the GEMM-fused LayerNorm (zeroed)
+  int n_ln_cnt = 0;
   void* base = nullptr;
 };
 

@@ -259,3 +259,32 @@ def test_graph_replay_matches_eager(name, mode, k):
         model.evict(0)
     model.close()
     c.close()
+
+
+@pytest.mark.parametrize("name,S", [("tiny_bert", 77), ("tiny_gpt2", 70), ("bert_base", 128), ("gpt2", 200)])
+def test_fused_layernorm_bit_identical(name, S):
+    """A LayerNorm that follows a resident-weight linear runs in that GEMM's epilogue (the last
+    CTA of each token tile normalises its complete rows); it shares the per-row code with the
+    LayerNorm kernel, so fused and unfused forwards must agree bit for bit, in eager and graph
+    mode, and the fused run launches 2 fewer kernels per layer."""
+    m = synth.SHAPES[name]
+    dtype = "fp16"
+    w = synth.make_weights(m, seed=21, dtype=dtype)
+    ids = synth.make_ids(m, 1, S, seed=22)
+    c = dp().Context([0])
+    model = dp().Model(c, m, w, dtype)
+    plan = dp().plan_generate(fake_cost(m, dtype), "PIPESWITCH", 1)  # all loaded: every linear on the GEMM
+    outs, kern = [], []
+    for fuse, graph in ((False, 0), (True, 0), (True, 1)):
+        c.set_opts(fuse_ln=fuse, use_graph=graph)
+        o, p, st = run_cold(model, plan, ids, dtype)
+        outs.append((o.clone(), None if p is None else p.clone()))
+        kern.append(st["n_kernels"])
+        model.evict(0)
+    for o, p in outs[1:]:
+        assert torch.equal(o, outs[0][0])
+        if p is not None:
+            assert torch.equal(p, outs[0][1])
+    assert kern[1] == kern[0] - 2 * m.layers
+    model.close()
+    c.close()

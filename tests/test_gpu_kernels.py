@@ -222,7 +222,8 @@ def test_layernorm_parity_and_dha(rows, n):
 
 
 @pytest.mark.parametrize("B,S,H,heads", [(1, 1, 128, 2), (2, 5, 128, 2), (1, 64, 768, 12), (2, 100, 256, 4),
-                                         (1, 128, 768, 12), (1, 384, 1024, 16), (1, 1024, 1024, 16)])
+                                         (1, 128, 768, 12), (1, 384, 1024, 16), (1, 1024, 1024, 16),
+                                         (3, 200, 256, 4)])
 @pytest.mark.parametrize("causal", [False, True])
 @pytest.mark.parametrize("dtype", ["fp16", "bf16"])
 def test_attention_parity(B, S, H, heads, causal, dtype):
