@@ -249,7 +249,7 @@ def main():
     # profile on the primary, plan, share the plan (the plan never names GPUs)
     # default plan: Algorithm 1 on the link-aware model (R19); the paper's own
     # Algorithm-1 plan ("DHA") and the other engine options are timed beside it below
-    mode = a.mode or ("PT_DHA_LINK" if world > 1 else "DHA_LINK")
+    mode = a.mode or ("PT_DHA_LINK_BAL" if world > 1 else "DHA_LINK")
     if rank == 0:
         cost = model.profile(local, a.batch, a.seq, a.profile_iters)
     else:

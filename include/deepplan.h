@@ -64,7 +64,12 @@ enum {
   /* NEXT-row extension, not the paper's (R19): Algorithm 1 on a
    * pipeline model where DHA reads occupy the primary link (cost.dha_link_ns) */
   DP_MODE_DHA_LINK = 6,
-  DP_MODE_PT_DHA_LINK = 7
+  DP_MODE_PT_DHA_LINK = 7,
+  /* NEXT-row extension f1(i)+(ii), R20: PT_DHA with the equal split taken over the
+   * bytes actually transferred (DHA units count 0) and Algorithm 1 re-run under the PT
+   * arrival model on partition 0 */
+  DP_MODE_PT_DHA_BAL = 8,
+  DP_MODE_PT_DHA_LINK_BAL = 9 /* the same on the link-aware model (R19 + R20) */
 };
 
 /* ---------------------------------------------------------------------------------

@@ -20,8 +20,8 @@ import numpy as np
 
 LOAD, DHA = 0, 1
 MODES = ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "PT", "PT_DHA")  # the paper's options
-EXT_MODES = ("DHA_LINK", "PT_DHA_LINK")  # NEXT-row extension (link-aware), R19
-LINK_AWARE = {"DHA_LINK", "PT_DHA_LINK"}
+EXT_MODES = ("DHA_LINK", "PT_DHA_LINK", "PT_DHA_BAL", "PT_DHA_LINK_BAL")  # NEXT-row extensions, R19 / R20
+LINK_AWARE = {"DHA_LINK", "PT_DHA_LINK", "PT_DHA_LINK_BAL"}
 INF_NS = 1 << 50
 
 
@@ -172,23 +172,25 @@ def algorithm1(cost):
     return method
 
 
-def algorithm1_link(cost):
+def algorithm1_link(cost, slot=None, k: int = 1, init=None):
     """NEXT-row extension (R19), not the paper's algorithm: the
     same loop as Algorithm 1 run on the link-aware simulator, where switching L_j to DHA frees
     only saved_j = Load_j - DhaLink_j of link time.  Line 9 still breaks on S < PerfDiff_j;
     a candidate with saved_j <= 0 is skipped (no link time freed: it cannot advance any later
     load); line 13 becomes S - saved_j - PerfDiff_j.  With DhaLink = 0 and every Load > 0
-    this is exactly algorithm1."""
+    this is exactly algorithm1.  ``slot``/``k``/``init``: the PT arrival model, slot-0
+    candidates and a kept DHA set, as in algorithm1_slots (R20)."""
     n = len(cost["load_ns"])
     load = _arr(cost, "load_ns")
     dlink = _arr(cost, "dha_link_ns") if "dha_link_ns" in cost else [0] * n
     pd = [d - m for d, m in zip(_arr(cost, "exe_dha_ns"), _arr(cost, "exe_mem_ns"))]
-    method = [LOAD] * n
+    method = [LOAD] * n if init is None else list(init)
     for i in range(n):
-        S = simulate(cost, method, link_aware=True)["stall"][i]
+        S = simulate(cost, method, slot, k, link_aware=True)["stall"][i]
         if not S > 0:
             continue
-        cand = sorted((j for j in range(i + 1) if method[j] == LOAD), key=lambda j: (pd[j], j))
+        cand = sorted((j for j in range(i + 1) if method[j] == LOAD and (slot is None or slot[j] == 0)),
+                      key=lambda j: (pd[j], j))
         for j in cand:
             if S < pd[j]:
                 break
@@ -197,6 +199,31 @@ def algorithm1_link(cost):
                 continue
             method[j] = DHA
             S = S - saved - pd[j]
+            if S <= 0:
+                break
+    return method
+
+
+def algorithm1_slots(cost, slot, k: int, init=None):
+    """NEXT-row extension f1(ii) (R20), not the paper's algorithm: Algorithm 1 run
+    under the PT arrival model -- stalls come from P1 with the given slots (a slot-s unit is
+    ready when its NVLink forward ends) and the candidates are the slot-0 units L_1..L_i not
+    yet DHA (the later partitions are loaded).  ``init``: DHA units kept from an
+    earlier pass (default none).  With k = 1 and no init this is exactly algorithm1."""
+    n = len(cost["load_ns"])
+    load = _arr(cost, "load_ns")
+    pd = [d - m for d, m in zip(_arr(cost, "exe_dha_ns"), _arr(cost, "exe_mem_ns"))]
+    method = [LOAD] * n if init is None else list(init)
+    for i in range(n):
+        S = simulate(cost, method, slot, k)["stall"][i]
+        if not S > 0:
+            continue
+        cand = sorted((j for j in range(i + 1) if method[j] == LOAD and slot[j] == 0), key=lambda j: (pd[j], j))
+        for j in cand:
+            if S < pd[j]:
+                break
+            method[j] = DHA
+            S = S - load[j] - pd[j]
             if S <= 0:
                 break
     return method
@@ -224,6 +251,13 @@ def partition(nbytes, k: int):
     return part
 
 
+def partition_transferred(nbytes, method, k: int):
+    """NEXT-row extension f1(i) (R20): the P3 rule applied to the bytes that are
+    actually transferred -- a DHA unit counts 0 -- so the primary's link carries its share
+    instead of idling behind DHA'd embeddings (BERT-Base k = 8: slot 0 = {word} under P3)."""
+    return partition([int(b) if m == LOAD else 0 for b, m in zip(nbytes, method)], k)
+
+
 def plan(cost, mode: str, k: int = 1):
     """Returns (method[n], slot[n], serial flag) for one of the five engine options
      plus the greedy comparison."""
@@ -248,6 +282,26 @@ def plan(cost, mode: str, k: int = 1):
                 slot[i] = part[i]
                 method[i] = LOAD
         return method, slot, False
+    if mode in ("PT_DHA_BAL", "PT_DHA_LINK_BAL"):
+        # (1) Algorithm 1 on one link; (2) the P3 rule on the transferred bytes, where a DHA
+        # unit that falls into a later partition is loaded there, so it is dropped from
+        # the DHA set and the split recomputed until the set is stable (it only shrinks);
+        # (3) Algorithm 1 continued under the PT arrival model on the slot-0 units (the DHA
+        # set of (1)-(2) is kept, so partition 0 only sheds bytes)
+        link = mode == "PT_DHA_LINK_BAL"
+        method = algorithm1_link(cost) if link else algorithm1(cost)
+        if k == 1:  # one link: nothing to split
+            return method, [0] * n, False
+        while True:
+            slot = partition_transferred(cost["bytes"], method, k)
+            moved = [i for i in range(n) if method[i] == DHA and slot[i] >= 1]
+            if not moved:
+                break
+            for i in moved:
+                method[i] = LOAD
+        if link:
+            return algorithm1_link(cost, slot, k, init=method), slot, False
+        return algorithm1_slots(cost, slot, k, init=method), slot, False
     raise ValueError(mode)
 
 
@@ -282,12 +336,14 @@ def simulate_batch(cost, methods: np.ndarray, slot=None, k: int = 1, link_aware:
     return t
 
 
-def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 18, link_aware: bool = False):
+def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 18, link_aware: bool = False,
+               slot=None):
     """Optimal method vector under P1 with the P3 partition fixed (units with part >= 1
     are LOAD on their slot).  ``free``: indices allowed to vary (default: all part-0
-    units); others keep ``base_method``.  Returns (latency, method, slot)."""
+    units); others keep ``base_method``.  ``slot``: a given partition instead of P3 (the
+    PT_DHA_BAL plans).  Returns (latency, method, slot)."""
     n = len(cost["load_ns"])
-    part = partition(cost["bytes"], k) if k > 1 else [0] * n
+    part = list(slot) if slot is not None else (partition(cost["bytes"], k) if k > 1 else [0] * n)
     slot = list(part)
     if free is None:
         free = [i for i in range(n) if part[i] == 0]

@@ -76,19 +76,24 @@ static Sim simulate(const dp_cost_table* c, const int8_t* method, const int8_t* 
 // remaining stall is below the candidate's PerfDiff (line 9); otherwise switch it to DHA
 // (line 12) and deduct Load + PerfDiff (line 13) until the stall is gone (lines 16-18).
 // Stalls are refreshed by re-simulating the current plan before each i (line 17).
-static void algorithm1(const dp_cost_table* c, int8_t* method) {
+// With `slot` (NEXT-row extension f1(ii), R20): stalls come from the PT arrival
+// model with those slots and only slot-0 units are candidates (later partitions are loaded).
+// keep_init: start from the DHA set already in `method` instead of all LOAD.
+static void algorithm1(const dp_cost_table* c, int8_t* method, const int8_t* slot = nullptr, int k = 1,
+                       bool keep_init = false) {
   const int n = c->n;
   std::vector<int64_t> pd(n);
   for (int i = 0; i < n; ++i) pd[i] = c->exe_dha_ns[i] - c->exe_mem_ns[i];
-  for (int i = 0; i < n; ++i) method[i] = DP_LOAD;
+  if (!keep_init)
+    for (int i = 0; i < n; ++i) method[i] = DP_LOAD;
   std::vector<int> cand;
   cand.reserve(n);
   for (int i = 0; i < n; ++i) {
-    int64_t S = simulate(c, method, nullptr, 1, false).stall[i];
+    int64_t S = simulate(c, method, slot, k, false).stall[i];
     if (S <= 0) continue;
     cand.clear();
     for (int j = 0; j <= i; ++j)
-      if (method[j] == DP_LOAD) cand.push_back(j);
+      if (method[j] == DP_LOAD && (slot == nullptr || slot[j] == 0)) cand.push_back(j);
     std::stable_sort(cand.begin(), cand.end(), [&](int a, int b) { return pd[a] < pd[b]; });
     for (int j : cand) {
       if (S < pd[j]) break;
@@ -102,19 +107,21 @@ static void algorithm1(const dp_cost_table* c, int8_t* method) {
 // Link-aware Algorithm 1 (NEXT-row extension, not the paper's; R19): the same loop
 // on the link-aware model; switching L_j frees only saved_j = Load_j - DhaLink_j of link
 // time, so a candidate with saved_j <= 0 is skipped and line 13 deducts saved_j.
-static void algorithm1_link(const dp_cost_table* c, int8_t* method) {
+static void algorithm1_link(const dp_cost_table* c, int8_t* method, const int8_t* slot = nullptr, int k = 1,
+                            bool keep_init = false) {
   const int n = c->n;
   std::vector<int64_t> pd(n);
   for (int i = 0; i < n; ++i) pd[i] = c->exe_dha_ns[i] - c->exe_mem_ns[i];
-  for (int i = 0; i < n; ++i) method[i] = DP_LOAD;
+  if (!keep_init)
+    for (int i = 0; i < n; ++i) method[i] = DP_LOAD;
   std::vector<int> cand;
   cand.reserve(n);
   for (int i = 0; i < n; ++i) {
-    int64_t S = simulate(c, method, nullptr, 1, false, true).stall[i];
+    int64_t S = simulate(c, method, slot, k, false, true).stall[i];
     if (S <= 0) continue;
     cand.clear();
     for (int j = 0; j <= i; ++j)
-      if (method[j] == DP_LOAD) cand.push_back(j);
+      if (method[j] == DP_LOAD && (slot == nullptr || slot[j] == 0)) cand.push_back(j);
     std::stable_sort(cand.begin(), cand.end(), [&](int a, int b) { return pd[a] < pd[b]; });
     for (int j : cand) {
       if (S < pd[j]) break;
@@ -127,7 +134,9 @@ static void algorithm1_link(const dp_cost_table* c, int8_t* method) {
   }
 }
 
-static bool link_mode(int mode) { return mode == DP_MODE_DHA_LINK || mode == DP_MODE_PT_DHA_LINK; }
+static bool link_mode(int mode) {
+  return mode == DP_MODE_DHA_LINK || mode == DP_MODE_PT_DHA_LINK || mode == DP_MODE_PT_DHA_LINK_BAL;
+}
 
 static void partition(const int64_t* bytes, int n, int k, int8_t* part) {
   int64_t total = 0;
@@ -191,6 +200,36 @@ static void generate(const dp_cost_table* c, int mode, int k, dp_plan* out) {
         }
       return;
     }
+    case DP_MODE_PT_DHA_BAL:
+    case DP_MODE_PT_DHA_LINK_BAL: {
+      const bool link = mode == DP_MODE_PT_DHA_LINK_BAL;
+      // NEXT-row extension f1(i)+(ii) (R20): Algorithm 1 on one link; the P3 rule
+      // on the bytes that are transferred (DHA units count 0); Algorithm 1 continued (its DHA
+      // set kept) under the PT arrival model on the slot-0 units
+      // (a DHA unit that falls into a later partition is loaded there, so it leaves the DHA
+      // set and the split is recomputed; the set only shrinks, so this terminates)
+      if (link)
+        algorithm1_link(c, out->method);
+      else
+        algorithm1(c, out->method);
+      if (k == 1) return;  // one link: nothing to split
+      std::vector<int64_t> tb(n);
+      for (bool moved = true; moved;) {
+        for (int i = 0; i < n; ++i) tb[i] = out->method[i] == DP_LOAD ? c->bytes[i] : 0;
+        partition(tb.data(), n, k, out->slot);
+        moved = false;
+        for (int i = 0; i < n; ++i)
+          if (out->method[i] == DP_DHA && out->slot[i] >= 1) {
+            out->method[i] = DP_LOAD;
+            moved = true;
+          }
+      }
+      if (link)
+        algorithm1_link(c, out->method, out->slot, k, true);
+      else
+        algorithm1(c, out->method, out->slot, k, true);
+      return;
+    }
     default:
       fail(DP_ERR_INVALID, "unknown plan mode");
   }
@@ -236,7 +275,14 @@ extern "C" dp_status dp_plan_exhaustive(const dp_cost_table* cost, const dp_plan
     DP_CHECK(nfree >= 0 && nfree <= 30 && (nfree == 0 || free_idx), DP_ERR_INVALID, "nfree out of range");
     const int n = cost->n, k = std::max(1, base->k);
     std::vector<int8_t> part(n, 0), m(base->method, base->method + n);
-    if (k > 1) partition(cost->bytes, n, k, part.data());
+    if (k > 1) {
+      if (base->mode == DP_MODE_PT_DHA_BAL || base->mode == DP_MODE_PT_DHA_LINK_BAL) {  // its own split
+        DP_CHECK(base->slot != nullptr, DP_ERR_INVALID, "bad base plan");
+        std::copy(base->slot, base->slot + n, part.begin());
+      } else {
+        partition(cost->bytes, n, k, part.data());
+      }
+    }
     for (int i = 0; i < n; ++i)
       if (part[i] >= 1) m[i] = DP_LOAD;
     for (int b = 0; b < nfree; ++b)
