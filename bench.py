@@ -52,6 +52,7 @@ def parse():
     ap.add_argument("--fuse-ln", action="store_true", help="LayerNorm in the preceding GEMM's epilogue")
     ap.add_argument("--profile-iters", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--quick", action="store_true", help="skip the other modes and per-kernel rooflines (sweeps)")
     return ap.parse_args()
 
 
@@ -159,7 +160,7 @@ def kernel_rooflines(dp, torch, m, T, peaks, peak_h2d, reps=50):
     return out
 
 
-def cpu_oracle_ms(m, w, ids, dtype, budget_s=15.0, max_runs=10):
+def cpu_oracle_ms(m, w, ids, dtype, budget_s=12.0, max_runs=60):
     """The oracle (fp64 numpy) timed on this host's cores, on a bounded sample."""
     from oracle import forward as F
     t0 = time.perf_counter()
@@ -382,7 +383,7 @@ def main():
     # the same cold start under the paper's other engine options (single GPU only), for the
     # paper's comparisons (e.g. PT+DHA / DHA vs PipeSwitch)
     other_modes = {}
-    if world == 1 and not os.environ.get("DP_BENCH_UNDER_NCU"):
+    if world == 1 and not os.environ.get("DP_BENCH_UNDER_NCU") and not a.quick:
         for om in ("DHA", "GREEDY", "PIPESWITCH", "BASELINE"):
             if om == mode:
                 continue
@@ -413,7 +414,8 @@ def main():
     R_lit = total_w / (peak_h2d * world * 1e9) * 1e3  # all weight bytes / aggregate H2D
     R_alg = per_link / (peak_h2d * 1e9) * 1e3          # busiest link's algorithmic bytes
     peaks, peaks_src = measured_peaks()
-    krl = None if os.environ.get("DP_BENCH_UNDER_NCU") else kernel_rooflines(dp, torch, m, T, peaks, peak_h2d)
+    krl = None if (os.environ.get("DP_BENCH_UNDER_NCU") or a.quick) else kernel_rooflines(dp, torch, m, T, peaks,
+                                                                                          peak_h2d)
 
     cpu = None
     if not a.no_cpu_baseline:

@@ -204,7 +204,7 @@ template <class T, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
                    const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io, int splits,
-                   const LnFuse lnf) {
+                   int nst, const LnFuse lnf) {
   constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
@@ -259,7 +259,9 @@ __global__ void __launch_bounds__(128, 1)
   // Weights never depend on the previous kernel: the producer puts the first ring's worth
   // of W tiles in flight BEFORE the grid-dependency wait (PDL), so their HBM latency
   // overlaps the predecessor's tail.  Activations (X, residual) and every store come after.
-  const int pre = num_kb < STAGES ? num_kb : STAGES;
+  // nst <= STAGES: the ring depth actually used (a shallower ring leaves room on the SM for
+  // the previous kernel's CTAs, so the PDL prologue overlap is not blocked on shared memory)
+  const int pre = num_kb < nst ? num_kb : nst;
   if (warp == 0 && lane == 0) {
     for (int kb = 0; kb < pre; ++kb) {
       mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
@@ -288,11 +290,11 @@ __global__ void __launch_bounds__(128, 1)
   if (warp == 0 && lane == 0) {
     // TMA producer
     for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % STAGES;
+      const int s = kb % nst;
       uint8_t* a = smem + s * STAGE_BYTES;
       uint8_t* b = a + A_BYTES;
       if (kb >= pre) {
-        mbar_wait(&empty_bar[s], ((kb / STAGES) - 1) & 1);
+        mbar_wait(&empty_bar[s], ((kb / nst) - 1) & 1);
         mbar_expect_tx(&full_bar[s], STAGE_BYTES);
         tma_load_2d(tmW, &full_bar[s], a, (kb_lo + kb) * BK, n0);
       }
@@ -301,8 +303,8 @@ __global__ void __launch_bounds__(128, 1)
   } else if (warp == 1 && lane == 0) {
     // MMA issuer
     for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % STAGES;
-      mbar_wait(&full_bar[s], (kb / STAGES) & 1);
+      const int s = kb % nst;
+      mbar_wait(&full_bar[s], (kb / nst) & 1);
       if (kb == 0) TRACE(3);
       asm volatile("tcgen05.fence::after_thread_sync;");
       const uint8_t* a = smem + s * STAGE_BYTES;
@@ -428,7 +430,7 @@ __global__ void __launch_bounds__(128, 1)
       const int nv = N / 8, esz = out32 ? 4 : 2;
       uint4* gb = reinterpret_cast<uint4*>(smem);  // [gamma | beta]
       uint8_t* zs = smem + ((2 * nv * 16 + 1023) & ~1023);
-      constexpr int RING = STAGES * STAGE_BYTES;
+      const int RING = nst * STAGE_BYTES;
       const int rows_per = (RING - (int)(zs - smem)) / (N * esz);
       for (int i = threadIdx.x; i < 2 * nv; i += 128)
         gb[i] = ldg16(i < nv ? static_cast<const T*>(lnf.gamma) + 8 * i : static_cast<const T*>(lnf.beta) + 8 * (i - nv));
@@ -487,11 +489,20 @@ template <class T, int BN>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
          const LnFuse& ln, cudaStream_t s) {
-  constexpr size_t smem = size_t(stages_for<BN>()) * (BM * BK * 2 + BN * BK * 2) + 1024;
-  static_assert(size_t(BM) * (BN + 1) * 4 + 1024 <= smem, "fp32 tile must fit the ring");
+  constexpr int STAGES = stages_for<BN>();
+  constexpr size_t STAGE_BYTES = BM * BK * 2 + BN * BK * 2;
+  constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
+  static_assert(size_t(BM) * (BN + 1) * 4 + 1024 <= smem_max, "fp32 tile must fit the ring");
+  constexpr int min_st = int((size_t(BM) * (BN + 1) * 4 + STAGE_BYTES - 1) / STAGE_BYTES);  // the tile fits
+  // ring depth: the full ring unless DP_GEMM_STAGES caps it (experiments), and never deeper
+  // than the K blocks a CTA streams
+  static const int env_st = getenv("DP_GEMM_STAGES") ? atoi(getenv("DP_GEMM_STAGES")) : 0;
+  int nst = env_st > 0 ? std::min(env_st, STAGES) : STAGES;
+  nst = std::max(nst, std::max(min_st, 1));
+  const size_t smem = size_t(nst) * STAGE_BYTES + 1024;
   static bool attr = false;
   if (!attr) {
-    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max));
     attr = true;
   }
   const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
@@ -505,7 +516,7 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
   const int mt = (M + BN - 1) / BN;
   launch_kernel_cluster(gemm_tc_kernel<T, BN>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem,
-                        dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, ln);
+                        dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, nst, ln);
 }
 
 template <class T>
