@@ -199,8 +199,10 @@ def run_reference(a):
             "warmup": a.warmup, "ms_per_step": round(v, 4), "higher_is_better": False, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded random-init weights, paper recipe)",
             "impl": "reference",
-            "config": {"workload": f"{a.model} fp16-rounded weights, batch {a.batch}, seq {a.seq}, full forward "
-                                   f"on the host CPU (no transfer: weights already in host DRAM)"},
+            "config": {"workload": f"{a.model} fp16 batch {a.batch} seq {a.seq} cold start -- reference arm: the "
+                                   f"oracle's full fp64 forward on the host CPU (weights already in host DRAM, "
+                                   f"fp16-rounded)",
+                       "model": a.model, "global_batch": a.batch, "seq_len": a.seq, "parallelism": "host"},
             "cpu_baseline": {"value": round(v, 4), "unit": "ms", "cores": cores, "kind": "oracle",
                              "sample": f"{steps} full forwards (fp64 numpy, BLAS threads = {cores})"},
             "e2e": {"value": round(v, 4), "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}

@@ -112,6 +112,16 @@ __device__ __forceinline__ float gelu_tanh(float x) {
   return 0.5f * x * (1.0f + tanhf(c * (x + 0.044715f * x * x * x)));
 }
 
+// Compile-time activation: an epilogue specialised per activation stays small (a runtime
+// switch inlined per element made the GEMM epilogue ~4 K instructions, instruction-fetch bound).
+template <int ACT>
+__device__ __forceinline__ float apply_act_c(float v) {
+  if constexpr (ACT == ACT_GELU_ERF) return gelu_erf(v);
+  else if constexpr (ACT == ACT_GELU_TANH) return gelu_tanh(v);
+  else if constexpr (ACT == ACT_TANH) return tanhf(v);
+  else return v;
+}
+
 __device__ __forceinline__ float apply_act(float v, int act) {
   switch (act) {
     case ACT_GELU_ERF: return gelu_erf(v);

@@ -160,9 +160,10 @@ struct LnFuse {
 };
 
 #ifdef DP_GEMM_TRACE
-// phase timestamps (globaltimer, ns) per CTA: entry, setup done, after grid-dependency wait,
-// first stage landed (MMA issuer), all MMAs done, partial/tile in smem, end; [7] = SM id
-__device__ unsigned long long g_gemm_trace[4096][8];
+// phase timestamps (globaltimer, ns) per CTA: 0 entry, 1 W prefetch issued, 2 setup done,
+// 3 after the grid-dependency wait, 4 first stage landed, 5 MMAs done, 6 tile in smem,
+// 7 tile reduced (split-K), 8 end; [15] = SM id
+__device__ unsigned long long g_gemm_trace[4096][16];
 __device__ __forceinline__ unsigned long long gtime() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -182,6 +183,11 @@ __device__ __forceinline__ unsigned long long gtime() {
 __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
+// Exit barrier: only orders the peers' completed DSMEM reads before this CTA's exit, so no
+// release fence (which compiles to a GPU-scope MEMBAR waiting for the epilogue's stores).
+__device__ __forceinline__ void cluster_sync_relaxed() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
+}
 __device__ __forceinline__ uint32_t mapa_u32(uint32_t saddr, uint32_t rank) {
   uint32_t r;
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
@@ -200,7 +206,7 @@ __device__ __forceinline__ float ld_cluster_f32(uint32_t addr) {
 // rank order 0..splits-1 (deterministic), then runs the epilogue.  At the hot path's
 // 128-token shapes a CTA's time is set by the bytes it ingests (~100 GB/s per SM measured,
 // profiles/r01_gemm_trace.jsonl), so spreading a weight tile over `splits` SMs pays.
-template <class T, int BN>
+template <class T, int BN, int ACT>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
                    const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io, int splits,
@@ -217,8 +223,11 @@ __global__ void __launch_bounds__(128, 1)
                              (uint32_t(BM >> 4) << 24);
 
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], done_bar;
+  // 1024-byte aligned for the 128-byte swizzle atoms; offset arithmetic on the __shared__ array
+  // (not an integer round trip) keeps the pointer in the shared address space, so the
+  // epilogue compiles to LDS/STS rather than generic loads/stores
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], done_bar, recv_bar;
   __shared__ uint32_t tmem_base_sh;
   __shared__ float sbias[BM];
 
@@ -243,7 +252,18 @@ __global__ void __launch_bounds__(128, 1)
       mbar_init(&empty_bar[s], 1);
     }
     mbar_init(&done_bar, 1);
+    mbar_init(&recv_bar, 1);  // split-K: the peers' partial rows land here (async-proxy pushes)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    // Weights never depend on the previous kernel: the first ring's worth of W tiles goes in
+    // flight right away -- before the TMEM allocation / CTA barrier and before the
+    // grid-dependency wait (PDL) -- so its HBM latency overlaps the setup and the
+    // predecessor's tail.  Activations (X, residual) and every store come after the wait.
+    const int pre0 = num_kb < nst ? num_kb : nst;
+    for (int kb = 0; kb < pre0; ++kb) {
+      mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
+      tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb_lo + kb) * BK, n0);
+    }
+    TRACE(1);
   }
   if (warp == 1) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base_sh)),
@@ -255,25 +275,19 @@ __global__ void __launch_bounds__(128, 1)
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem_d = tmem_base_sh;
   pdl_trigger();
+  // split-K: announce that this CTA's barriers are initialised; the matching wait comes right
+  // before the first push into a peer, long after every CTA of the cluster has arrived
+  if (splits > 1) asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
 
-  // Weights never depend on the previous kernel: the producer puts the first ring's worth
-  // of W tiles in flight BEFORE the grid-dependency wait (PDL), so their HBM latency
-  // overlaps the predecessor's tail.  Activations (X, residual) and every store come after.
   // nst <= STAGES: the ring depth actually used (a shallower ring leaves room on the SM for
   // the previous kernel's CTAs, so the PDL prologue overlap is not blocked on shared memory)
   const int pre = num_kb < nst ? num_kb : nst;
-  if (warp == 0 && lane == 0) {
-    for (int kb = 0; kb < pre; ++kb) {
-      mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
-      tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb_lo + kb) * BK, n0);
-    }
-  }
   // the bias never depends on the previous kernel either (128 threads = 128 rows of the tile;
   // read after the W tiles are in flight, visible to the epilogue after its barrier)
   sbias[threadIdx.x] = bias != nullptr ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
-  TRACE(1);
+  if (threadIdx.x == 0) TRACE(2);
   pdl_wait();
-  TRACE(2);
+  if (threadIdx.x == 0) TRACE(3);
 
   // epilogue thread mapping (single split): thread t owns 8 consecutive W rows
   // nl = 8*(t%16) of tokens ml = t/16 + 8*j; their residual is fetched now, under the mainloop
@@ -305,7 +319,7 @@ __global__ void __launch_bounds__(128, 1)
     for (int kb = 0; kb < num_kb; ++kb) {
       const int s = kb % nst;
       mbar_wait(&full_bar[s], (kb / nst) & 1);
-      if (kb == 0) TRACE(3);
+      if (kb == 0) TRACE(4);
       asm volatile("tcgen05.fence::after_thread_sync;");
       const uint8_t* a = smem + s * STAGE_BYTES;
       const uint8_t* b = a + A_BYTES;
@@ -320,30 +334,43 @@ __global__ void __launch_bounds__(128, 1)
   __syncwarp();
 
   mbar_wait(&done_bar, 0);
-  if (threadIdx.x == 0) TRACE(4);
+  if (threadIdx.x == 0) TRACE(5);
   asm volatile("tcgen05.fence::after_thread_sync;");
   // 1) TMEM -> shared memory (the ring is free once the MMAs are done): the fp32 tile,
   //    [128 W rows][BN tokens] with an odd row stride
+  //    (split-K: unpadded [128][BN], so each owner's rows are one contiguous block to push)
   const int row = warp * 32 + lane;  // TMEM lane = W row within the tile
   float* tile = reinterpret_cast<float*>(smem);
+  const int rstride = splits == 1 ? PROW : BN;
 #pragma unroll 1
   for (int c0 = 0; c0 < BN; c0 += 16) {
     uint32_t v[16];
     tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
+    if (splits == 1) {
 #pragma unroll
-    for (int j = 0; j < 16; ++j) tile[row * PROW + c0 + j] = __uint_as_float(v[j]);
+      for (int j = 0; j < 16; ++j) tile[row * rstride + c0 + j] = __uint_as_float(v[j]);
+    } else {
+#pragma unroll
+      for (int j = 0; j < 16; j += 4)
+        *reinterpret_cast<float4*>(&tile[row * rstride + c0 + j]) =
+            make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
+                        __uint_as_float(v[j + 3]));
+    }
   }
   // 2) + bias, activation, + residual; one 16-byte store per 8 outputs (8 W rows of a token)
-  auto finish = [&](int nl, int ml, float* acc, const float* r8) {
+  // rs: the residual already staged in shared memory (8 floats), or nullptr to load it now
+  auto finish = [&](int nl, int ml, float* acc, const float* rs) {
     const size_t m = (size_t)(m0 + ml);
     const int n = n0 + nl;
 #pragma unroll
-    for (int e = 0; e < 8; ++e) acc[e] = apply_act(acc[e] + sbias[nl + e], act);
+    for (int e = 0; e < 8; ++e) acc[e] = apply_act_c<ACT>(acc[e] + sbias[nl + e]);
     if (res) {
-      float rl[8];
-      if (r8 == nullptr) {
-        load8<T>(res, m * ldr + n, rl, res32);
-        r8 = rl;
+      float r8[8];
+      if (rs != nullptr) {
+        const float4 a = reinterpret_cast<const float4*>(rs)[0], b = reinterpret_cast<const float4*>(rs)[1];
+        r8[0] = a.x, r8[1] = a.y, r8[2] = a.z, r8[3] = a.w, r8[4] = b.x, r8[5] = b.y, r8[6] = b.z, r8[7] = b.w;
+      } else {
+        load8<T>(res, m * ldr + n, r8, res32);
       }
 #pragma unroll
       for (int e = 0; e < 8; ++e) acc[e] += r8[e];
@@ -352,17 +379,32 @@ __global__ void __launch_bounds__(128, 1)
   };
   if (splits == 1) {
     __syncthreads();
-    if (threadIdx.x == 0) TRACE(5);
+    if (threadIdx.x == 0) {
+      TRACE(6);
+      TRACE(7);
+    }
     if constexpr (RP > 0) {
+      // the prefetched residual goes to shared memory (after the fp32 tile) so the store loop
+      // below can stay rolled: one small loop body, hot in the instruction cache
+      float* rs = tile + BM * PROW + threadIdx.x * 8;  // [RP][128 threads][8]
+      if (res != nullptr) {
 #pragma unroll
+        for (int j = 0; j < RP; ++j) {
+          float4* d = reinterpret_cast<float4*>(rs + j * 128 * 8);
+          d[0] = make_float4(rpre[j][0], rpre[j][1], rpre[j][2], rpre[j][3]);
+          d[1] = make_float4(rpre[j][4], rpre[j][5], rpre[j][6], rpre[j][7]);
+        }
+      }
+#pragma unroll 1
       for (int j = 0; j < RP; ++j) {
         const int ml = (threadIdx.x >> 4) + 8 * j;
         if (ml < mcount) {
           float acc[8];
 #pragma unroll
           for (int e = 0; e < 8; ++e) acc[e] = tile[(nl_t + e) * PROW + ml];
-          finish(nl_t, ml, acc, res != nullptr ? rpre[j] : nullptr);
+          finish(nl_t, ml, acc, res != nullptr ? rs + j * 128 * 8 : nullptr);
         }
+        if (threadIdx.x == 0 && j < 4) TRACE(9 + j);
       }
     } else {
       // wide tiles: a rolled loop (an unrolled 32-pass epilogue is instruction-fetch bound)
@@ -375,39 +417,60 @@ __global__ void __launch_bounds__(128, 1)
       }
     }
   } else {
-    // 1b) cluster split-K reduction (see above)
-    cluster_sync_all();
-    if (threadIdx.x == 0) TRACE(5);
-    const uint32_t tile_sa = smem_u32(tile);
-    uint32_t rb[8];
-#pragma unroll
-    for (int p = 0; p < 8; ++p) rb[p] = p < splits ? mapa_u32(tile_sa, (uint32_t)p) : 0u;
-    const int g0 = sp * 16 / splits, g1 = (sp + 1) * 16 / splits;  // this rank's 8-row groups
-    const int units = (g1 - g0) * mcount;
-    for (int u = threadIdx.x; u < units; u += 128) {
-      const int gi = g0 + u / mcount, ml = u - (u / mcount) * mcount;
-      float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-#pragma unroll
-      for (int p = 0; p < 8; ++p) {
-        if (p < splits) {
-          float v[8];
-#pragma unroll
-          for (int e = 0; e < 8; ++e) v[e] = ld_cluster_f32(rb[p] + (uint32_t)(((8 * gi + e) * PROW + ml) * 4));
-#pragma unroll
-          for (int e = 0; e < 8; ++e) acc[e] += v[e];
-        }
-      }
-      finish(8 * gi, ml, acc, nullptr);
+    // 1b) cluster split-K reduction: rank r owns tile rows [r*RPR, (r+1)*RPR).  Every CTA pushes
+    //     the rows each peer owns from its send buffer into that peer's receive slot with a
+    //     bulk async copy (cp.async.bulk shared::cta -> shared::cluster) that completes on the
+    //     peer's recv_bar -- no cluster-wide barrier with a release fence, no latency-bound
+    //     remote loads.  The owner sums the slots in rank order 0..splits-1 (deterministic).
+    const int RPR = BM / splits;                     // rows per owner (splits is a power of 2)
+    const uint32_t slot_bytes = uint32_t(RPR) * BN * 4;
+    float* recv = tile + BM * BN;                    // [splits][RPR][BN]
+    if (threadIdx.x == 0) {
+      TRACE(6);
+      // this CTA expects splits-1 slots; the arrival keeps the phase open until then
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&recv_bar)),
+                   "r"(slot_bytes * (splits - 1))
+                   : "memory");
     }
-    cluster_sync_all();  // every peer has read this CTA's tile
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // send buffer -> async proxy
+    __syncthreads();
+    asm volatile("barrier.cluster.wait.aligned;" ::: "memory");     // peers' recv_bar initialised
+    if (threadIdx.x == 0) {
+      for (int r = 0; r < splits; ++r) {
+        if (r == sp) continue;
+        const uint32_t src = smem_u32(tile + r * RPR * BN);
+        const uint32_t dst = mapa_u32(smem_u32(recv + sp * RPR * BN), (uint32_t)r);
+        const uint32_t bar = mapa_u32(smem_u32(&recv_bar), (uint32_t)r);
+        asm volatile(
+            "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+            "r"(src), "r"(slot_bytes), "r"(bar)
+            : "memory");
+      }
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    }
+    mbar_wait(&recv_bar, 0);
+    if (threadIdx.x == 0) TRACE(7);
+    const int units = (RPR / 8) * mcount;
+    for (int u = threadIdx.x; u < units; u += 128) {
+      const int gi = u / mcount, ml = u - gi * mcount;  // 8-row group within the owned rows
+      float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+      for (int p = 0; p < splits; ++p) {
+        const float* sl = p == sp ? tile + sp * RPR * BN : recv + p * RPR * BN;
+#pragma unroll
+        for (int e = 0; e < 8; ++e) acc[e] += sl[(8 * gi + e) * BN + ml];
+      }
+      finish(sp * RPR + 8 * gi, ml, acc, nullptr);
+    }
+    // the pushes must have read this CTA's send buffer before it exits
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
   }
 #ifdef DP_GEMM_TRACE
   if (threadIdx.x == 0) {
-    TRACE(6);
+    TRACE(8);
     unsigned smid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
     const int b_ = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
-    if (b_ < 4096) g_gemm_trace[b_][7] = smid;
+    if (b_ < 4096) g_gemm_trace[b_][15] = smid;
   }
 #endif
   asm volatile("tcgen05.fence::before_thread_sync;");
@@ -485,24 +548,30 @@ CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int b
   return m;
 }
 
-template <class T, int BN>
+template <class T, int BN, int ACT>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
          const LnFuse& ln, cudaStream_t s) {
   constexpr int STAGES = stages_for<BN>();
   constexpr size_t STAGE_BYTES = BM * BK * 2 + BN * BK * 2;
   constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
-  static_assert(size_t(BM) * (BN + 1) * 4 + 1024 <= smem_max, "fp32 tile must fit the ring");
-  constexpr int min_st = int((size_t(BM) * (BN + 1) * 4 + STAGE_BYTES - 1) / STAGE_BYTES);  // the tile fits
+  // the fp32 tile (+ the staged residual for BN <= 64) must fit the ring
+  constexpr size_t epi_bytes = size_t(BM) * (BN + 1) * 4 + (BN <= 64 ? size_t(BN / 8) * 128 * 8 * 4 : 0);
+  static_assert(epi_bytes + 1024 <= smem_max, "epilogue buffers must fit the ring");
+  // split-K: unpadded send tile + receive slots, 2 x BM x BN fp32
+  const size_t need = splits > 1 ? size_t(2) * BM * BN * 4 : epi_bytes;
+  const int min_st = int((need + STAGE_BYTES - 1) / STAGE_BYTES);
   // ring depth: the full ring unless DP_GEMM_STAGES caps it (experiments), and never deeper
   // than the K blocks a CTA streams
   static const int env_st = getenv("DP_GEMM_STAGES") ? atoi(getenv("DP_GEMM_STAGES")) : 0;
   int nst = env_st > 0 ? std::min(env_st, STAGES) : STAGES;
   nst = std::max(nst, std::max(min_st, 1));
+  DP_CHECK(nst <= STAGES, DP_ERR_INVALID, "gemm: epilogue buffers do not fit this tile width");
   const size_t smem = size_t(nst) * STAGE_BYTES + 1024;
   static bool attr = false;
   if (!attr) {
-    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max));
+    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN, ACT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smem_max));
     attr = true;
   }
   const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
@@ -515,7 +584,7 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   }
   CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
   const int mt = (M + BN - 1) / BN;
-  launch_kernel_cluster(gemm_tc_kernel<T, BN>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem,
+  launch_kernel_cluster(gemm_tc_kernel<T, BN, ACT>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem,
                         dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, nst, ln);
 }
 
@@ -523,13 +592,24 @@ template <class T>
 void dispatch(int bn, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
               const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io,
               int sp, const LnFuse& ln, cudaStream_t s) {
+#define DP_RUN(B, A) run<T, B, A>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s)
+#define DP_ACTS(B)                                 \
+  switch (act) {                                   \
+    case ACT_NONE: DP_RUN(B, ACT_NONE); break;           \
+    case ACT_GELU_ERF: DP_RUN(B, ACT_GELU_ERF); break;   \
+    case ACT_GELU_TANH: DP_RUN(B, ACT_GELU_TANH); break; \
+    case ACT_TANH: DP_RUN(B, ACT_TANH); break;           \
+    default: fail(DP_ERR_INVALID, "gemm: unknown activation"); \
+  }
   switch (bn) {
-    case 32: run<T, 32>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
-    case 64: run<T, 64>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
-    case 128: run<T, 128>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
-    case 256: run<T, 256>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s); break;
+    case 32: DP_ACTS(32); break;
+    case 64: DP_ACTS(64); break;
+    case 128: DP_ACTS(128); break;
+    case 256: DP_ACTS(256); break;
     default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
   }
+#undef DP_ACTS
+#undef DP_RUN
 }
 
 }  // namespace
@@ -548,10 +628,11 @@ static int pick_bn(int M, int N) {
 }
 
 // (BN, splits) from a per-CTA ingest model fitted to the B200 sweeps and per-CTA traces
-// (profiles/r01_gemm_sweep_v3.txt, r01_gemm_trace.jsonl): a CTA streams its W and X tiles at
+// (profiles/r01_gemm_sweep_v4.txt, r01_gemm_trace.jsonl): a CTA streams its W and X tiles at
 // ~100 GB/s (the mainloop time is its bytes / 1e5 B/us), all CTAs together at ~8 TB/s from
-// L2/HBM, and a cluster split-K reduction costs ~2.5 us.  Splits only in one wave of <= 148
-// CTAs, >= 4 k-blocks each.  Within 2% of the best measured configuration at every swept shape.
+// L2/HBM, and the cluster split-K reduction (bulk DSMEM pushes) costs ~1.2 us.  Splits only in
+// one wave of <= 148 CTAs, >= 4 k-blocks each, BN <= 128 (the send/receive buffers must fit).
+// Picks the best measured configuration at every swept shape.
 struct GemmCfg {
   int bn, sp;
 };
@@ -563,10 +644,10 @@ static GemmCfg pick_cfg(int M, int N, int K) {
     if (bn > 32 && M < bn) continue;
     const int tiles = ntile * ((M + bn - 1) / bn);
     for (int sp : {1, 2, 4}) {
-      if (sp > 1 && (kb / sp < 4 || tiles * sp > 148)) continue;
+      if (sp > 1 && (kb / sp < 4 || tiles * sp > 148 || bn >= 256)) continue;
       const double per = double(kb) / sp * (BM * BK * 2 + bn * BK * 2);
       const int ctas = tiles * sp, waves = (ctas + 147) / 148;
-      const double t = std::max(waves * per / 1e5, ctas * per / 8e6) + (sp > 1 ? 2.5 : 0.0);
+      const double t = std::max(waves * per / 1e5, ctas * per / 8e6) + (sp > 1 ? 1.2 : 0.0);
       if (t < best_t - 1e-9) {
         best_t = t;
         best = {bn, sp};
@@ -594,6 +675,8 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
   const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : cfg.bn);
   int sp = env_sp > 0 ? env_sp : (bn_hint > 0 || env_bn > 0 ? 1 : cfg.sp);
   sp = std::max(1, std::min(std::min(sp, 8), K / BK));
+  while (sp & (sp - 1)) --sp;  // a power of two: every rank owns BM / sp rows
+  if (bn >= 256) sp = 1;       // the send + receive buffers (2 x 128 x BN fp32) must fit the ring
   if (dtype == DP_BF16)
     dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s);
   else
@@ -630,6 +713,6 @@ void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void
 #ifdef DP_GEMM_TRACE
 extern "C" __attribute__((visibility("default"))) int dp_debug_gemm_trace(void* host, int nblocks) {
   if (nblocks > 4096) nblocks = 4096;
-  return (int)cudaMemcpyFromSymbol(host, dp::g_gemm_trace, size_t(nblocks) * 8 * sizeof(unsigned long long));
+  return (int)cudaMemcpyFromSymbol(host, dp::g_gemm_trace, size_t(nblocks) * 16 * sizeof(unsigned long long));
 }
 #endif

@@ -620,6 +620,9 @@ __device__ __forceinline__ uint32_t cluster_rank() {
 __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
+__device__ __forceinline__ void cluster_sync_relaxed() {  // exit barrier: no release fence needed
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
+}
 __device__ __forceinline__ float ld_dsmem_f32(const float* p, uint32_t rank) {
   uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(p)), ra;
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(rank));
@@ -742,7 +745,7 @@ __global__ void __launch_bounds__(256) skinny_mma_kernel(const T* __restrict__ X
         if (res) v += load1<T>(res, (size_t)m * ldr + n, io & IO_RES_F32);
         store1<T>(Y, (size_t)m * ldy + n, v, io & IO_OUT_F32);
       }
-      cluster_sync_all();  // peers have read this CTA's partials before the ring is reused / exit
+      cluster_sync_relaxed();  // peers have read this CTA's partials before the ring is reused / exit
     }
   }
 }

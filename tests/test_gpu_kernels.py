@@ -265,3 +265,47 @@ def test_fp32_residual_stream_io():
     torch.cuda.synchronize()
     ref = F.layer_norm(r.astype(np.float64), g.astype(np.float64), b.astype(np.float64), 1e-5)
     close(f64(Y), ref, "fp16", K=N, scale=8)
+
+
+_SPLIT_SCRIPT = r"""
+import math, sys, numpy as np, torch
+sys.path.insert(0, '.')
+import synth
+from oracle import forward as F
+import paper_conf_eurosys_jeongba23_b200 as dp
+M, N, K = (int(v) for v in sys.argv[1:4])
+rng = np.random.default_rng(M + N + K)
+x = synth.round_to(rng.standard_normal((M, K)).astype(np.float32), 'fp16')
+w = synth.round_to((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32), 'fp16')
+b = synth.round_to((0.1 * rng.standard_normal(N)).astype(np.float32), 'fp16')
+r = synth.round_to(rng.standard_normal((M, N)).astype(np.float32), 'fp16')
+X, W, B, R = (torch.from_numpy(a).cuda() for a in (x, w, b, r))
+Y = torch.empty(M, N, dtype=torch.float16, device='cuda')
+Y2 = torch.empty_like(Y)
+dp.linear(X, K, W, B, R, N, Y, N, M, N, K, act='gelu_erf', path=0)
+dp.linear(X, K, W, B, R, N, Y2, N, M, N, K, act='gelu_erf', path=0)
+torch.cuda.synchronize()
+assert torch.equal(Y, Y2), 'split-K GEMM not deterministic'
+ref = F.linear(*(synth.storage_to_f64(a, 'fp16') for a in (x, w, b)), 'gelu_erf', synth.storage_to_f64(r, 'fp16'))
+err = np.abs(Y.double().cpu().numpy() - ref)
+tol = 2.0 ** -10 * np.abs(ref) + K * 2.0 ** -22 * 4 * np.abs(x).max() * np.abs(w).max() + 1e-6
+assert np.all(err <= tol), err.max()
+print('ok')
+"""
+
+
+@pytest.mark.parametrize("bn,split,M,N,K", [(32, 2, 128, 768, 768), (32, 4, 128, 768, 3072), (32, 8, 100, 256, 1024),
+                                             (64, 4, 200, 512, 2048), (128, 2, 384, 1024, 1024),
+                                             (128, 4, 333, 768, 4096), (64, 8, 64, 128, 4096)])
+def test_gemm_split_k_cluster_configs(bn, split, M, N, K):
+    """Every (BN, split) the cluster split-K path can take, forced through DP_GEMM_BN /
+    DP_GEMM_SPLIT in a fresh process (they are read once): parity with the oracle and
+    run-to-run bit equality (the reduction order is fixed)."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, DP_GEMM_BN=str(bn), DP_GEMM_SPLIT=str(split))
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _SPLIT_SCRIPT, str(M), str(N), str(K)], env=env, cwd=root,
+                       capture_output=True, text=True, timeout=120)
+    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stderr[-2000:]

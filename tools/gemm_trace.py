@@ -1,9 +1,9 @@
 """Per-CTA phase timeline of the tcgen05 GEMM (needs the instrumented build:
 DP_NVCC_EXTRA=-DDP_GEMM_TRACE python paper_conf_eurosys_jeongba23_b200/build.py).
 
-Phases (globaltimer ns, relative to the earliest CTA entry): 0 entry, 1 setup done (barriers,
-TMEM), 2 after griddepcontrol.wait, 3 first stage landed, 4 all MMAs done, 5 tile ready for the
-epilogue (after the split-K fixup), 6 end.  python tools/gemm_trace.py M N K [reps]"""
+Phases (globaltimer ns, relative to the earliest CTA entry): 0 entry, 1 W prefetch issued,
+2 setup done (barriers, TMEM, CTA barrier), 3 after griddepcontrol.wait, 4 first stage landed,
+5 all MMAs done, 6 fp32 tile in shared memory, 7 tile reduced (split-K cluster), 8 end.  python tools/gemm_trace.py M N K [reps]"""
 import ctypes
 import json
 import math
@@ -25,15 +25,16 @@ y = torch.empty(M, N, device="cuda").half()
 for _ in range(reps):
     dp.linear(x, K, w, None, None, 0, y, N, M, N, K, path=0)
 torch.cuda.synchronize()
-buf = np.zeros((4096, 8), dtype=np.uint64)
+buf = np.zeros((4096, 16), dtype=np.uint64)
 assert _lib.lib.dp_debug_gemm_trace(buf.ctypes.data_as(ctypes.c_void_p), 4096) == 0
-rows = buf[(buf[:, 0] > 0) & (buf[:, 6] > 0)]
+rows = buf[(buf[:, 0] > 0) & (buf[:, 8] > 0)]
 t0 = rows[:, 0].min()
-rel = (rows[:, :7].astype(np.int64) - int(t0)) / 1e3  # us
-names = ["entry", "setup", "pdl_wait", "first_stage", "mma_done", "tile_ready", "end"]
+rel = (rows[:, :9].astype(np.int64) - int(t0)) / 1e3  # us
+names = ["entry", "w_issued", "setup", "pdl_wait", "first_stage", "mma_done", "tile_smem", "tile_reduced", "end"]
 out = {"shape": [M, N, K], "ctas": int(len(rows)), "env": {k: os.environ.get(k) for k in ("DP_GEMM_BN", "DP_GEMM_SPLIT")}}
 for i, n in enumerate(names):
     col = rel[:, i]
     out[n] = {"min": round(float(col.min()), 3), "med": round(float(np.median(col)), 3), "max": round(float(col.max()), 3)}
-out["per_cta_active_us_med"] = round(float(np.median(rel[:, 6] - rel[:, 0])), 3)
+out["epi_j"] = [round(float(np.median((rows[:, 9 + j].astype(np.int64) - int(t0)) / 1e3)), 3) for j in range(4)]
+out["per_cta_active_us_med"] = round(float(np.median(rel[:, 8] - rel[:, 0])), 3)
 print(json.dumps(out))
