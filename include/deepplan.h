@@ -162,7 +162,10 @@ typedef struct {
   int64_t tail_bytes;     /* the last DMA piece of a link carries at most this many bytes
                              (a unit suffix), so little compute remains after the last byte
                              lands [2 MiB]; 0 = off */
-  int32_t reserved[2];
+  int32_t persistent;     /* 1 = warm runs execute every layer in ONE persistent kernel (K6: grid =
+                             #SMs, grid barriers between ops, next GEMM's weights prefetched under
+                             the current op) when all layer units are resident [0] */
+  int32_t reserved[1];
 } dp_engine_opts;
 dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* opts);
 dp_status dp_context_get_opts(dp_context* ctx, dp_engine_opts* out);

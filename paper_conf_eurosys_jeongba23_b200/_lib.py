@@ -51,7 +51,7 @@ class EngineOpts(C.Structure):
     _fields_ = [("chunk_bytes", C.c_int64), ("n_h2d_streams", C.c_int32), ("use_graph", C.c_int32),
                 ("gemm_bn", C.c_int32), ("debug_delay_us", C.c_int32), ("debug_poison", C.c_int32),
                 ("use_pdl", C.c_int32), ("fuse_ln", C.c_int32), ("tail_bytes", C.c_int64),
-                ("reserved", C.c_int32 * 2)]
+                ("persistent", C.c_int32), ("reserved", C.c_int32 * 1)]
 
 
 class ModelConfig(C.Structure):
@@ -273,7 +273,7 @@ class Context:
         self.devs = list(devs)
 
     def set_opts(self, chunk_bytes=None, n_h2d_streams=None, use_graph=None, gemm_bn=None, debug_delay_us=None,
-                 debug_poison=None, use_pdl=None, tail_bytes=None, fuse_ln=None):
+                 debug_poison=None, use_pdl=None, tail_bytes=None, fuse_ln=None, persistent=None):
         o = EngineOpts()
         _check(lib.dp_context_get_opts(self.h, C.byref(o)))
         if chunk_bytes is not None:
@@ -294,6 +294,8 @@ class Context:
             o.tail_bytes = int(tail_bytes)
         if fuse_ln is not None:
             o.fuse_ln = 1 if fuse_ln else 0
+        if persistent is not None:
+            o.persistent = 1 if persistent else 0
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))
 
     def peer_init(self, uid: bytes, rank: int, nranks: int):

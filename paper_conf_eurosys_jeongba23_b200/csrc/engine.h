@@ -59,6 +59,7 @@ struct ForwardArgs {
   int bn_hint = 0;
   bool pdl = false;  // chain kernels with programmatic dependent launch (opts.use_pdl)
   bool fuse_ln = false;  // LayerNorm in the preceding GEMM's epilogue (opts.fuse_ln)
+  bool persistent = false;  // all layers in one K6 launch when every layer unit is resident
 };
 
 void ensure_workspace(dp_model* m, int dev, int64_t tokens);

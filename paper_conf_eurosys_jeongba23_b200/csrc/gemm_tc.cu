@@ -37,96 +37,60 @@
 #include "kernels.h"
 #include "launch.cuh"
 #include "ln.cuh"
+#include "tc.cuh"
 
 namespace dp {
+
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  DP_CHECK(fn != nullptr, DP_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  return fn;
+}
+
+CUtensorMap make_kmajor_map(const void* base, int dtype, int rows, int K, int ld, int box_rows) {
+  CUtensorMap m;
+  std::memset(&m, 0, sizeof(m));
+  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
+  cuuint32_t box[2] = {64u, (cuuint32_t)box_rows};  // 64 elements = one 128-byte swizzle row
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = get_encode()(&m, dtype == DP_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16,
+                            2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  DP_CHECK(r == CUDA_SUCCESS, DP_ERR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+  return m;
+}
+
+// Generic tiled map (no swizzle): rank 1..3, dims/strides in elements / bytes (strides of
+// dims 1.., as cuTensorMapEncodeTiled takes them).  Used for K6's TMA stores.
+CUtensorMap make_plain_map(const void* base, CUtensorMapDataType dt, int rank, const uint64_t* dims,
+                           const uint64_t* strides_bytes, const uint32_t* box) {
+  CUtensorMap m;
+  std::memset(&m, 0, sizeof(m));
+  cuuint64_t d[3], st[2];
+  cuuint32_t bx[3], es[3] = {1, 1, 1};
+  for (int i = 0; i < rank; ++i) d[i] = dims[i], bx[i] = box[i];
+  for (int i = 0; i + 1 < rank; ++i) st[i] = strides_bytes[i];
+  CUresult r = get_encode()(&m, dt, rank, const_cast<void*>(base), d, st, bx, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  DP_CHECK(r == CUDA_SUCCESS, DP_ERR_CUDA, "cuTensorMapEncodeTiled (plain) failed (" + std::to_string((int)r) + ")");
+  return m;
+}
 
 namespace {
 
 constexpr int BM = 128;  // W rows per tile (MMA M)
 constexpr int BK = 64;   // K per stage: 64 x 2 B = one 128-byte swizzle row
-
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
-}
-
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-               : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
-  const uint32_t a = smem_u32(bar);
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@!P1 bra WAIT_%=;\n"
-      "}\n" ::"r"(a),
-      "r"(phase)
-      : "memory");
-}
-
-__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-          smem_u32(dst)),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar))
-      : "memory");
-}
-
-__device__ __forceinline__ uint64_t sw128_desc(const void* smem_tile) {
-  const uint64_t addr = smem_u32(smem_tile);
-  uint64_t d = 0;
-  d |= (addr & 0x3FFFFull) >> 4;  // start address
-  d |= uint64_t(1) << 16;          // LBO (unused for swizzled K-major)
-  d |= uint64_t(1024 >> 4) << 32;  // SBO: 8 rows x 128 B
-  d |= uint64_t(1) << 46;          // descriptor version (sm_100)
-  d |= uint64_t(2) << 61;          // SWIZZLE_128B
-  return d;
-}
-
-__device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "setp.ne.b32 p, %4, 0;\n"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
-      "}\n" ::"r"(tmem_d),
-      "l"(a), "l"(b), "r"(idesc), "r"(acc));
-}
-
-__device__ __forceinline__ void umma_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
-               : "memory");
-}
-
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-        "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-      : "r"(taddr));
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-}
-
-
-
-
-template <class T>
-struct FmtBits;
-template <>
-struct FmtBits<__half> {
-  static constexpr uint32_t v = 0;
-};
-template <>
-struct FmtBits<__nv_bfloat16> {
-  static constexpr uint32_t v = 1;
-};
 
 // Ring depth per tile width: as many stages as ~224 KB of shared memory holds (<= 12), so a
 // K = 768 layer (12 k-blocks) has its whole weight slice in flight at once.
@@ -180,14 +144,6 @@ __device__ __forceinline__ unsigned long long gtime() {
   } while (0)
 #endif
 
-__device__ __forceinline__ void cluster_sync_all() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-// Exit barrier: only orders the peers' completed DSMEM reads before this CTA's exit, so no
-// release fence (which compiles to a GPU-scope MEMBAR waiting for the epilogue's stores).
-__device__ __forceinline__ void cluster_sync_relaxed() {
-  asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
-}
 __device__ __forceinline__ uint32_t mapa_u32(uint32_t saddr, uint32_t rank) {
   uint32_t r;
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
@@ -518,36 +474,6 @@ __global__ void __launch_bounds__(128, 1)
   }
 }
 
-PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-  static std::once_flag once;
-  std::call_once(once, [] {
-    void* p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
-  });
-  DP_CHECK(fn != nullptr, DP_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
-  return fn;
-}
-
-// 2D K-major tile map: rows x K elements with row stride ld (elements), box {64, box_rows}.
-CUtensorMap make_map(const void* base, int dtype, int rows, int K, int ld, int box_rows) {
-  CUtensorMap m;
-  std::memset(&m, 0, sizeof(m));
-  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
-  cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
-  cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)box_rows};
-  cuuint32_t estr[2] = {1, 1};
-  CUresult r = get_encode()(&m, dtype == DP_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16,
-                            2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  DP_CHECK(r == CUDA_SUCCESS, DP_ERR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
-  return m;
-}
-
 template <class T, int BN, int ACT>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
@@ -578,11 +504,11 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   GemmGroup g;
   std::memset(&g, 0, sizeof(g));
   for (int i = 0; i < ngroups; ++i) {
-    g.w[i] = make_map(w[i], dtype, N, K, K, BM);
+    g.w[i] = make_kmajor_map(w[i], dtype, N, K, K, BM);
     g.bias[i] = bias ? bias[i] : nullptr;
     g.ycol[i] = ycol ? ycol[i] : 0;
   }
-  CUtensorMap mx = make_map(x, dtype, M, K, ldx, BN);
+  CUtensorMap mx = make_kmajor_map(x, dtype, M, K, ldx, BN);
   const int mt = (M + BN - 1) / BN;
   launch_kernel_cluster(gemm_tc_kernel<T, BN, ACT>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem,
                         dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, nst, ln);

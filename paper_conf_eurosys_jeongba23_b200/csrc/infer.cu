@@ -561,8 +561,9 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.bn_hint = ctx->opts.gemm_bn;
     a.pdl = ctx->opts.use_pdl != 0;
     a.fuse_ln = ctx->opts.fuse_ln != 0;
+    a.persistent = ctx->opts.persistent != 0;
     if (ctx->opts.use_graph) {
-      std::string key = "warm|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
+      std::string key = "warm|" + std::to_string(a.persistent) + "|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
                         graph_key(ctx, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);
       dp_run_stats gs = run_graph(ds, key, (cudaStream_t)stream, [&](cudaStream_t cs) {
         a.stream = cs;
@@ -615,6 +616,7 @@ extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
         cudaDeviceSynchronize();
         for (auto& kv : ds.graphs) cudaGraphExecDestroy(kv.second.exec);
         ds.graphs.clear();
+        ds.persist.clear();
         if (ds.capture) cudaStreamDestroy(ds.capture);
         if (ds.dbase) cudaFree(ds.dbase);
         if (ds.ws.base) cudaFree(ds.ws.base);

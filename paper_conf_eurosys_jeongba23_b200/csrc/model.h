@@ -52,6 +52,8 @@ struct Workspace {
   void* base = nullptr;
 };
 
+struct PersistProgram;  // K6 (persist.h)
+
 struct GraphEntry {
   cudaGraphExec_t exec = nullptr;
   dp_run_stats stats{};
@@ -64,6 +66,8 @@ struct DevState {
   Workspace ws;
   std::map<std::string, GraphEntry> graphs;  // captured cold / warm runs (opts.use_graph)
   cudaStream_t capture = nullptr;            // private stream the graphs are captured on
+  // K6 programs per (batch, seq, workspace): their tensor maps point into dbase and ws
+  std::map<std::string, std::shared_ptr<PersistProgram>> persist;
 };
 
 std::vector<ParamDesc> config_params(const dp_model_config& c);
