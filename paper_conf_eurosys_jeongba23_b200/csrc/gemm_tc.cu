@@ -121,6 +121,7 @@ struct LnFuse {
   int ldo;
   float eps;
   int* cnt;           // per m-tile arrival counters, zero between launches (the last CTA resets)
+  float* out32;       // optional fp32 copy of the LN output (BERT's residual stream), [M, ldo]
 };
 
 #ifdef DP_GEMM_TRACE
@@ -467,7 +468,7 @@ __global__ void __launch_bounds__(128, 1)
         __syncthreads();
         for (int tk = warp; tk < nr; tk += 4)
           ln_row_warp<T, 6, 2>(zs, nullptr, (size_t)tk * N, N, lnf.eps, out32, gb, static_cast<T*>(lnf.out),
-                               (size_t)(m0 + r0 + tk) * lnf.ldo);
+                               (size_t)(m0 + r0 + tk) * lnf.ldo, lnf.out32);
       }
       if (threadIdx.x == 0) lnf.cnt[blockIdx.y] = 0;
     }
@@ -612,7 +613,7 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
 void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
                           const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
                           int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
-  const LnFuse none{nullptr, nullptr, nullptr, 0, 0.f, nullptr};
+  const LnFuse none{nullptr, nullptr, nullptr, 0, 0.f, nullptr, nullptr};
   gemm_impl(dtype, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, bn_hint, none, s);
 }
 
@@ -621,11 +622,11 @@ bool gemm_ln_supported(int N) { return N % 8 == 0 && N <= 6 * 256; }
 void launch_gemm_tc_ln(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                        void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, const void* gamma,
                        const void* beta, float eps, void* ln_out, int ldo, int* counters, int ncounters,
-                       cudaStream_t s) {
+                       cudaStream_t s, void* ln_out32) {
   DP_CHECK(gamma && beta && ln_out && counters, DP_ERR_INVALID, "fused LayerNorm: missing buffers");
   DP_CHECK(gemm_ln_supported(N) && ldo % 8 == 0, DP_ERR_UNSUPPORTED, "fused LayerNorm: N <= 1536, multiple of 8");
   DP_CHECK((M + 31) / 32 <= ncounters, DP_ERR_INVALID, "fused LayerNorm: too few m-tile counters");
-  const LnFuse ln{gamma, beta, ln_out, ldo, eps, counters};
+  const LnFuse ln{gamma, beta, ln_out, ldo, eps, counters, static_cast<float*>(ln_out32)};
   gemm_impl(dtype, x, ldx, 1, &w, &bias, nullptr, res, ldr, y, ldy, M, N, K, act, io, bn_hint, ln, s);
 }
 

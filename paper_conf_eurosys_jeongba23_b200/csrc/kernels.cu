@@ -33,7 +33,7 @@ template <class T, int VPL>
 __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ ids, int ntok, int seq, int pos_off,
                                                     const T* word, const T* pos, const T* type, const T* g,
                                                     const T* b, int H, float eps, void* __restrict__ out_,
-                                                    int out_f32) {
+                                                    int out_f32, float* __restrict__ out32) {
   extern __shared__ uint4 sm[];  // [type0 | gamma | beta] as 16-byte vectors
   pdl_trigger();
   const int nv = H / 8;
@@ -131,6 +131,7 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
 #pragma unroll
       for (int e = 0; e < 8; ++e) y[e] = (x[v][e] - mean) * rstd * gg[e] + bb[e];
       store8<T>(out_, (size_t)t * H + 8 * c, y, out_f32);
+      if (out32 != nullptr) store8<T>(out32, (size_t)t * H + 8 * c, y, 1);  // fp32 residual-stream copy
     }
   }
 }
@@ -138,14 +139,14 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
 template <class T>
 static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                     const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
-                    cudaStream_t s) {
+                    float* out32, cudaStream_t s) {
   const int warps = 8;
   dim3 grid((ntok + warps - 1) / warps);
   const size_t sm = size_t(3) * (H / 8) * 16;
   const int vpl = (H / 8 + 31) / 32;
 #define DP_EMB(V)                                                                                      \
   launch_kernel(embed_kernel<T, V>, grid, dim3(warps * 32), sm, s, ids, ntok, seq, pos_off, (const T*)word, \
-                (const T*)pos, (const T*)type, (const T*)g, (const T*)b, H, eps, out, (int)out_f32)
+                (const T*)pos, (const T*)type, (const T*)g, (const T*)b, H, eps, out, (int)out_f32, out32)
   switch (vpl) {
     case 1: DP_EMB(1); break;
     case 2: DP_EMB(2); break;
@@ -161,14 +162,16 @@ static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const vo
 
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                   const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
-                  cudaStream_t s) {
+                  cudaStream_t s, void* out32) {
   DP_CHECK(H % 8 == 0 && H > 0, DP_ERR_INVALID, "hidden must be a multiple of 8");
   DP_CHECK(seq > 0 && ntok >= 0, DP_ERR_INVALID, "bad token counts");
   if (ntok == 0) return;
   if (dtype == DP_BF16)
-    embed_t<__nv_bfloat16>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, s);
+    embed_t<__nv_bfloat16>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32,
+                           static_cast<float*>(out32), s);
   else
-    embed_t<__half>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, s);
+    embed_t<__half>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, static_cast<float*>(out32),
+                    s);
 }
 
 // -------------------------------------------------------------------------------------
@@ -177,7 +180,7 @@ void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off,
 template <class T, int VPL>
 __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__ x, const void* __restrict__ r,
                                                         const T* g, const T* b, T* __restrict__ y, int rows,
-                                                        int n, float eps, int in_f32) {
+                                                        int n, float eps, int in_f32, float* __restrict__ y32) {
   extern __shared__ uint4 sm[];  // [gamma | beta]
   pdl_trigger();
   const int nv = n / 8;
@@ -187,12 +190,12 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__
   const int lane = threadIdx.x & 31;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
   for (int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); row < rows; row += nwarps)
-    ln_row_warp<T, VPL, 0>(x, r, (size_t)row * n, n, eps, in_f32, sm, y, (size_t)row * n);
+    ln_row_warp<T, VPL, 0>(x, r, (size_t)row * n, n, eps, in_f32, sm, y, (size_t)row * n, y32);
 }
 
 template <class T>
 static void layernorm_t(const void* x, const void* r, const void* g, const void* b, void* y, int rows, int n,
-                        float eps, bool in_f32, cudaStream_t s) {
+                        float eps, bool in_f32, float* y32, cudaStream_t s) {
   // one row per warp (latency: every row's loads in flight at once); gamma/beta are read
   // once per CTA, so a DHA LayerNorm costs rows/8 x 4H bytes of host reads
   const int warps = 8;
@@ -203,7 +206,7 @@ static void layernorm_t(const void* x, const void* r, const void* g, const void*
   const int vpl = (n / 8 + 31) / 32;
 #define DP_LN(V)                                                                                       \
   launch_kernel(layernorm_kernel<T, V>, dim3(grid), dim3(warps * 32), sm, s, x, r, (const T*)g, (const T*)b, (T*)y, \
-                rows, n, eps, (int)in_f32)
+                rows, n, eps, (int)in_f32, y32)
   switch (vpl) {
     case 1: DP_LN(1); break;
     case 2: DP_LN(2); break;
@@ -218,13 +221,13 @@ static void layernorm_t(const void* x, const void* r, const void* g, const void*
 }
 
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
-                      int n, float eps, bool in_f32, cudaStream_t s) {
+                      int n, float eps, bool in_f32, cudaStream_t s, void* y32) {
   DP_CHECK(n % 8 == 0 && n > 0, DP_ERR_INVALID, "LN width must be a multiple of 8");
   if (rows <= 0) return;
   if (dtype == DP_BF16)
-    layernorm_t<__nv_bfloat16>(x, r, g, b, y, rows, n, eps, in_f32, s);
+    layernorm_t<__nv_bfloat16>(x, r, g, b, y, rows, n, eps, in_f32, static_cast<float*>(y32), s);
   else
-    layernorm_t<__half>(x, r, g, b, y, rows, n, eps, in_f32, s);
+    layernorm_t<__half>(x, r, g, b, y, rows, n, eps, in_f32, static_cast<float*>(y32), s);
 }
 
 // -------------------------------------------------------------------------------------

@@ -14,11 +14,11 @@ enum Io { IO_RES_F32 = 1, IO_OUT_F32 = 2 };
 // host-mapped (direct-host-access).  ln_g == nullptr -> no LN (GPT-2).
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                   const void* type, const void* ln_g, const void* ln_b, int H, float eps, void* out, bool out_f32,
-                  cudaStream_t s);
+                  cudaStream_t s, void* out32 = nullptr);  // out32: optional fp32 copy of the LN output
 
 // K4: y = LN(x (+ r)) * g + b; g/b may be host-mapped.
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
-                      int n, float eps, bool in_f32, cudaStream_t s);
+                      int n, float eps, bool in_f32, cudaStream_t s, void* y32 = nullptr);  // y32: optional fp32 copy
 
 // K3: skinny linear reading W exactly once (W may be host-mapped) -- a11.
 void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
@@ -36,7 +36,7 @@ bool gemm_ln_supported(int N);
 void launch_gemm_tc_ln(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                        void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, const void* gamma,
                        const void* beta, float eps, void* ln_out, int ldo, int* counters, int ncounters,
-                       cudaStream_t s);
+                       cudaStream_t s, void* ln_out32 = nullptr);
 bool gemm_tc_supported(int N, int K);
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);

@@ -37,7 +37,7 @@ __device__ __forceinline__ void load8_generic(const void* base, size_t i, float*
 // SRC: 0 = read-only global path, 1 = L2-coherent global, 2 = generic (shared memory).
 template <class T, int VPL, int SRC>
 __device__ __forceinline__ void ln_row_warp(const void* x, const void* r, size_t off, int n, float eps, int in_f32,
-                                            const uint4* gb, T* y, size_t yoff) {
+                                            const uint4* gb, T* y, size_t yoff, float* y32 = nullptr) {
   const int lane = threadIdx.x & 31, nv = n / 8;
   float v[VPL][8];
   float sum = 0.f;
@@ -85,6 +85,7 @@ __device__ __forceinline__ void ln_row_warp(const void* x, const void* r, size_t
 #pragma unroll
       for (int e = 0; e < 8; ++e) o[e] = (v[k][e] - mean) * rstd * gg[e] + bb[e];
       reinterpret_cast<uint4*>(y + yoff)[c] = pack8<T>(o);
+      if (y32 != nullptr) store8<T>(y32, yoff + 8 * c, o, 1);  // fp32 residual-stream copy
     }
   }
 }

@@ -44,9 +44,11 @@ struct Workspace {
   void* x = nullptr;    // [T, H]
   void* qkv = nullptr;  // [T, 3H]
   void* ctx = nullptr;  // [T, H]
-  void* tmp = nullptr;  // [T, H]
+  void* tmp = nullptr;  // [T, H] fp32 (pre-LayerNorm sums)
   void* x1 = nullptr;   // [T, H]
   void* h = nullptr;    // [T, F]
+  void* xr = nullptr;   // [T, H] fp32: BERT/RoBERTa residual stream (copy of x)
+  void* x1r = nullptr;  // [T, H] fp32: copy of x1
   int* ln_cnt = nullptr;  // per-32-token-tile counters of the GEMM-fused LayerNorm (zeroed)
   int n_ln_cnt = 0;
   void* base = nullptr;

@@ -81,6 +81,7 @@ struct POp {
   const void* beta;
   float eps;
   void* zout;              // optional z (pre-LN) [rows][cols]
+  float* out32;            // optional fp32 copy of the LayerNorm output (BERT residual stream)
   void* out;               // [rows][cols] storage dtype (out_final: the kernel's `final_out`)
   // ATTN
   const void* qkv;
@@ -273,7 +274,9 @@ __device__ __forceinline__ void reduce_ln_rows(const POp& op, int b, int G, void
       const int c = t + 128 * e;
       const float g = Cvt<T>::to1(static_cast<const T*>(op.gamma)[c]);
       const float be = Cvt<T>::to1(static_cast<const T*>(op.beta)[c]);
-      static_cast<T*>(out)[row + c] = Cvt<T>::from1((z[e] - mean) * rstd * g + be);
+      const float y = (z[e] - mean) * rstd * g + be;
+      static_cast<T*>(out)[row + c] = Cvt<T>::from1(y);
+      if (op.out32 != nullptr) op.out32[row + c] = y;
     }
     named_sync(1, 128);  // red[] free for the next row
   }
@@ -758,10 +761,13 @@ std::shared_ptr<PersistProgram> build_persist_program(dp_model* m, int dev, int 
       gemm(ws.x, H, {q, k, v}, H, H, true, {second(q), second(k), second(v)}, ACT_NONE, ws.qkv, 3 * H);
       attn(false);
       int sp = gemm(ws.ctx, H, {ao}, H, H, false, {}, 0, nullptr, 0);
-      reduce(sp, H, {second(ao)}, ACT_NONE, ws.x, 0, ln1, nullptr, 0, ws.x1, false);
+      // fp32 residual stream (xr / x1r), as in the per-kernel path (R21)
+      ops[reduce(sp, H, {second(ao)}, ACT_NONE, ws.xr, 1, ln1, nullptr, 0, ws.x1, false)].out32 =
+          static_cast<float*>(ws.x1r);
       gemm(ws.x1, H, {fc1}, F, H, true, {second(fc1)}, ACT_GELU_ERF, ws.h, F);
       sp = gemm(ws.h, F, {fc2}, H, F, false, {}, 0, nullptr, 0);
-      reduce(sp, H, {second(fc2)}, ACT_NONE, ws.x1, 0, ln2, nullptr, 0, ws.x, l == L - 1);
+      ops[reduce(sp, H, {second(fc2)}, ACT_NONE, ws.x1r, 1, ln2, nullptr, 0, ws.x, l == L - 1)].out32 =
+          l == L - 1 ? nullptr : static_cast<float*>(ws.xr);
     }
   } else {
     const int first_ln = 2;  // wte, wpe, then ln_1 of block 0

@@ -289,3 +289,21 @@ def test_fused_layernorm_bit_identical(name, S):
     assert kern[1] == kern[0] - 2 * m.layers
     model.close()
     c.close()
+
+
+def test_bert_base_batched_cold_start():
+    """Batching (Fig. 12): BERT-Base fp16, batch 4 x seq 128, the default link-aware
+    plan from a live profile at that batch, vs the fp64 oracle."""
+    m = synth.SHAPES["bert_base"]
+    dtype = "fp16"
+    w = synth.make_weights(m, seed=2, dtype=dtype)
+    ids = synth.make_ids(m, 4, 128, seed=3)
+    ref, ref_pool = F.forward(m, w, ids, dtype)
+    model = dp().Model(ctx(), m, w, dtype)
+    cost = model.profile(0, 4, 128, iters=3)
+    plan = dp().plan_generate(cost, "DHA_LINK", 1)
+    out, pool, st = run_cold(model, plan, ids, dtype)
+    model.evict(0)
+    assert np.abs(f64(out) - ref.reshape(4 * 128, -1)).max() <= 1e-2
+    assert np.abs(f64(pool) - ref_pool).max() <= 1e-2
+    model.close()
