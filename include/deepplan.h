@@ -289,6 +289,17 @@ dp_status dp_infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int32
 dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, const int32_t* d_ids, int32_t batch,
                         int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats);
 
+/* GPT-2 tied language-model head ("logits", R14): logits[r][v] =
+ * sum_h hidden[r][h] * wte[v][h] for r < rows, fp32, row stride = vocab.  d_hidden: rows
+ * vectors of `hidden` storage-dtype elements with row stride ld_hidden (e.g. the last
+ * position of every sequence of a forward's d_out: ld_hidden = seq*hidden, d_hidden pointing
+ * at token seq-1).  wte is read from HBM when the model is resident on dev with its wte unit
+ * loaded, else in place from the pinned host arena (direct-host-access: every byte of the
+ * table crosses the link once).  Enqueued on `stream`.  DP_ERR_UNSUPPORTED for
+ * BERT/RoBERTa; DP_ERR_INVALID on bad arguments. */
+dp_status dp_lm_head(dp_context* ctx, dp_model* m, int32_t dev, const void* d_hidden, int32_t ld_hidden,
+                     int32_t rows, float* d_logits, void* stream);
+
 /* Residency: make the model non-resident on dev (its HBM slots return to the pool).
  * Synchronises the device's streams first. */
 dp_status dp_model_evict(dp_context* ctx, dp_model* m, int32_t dev);

@@ -148,3 +148,11 @@ def linear(x: np.ndarray, w_nk: np.ndarray, b: np.ndarray | None = None, act: st
     if residual is not None:
         y = y + residual
     return y
+
+
+def lm_head(m: ModelShape, weights, hidden: np.ndarray, dtype: str = "fp16") -> np.ndarray:
+    """GPT-2's tied language-model head (the "logits" of P:241 read literally):
+    logits = hidden . wte^T over the whole vocabulary, f64.  hidden: [..., H]."""
+    if m.family != "gpt2":
+        raise ValueError("tied LM head: GPT-2 only")
+    return np.asarray(hidden, dtype=np.float64) @ _w(weights, "wte.weight", dtype).T

@@ -133,6 +133,7 @@ _sig("dp_infer_cold", [vp, vp, C.POINTER(Plan), C.c_int32, i32p, C.c_int32, vp, 
                        C.POINTER(RunStats)])
 _sig("dp_infer_warm", [vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp, vp, C.POINTER(RunStats)])
 _sig("dp_model_evict", [vp, vp, C.c_int32])
+_sig("dp_lm_head", [vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp])
 _sig("dp_model_is_resident", [vp, C.c_int32])
 _sig("dp_host_alloc", [C.c_int64, C.POINTER(vp)])
 _sig("dp_host_free", [vp])
@@ -435,6 +436,15 @@ class Model:
         _check(lib.dp_infer_warm(self.ctx.h, self.h, int(dev), _dptr(ids), B, S, _dptr(out), _dptr(pooled),
                                  _stream_ptr(stream), C.byref(st)))
         return _stats(st)
+
+    def lm_head(self, dev: int, hidden, logits, rows: int | None = None, ld_hidden: int | None = None,
+                stream=None):
+        """GPT-2 tied LM head (dp_lm_head): logits[r] = hidden_row_r . wte^T (fp32).  `hidden` is a
+        device tensor whose first element is row 0; rows are ld_hidden elements apart."""
+        rows = rows if rows is not None else logits.shape[0]
+        ld = ld_hidden if ld_hidden is not None else self.shape.hidden
+        _check(lib.dp_lm_head(self.ctx.h, self.h, int(dev), _dptr(hidden), int(ld), int(rows), _dptr(logits),
+                              _stream_ptr(stream)))
 
     def evict(self, dev: int):
         _check(lib.dp_model_evict(self.ctx.h, self.h, int(dev)))

@@ -587,6 +587,23 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
   });
 }
 
+extern "C" dp_status dp_lm_head(dp_context* ctx, dp_model* m, int32_t dev, const void* d_hidden, int32_t ld_hidden,
+                                int32_t rows, float* d_logits, void* stream) {
+  return guard([&] {
+    DP_CHECK(ctx && m && d_hidden && d_logits, DP_ERR_INVALID, "NULL argument");
+    DP_CHECK(m->cfg.family == DP_FAMILY_GPT2, DP_ERR_UNSUPPORTED, "tied LM head: GPT-2 models only");
+    DP_CHECK(rows >= 0 && ld_hidden >= m->cfg.hidden && ld_hidden % 8 == 0, DP_ERR_INVALID, "bad rows / ld_hidden");
+    ctx->on(dev);
+    DeviceGuard g(dev);
+    const DevState& ds = m->dev[dev];
+    // unit 0 = wte; its weight is the first parameter of the unit
+    const bool in_hbm = ds.resident && !ds.method.empty() && ds.method[0] == DP_LOAD;
+    const void* wte = in_hbm ? static_cast<const void*>(m->device(dev, 0)) : static_cast<const void*>(m->host(0));
+    launch_skinny_linear(m->cfg.dtype, d_hidden, ld_hidden, wte, nullptr, nullptr, 0, d_logits, m->cfg.vocab, rows,
+                         m->cfg.vocab, m->cfg.hidden, ACT_NONE, IO_OUT_F32, (cudaStream_t)stream);
+  });
+}
+
 extern "C" dp_status dp_model_evict(dp_context* ctx, dp_model* m, int32_t dev) {
   return guard([&] {
     DP_CHECK(ctx && m, DP_ERR_INVALID, "NULL context/model");

@@ -314,6 +314,119 @@ __global__ void __launch_bounds__(256) skinny_linear_kernel(const T* __restrict_
   }
 }
 
+// K3 variant for M <= 8 rows and K = 256 * VPL <= 1024 (the pooler, GPT-2's LM head): a
+// streaming GEMV.  One warp per output column n (a W row), two rows per iteration: every lane
+// issues its 2 x VPL 16-byte loads of the two rows before any FMA, so ~2 x K x 2 bytes per warp
+// are in flight; X sits in shared memory as fp32.  W is read exactly once (host-mapped or HBM),
+// no shared-memory staging of W (the skinny kernel above stages W as fp32 for reuse across
+// many tokens, which a 1..4-row GEMV does not need).
+template <class T, int MR, int VPL>
+__global__ void __launch_bounds__(256) gemv_kernel(const T* __restrict__ X, int ldx, const T* W, const T* bias,
+                                                   const void* res, int ldr, void* Y, int ldy, int M, int N,
+                                                   int act, int io) {
+  constexpr int K = 256 * VPL;
+  extern __shared__ float xs[];  // [MR][K]
+  pdl_trigger();
+  const int lane = threadIdx.x & 31;
+  const int gw = blockIdx.x * 8 + (threadIdx.x >> 5), nw = gridDim.x * 8;
+  // weights never depend on the previous kernel: the first two rows are in flight before the
+  // grid-dependency wait
+  uint4 wa[VPL], wb[VPL];
+  int n = gw;
+  auto fetch = [&](uint4* dst, int row) {
+#pragma unroll
+    for (int v = 0; v < VPL; ++v)
+      if (row < N) dst[v] = ldg16(W + (size_t)row * K + 8 * (lane + 32 * v));
+  };
+  fetch(wa, n);
+  fetch(wb, n + nw);
+  pdl_wait();
+  for (int i = threadIdx.x; i < MR * K / 8; i += 256) {
+    const int m = i / (K / 8), c = i - m * (K / 8);
+    float f[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+    if (m < M) unpack8<T>(ldg16(X + (size_t)m * ldx + 8 * c), f);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) xs[m * K + 8 * c + e] = f[e];
+  }
+  __syncthreads();
+  for (; n < N; n += 2 * nw) {
+    float acc[2][MR];
+#pragma unroll
+    for (int t = 0; t < 2; ++t)
+#pragma unroll
+      for (int m = 0; m < MR; ++m) acc[t][m] = 0.f;
+#pragma unroll
+    for (int v = 0; v < VPL; ++v) {
+      float a[8], b[8];
+      unpack8<T>(wa[v], a);
+      unpack8<T>(wb[v], b);
+#pragma unroll
+      for (int m = 0; m < MR; ++m) {
+        const float4* xp = reinterpret_cast<const float4*>(xs + m * K + 8 * (lane + 32 * v));
+        const float4 x0 = xp[0], x1 = xp[1];
+        const float xv[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          acc[0][m] = fmaf(xv[e], a[e], acc[0][m]);
+          acc[1][m] = fmaf(xv[e], b[e], acc[1][m]);
+        }
+      }
+    }
+    const int n0 = n, n1 = n + nw;
+    fetch(wa, n + 2 * nw);  // the next two rows stream while this pair is reduced and stored
+    fetch(wb, n + 3 * nw);
+#pragma unroll
+    for (int t = 0; t < 2; ++t) {
+      const int row = t == 0 ? n0 : n1;
+#pragma unroll
+      for (int m = 0; m < MR; ++m) acc[t][m] = warp_sum(acc[t][m]);
+      if (lane == 0 && row < N) {
+        const float bz = bias ? Cvt<T>::to1(bias[row]) : 0.f;
+#pragma unroll
+        for (int m = 0; m < MR; ++m) {
+          if (m < M) {
+            float v = apply_act(acc[t][m] + bz, act);
+            if (res) v += load1<T>(res, (size_t)m * ldr + row, io & IO_RES_F32);
+            store1<T>(Y, (size_t)m * ldy + row, v, io & IO_OUT_F32);
+          }
+        }
+      }
+    }
+  }
+}
+
+template <class T, int MR>
+static void gemv_mr(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
+                    int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
+  const size_t sm = size_t(MR) * K * 4;
+  int grid = (N + 15) / 16;  // 8 warps x 2 rows per CTA per pass
+  if (grid > 148 * 8) grid = 148 * 8;
+#define DP_GEMV(V)                                                                                           \
+  launch_kernel(gemv_kernel<T, MR, V>, dim3(grid), dim3(256), sm, s, (const T*)x, ldx, (const T*)w, (const T*)bias, \
+                res, ldr, y, ldy, M, N, act, io)
+  switch (K / 256) {
+    case 1: DP_GEMV(1); break;
+    case 2: DP_GEMV(2); break;
+    case 3: DP_GEMV(3); break;
+    case 4: DP_GEMV(4); break;
+    default: fail(DP_ERR_UNSUPPORTED, "gemv: K must be 256..1024");
+  }
+#undef DP_GEMV
+}
+
+bool gemv_supported(int M, int K, int ldx, const void* x) {
+  return M >= 1 && M <= 8 && K % 256 == 0 && K <= 1024 && ldx % 8 == 0 && ((uintptr_t)x % 16) == 0;
+}
+
+template <class T>
+static void gemv_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y, int ldy,
+                   int M, int N, int K, int act, int io, cudaStream_t s) {
+  if (M == 1) gemv_mr<T, 1>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+  else if (M == 2) gemv_mr<T, 2>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+  else if (M <= 4) gemv_mr<T, 4>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+  else gemv_mr<T, 8>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+}
+
 template <class T>
 static void skinny_t(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
                      int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
@@ -346,6 +459,13 @@ void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, cons
       skinny_mma_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
     else
       skinny_mma_t<__half>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+    return;
+  }
+  if (gemv_supported(M, K, ldx, x)) {
+    if (dtype == DP_BF16)
+      gemv_t<__nv_bfloat16>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
+    else
+      gemv_t<__half>(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, io, s);
     return;
   }
   DP_CHECK(size_t(8) * K * 4 <= 200 * 1024, DP_ERR_UNSUPPORTED, "skinny linear: K too large");

@@ -229,6 +229,55 @@ def make_poisson_trace(n_req: int, rate_per_s: float, n_instances: int, seed: in
     return arrival_ns, inst
 
 
+def make_maf_like_trace(duration_s: float, rate_per_s: float, n_instances: int, seed: int = 7, *,
+                        zipf_a: float = 1.1, swing: float = 0.5, period_s: float | None = None,
+                        spikes_per_min: float = 6.0, spike_s: float = 1.5, spike_gain: float = 20.0,
+                        spike_frac: float = 0.05, bin_s: float = 0.05):
+    """A synthetic stand-in for the Azure Functions (MAF) trace of P:342-350 (the real trace
+    is not available offline): "heavy sustained requests, fluctuations in request rates, and
+    spikes in requests", mapped to the n instances.
+
+    * popularity: instance i gets share ~ 1 / (rank_i)^zipf_a (a random permutation of ranks),
+      so a few instances are hot and sustained and most are rare;
+    * fluctuation: the offered load is rate * (1 + swing * sin(2 pi t / period)) (period =
+      duration / 3 by default);
+    * spikes: Poisson spike events (spikes_per_min); each multiplies the rate of a random
+      spike_frac of the instances by spike_gain for spike_s seconds.
+    The base load is normalised so the mean offered rate (without spikes) is rate_per_s.
+    Arrivals are a piecewise-constant-rate Poisson process on bins of bin_s seconds.
+    Returns (arrival_ns int64[n], instance int32[n]), sorted by arrival."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    period_s = period_s or duration_s / 3.0
+    ranks = rng.permutation(n_instances) + 1
+    share = 1.0 / ranks.astype(np.float64) ** zipf_a
+    share /= share.sum()
+    nb = int(np.ceil(duration_s / bin_s))
+    t0 = np.arange(nb) * bin_s
+    g = 1.0 + swing * np.sin(2 * np.pi * (t0 + 0.5 * bin_s) / period_s)
+    lam = np.outer(g * rate_per_s * bin_s, share)  # [bins, instances] expected counts
+    n_spikes = rng.poisson(spikes_per_min * duration_s / 60.0)
+    for _ in range(n_spikes):
+        start = rng.uniform(0, duration_s)
+        b0, b1 = int(start / bin_s), int(min(duration_s, start + spike_s) / bin_s) + 1
+        hot = rng.choice(n_instances, size=max(1, int(round(spike_frac * n_instances))), replace=False)
+        lam[b0:b1, hot] *= spike_gain
+    counts = rng.poisson(lam)
+    times, insts = [], []
+    for b in range(nb):
+        row = counts[b]
+        nz = np.nonzero(row)[0]
+        for i in nz:
+            k = int(row[i])
+            times.append(t0[b] + rng.uniform(0, bin_s, size=k))
+            insts.append(np.full(k, i, dtype=np.int32))
+    if not times:
+        return np.zeros(0, np.int64), np.zeros(0, np.int32)
+    t = np.concatenate(times)
+    inst = np.concatenate(insts)
+    order = np.argsort(t, kind="stable")
+    return np.round(t[order] * 1e9).astype(np.int64), inst[order]
+
+
 def instance_models(n_instances: int, ratio=(4, 4, 1)) -> np.ndarray:
     """Model index per instance following a mix ratio (4:4:1 BERT/RoBERTa/GPT-2)."""
     tot = sum(ratio)

@@ -126,7 +126,9 @@ def test_linear_tcgen05_parity(M, N, K, dtype):
 
 
 @pytest.mark.parametrize("M,N,K", [(1, 768, 768), (5, 128, 64), (128, 768, 768), (128, 3072, 768),
-                                   (128, 768, 3072), (384, 1024, 4096), (17, 2304, 768)])
+                                   (128, 768, 3072), (384, 1024, 4096), (17, 2304, 768),
+                                   # M <= 8, K in 256..1024: the streaming GEMV (pooler, LM head), ragged N
+                                   (2, 1001, 256), (3, 50257, 1024), (4, 129, 512), (6, 3072, 1024), (8, 777, 768)])
 @pytest.mark.parametrize("dtype", ["fp16", "bf16"])
 def test_linear_skinny_dha_parity_and_bit_identity(M, N, K, dtype):
     rng = np.random.default_rng(M + 3 * N + K)

@@ -200,3 +200,29 @@ def test_unit_counts_and_fp16_bytes():
         m = synth.SHAPES[name]
         assert len(U.unit_params(m)) == n
         assert U.model_bytes(m, "fp16") == nb
+
+
+def test_lm_head_matches_transformers_gpt2_lm_head():
+    """The oracle's tied LM head = transformers' GPT2LMHeadModel logits (same state dict, f64)."""
+    import torch
+    from transformers import GPT2Config, GPT2LMHeadModel
+    m = synth.SHAPES["tiny_gpt2"]
+    dtype = "fp16"
+    w = synth.make_weights(m, seed=9, dtype=dtype)
+    ids = synth.make_ids(m, 2, 19, seed=4)
+    x, _ = F.forward(m, w, ids, dtype)
+    logits = F.lm_head(m, w, x, dtype)
+    cfg = GPT2Config(vocab_size=m.vocab, n_embd=m.hidden, n_layer=m.layers, n_head=m.heads, n_positions=m.max_pos,
+                     n_inner=m.ffn, activation_function="gelu_new", layer_norm_epsilon=m.ln_eps, resid_pdrop=0.0,
+                     embd_pdrop=0.0, attn_pdrop=0.0, attn_implementation="eager", tie_word_embeddings=True)
+    model = GPT2LMHeadModel(cfg).double().eval()
+    sd = {"transformer." + k: torch.from_numpy(synth.storage_to_f64(v, dtype)) for k, v in w.items()}
+    missing, unexpected = model.load_state_dict(sd, strict=False)
+    assert not unexpected, unexpected
+    assert model.lm_head.weight.data_ptr() == model.transformer.wte.weight.data_ptr()  # tied
+    with torch.no_grad():
+        ref = model(input_ids=torch.from_numpy(ids.astype(np.int64))).logits.numpy()
+    assert logits.shape == (2, 19, m.vocab)
+    assert np.max(np.abs(logits - ref)) < 1e-9
+    with pytest.raises(ValueError):
+        F.lm_head(synth.SHAPES["tiny_bert"], w, x, dtype)

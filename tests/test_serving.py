@@ -59,3 +59,39 @@ def test_metrics():
     r = {"finish_ns": np.array([10, 30, 200]), "cold": np.array([1, 0, 1])}
     m = OS.metrics([0, 0, 0], r, slo_ns=100)
     assert m["goodput"] == pytest.approx(2 / 3) and m["cold_rate"] == pytest.approx(2 / 3)
+
+
+def test_maf_like_trace_properties():
+    """The synthetic MAF-like trace: deterministic per seed, mean rate
+    near the requested one, heavy-tailed popularity (hot sustained instances), and burstier
+    than Poisson (index of dispersion of per-second counts > 1)."""
+    arr, inst = synth.make_maf_like_trace(60.0, 150.0, 200, seed=3, spikes_per_min=0)
+    arr2, inst2 = synth.make_maf_like_trace(60.0, 150.0, 200, seed=3, spikes_per_min=0)
+    assert np.array_equal(arr, arr2) and np.array_equal(inst, inst2)
+    assert np.all(np.diff(arr) >= 0) and arr[0] >= 0 and arr[-1] < 60e9
+    assert abs(len(arr) / 60.0 - 150.0) < 0.1 * 150.0
+    counts = np.bincount(inst, minlength=200)
+    top = np.sort(counts)[::-1]
+    assert top[:20].sum() > 0.5 * len(arr)  # the hottest 10% of instances carry most requests
+    per_s = np.bincount((arr // 1_000_000_000).astype(np.int64), minlength=60)
+    assert per_s.var() / per_s.mean() > 3.0  # rate swings: far from Poisson (dispersion 1)
+    # spikes add load on a few instances for a short time
+    arr_s, inst_s = synth.make_maf_like_trace(60.0, 150.0, 200, seed=3, spikes_per_min=10)
+    assert len(arr_s) > len(arr)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_dry_run_matches_oracle_maf_like(seed):
+    rng = np.random.default_rng(100 + seed)
+    ninst = int(rng.integers(50, 300))
+    ngpu = int(rng.integers(1, 9))
+    cold, warm, rb = _table(3, rng)
+    moi = synth.instance_models(ninst, (4, 4, 1))
+    arr, inst = synth.make_maf_like_trace(8.0, float(rng.integers(50, 300)), ninst, seed=seed)
+    budget = int(rb.max() * rng.integers(1, 30))
+    kw = dict(ngpu=ngpu, per_gpu_budget_bytes=budget, cold_ns=cold, warm_ns=warm, resident_bytes=rb,
+              model_of_instance=moi)
+    got = dp.serve_run(arr, inst, dry_run=True, **kw)
+    ref = OS.replay(arr, inst, **kw)
+    for k in ref:
+        assert np.array_equal(got[k], ref[k]), k

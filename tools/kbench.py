@@ -1,7 +1,7 @@
 """Per-kernel device timings through the C-ABI hooks (CUDA events around back-to-back
 launches on one stream, after warm-up).  Used with ncu too:
   ncu --set full -k regex:gemm_tc -c 3 python tools/kbench.py gemm
-python tools/kbench.py [all|gemm|ln|attn|skinny|embed] [reps]"""
+python tools/kbench.py [all|gemm|ln|attn|skinny|embed|lmhead] [reps]"""
 import json
 import math
 import os
@@ -75,6 +75,18 @@ if which in ("all", "skinny"):
         us_d = timeit(lambda: dp.linear(x, K, wd, None, None, 0, y, N, M, N, K, path=1), n=20)
         res[f"skinny M{M} N{N} K{K}"] = {"us_host": round(us_h, 2), "pcie_gbs": round(N * K * 2 / us_h / 1e3, 1),
                                         "us_hbm": round(us_d, 2)}
+        dp.host_free(wh)
+if which in ("all", "lmhead"):
+    # GPT-2 tied LM head (dp_lm_head's kernel): wte [V, H] read once, from HBM or from host
+    for (V, H, M) in [(50257, 768, 1), (50257, 1024, 1), (50257, 1024, 8)]:
+        x = torch.randn(M, H, device="cuda").half()
+        wh = dp.host_alloc(V * H * 2)
+        wd = (torch.randn(V, H, device="cuda") * 0.02).half()
+        y = torch.empty(M, V, device="cuda", dtype=torch.float32)
+        us_h = timeit(lambda: dp.linear(x, H, wh, None, None, 0, y, V, M, V, H, path=1, io=2), n=10)
+        us_d = timeit(lambda: dp.linear(x, H, wd, None, None, 0, y, V, M, V, H, path=1, io=2), n=20)
+        res[f"lm_head V{V} H{H} rows{M}"] = {"us_host": round(us_h, 1), "pcie_gbs": round(V * H * 2 / us_h / 1e3, 1),
+                                            "us_hbm": round(us_d, 2), "hbm_gbs": round(V * H * 2 / us_d / 1e3, 1)}
         dp.host_free(wh)
 if which in ("all", "embed"):
     V, P, H, S = 30522, 512, 768, 128

@@ -47,6 +47,10 @@ def main():
     ap.add_argument("--requests", type=int, default=600)
     ap.add_argument("--slo-ms", type=float, default=10.0)
     ap.add_argument("--modes", default="PIPESWITCH,DHA,DHA_LINK")
+    ap.add_argument("--trace", default="poisson", choices=["poisson", "maf"],
+                    help="poisson (P:328) or the synthetic MAF-like bursty trace (P:342-350, SURVEY f2)")
+    ap.add_argument("--duration", type=float, default=20.0, help="maf: trace seconds (rate x duration requests)")
+    ap.add_argument("--window", type=float, default=1.0, help="maf: seconds per timeline window (Fig. 15)")
     a = ap.parse_args()
     mix = [(n, int(s), int(wt)) for n, s, wt in (x.split(":") for x in a.mix.split(","))]
     ctx = dp.Context(list(range(a.gpus)))
@@ -65,8 +69,12 @@ def main():
         else np.zeros(a.instances, np.int32)
     insts = [bases[moi[i]].clone() for i in range(a.instances)]  # the bases are profiling-only
     budget = int(a.fit * bases[0].nbytes)
-    arr, inst = synth.make_poisson_trace(a.requests, a.rate, a.instances, seed=11)
-    report = {"mix": a.mix, "gpus": a.gpus, "instances": a.instances, "rate_rps": a.rate, "requests": a.requests,
+    if a.trace == "maf":
+        arr, inst = synth.make_maf_like_trace(a.duration, a.rate, a.instances, seed=11)
+        a.requests = len(arr)
+    else:
+        arr, inst = synth.make_poisson_trace(a.requests, a.rate, a.instances, seed=11)
+    report = {"trace": a.trace, "mix": a.mix, "gpus": a.gpus, "instances": a.instances, "rate_rps": a.rate, "requests": a.requests,
               "slo_ms": a.slo_ms, "per_gpu_budget_bytes": budget, "modes": {}}
     for mode in a.modes.split(","):
         k = a.gpus if mode.startswith("PT") else 1
@@ -96,17 +104,25 @@ def main():
                 if i.is_resident(g):
                     i.evict(g)
 
-        def summarize(r):
+        def summarize(r, timeline=False):
             lat = (r["finish_ns"] - arr) / 1e6
-            return {"p99_ms": round(float(np.percentile(lat, 99)), 3), "p50_ms": round(float(np.median(lat)), 3),
-                    "goodput": round(float(np.mean(lat <= a.slo_ms)), 4),
-                    "cold_rate": round(float(np.mean(r["cold"])), 4),
-                    "throughput_rps": round(len(lat) / ((r["finish_ns"].max() - arr.min()) / 1e9), 1)}
+            out = {"p99_ms": round(float(np.percentile(lat, 99)), 3), "p50_ms": round(float(np.median(lat)), 3),
+                   "goodput": round(float(np.mean(lat <= a.slo_ms)), 4),
+                   "cold_rate": round(float(np.mean(r["cold"])), 4),
+                   "throughput_rps": round(len(lat) / ((r["finish_ns"].max() - arr.min()) / 1e9), 1)}
+            if timeline and a.trace == "maf":  # Fig. 15: offered load and p99 / goodput per window
+                w = (arr // int(a.window * 1e9)).astype(np.int64)
+                out["timeline"] = [{"t_s": int(k * a.window), "offered_rps": round(float(np.sum(w == k)) / a.window, 1),
+                                    "p99_ms": round(float(np.percentile(lat[w == k], 99)), 3),
+                                    "goodput": round(float(np.mean(lat[w == k] <= a.slo_ms)), 4),
+                                    "cold_rate": round(float(np.mean(r["cold"][w == k])), 4)}
+                                   for k in np.unique(w)]
+            return out
         report["modes"][mode] = {
             "per_model": {mix[mi][0]: {"cold_ms": cold[mi] / 1e6, "warm_ms": warm[mi] / 1e6,
                                        "resident_mb": round(resident[mi] / 2 ** 20, 1),
                                        "dha_units": int(plans[mi].method.sum())} for mi in range(len(mix))},
-            "live": summarize(live), "replay": summarize(dry)}
+            "live": summarize(live, timeline=True), "replay": summarize(dry)}
     print(json.dumps(report))
 
 
