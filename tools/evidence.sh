@@ -26,6 +26,7 @@ full skinny_dha skinny skinny 3
 full embed_dha embed embed 3
 full attention attn attention 3
 full layernorm ln layernorm 3
+full lmhead_hbm lmhead gemv 16
 timeout 900 python tools/plan_compare.py > $o/plan_compare.json 2> $o/plan_compare.err
 timeout 600 python tools/serve_bench.py --mix bert_base:128:4,roberta_base:384:4,gpt2:1024:1 --instances 45 \
   --fit 8 --rate 200 --requests 600 --slo-ms 20 > $o/serve_mix.json 2> $o/serve_mix.err

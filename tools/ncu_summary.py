@@ -52,7 +52,10 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 
 
 def report(path):
-    txt = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    if path.endswith(".csv"):  # the raw page exported on the GPU box (the .ncu-rep may not travel back)
+        txt = open(path).read()
+    else:
+        txt = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(txt)))
     hdr, units = rows[0], rows[1]
     out = []
@@ -77,6 +80,8 @@ ALGO = {
     "embed_dha": {"shape": "S128 H768, tables in pinned host memory", "host_bytes": (2 * 128 + 3) * 768 * 2},
     "attention": {"shape": "B1 S128 H768 12 heads", "flops": 4 * 128 * 128 * 768},
     "layernorm": {"shape": "128 x 768", "bytes": 2 * 2 * 128 * 768},
+    "lmhead_hbm": {"shape": "GPT-2 tied LM head, 1 row, V50257 H768, wte in HBM (streaming GEMV)",
+                   "bytes": 2 * 50257 * 768},
 }
 
 
@@ -86,6 +91,9 @@ def bundle(d, launches_csv, peaks):
     out = {"kernels": {}, "bench_step_launches": launches(launches_csv, 86) if launches_csv else None}
     for name, algo in ALGO.items():
         path = f"{d}/full_{name}.ncu-rep"
+        import os
+        if not os.path.exists(path):
+            path = f"{d}/full_{name}.raw.csv"
         try:
             r = report(path)[0]
         except Exception as e:  # noqa: BLE001
