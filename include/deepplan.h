@@ -157,8 +157,9 @@ typedef struct {
   int32_t use_pdl;        /* chain consecutive kernels with programmatic dependent launch:
                              a kernel's weight prefetch overlaps its predecessor [1] */
   int32_t fuse_ln;        /* 1 = a LayerNorm that follows a resident-weight linear runs in
-                             that GEMM's epilogue (bit-identical results; measured slower on
-                             B200 at 128 tokens: the last CTA's row tail is serial) [0] */
+                             that GEMM's epilogue (a cluster along N exchanges per-token
+                             statistics over DSMEM; deterministic; measured slower on B200 at
+                             128 tokens) [0] */
   int64_t tail_bytes;     /* the last DMA piece of a link carries at most this many bytes
                              (a unit suffix), so little compute remains after the last byte
                              lands [2 MiB]; 0 = off */

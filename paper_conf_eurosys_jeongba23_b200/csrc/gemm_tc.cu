@@ -109,21 +109,6 @@ struct GemmGroup {
   long long ycol[3];
 };
 
-// Optional LayerNorm over complete output rows (K2 + K4 fused; BERT's post-LN after
-// attn-out / fc2, GPT-2's pre-LN after the residual projections): every CTA of an m-tile
-// bumps that tile's counter once its outputs are stored; the LAST one normalises the m-tile's
-// BN rows (z = the stored GEMM output, full N) with the same per-row code as the LayerNorm
-// kernel (ln.cuh), so fused and unfused results are bit-identical.
-struct LnFuse {
-  const void* gamma;  // [N] (T); nullptr = no LayerNorm
-  const void* beta;
-  void* out;          // [M, ldo] (T)
-  int ldo;
-  float eps;
-  int* cnt;           // per m-tile arrival counters, zero between launches (the last CTA resets)
-  float* out32;       // optional fp32 copy of the LN output (BERT's residual stream), [M, ldo]
-};
-
 #ifdef DP_GEMM_TRACE
 // phase timestamps (globaltimer, ns) per CTA: 0 entry, 1 W prefetch issued, 2 setup done,
 // 3 after the grid-dependency wait, 4 first stage landed, 5 MMAs done, 6 tile in smem,
@@ -167,7 +152,7 @@ template <class T, int BN, int ACT>
 __global__ void __launch_bounds__(128, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
                    const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io, int splits,
-                   int nst, const LnFuse lnf) {
+                   int nst) {
   constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
@@ -435,50 +420,12 @@ __global__ void __launch_bounds__(128, 1)
   if (warp == 1) {
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_d), "r"(TMEM_COLS));
   }
-  if (lnf.gamma != nullptr) {
-    // 3) fused LayerNorm of complete rows (see LnFuse)
-    __shared__ int ln_last;
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) ln_last = atomicAdd(&lnf.cnt[blockIdx.y], 1) == (int)(gridDim.x * gridDim.z) - 1;
-    __syncthreads();
-    if (ln_last) {
-      __threadfence();
-      // the m-tile's complete rows (written by every CTA of the tile) are staged into shared
-      // memory with cp.async -- all in flight at once, one L2 round trip -- then normalised
-      // row by row from there (the ring is free)
-      const int nv = N / 8, esz = out32 ? 4 : 2;
-      uint4* gb = reinterpret_cast<uint4*>(smem);  // [gamma | beta]
-      uint8_t* zs = smem + ((2 * nv * 16 + 1023) & ~1023);
-      const int RING = nst * STAGE_BYTES;
-      const int rows_per = (RING - (int)(zs - smem)) / (N * esz);
-      for (int i = threadIdx.x; i < 2 * nv; i += 128)
-        gb[i] = ldg16(i < nv ? static_cast<const T*>(lnf.gamma) + 8 * i : static_cast<const T*>(lnf.beta) + 8 * (i - nv));
-      const int vrow = N * esz / 16;  // 16-byte vectors per row
-      for (int r0 = 0; r0 < mcount; r0 += rows_per) {
-        const int nr = min(rows_per, mcount - r0);
-        __syncthreads();  // previous chunk consumed
-        for (int i = threadIdx.x; i < nr * vrow; i += 128) {
-          const int r = i / vrow, c = i - r * vrow;
-          const uint8_t* src = static_cast<const uint8_t*>(Y) + ((size_t)(m0 + r0 + r) * ldy) * esz + (size_t)c * 16;
-          const uint32_t dst = smem_u32(zs + (size_t)r * N * esz + (size_t)c * 16);
-          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
-        }
-        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-        __syncthreads();
-        for (int tk = warp; tk < nr; tk += 4)
-          ln_row_warp<T, 6, 2>(zs, nullptr, (size_t)tk * N, N, lnf.eps, out32, gb, static_cast<T*>(lnf.out),
-                               (size_t)(m0 + r0 + tk) * lnf.ldo, lnf.out32);
-      }
-      if (threadIdx.x == 0) lnf.cnt[blockIdx.y] = 0;
-    }
-  }
 }
 
 template <class T, int BN, int ACT>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
-         const LnFuse& ln, cudaStream_t s) {
+         cudaStream_t s) {
   constexpr int STAGES = stages_for<BN>();
   constexpr size_t STAGE_BYTES = BM * BK * 2 + BN * BK * 2;
   constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
@@ -512,14 +459,14 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   CUtensorMap mx = make_kmajor_map(x, dtype, M, K, ldx, BN);
   const int mt = (M + BN - 1) / BN;
   launch_kernel_cluster(gemm_tc_kernel<T, BN, ACT>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem,
-                        dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, nst, ln);
+                        dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, nst);
 }
 
 template <class T>
 void dispatch(int bn, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
               const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io,
-              int sp, const LnFuse& ln, cudaStream_t s) {
-#define DP_RUN(B, A) run<T, B, A>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s)
+              int sp, cudaStream_t s) {
+#define DP_RUN(B, A) run<T, B, A>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s)
 #define DP_ACTS(B)                                 \
   switch (act) {                                   \
     case ACT_NONE: DP_RUN(B, ACT_NONE); break;           \
@@ -586,7 +533,7 @@ static GemmCfg pick_cfg(int M, int N, int K) {
 
 static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
                       const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act,
-                      int io, int bn_hint, const LnFuse& ln, cudaStream_t s) {
+                      int io, int bn_hint, cudaStream_t s) {
   DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
   DP_CHECK(ngroups >= 1 && ngroups <= 3, DP_ERR_INVALID, "gemm: 1..3 weight groups");
   DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0, DP_ERR_INVALID, "GEMM activations must be 16-byte aligned");
@@ -605,29 +552,15 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
   while (sp & (sp - 1)) --sp;  // a power of two: every rank owns BM / sp rows
   if (bn >= 256) sp = 1;       // the send + receive buffers (2 x 128 x BN fp32) must fit the ring
   if (dtype == DP_BF16)
-    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s);
+    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
   else
-    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, ln, s);
+    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
 }
 
 void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
                           const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
                           int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
-  const LnFuse none{nullptr, nullptr, nullptr, 0, 0.f, nullptr, nullptr};
-  gemm_impl(dtype, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, bn_hint, none, s);
-}
-
-bool gemm_ln_supported(int N) { return N % 8 == 0 && N <= 6 * 256; }
-
-void launch_gemm_tc_ln(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
-                       void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, const void* gamma,
-                       const void* beta, float eps, void* ln_out, int ldo, int* counters, int ncounters,
-                       cudaStream_t s, void* ln_out32) {
-  DP_CHECK(gamma && beta && ln_out && counters, DP_ERR_INVALID, "fused LayerNorm: missing buffers");
-  DP_CHECK(gemm_ln_supported(N) && ldo % 8 == 0, DP_ERR_UNSUPPORTED, "fused LayerNorm: N <= 1536, multiple of 8");
-  DP_CHECK((M + 31) / 32 <= ncounters, DP_ERR_INVALID, "fused LayerNorm: too few m-tile counters");
-  const LnFuse ln{gamma, beta, ln_out, ldo, eps, counters, static_cast<float*>(ln_out32)};
-  gemm_impl(dtype, x, ldx, 1, &w, &bias, nullptr, res, ldr, y, ldy, M, N, K, act, io, bn_hint, ln, s);
+  gemm_impl(dtype, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, bn_hint, s);
 }
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,

@@ -49,8 +49,6 @@ struct Workspace {
   void* h = nullptr;    // [T, F]
   void* xr = nullptr;   // [T, H] fp32: BERT/RoBERTa residual stream (copy of x)
   void* x1r = nullptr;  // [T, H] fp32: copy of x1
-  int* ln_cnt = nullptr;  // per-32-token-tile counters of the GEMM-fused LayerNorm (zeroed)
-  int n_ln_cnt = 0;
   void* base = nullptr;
 };
 

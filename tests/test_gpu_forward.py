@@ -262,16 +262,20 @@ def test_graph_replay_matches_eager(name, mode, k):
     c.close()
 
 
-@pytest.mark.parametrize("name,S", [("tiny_bert", 77), ("tiny_gpt2", 70), ("bert_base", 128), ("gpt2", 200)])
-def test_fused_layernorm_bit_identical(name, S):
-    """A LayerNorm that follows a resident-weight linear runs in that GEMM's epilogue (the last
-    CTA of each token tile normalises its complete rows); it shares the per-row code with the
-    LayerNorm kernel, so fused and unfused forwards must agree bit for bit, in eager and graph
-    mode, and the fused run launches 2 fewer kernels per layer."""
+@pytest.mark.parametrize("name,B,S", [("tiny_bert", 1, 77), ("tiny_gpt2", 1, 70), ("bert_base", 1, 128),
+                                      ("gpt2", 1, 200), ("tiny_roberta", 3, 50), ("bert_large", 1, 96)])
+@pytest.mark.parametrize("dtype", ["fp16", "bf16"])
+def test_fused_layernorm(name, B, S, dtype):
+    """A LayerNorm that follows a resident-weight linear runs in that GEMM's epilogue (K2+K4,
+    gemm_ln.cu: a cluster along N exchanges per-token statistics over DSMEM).  The fused forward
+    matches the oracle within the north_star tolerance, stays close to the unfused one (same
+    math, another summation order), is deterministic (eager == graph replay, bit for bit), and
+    launches 2 fewer kernels per layer."""
     m = synth.SHAPES[name]
-    dtype = "fp16"
     w = synth.make_weights(m, seed=21, dtype=dtype)
-    ids = synth.make_ids(m, 1, S, seed=22)
+    ids = synth.make_ids(m, B, S, seed=22)
+    ref, ref_pool = F.forward(m, w, ids, dtype)
+    ref = ref.reshape(B * S, -1)
     c = dp().Context([0])
     model = dp().Model(c, m, w, dtype)
     plan = dp().plan_generate(fake_cost(m, dtype), "PIPESWITCH", 1)  # all loaded: every linear on the GEMM
@@ -282,10 +286,13 @@ def test_fused_layernorm_bit_identical(name, S):
         outs.append((o.clone(), None if p is None else p.clone()))
         kern.append(st["n_kernels"])
         model.evict(0)
-    for o, p in outs[1:]:
-        assert torch.equal(o, outs[0][0])
+    tol = tolerance(dtype, "paper", ref)
+    for o, p in outs:
+        assert np.all(np.abs(f64(o) - ref) <= tol)
         if p is not None:
-            assert torch.equal(p, outs[0][1])
+            assert np.all(np.abs(f64(p) - ref_pool) <= tolerance(dtype, "paper", ref_pool))
+    assert np.abs(f64(outs[1][0]) - f64(outs[0][0])).max() <= tol.max()
+    assert torch.equal(outs[1][0], outs[2][0])  # deterministic
     assert kern[1] == kern[0] - 2 * m.layers
     model.close()
     c.close()
