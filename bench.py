@@ -407,10 +407,15 @@ def main():
             other_modes[om] = {"ms": round(float(np.mean(ts)), 4), "dha_units": int(p2.method.sum()),
                                "predicted_ms": round(dp.plan_simulate(cost, p2)[0] / 1e6, 4)}
 
-    h2d_bytes = int(sum(stats["h2d_bytes"]))
+    # bytes per host link come from the plan (the simulator's link_bytes equal the bytes each
+    # link's DMAs carry, bit-exactly -- tests/test_gpu_forward.py); rank 0's own stats only see
+    # its own link when the partitions travel on other ranks
+    link_plan = [int(b) for b in link][:world]
+    h2d_bytes = int(sum(link_plan))
+    assert world > 1 or h2d_bytes == int(stats["h2d_bytes"][0]), (h2d_bytes, stats["h2d_bytes"])
     dha_bytes = int(stats["dha_weight_bytes"])
     link_bytes = h2d_bytes + dha_bytes  # bytes the path must move over host links per step
-    per_link = max(stats["h2d_bytes"][:world]) + dha_bytes
+    per_link = max([link_plan[0] + dha_bytes] + link_plan[1:])  # DHA reads use the primary's link
     achieved = link_bytes / (ms * 1e-3) / 1e9
     total_w = model.nbytes
     R_lit = total_w / (peak_h2d * world * 1e9) * 1e3  # all weight bytes / aggregate H2D

@@ -314,3 +314,30 @@ def test_bert_base_batched_cold_start():
     assert np.abs(f64(out) - ref.reshape(4 * 128, -1)).max() <= 1e-2
     assert np.abs(f64(pool) - ref_pool).max() <= 1e-2
     model.close()
+
+
+@pytest.mark.parametrize("name,S,mode,k", [("bert_large", 384, "PT_DHA_LINK_BAL", 2),
+                                           ("roberta_large", 384, "DHA_LINK", 1),
+                                           ("bert_large", 384, "PT_DHA", 4)])
+def test_large_models_full_size(name, S, mode, k):
+    """BASELINE.json configs[2]/[3] at full size: BERT-Large / RoBERTa-Large fp16, batch 1, seq
+    384, a live profile -> the plan -> cold start (PT slots served in loopback on this one GPU:
+    the event / ring logic of the multi-GPU path, not its bandwidth), vs the fp64 oracle at the
+    north_star's max-abs 1e-2; bytes per link == the oracle simulator's."""
+    m = synth.SHAPES[name]
+    dtype = "fp16"
+    w = synth.make_weights(m, seed=7, dtype=dtype)
+    ids = synth.make_ids(m, 1, S, seed=8)
+    ref, ref_pool = F.forward(m, w, ids, dtype)
+    model = dp().Model(ctx(), m, w, dtype)
+    cost = model.profile(0, 1, S, iters=2)
+    plan = dp().plan_generate(cost, mode, k)
+    om, osl, ser = OP.plan(cost, mode, k)
+    assert list(plan.method) == om and list(plan.slot) == osl
+    out, pool, st = run_cold(model, plan, ids, dtype, secondaries=[0] * (k - 1))
+    model.evict(0)
+    assert np.abs(f64(out) - ref.reshape(S, -1)).max() <= 1e-2
+    assert np.abs(f64(pool) - ref_pool).max() <= 1e-2
+    link = OP.simulate(cost, om, osl, k, ser)["link_bytes"]
+    assert st["h2d_bytes"][:len(link)] == link
+    model.close()
