@@ -51,6 +51,10 @@ def parse():
     ap.add_argument("--no-pdl", action="store_true")
     ap.add_argument("--fuse-ln", action="store_true", help="LayerNorm in the preceding GEMM's epilogue")
     ap.add_argument("--profile-iters", type=int, default=10)
+    ap.add_argument("--pt-transport", default="dma", choices=["dma", "sm", "ce"],
+                    help="PT slots at N>1: dma = copy engine into a staging ring + NCCL send/recv (the paper's "
+                         "two hops); sm = SURVEY f4 forwarder kernel (host -> primary HBM over CUDA IPC); "
+                         "ce = one copy-engine DMA per piece straight into the primary's slot (CUDA IPC)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--quick", action="store_true", help="skip the other modes and per-kernel rooflines (sweeps)")
     return ap.parse_args()
@@ -237,13 +241,18 @@ def main():
     ctx = dp.Context([local])
     ctx.set_opts(chunk_bytes=int(a.chunk_mb * (1 << 20)), n_h2d_streams=a.h2d_streams,
                  tail_bytes=int(a.tail_mb * (1 << 20)), use_graph=0 if (a.no_graph or world > 1) else 1,
-                 use_pdl=0 if a.no_pdl else 1, fuse_ln=a.fuse_ln)
+                 use_pdl=0 if a.no_pdl else 1, fuse_ln=a.fuse_ln, pt_transport=a.pt_transport)
     model = dp.Model(ctx, m, w, dtype)
-    if dist_on:
+    if dist_on and a.pt_transport == "dma":
         uid = dp.peer_unique_id() if rank == 0 else None
         box = [uid]
         dist.broadcast_object_list(box, src=0)
         ctx.peer_init(box[0], rank, world)
+    elif dist_on:  # single-hop transports: CUDA IPC handles of the slots + mailboxes, no NCCL
+        ctx.peer_init_ipc(rank, world)
+        blocks = [None] * world
+        dist.all_gather_object(blocks, model.ipc_export())
+        model.ipc_import(blocks)
 
     # roofline denominator: pinned H2D bandwidth of this GPU's link, measured now with the
     # library's own pinned+mapped allocation (256 MiB, best of 5, CUDA events)
@@ -440,6 +449,7 @@ def main():
                    "model": a.model, "global_batch": a.batch, "seq_len": a.seq, "parallelism": f"pt{world}",
                    "plan_mode": mode, "dha_units": int(plan.method.sum()), "units": int(len(plan.method)),
                    "chunk_bytes": int(a.chunk_mb * (1 << 20)), "h2d_streams": a.h2d_streams,
+                   "pt_transport": a.pt_transport if world > 1 else None,
                    "l2": "flushed between steps (256 MiB write)"},
         "roofline": {"bound": "pcie", "achieved": round(achieved, 2), "peak": round(peak_h2d, 2), "unit": "GB/s",
                      "frac": round(achieved / (peak_h2d * world), 4), "traffic": None,

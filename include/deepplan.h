@@ -166,8 +166,23 @@ typedef struct {
   int32_t persistent;     /* 1 = warm runs execute every layer in ONE persistent kernel (K6: grid =
                              #SMs, grid barriers between ops, next GEMM's weights prefetched under
                              the current op) when all layer units are resident [0] */
-  int32_t reserved[1];
+  int32_t pt_transport;   /* how a PT slot's units reach the primary:
+                             DP_PT_DMA = the secondary's copy engine DMAs each piece over its
+                             own PCIe link into a staging ring, then a peer copy (NCCL send/recv
+                             across processes) forwards it over NVLink [default];
+                             DP_PT_SM = SURVEY f4: a forwarder kernel on the secondary reads
+                             the piece from the pinned arena in place (16-byte zero-copy loads
+                             over the secondary's PCIe link) and stores it straight into the
+                             primary's HBM slot over NVLink -- no staging ring, no second copy;
+                             across processes completion is a flag the kernel releases into
+                             the primary's memory (dp_peer_ipc_*), not an NCCL call;
+                             DP_PT_CE = the same single hop driven by the secondary's copy
+                             engine: one DMA per piece from the arena straight into the
+                             primary's slot through the peer / IPC mapping (no staging ring) */
 } dp_engine_opts;
+#define DP_PT_DMA 0
+#define DP_PT_SM 1
+#define DP_PT_CE 2
 dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* opts);
 dp_status dp_context_get_opts(dp_context* ctx, dp_engine_opts* out);
 
@@ -177,6 +192,28 @@ dp_status dp_context_get_opts(dp_context* ctx, dp_engine_opts* out);
  * gather uses ncclSend/ncclRecv only.  DP_ERR_NCCL on failure. */
 dp_status dp_peer_unique_id(void* out128);
 dp_status dp_peer_init(dp_context* ctx, const void* uid128, int32_t rank, int32_t nranks);
+
+/* Multi-process PT without NCCL (opts.pt_transport = DP_PT_SM / DP_PT_CE): records
+ * this process's rank among nranks (one device per context).  Either this or dp_peer_init
+ * makes dp_infer_cold multi-process: `primary` is then a rank.  DP_ERR_STATE if already
+ * initialised. */
+dp_status dp_peer_init_ipc(dp_context* ctx, int32_t rank, int32_t nranks);
+
+/* CUDA IPC exchange for the SM forwarder across processes.  dp_peer_ipc_export allocates
+ * (once) this rank's HBM slots for `m` and its 16 KiB mailbox (a go word the primary
+ * releases at the start of a cold start, and one done word per (slot, piece) the secondaries
+ * release when a piece has landed), and writes DP_IPC_HANDLE_BYTES of cudaIpcMemHandle_t
+ * data to `out` (caller-owned).  The caller distributes every rank's block (e.g.
+ * torch.distributed all_gather); dp_peer_ipc_import takes all nranks blocks concatenated in
+ * rank order and opens the other ranks' handles (own block ignored; ranks on the same
+ * device are allowed -- loopback across processes).  Both are collective in the sense that
+ * every rank calls them for the same model; the handles stay open until dp_model_destroy /
+ * dp_context_destroy.  DP_ERR_STATE before dp_peer_init[_ipc]; DP_ERR_CUDA if an IPC call
+ * fails. */
+#define DP_IPC_HANDLE_BYTES 128
+typedef struct dp_model dp_model;
+dp_status dp_peer_ipc_export(dp_context* ctx, dp_model* m, void* out);
+dp_status dp_peer_ipc_import(dp_context* ctx, dp_model* m, const void* all_handles);
 
 /* ---------------------------------------------------------------------------------
  * Model registration: host weight arena ("we allocate the pinned memory for the
@@ -259,7 +296,8 @@ dp_status dp_measure_h2d(int32_t dev, int64_t bytes, int32_t reps, double* gbs);
  * --------------------------------------------------------------------------------- */
 #define DP_STATS_MAX_UNITS 512
 typedef struct {
-  int64_t h2d_bytes[DP_MAX_DEVICES];    /* bytes DMA'd host->device over each slot's link */
+  int64_t h2d_bytes[DP_MAX_DEVICES];    /* bytes moved host->device over each slot's link
+                                           (copy-engine DMAs, or the SM forwarder's reads) */
   int64_t nvlink_bytes[DP_MAX_DEVICES]; /* bytes gathered from slot s into the primary */
   int64_t dha_weight_bytes;             /* weight bytes DHA kernels must read (algorithmic) */
   int32_t n_copies;                     /* DMA operations issued */
@@ -314,6 +352,13 @@ int32_t dp_model_is_resident(const dp_model* m, int32_t dev);
 /* Pinned, mapped, portable host memory (cudaHostAlloc) and its release. */
 dp_status dp_host_alloc(int64_t bytes, void** out);
 dp_status dp_host_free(void* p);
+
+/* SM-driven PT forwarder (the design alternative of P:182): copies `bytes`
+ * from `src` (host-mapped pinned memory, read in place with 16-byte loads over the link of
+ * the device owning `stream`'s context) to `dst` (device memory of that device or a peer's,
+ * written over NVLink) with one kernel; `bytes` may be any size (a sub-16-byte tail is
+ * copied bytewise).  src/dst must be 16-byte aligned.  Enqueued on `stream`. */
+dp_status dp_pt_forward(const void* src, void* dst, int64_t bytes, void* stream);
 
 /* Embedding: x[t,:] = LN(word[ids[t]] + pos[p(t)] + type[0]) for BERT/
  * RoBERTa (ln_g/ln_b non-NULL), or wte[ids[t]] + wpe[p(t)] for GPT-2 (type, ln NULL).

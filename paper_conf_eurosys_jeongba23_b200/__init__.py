@@ -9,12 +9,12 @@ built, importing this package raises.
 from ._lib import (  # noqa: F401
     DHA, LOAD, MODES, UNIT_KINDS, Context, DeepPlanError, Model, attention, embed, host_alloc, host_free,
     layernorm, lib, linear, plan_exhaustive, plan_generate, plan_partition, plan_simulate, serve_run,
-    peer_unique_id, measure_h2d, transfer_schedule, config_units,
+    peer_unique_id, measure_h2d, transfer_schedule, config_units, pt_forward,
 )
 
 __all__ = [
     "DHA", "LOAD", "MODES", "UNIT_KINDS", "Context", "DeepPlanError", "Model", "attention", "embed",
     "host_alloc", "host_free", "layernorm", "lib", "linear", "plan_exhaustive", "plan_generate",
     "plan_partition", "plan_simulate", "serve_run", "peer_unique_id", "measure_h2d", "transfer_schedule",
-    "config_units",
+    "config_units", "pt_forward",
 ]

@@ -16,6 +16,7 @@ UNIT_KINDS = {0: "emb", 1: "ln", 2: "linear"}
 FAMILIES = {"bert": 0, "roberta": 1, "gpt2": 2}
 DTYPES = {"fp16": 0, "bf16": 1}
 ACTS = {"none": 0, "gelu_erf": 1, "gelu_tanh": 2, "tanh": 3}
+PT_TRANSPORTS = {"dma": 0, "sm": 1, "ce": 2}  # dp_engine_opts.pt_transport: DP_PT_DMA / _SM / _CE
 DP_MAX_DEVICES = 8
 
 
@@ -51,7 +52,7 @@ class EngineOpts(C.Structure):
     _fields_ = [("chunk_bytes", C.c_int64), ("n_h2d_streams", C.c_int32), ("use_graph", C.c_int32),
                 ("gemm_bn", C.c_int32), ("debug_delay_us", C.c_int32), ("debug_poison", C.c_int32),
                 ("use_pdl", C.c_int32), ("fuse_ln", C.c_int32), ("tail_bytes", C.c_int64),
-                ("persistent", C.c_int32), ("reserved", C.c_int32 * 1)]
+                ("persistent", C.c_int32), ("pt_transport", C.c_int32)]
 
 
 class ModelConfig(C.Structure):
@@ -117,6 +118,10 @@ _sig("dp_context_set_opts", [vp, C.POINTER(EngineOpts)])
 _sig("dp_context_get_opts", [vp, C.POINTER(EngineOpts)])
 _sig("dp_peer_unique_id", [vp])
 _sig("dp_peer_init", [vp, vp, C.c_int32, C.c_int32])
+_sig("dp_peer_init_ipc", [vp, C.c_int32, C.c_int32])
+_sig("dp_peer_ipc_export", [vp, vp, vp])
+_sig("dp_peer_ipc_import", [vp, vp, vp])
+_sig("dp_pt_forward", [vp, vp, C.c_int64, vp])
 _sig("dp_config_params", [C.POINTER(ModelConfig), C.POINTER(ParamInfo), C.c_int32, i32p])
 _sig("dp_model_create", [vp, C.POINTER(ModelConfig), C.POINTER(vp), C.c_int32, C.POINTER(vp)])
 _sig("dp_model_destroy", [vp, vp])
@@ -274,7 +279,8 @@ class Context:
         self.devs = list(devs)
 
     def set_opts(self, chunk_bytes=None, n_h2d_streams=None, use_graph=None, gemm_bn=None, debug_delay_us=None,
-                 debug_poison=None, use_pdl=None, tail_bytes=None, fuse_ln=None, persistent=None):
+                 debug_poison=None, use_pdl=None, tail_bytes=None, fuse_ln=None, persistent=None,
+                 pt_transport=None):
         o = EngineOpts()
         _check(lib.dp_context_get_opts(self.h, C.byref(o)))
         if chunk_bytes is not None:
@@ -297,11 +303,17 @@ class Context:
             o.fuse_ln = 1 if fuse_ln else 0
         if persistent is not None:
             o.persistent = 1 if persistent else 0
+        if pt_transport is not None:
+            o.pt_transport = PT_TRANSPORTS[pt_transport] if isinstance(pt_transport, str) else int(pt_transport)
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))
 
     def peer_init(self, uid: bytes, rank: int, nranks: int):
         buf = C.create_string_buffer(uid, 128)
         _check(lib.dp_peer_init(self.h, C.cast(buf, vp), int(rank), int(nranks)))
+
+    def peer_init_ipc(self, rank: int, nranks: int):
+        """Multi-process PT without NCCL (SM forwarder over CUDA IPC)."""
+        _check(lib.dp_peer_init_ipc(self.h, int(rank), int(nranks)))
 
     def close(self):
         if self.h:
@@ -446,6 +458,18 @@ class Model:
         _check(lib.dp_lm_head(self.ctx.h, self.h, int(dev), _dptr(hidden), int(ld), int(rows), _dptr(logits),
                               _stream_ptr(stream)))
 
+    def ipc_export(self) -> bytes:
+        """This rank's DP_IPC_HANDLE_BYTES block (HBM slots + mailbox) for the SM forwarder."""
+        buf = C.create_string_buffer(128)
+        _check(lib.dp_peer_ipc_export(self.ctx.h, self.h, C.cast(buf, vp)))
+        return buf.raw
+
+    def ipc_import(self, blocks):
+        """Open the other ranks' blocks (a list of bytes in rank order)."""
+        data = b"".join(bytes(b) for b in blocks)
+        buf = C.create_string_buffer(data, len(data))
+        _check(lib.dp_peer_ipc_import(self.ctx.h, self.h, C.cast(buf, vp)))
+
     def evict(self, dev: int):
         _check(lib.dp_model_evict(self.ctx.h, self.h, int(dev)))
 
@@ -473,6 +497,11 @@ def measure_h2d(dev: int, nbytes: int = 256 << 20, reps: int = 5) -> float:
     g = C.c_double()
     _check(lib.dp_measure_h2d(int(dev), int(nbytes), int(reps), C.byref(g)))
     return float(g.value)
+
+
+def pt_forward(src, dst, nbytes: int, stream=None):
+    """SM-driven PT forwarder kernel (host-mapped src -> local or peer HBM dst)."""
+    _check(lib.dp_pt_forward(_dptr(src), _dptr(dst), int(nbytes), _stream_ptr(stream)))
 
 
 def host_alloc(nbytes: int) -> int:

@@ -76,9 +76,13 @@ struct dp_context {
   dp::DevCtx dc[DP_MAX_DEVICES];
   dp_engine_opts opts{};
   std::map<std::pair<int, int>, dp::SlotRes> slots;  // (slot, device) -> resources
-  // multi-process PT (NCCL)
+  // multi-process PT: NCCL (dp_peer_init) or CUDA IPC + SM forwarder (dp_peer_init_ipc)
   void* comm = nullptr;
-  int rank = -1, nranks = 0;
+  int rank = -1, nranks = 0;  // nranks > 0: multi-process (`primary` is a rank)
   cudaStream_t comm_stream = nullptr;
+  uint32_t* mailbox = nullptr;                    // this rank's (pt_forward.cu layout)
+  uint32_t* peer_mailbox[DP_MAX_DEVICES] = {};     // other ranks' (IPC-mapped), by rank
+  uint32_t pt_epoch = 0;                          // cold starts run in SM/IPC mode so far
+  bool multiproc() const { return nranks > 0; }
   dp::DevCtx& on(int dev);
 };

@@ -217,9 +217,6 @@ __global__ void __launch_bounds__(128, 1)
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem_d = tmem_base_sh;
   pdl_trigger();
-  // split-K: announce that this CTA's barriers are initialised; the matching wait comes right
-  // before the first push into a peer, long after every CTA of the cluster has arrived
-  if (splits > 1) asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
 
   // nst <= STAGES: the ring depth actually used (a shallower ring leaves room on the SM for
   // the previous kernel's CTAs, so the PDL prologue overlap is not blocked on shared memory)
@@ -277,6 +274,13 @@ __global__ void __launch_bounds__(128, 1)
 
   mbar_wait(&done_bar, 0);
   if (threadIdx.x == 0) TRACE(5);
+  // split-K: announce that this CTA's MMAs are done, i.e. its TMA ring -- which the receive
+  // slots below overlap -- is free.  Peers push into our receive slots only after the
+  // matching wait.  (An arrive right after setup let a fast peer push while a slow CTA was
+  // still streaming stages into that memory: a corrupted operand under SM contention, caught
+  // by tools/stress_concurrency.py.)  Release orders our tensor-core reads of the ring before
+  // the peers' async-proxy writes into it.
+  if (splits > 1) asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
   asm volatile("tcgen05.fence::after_thread_sync;");
   // 1) TMEM -> shared memory (the ring is free once the MMAs are done): the fp32 tile,
   //    [128 W rows][BN tokens] with an odd row stride
@@ -376,7 +380,7 @@ __global__ void __launch_bounds__(128, 1)
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // send buffer -> async proxy
     __syncthreads();
-    asm volatile("barrier.cluster.wait.aligned;" ::: "memory");     // peers' recv_bar initialised
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");  // peers' rings free, recv_bar ready
     if (threadIdx.x == 0) {
       for (int r = 0; r < splits; ++r) {
         if (r == sp) continue;

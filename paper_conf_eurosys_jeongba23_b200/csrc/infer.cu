@@ -87,7 +87,7 @@ static SlotRes& slot_res(dp_context* ctx, int slot, int dev, int64_t ring_bytes)
   return r;
 }
 
-static void ensure_slots(dp_model* m, int dev) {
+void dp::ensure_slots(dp_model* m, int dev) {
   DevState& ds = m->dev[dev];
   if (ds.dbase) return;
   DeviceGuard g(dev);
@@ -95,6 +95,24 @@ static void ensure_slots(dp_model* m, int dev) {
     ds.dbase = nullptr;
     fail(DP_ERR_OOM, "HBM slot allocation for the model failed");
   }
+}
+
+// Single-process SM forwarding to another GPU stores through the peer mapping.
+static void ensure_peer_access(int from, int to) {
+  static bool done[DP_MAX_DEVICES][DP_MAX_DEVICES] = {};
+  if (from == to || done[from][to]) return;
+  int ok = 0;
+  DP_CUDA(cudaDeviceCanAccessPeer(&ok, from, to));
+  DP_CHECK(ok, DP_ERR_UNSUPPORTED, "SM PT forwarder: device " + std::to_string(from) + " cannot access device " +
+                                       std::to_string(to) + "'s memory");
+  DeviceGuard g(from);
+  cudaError_t e = cudaDeviceEnablePeerAccess(to, 0);
+  if (e == cudaErrorPeerAccessAlreadyEnabled) {
+    cudaGetLastError();
+  } else {
+    DP_CUDA(e);
+  }
+  done[from][to] = true;
 }
 
 extern "C" const char* dp_last_error(void) { return g_last_error.c_str(); }
@@ -143,6 +161,10 @@ extern "C" dp_status dp_context_destroy(dp_context* ctx) {
       if (kv.second.mig) cudaStreamDestroy(kv.second.mig);
       if (kv.second.ring) cudaFree(kv.second.ring);
     }
+    if (!ctx->devs.empty()) {
+      DeviceGuard g(ctx->devs[0]);
+      ipc_close(ctx);
+    }
     peer_destroy(ctx);
     delete ctx;
   });
@@ -155,6 +177,8 @@ extern "C" dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* 
     DP_CHECK(o->n_h2d_streams >= 1 && o->n_h2d_streams <= 8, DP_ERR_INVALID, "n_h2d_streams must be 1..8");
     DP_CHECK(o->gemm_bn == 0 || o->gemm_bn == 32 || o->gemm_bn == 64 || o->gemm_bn == 128 || o->gemm_bn == 256,
              DP_ERR_INVALID, "gemm_bn must be 0/32/64/128/256");
+    DP_CHECK(o->pt_transport == DP_PT_DMA || o->pt_transport == DP_PT_SM || o->pt_transport == DP_PT_CE,
+             DP_ERR_INVALID, "pt_transport must be DP_PT_DMA, DP_PT_SM or DP_PT_CE");
     ctx->opts = *o;
   });
 }
@@ -311,7 +335,8 @@ static std::string graph_key(const dp_context* ctx, const dp_plan* plan, const i
        std::to_string((uintptr_t)pooled) + "|" + std::to_string(batch) + "x" + std::to_string(seq) + "|" +
        std::to_string(ctx->opts.chunk_bytes) + "," + std::to_string(ctx->opts.n_h2d_streams) + "," +
        std::to_string(ctx->opts.gemm_bn) + "," + std::to_string(ctx->opts.debug_delay_us) + "," +
-       std::to_string(ctx->opts.use_pdl) + "," + std::to_string(ctx->opts.fuse_ln);
+       std::to_string(ctx->opts.use_pdl) + "," + std::to_string(ctx->opts.fuse_ln) + "," +
+       std::to_string(ctx->opts.pt_transport);
   return k;
 }
 
@@ -355,7 +380,7 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   ctx->on(primary);
   DevState& ds = m->dev[primary];
   DP_CHECK(!ds.resident, DP_ERR_STATE, "model already resident on the primary; evict it first");
-  DP_CHECK(ctx->comm || nsec >= plan->k - 1, DP_ERR_INVALID, "need k-1 secondaries for the plan");
+  DP_CHECK(ctx->multiproc() || nsec >= plan->k - 1, DP_ERR_INVALID, "need k-1 secondaries for the plan");
   DP_CHECK(batch > 0 && seq > 0 && ids && out, DP_ERR_INVALID, "bad inference arguments");
   DP_CHECK(seq + (m->cfg.family == DP_FAMILY_ROBERTA ? m->cfg.pad_idx + 1 : 0) <= m->cfg.max_pos, DP_ERR_INVALID,
            "sequence longer than the position table");
@@ -363,7 +388,7 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   ensure_slots(m, primary);
   ensure_h2d_streams(ctx, primary);
   ensure_workspace(m, primary, int64_t(batch) * seq);
-  bool graph = ctx->opts.use_graph != 0 && !ctx->comm;
+  bool graph = ctx->opts.use_graph != 0 && !ctx->multiproc();
   for (int s = 1; s < plan->k && graph; ++s) graph = secondaries[s - 1] == primary;  // single-device graphs only
   dp_run_stats st;
   if (graph) {
@@ -418,26 +443,75 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   }
 
   // (2) PT slots
-  if (!ctx->comm)
+  const bool one_hop = ctx->opts.pt_transport != DP_PT_DMA;  // single hop: SM forwarder or direct DMA
+  const bool ce_fwd = ctx->opts.pt_transport == DP_PT_CE;
+  // across processes with the SM forwarder: (slot, piece) a loaded unit arrives in
+  std::vector<std::pair<int, int>> unit_piece(n, {-1, -1});
+  std::vector<size_t> slot_npieces(plan->k, 0);
+  uint32_t epoch = 0;
+  if (!ctx->multiproc())
     for (int s = 1; s < plan->k; ++s) {
       const int sdev = secondaries[s - 1];
       DP_CHECK(sdev >= 0 && sdev < DP_MAX_DEVICES && ctx->dc[sdev].ready, DP_ERR_INVALID,
                "secondary device not in the context");
       if (sdev != primary) ctx->dc[sdev].events.reset();
     }
-  if (ctx->comm && plan->k > 1) peer_recv_all(ctx, m, plan, prim_rank, primary, fork, unit_ev, st);
-  for (int s = 1; s < plan->k && !ctx->comm; ++s) {
+  if (ctx->multiproc() && plan->k > 1 && !one_hop) {
+    DP_CHECK(ctx->comm, DP_ERR_STATE, "DMA transport across processes needs dp_peer_init (NCCL)");
+    peer_recv_all(ctx, m, plan, prim_rank, primary, fork, unit_ev, st);
+  }
+  if (ctx->multiproc() && one_hop) {
+    // go to every secondary; their forwarders store into our slots and release done words
+    ipc_check_primary(ctx);
+    epoch = ++ctx->pt_epoch;
+    ipc_primary_begin(ctx, plan, prim_rank, stream, epoch);
+    for (int s = 1; s < plan->k; ++s) {
+      auto pcs = slot_pieces(m, plan, s, cap, opt_tail(ctx));
+      slot_npieces[s] = pcs.size();
+      for (size_t r = 0; r < pcs.size(); ++r) {
+        for (int u = pcs[r].first_unit; u <= pcs[r].last_unit; ++u) unit_piece[u] = {s, (int)r};
+        st.nvlink_bytes[s] += pcs[r].bytes;
+      }
+    }
+  }
+  for (int s = 1; s < plan->k && !ctx->multiproc(); ++s) {
     auto pcs = slot_pieces(m, plan, s, cap, opt_tail(ctx));
     if (pcs.empty()) continue;
     const int sdev = secondaries[s - 1];
     const int64_t ring_slots = 3;
     int64_t slot_bytes = 0;
     for (const auto& p : pcs) slot_bytes = std::max(slot_bytes, p.bytes);
-    SlotRes& r = slot_res(ctx, s, sdev, ring_slots * slot_bytes);
+    SlotRes& r = slot_res(ctx, s, sdev, one_hop ? 0 : ring_slots * slot_bytes);
     DevCtx& sd = ctx->dc[sdev];
     {
       DeviceGuard gs(sdev);
       DP_CUDA(cudaStreamWaitEvent(r.h2d, fork, 0));
+    }
+    if (one_hop) {  // one hop per piece on the secondary, host -> primary HBM
+      if (!ce_fwd) ensure_peer_access(sdev, primary);
+      DeviceGuard gs(sdev);
+      for (const Piece& p : pcs) {
+        if (ctx->opts.debug_delay_us > 0) launch_spin((long long)ctx->opts.debug_delay_us * 2000, r.h2d);
+        if (ce_fwd) {
+          DP_CUDA(cudaMemcpyAsync(static_cast<uint8_t*>(ds.dbase) + p.off, static_cast<const uint8_t*>(m->arena) + p.off,
+                                  p.bytes, cudaMemcpyDefault, r.h2d));
+          ++st.n_copies;
+        } else {
+          launch_pt_forward(static_cast<const uint8_t*>(m->arena) + p.off, static_cast<uint8_t*>(ds.dbase) + p.off,
+                            p.bytes, r.h2d, nullptr, 0, nullptr, nullptr);
+        }
+        st.h2d_bytes[s] += p.bytes;
+        st.nvlink_bytes[s] += p.bytes;
+        cudaEvent_t done = sd.events.get();
+        DP_CUDA(cudaEventRecord(done, r.h2d));
+        ++st.n_events;
+        bind_units(unit_ev, p, done);
+      }
+      // the end-of-cold-start join waits on the migration stream: chain it behind the loads
+      cudaEvent_t last = sd.events.get();
+      DP_CUDA(cudaEventRecord(last, r.h2d));
+      DP_CUDA(cudaStreamWaitEvent(r.mig, last, 0));
+      continue;
     }
     std::vector<cudaEvent_t> fwd_done(pcs.size(), nullptr);
     for (size_t c = 0; c < pcs.size(); ++c) {
@@ -482,8 +556,16 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   a.pooled = pooled;
   a.stream = stream;
   a.bn_hint = ctx->opts.gemm_bn;
+  std::pair<int, int> last_piece{-1, -1};
   a.before_unit = [&](int u) {
     if (method[u] == DP_DHA) return;  // DHA layers skip the dependency check
+    if (unit_piece[u].first > 0) {    // across processes: acquire the piece's done word
+      if (unit_piece[u] == last_piece) return;
+      ipc_primary_wait(ctx, unit_piece[u].first, (size_t)unit_piece[u].second, epoch, stream);
+      pdl_state().block_next = true;
+      last_piece = unit_piece[u];
+      return;
+    }
     cudaEvent_t e = unit_ev[u];
     DP_CHECK(e != nullptr, DP_ERR_STATE, "internal: loaded unit has no completion event");
     if (e == last_waited) return;
@@ -501,7 +583,9 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
     ++st.n_events;
   }
-  for (int s = 1; s < plan->k && !ctx->comm; ++s) {
+  for (int s = 1; s < plan->k && ctx->multiproc() && one_hop; ++s)  // every piece landed
+    if (slot_npieces[s] > 0) ipc_primary_wait(ctx, s, slot_npieces[s] - 1, epoch, stream);
+  for (int s = 1; s < plan->k && !ctx->multiproc(); ++s) {
     auto it = ctx->slots.find({s, secondaries[s - 1]});
     if (it == ctx->slots.end()) continue;
     DeviceGuard gs(it->second.dev);
@@ -510,7 +594,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     DeviceGuard gp(primary);
     DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
   }
-  if (ctx->comm) peer_join(ctx, stream);
+  if (ctx->comm && !one_hop) peer_join(ctx, stream);
   st.n_kernels = a.kernels;
   st.dha_weight_bytes = dha_bytes(m, method, batch * seq, seq);
   return st;
@@ -523,10 +607,17 @@ extern "C" dp_status dp_infer_cold(dp_context* ctx, dp_model* m, const dp_plan* 
                                    int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats) {
   return guard([&] {
     DP_CHECK(ctx && m, DP_ERR_INVALID, "NULL context/model");
-    if (ctx->comm) {  // multi-process PT: `primary` is a rank, each process has one device
+    if (ctx->multiproc()) {  // multi-process PT: `primary` is a rank, each process has one device
       validate_plan(m, plan);
+      DP_CHECK(primary >= 0 && primary < ctx->nranks, DP_ERR_INVALID, "primary rank out of range");
       if (ctx->rank != primary) {  // secondary rank: only its transfers
-        peer_send_rank(ctx, m, plan, primary, stats);
+        DeviceGuard g(ctx->devs[0]);
+        if (ctx->opts.pt_transport != DP_PT_DMA) {
+          ipc_send_rank(ctx, m, plan, primary, stats);
+        } else {
+          DP_CHECK(ctx->comm, DP_ERR_STATE, "DMA transport across processes needs dp_peer_init (NCCL)");
+          peer_send_rank(ctx, m, plan, primary, stats);
+        }
         return;
       }
       infer_cold(ctx, m, plan, ctx->devs[0], primary, nullptr, 0, d_ids, batch, seq, d_out, d_pooled,
@@ -639,6 +730,7 @@ extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
         if (ds.ws.base) cudaFree(ds.ws.base);
       }
     }
+    ipc_close_model(m);
     delete m;  // the last instance sharing the arena frees it
   });
 }

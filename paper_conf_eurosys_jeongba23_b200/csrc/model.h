@@ -89,6 +89,7 @@ struct dp_model {
   std::shared_ptr<void> arena_owner;  // shared by dp_model_clone instances
   int64_t arena_bytes = 0;
   dp::DevState dev[DP_MAX_DEVICES];
+  void* peer_dbase[DP_MAX_DEVICES] = {};  // other ranks' HBM slots, IPC-mapped (by rank)
 
   const uint8_t* host(int u) const { return static_cast<const uint8_t*>(arena) + units[u].off; }
   uint8_t* device(int d, int u) const { return static_cast<uint8_t*>(dev[d].dbase) + units[u].off; }

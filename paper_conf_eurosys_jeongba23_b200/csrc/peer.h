@@ -25,4 +25,18 @@ inline int64_t opt_cap(const dp_context* ctx) { return ctx->opts.chunk_bytes < 4
 inline int64_t opt_tail(const dp_context* ctx) { return ctx->opts.tail_bytes; }
 void bind_units(std::vector<cudaEvent_t>& unit_ev, const Piece& p, cudaEvent_t e);
 
+// SM-driven forwarder (pt_forward.cu).  go/counter/done are null in one process.
+void launch_pt_forward(const void* src, void* dst, int64_t bytes, cudaStream_t s, const uint32_t* go,
+                       uint32_t epoch, uint32_t* counter, uint32_t* done);
+// Across processes (CUDA IPC mailboxes): the primary releases `go` to its secondaries, then
+// waits on done[slot][piece] before the units of that piece; a secondary forwards its slot.
+void ipc_check_primary(dp_context* ctx);
+void ipc_primary_begin(dp_context* ctx, const dp_plan* plan, int prim_rank, cudaStream_t exec, uint32_t epoch);
+void ipc_primary_wait(dp_context* ctx, int slot, size_t piece, uint32_t epoch, cudaStream_t exec);
+void ipc_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, dp_run_stats* stats);
+void ipc_close(dp_context* ctx);
+void ipc_close_model(dp_model* m);
+// The model's HBM slots on dev (infer.cu).
+void ensure_slots(dp_model* m, int dev);
+
 }  // namespace dp

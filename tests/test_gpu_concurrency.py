@@ -1,0 +1,75 @@
+"""Kernel determinism under SM contention (GPU).
+
+A kernel's result must not depend on what else runs on the GPU: with the PT forwarder
+streaming a pinned buffer from another stream (2 CTAs per SM -- exactly what a cold start
+with opts.pt_transport = "sm" runs beside the forward in loopback, and what a serving GPU
+runs beside a foreign request), every hot kernel is repeated and compared bit for bit with
+its noise-free output.  This caught a real race: the cluster split-K GEMM let a fast CTA
+push its partial rows into a slow peer's receive slots -- which overlap the peer's TMA ring
+-- before the peer's mainloop had finished (BERT-Large fc2, M384 N1024 K4096: 1 NaN tile in
+200 runs).  The arrive now follows the MMAs (gemm_tc.cu)."""
+import math
+
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+def dp():
+    import paper_conf_eurosys_jeongba23_b200 as m
+    return m
+
+
+def _stress(fn, out, reps, noise_src, noise_dst, side, main):
+    with torch.cuda.stream(main):
+        fn()
+    torch.cuda.synchronize()
+    ref = out.clone()
+    bad = 0
+    for i in range(reps):
+        with torch.cuda.stream(side):
+            dp().pt_forward(noise_src, noise_dst, (16 << 20) + (i % 7) * 4096, stream=side)
+        with torch.cuda.stream(main):
+            if i % 2:
+                out.fill_(0)
+            fn()
+        torch.cuda.current_stream().wait_stream(main)
+        if not torch.equal(out, ref):
+            bad += 1
+    torch.cuda.synchronize()
+    return bad
+
+
+@pytest.fixture(scope="module")
+def noise():
+    return (torch.empty(32 << 20, dtype=torch.uint8).pin_memory(),
+            torch.empty(32 << 20, dtype=torch.uint8, device="cuda"), torch.cuda.Stream(), torch.cuda.Stream())
+
+
+@pytest.mark.parametrize("M,N,K", [(384, 1024, 4096), (128, 768, 3072), (1024, 1024, 4096), (384, 1024, 1024),
+                                   (128, 3072, 768)])
+def test_gemm_deterministic_under_contention(M, N, K, noise):
+    torch.manual_seed(M + N + K)
+    x = torch.randn(M, K, device="cuda").half()
+    w = (torch.randn(N, K, device="cuda") / math.sqrt(K)).half()
+    b = torch.randn(N, device="cuda").half()
+    r = torch.randn(M, N, device="cuda").half()
+    y = torch.empty(M, N, device="cuda").half()
+    main = noise[3]
+    bad = _stress(lambda: dp().linear(x, K, w, b, r, N, y, N, M, N, K, path=0, stream=main), y, 600, *noise)
+    assert bad == 0
+
+
+@pytest.mark.parametrize("S,H,heads,causal", [(384, 1024, 16, 0), (1024, 1024, 16, 1)])
+def test_attention_and_skinny_deterministic_under_contention(S, H, heads, causal, noise):
+    torch.manual_seed(S)
+    qkv = torch.randn(S, 3 * H, device="cuda").half()
+    o = torch.empty(S, H, device="cuda").half()
+    main = noise[3]
+    assert _stress(lambda: dp().attention(qkv, 3 * H, o, 1, S, H, heads, causal, stream=main), o, 200, *noise) == 0
+    x = torch.randn(128, 3072, device="cuda").half()
+    w = (torch.randn(768, 3072, device="cuda") / 50).half()
+    y = torch.empty(128, 768, device="cuda").half()
+    assert _stress(lambda: dp().linear(x, 3072, w, None, None, 0, y, 768, 128, 768, 3072, path=1, stream=main), y,
+                   200, *noise) == 0

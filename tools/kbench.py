@@ -1,7 +1,7 @@
 """Per-kernel device timings through the C-ABI hooks (CUDA events around back-to-back
 launches on one stream, after warm-up).  Used with ncu too:
   ncu --set full -k regex:gemm_tc -c 3 python tools/kbench.py gemm
-python tools/kbench.py [all|gemm|ln|attn|skinny|embed|lmhead] [reps]"""
+python tools/kbench.py [all|gemm|ln|attn|skinny|embed|lmhead|ptfwd] [reps]"""
 import json
 import math
 import os
@@ -99,4 +99,19 @@ if which in ("all", "embed"):
     out = torch.empty(S, H, device="cuda").half()
     us = timeit(lambda: dp.embed(ids, S, word, pos, typ, g, bb, H, 1e-12, out), n=20)
     res["embed DHA S128 H768"] = {"us": round(us, 2), "pcie_gbs": round((2 * S + 3) * H * 2 / us / 1e3, 1)}
+
+if which in ("all", "ptfwd"):
+    # SM-driven PT forwarder vs the copy engine, host -> this GPU's HBM (on one GPU
+    # the NVLink hop of the multi-GPU case is a local store): the per-link read side of PT.
+    for mb in (1, 4, 32, 128):
+        nb = mb << 20
+        src = torch.empty(nb, dtype=torch.uint8).pin_memory()
+        src.random_(0, 255)
+        dst = torch.empty(nb, dtype=torch.uint8, device="cuda")
+        us_f = timeit(lambda: dp.pt_forward(src, dst, nb), n=max(3, min(reps, 2048 // mb)))
+        us_d = timeit(lambda: dst.copy_(src, non_blocking=True), n=max(3, min(reps, 2048 // mb)))
+        assert torch.equal(dst.cpu(), src)
+        res[f"pt_forward {mb} MiB"] = {"us": round(us_f, 2), "gbs": round(nb / us_f / 1e3, 2),
+                                       "dma_us": round(us_d, 2), "dma_gbs": round(nb / us_d / 1e3, 2)}
+
 print(json.dumps(res, indent=1))
