@@ -228,11 +228,22 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # DP_BENCH_ONE_GPU=1 (tests only): every rank on device 0 and a gloo process group -- the
+    # N > 1 control flow with the IPC transports (sm / ce) on a one-GPU box; NCCL refuses two
+    # ranks on one device, so --pt-transport dma is not available there
+    one_gpu = os.environ.get("DP_BENCH_ONE_GPU") == "1"
+    if one_gpu:
+        local = 0
+        assert a.pt_transport != "dma" or world == 1, "DP_BENCH_ONE_GPU needs --pt-transport sm or ce"
     assert world == a.gpus, f"--gpus {a.gpus} but WORLD_SIZE {world}"
     torch.cuda.set_device(local)
     dist_on = world > 1
     if dist_on:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    red_dev = "cpu" if one_gpu else "cuda"  # gloo reduces host tensors
 
     m = synth.SHAPES[a.model]
     dtype = "fp16"
@@ -330,7 +341,7 @@ def main():
     ck = clocks.stop()
     lat = [ev0[i].elapsed_time(ev1[i]) for i in range(a.steps)]
     my_ms = float(np.mean(lat))
-    t = torch.tensor([my_ms], dtype=torch.float64, device="cuda")
+    t = torch.tensor([my_ms], dtype=torch.float64, device=red_dev)
     if dist_on:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms = float(t.item())
@@ -365,7 +376,7 @@ def main():
             e2e.append(s0.elapsed_time(s1))
             if dist_on:
                 dist.barrier()
-        t = torch.tensor([float(np.mean(e2e))], dtype=torch.float64, device="cuda")
+        t = torch.tensor([float(np.mean(e2e))], dtype=torch.float64, device=red_dev)
         if dist_on:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
@@ -375,9 +386,12 @@ def main():
             dist.destroy_process_group()
         return
 
-    # warm latency (the compute-only term of the north-star roofline)
+    # warm latency (the compute-only term of the north-star roofline).  The secondaries have
+    # left, so at N > 1 the model is made resident by a local cold start with the SAME method
+    # vector (same DHA set, every loaded unit over this GPU's own link, k = 1)
     model.evict(local) if model.is_resident(local) else None
-    model.infer_cold(plan, 0, ids, out, pooled, stream=stream)
+    plan_local = plan if world == 1 else dp._lib.PlanArrays(len(plan.method), plan.method, None, plan.s.mode, 1)
+    model.infer_cold(plan_local, 0, ids, out, pooled, stream=stream)
     torch.cuda.synchronize()
     wl = []
     for i in range(10):

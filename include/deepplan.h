@@ -195,8 +195,10 @@ dp_status dp_peer_init(dp_context* ctx, const void* uid128, int32_t rank, int32_
 
 /* Multi-process PT without NCCL (opts.pt_transport = DP_PT_SM / DP_PT_CE): records
  * this process's rank among nranks (one device per context).  Either this or dp_peer_init
- * makes dp_infer_cold multi-process: `primary` is then a rank.  DP_ERR_STATE if already
- * initialised. */
+ * makes dp_infer_cold multi-process: `primary` is then a rank.  With the IPC transports every
+ * rank must call dp_infer_cold for every plan with k > 1 (in the same order: the ranks count
+ * these cold starts as the epochs of their go / done words); a k = 1 plan is local to the
+ * primary.  DP_ERR_STATE if already initialised. */
 dp_status dp_peer_init_ipc(dp_context* ctx, int32_t rank, int32_t nranks);
 
 /* CUDA IPC exchange for the SM forwarder across processes.  dp_peer_ipc_export allocates

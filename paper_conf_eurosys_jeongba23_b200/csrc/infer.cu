@@ -460,7 +460,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     DP_CHECK(ctx->comm, DP_ERR_STATE, "DMA transport across processes needs dp_peer_init (NCCL)");
     peer_recv_all(ctx, m, plan, prim_rank, primary, fork, unit_ev, st);
   }
-  if (ctx->multiproc() && one_hop) {
+  if (ctx->multiproc() && one_hop && plan->k > 1) {
     // go to every secondary; their forwarders store into our slots and release done words
     ipc_check_primary(ctx);
     epoch = ++ctx->pt_epoch;

@@ -215,7 +215,11 @@ void ipc_check_primary(dp_context* ctx) {
 void ipc_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, dp_run_stats* stats) {
   dp_run_stats st;
   std::memset(&st, 0, sizeof(st));
-  const uint32_t epoch = ++ctx->pt_epoch;  // every rank counts the same cold starts
+  if (plan->k <= 1) {  // no PT slots: not a rendezvous, no epoch
+    if (stats) *stats = st;
+    return;
+  }
+  const uint32_t epoch = ++ctx->pt_epoch;  // every rank counts the same k > 1 cold starts
   int slot = -1;
   for (int s = 1; s < plan->k; ++s)
     if (peer_rank_of_slot(ctx, primary, s) == ctx->rank) slot = s;
