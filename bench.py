@@ -335,7 +335,13 @@ def main():
             dist.barrier()
     sync_all()
     pad_s = 0.0 if os.environ.get("DP_BENCH_UNDER_NCU") else 1.0
-    while time.perf_counter() - t_start < pad_s:  # keep the GPU busy for the clock samples
+    while True:  # keep the GPU busy for the clock samples; rank 0 decides for every rank so
+        # all ranks run the same number of cold starts (each k > 1 one is a rendezvous)
+        go_on = torch.tensor([1 if time.perf_counter() - t_start < pad_s else 0], device=red_dev)
+        if dist_on:
+            dist.broadcast(go_on, src=0)
+        if not int(go_on.item()):
+            break
         step()
         sync_all()
     ck = clocks.stop()

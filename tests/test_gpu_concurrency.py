@@ -10,6 +10,8 @@ push its partial rows into a slow peer's receive slots -- which overlap the peer
 200 runs).  The arrive now follows the MMAs (gemm_tc.cu)."""
 import math
 
+import numpy as np
+
 import pytest
 
 torch = pytest.importorskip("torch")
@@ -73,3 +75,29 @@ def test_attention_and_skinny_deterministic_under_contention(S, H, heads, causal
     y = torch.empty(128, 768, device="cuda").half()
     assert _stress(lambda: dp().linear(x, 3072, w, None, None, 0, y, 768, 128, 768, 3072, path=1, stream=main), y,
                    200, *noise) == 0
+
+
+@pytest.mark.parametrize("name,S,opts", [("bert_base", 128, {}), ("bert_large", 384, {}), ("gpt2", 256, {}),
+                                         ("bert_base", 128, {"fuse_ln": True}),
+                                         ("bert_base", 128, {"persistent": True})])
+def test_warm_forward_deterministic_under_contention(name, S, opts, noise):
+    """The whole warm forward (every kernel of the chain, PDL overlap included) beside the
+    noise kernel: bit-identical to the quiet run, 40 times."""
+    import synth
+    m = synth.SHAPES[name]
+    w = synth.make_weights(m, seed=41, dtype="fp16")
+    ids = torch.from_numpy(synth.make_ids(m, 1, S, seed=42)).cuda()
+    c = dp().Context([0])
+    c.set_opts(**opts)
+    model = dp().Model(c, m, w, "fp16")
+    plan = dp()._lib.PlanArrays(model.n, np.zeros(model.n, np.int8), None, 1, 1)
+    out = torch.empty(S, m.hidden, dtype=torch.float16, device="cuda")
+    pooled = torch.empty(1, m.hidden, dtype=torch.float16, device="cuda") if m.family != "gpt2" else None
+    model.infer_cold(plan, 0, ids, out, pooled)
+    torch.cuda.synchronize()
+    main = noise[3]
+    bad = _stress(lambda: model.infer_warm(0, ids, out, pooled, stream=main), out, 40, *noise)
+    model.evict(0)
+    model.close()
+    c.close()
+    assert bad == 0
