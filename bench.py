@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--no-pdl", action="store_true")
     ap.add_argument("--fuse-ln", action="store_true", help="LayerNorm in the preceding GEMM's epilogue")
     ap.add_argument("--profile-iters", type=int, default=10)
-    ap.add_argument("--pt-transport", default="dma", choices=["dma", "sm", "ce"],
+    ap.add_argument("--pt-transport", default="ce", choices=["dma", "sm", "ce"],
                     help="PT slots at N>1: dma = copy engine into a staging ring + NCCL send/recv (the paper's "
                          "two hops); sm = SURVEY f4 forwarder kernel (host -> primary HBM over CUDA IPC); "
                          "ce = one copy-engine DMA per piece straight into the primary's slot (CUDA IPC)")
@@ -272,7 +272,7 @@ def main():
     # profile on the primary, plan, share the plan (the plan never names GPUs)
     # default plan: Algorithm 1 on the link-aware model (R19); the paper's own
     # Algorithm-1 plan ("DHA") and the other engine options are timed beside it below
-    mode = a.mode or ("PT_DHA_LINK_BAL" if world > 1 else "DHA_LINK")
+    mode = a.mode or ("PT_DHA_LINK_STRIPE" if world > 1 else "DHA_LINK")
     if rank == 0:
         cost = model.profile(local, a.batch, a.seq, a.profile_iters)
     else:

@@ -69,7 +69,12 @@ enum {
    * bytes actually transferred (DHA units count 0) and Algorithm 1 re-run under the PT
    * arrival model on partition 0 */
   DP_MODE_PT_DHA_BAL = 8,
-  DP_MODE_PT_DHA_LINK_BAL = 9 /* the same on the link-aware model (R19 + R20) */
+  DP_MODE_PT_DHA_LINK_BAL = 9, /* the same on the link-aware model (R19 + R20) */
+  /* NEXT-row extension, R22: instead of contiguous partitions, the loaded units are
+   * striped over the k links by earliest arrival at the primary (so the links deliver the
+   * model front to back together), with Algorithm 1 run under that PT arrival model */
+  DP_MODE_PT_DHA_STRIPE = 10,
+  DP_MODE_PT_DHA_LINK_STRIPE = 11 /* the same on the link-aware model (R19 + R22) */
 };
 
 /* ---------------------------------------------------------------------------------

@@ -20,8 +20,9 @@ import numpy as np
 
 LOAD, DHA = 0, 1
 MODES = ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "PT", "PT_DHA")  # the paper's options
-EXT_MODES = ("DHA_LINK", "PT_DHA_LINK", "PT_DHA_BAL", "PT_DHA_LINK_BAL")  # NEXT-row extensions, R19 / R20
-LINK_AWARE = {"DHA_LINK", "PT_DHA_LINK", "PT_DHA_LINK_BAL"}
+EXT_MODES = ("DHA_LINK", "PT_DHA_LINK", "PT_DHA_BAL", "PT_DHA_LINK_BAL",  # NEXT-row extensions, R19 / R20
+             "PT_DHA_STRIPE", "PT_DHA_LINK_STRIPE")                              # R22
+LINK_AWARE = {"DHA_LINK", "PT_DHA_LINK", "PT_DHA_LINK_BAL", "PT_DHA_LINK_STRIPE"}
 INF_NS = 1 << 50
 
 
@@ -258,6 +259,37 @@ def partition_transferred(nbytes, method, k: int):
     return partition([int(b) if m == LOAD else 0 for b, m in zip(nbytes, method)], k)
 
 
+def stripe(cost, method, k: int, link_aware: bool = False):
+    """NEXT-row extension (R22), not the paper's rule: instead of contiguous equal
+    partitions, every loaded unit, in forward order, goes to the link on which it
+    would reach the primary first under the P1 model, given the units already assigned:
+      arrival(0) = link[0] + Load_i;  arrival(s >= 1) = max(link[s] + Load_i, fwd[s]) + Fwd_i
+    (ties -> the lowest slot).  The k links then deliver the model front to back together, so
+    the compute can follow the arrivals instead of waiting for a whole later partition.
+    DHA units stay in slot 0; on the link-aware model (R19) their reads occupy link 0 in
+    forward order, as in the simulator.  Returns slot[n]."""
+    n = len(cost["load_ns"])
+    load, fwd = _arr(cost, "load_ns"), _arr(cost, "fwd_ns")
+    dlink = _arr(cost, "dha_link_ns") if (link_aware and "dha_link_ns" in cost) else [0] * n
+    link = [0] * k
+    fw = [0] * k
+    slot = [0] * n
+    for i in range(n):
+        if method[i] == DHA:
+            link[0] += dlink[i]
+            continue
+        best, best_t = 0, None
+        for s in range(k):
+            t = link[0] + load[i] if s == 0 else max(link[s] + load[i], fw[s]) + fwd[i]
+            if best_t is None or t < best_t:
+                best, best_t = s, t
+        slot[i] = best
+        link[best] += load[i]
+        if best >= 1:
+            fw[best] = best_t
+    return slot
+
+
 def plan(cost, mode: str, k: int = 1):
     """Returns (method[n], slot[n], serial flag) for one of the five engine options
      plus the greedy comparison."""
@@ -302,6 +334,17 @@ def plan(cost, mode: str, k: int = 1):
         if link:
             return algorithm1_link(cost, slot, k, init=method), slot, False
         return algorithm1_slots(cost, slot, k, init=method), slot, False
+    if mode in ("PT_DHA_STRIPE", "PT_DHA_LINK_STRIPE"):
+        # R22: (1) every unit loaded, striped over the k links by earliest arrival; (2) Algorithm
+        # 1 (or its link-aware form) under that PT arrival model, candidates the slot-0 units
+        # (as R20 step 3); (3) the units still loaded re-striped around the chosen DHA set.
+        # With k = 1 this is exactly Algorithm 1.  (Starting from the one-link DHA set instead
+        # keeps DHA linears that only paid while one link carried everything.)
+        link = mode == "PT_DHA_LINK_STRIPE"
+        method = [LOAD] * n
+        slot = stripe(cost, method, k, link)
+        method = algorithm1_link(cost, slot, k, init=method) if link else algorithm1_slots(cost, slot, k, init=method)
+        return method, stripe(cost, method, k, link), False
     raise ValueError(mode)
 
 

@@ -11,7 +11,7 @@ _LIB_PATH = os.path.join(_HERE, "libdeepplan.so")
 
 LOAD, DHA = 0, 1
 MODES = {"BASELINE": 0, "PIPESWITCH": 1, "GREEDY": 2, "DHA": 3, "PT": 4, "PT_DHA": 5, "DHA_LINK": 6,
-         "PT_DHA_LINK": 7, "PT_DHA_BAL": 8, "PT_DHA_LINK_BAL": 9}
+         "PT_DHA_LINK": 7, "PT_DHA_BAL": 8, "PT_DHA_LINK_BAL": 9, "PT_DHA_STRIPE": 10, "PT_DHA_LINK_STRIPE": 11}
 UNIT_KINDS = {0: "emb", 1: "ln", 2: "linear"}
 FAMILIES = {"bert": 0, "roberta": 1, "gpt2": 2}
 DTYPES = {"fp16": 0, "bf16": 1}

@@ -135,7 +135,38 @@ static void algorithm1_link(const dp_cost_table* c, int8_t* method, const int8_t
 }
 
 static bool link_mode(int mode) {
-  return mode == DP_MODE_DHA_LINK || mode == DP_MODE_PT_DHA_LINK || mode == DP_MODE_PT_DHA_LINK_BAL;
+  return mode == DP_MODE_DHA_LINK || mode == DP_MODE_PT_DHA_LINK || mode == DP_MODE_PT_DHA_LINK_BAL ||
+         mode == DP_MODE_PT_DHA_LINK_STRIPE;
+}
+
+// Striped PT assignment (NEXT-row extension, R22; not the paper's contiguous rule):
+// each loaded unit, in forward order, goes to the link on which it reaches the primary first
+// under the pipeline model, given the units already assigned -- arrival on link 0 = link_0 +
+// Load_i, on link s >= 1 = max(link_s + Load_i, fwd_s) + Fwd_i; ties -> the lowest link.  DHA
+// units stay in slot 0; on the link-aware model their reads occupy link 0 in forward order.
+static void stripe(const dp_cost_table* c, const int8_t* method, int k, bool link_aware, int8_t* slot) {
+  const int n = c->n;
+  std::vector<int64_t> link(k, 0), fw(k, 0);
+  const bool la = link_aware && c->dha_link_ns != nullptr;
+  for (int i = 0; i < n; ++i) {
+    slot[i] = 0;
+    if (method[i] == DP_DHA) {
+      if (la) link[0] += c->dha_link_ns[i];
+      continue;
+    }
+    int best = 0;
+    int64_t best_t = 0;
+    for (int s = 0; s < k; ++s) {
+      const int64_t t = s == 0 ? link[0] + c->load_ns[i] : std::max(link[s] + c->load_ns[i], fw[s]) + c->fwd_ns[i];
+      if (s == 0 || t < best_t) {
+        best = s;
+        best_t = t;
+      }
+    }
+    slot[i] = int8_t(best);
+    link[best] += c->load_ns[i];
+    if (best >= 1) fw[best] = best_t;
+  }
 }
 
 static void partition(const int64_t* bytes, int n, int k, int8_t* part) {
@@ -230,6 +261,21 @@ static void generate(const dp_cost_table* c, int mode, int k, dp_plan* out) {
         algorithm1(c, out->method, out->slot, k, true);
       return;
     }
+    case DP_MODE_PT_DHA_STRIPE:
+    case DP_MODE_PT_DHA_LINK_STRIPE: {
+      // R22: (1) all units loaded, striped by earliest arrival; (2) Algorithm 1 (or its
+      // link-aware form) under that PT arrival model on the slot-0 units; (3) the units still
+      // loaded re-striped around the chosen DHA set.  k = 1 is exactly Algorithm 1.
+      const bool link = mode == DP_MODE_PT_DHA_LINK_STRIPE;
+      std::memset(out->method, DP_LOAD, n);
+      stripe(c, out->method, k, link, out->slot);
+      if (link)
+        algorithm1_link(c, out->method, out->slot, k, true);
+      else
+        algorithm1(c, out->method, out->slot, k, true);
+      stripe(c, out->method, k, link, out->slot);
+      return;
+    }
     default:
       fail(DP_ERR_INVALID, "unknown plan mode");
   }
@@ -276,7 +322,8 @@ extern "C" dp_status dp_plan_exhaustive(const dp_cost_table* cost, const dp_plan
     const int n = cost->n, k = std::max(1, base->k);
     std::vector<int8_t> part(n, 0), m(base->method, base->method + n);
     if (k > 1) {
-      if (base->mode == DP_MODE_PT_DHA_BAL || base->mode == DP_MODE_PT_DHA_LINK_BAL) {  // its own split
+      if (base->mode == DP_MODE_PT_DHA_BAL || base->mode == DP_MODE_PT_DHA_LINK_BAL ||
+          base->mode == DP_MODE_PT_DHA_STRIPE || base->mode == DP_MODE_PT_DHA_LINK_STRIPE) {  // its own split
         DP_CHECK(base->slot != nullptr, DP_ERR_INVALID, "bad base plan");
         std::copy(base->slot, base->slot + n, part.begin());
       } else {

@@ -98,7 +98,7 @@ def test_all_modes_match_oracle(name, B, S, dtype, recipe):
     tol = tolerance(dtype, recipe, ref)
     outs = {}
     for mode in ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "PT", "PT_DHA", "DHA_LINK", "PT_DHA_LINK", "PT_DHA_BAL",
-                 "PT_DHA_LINK_BAL"):
+                 "PT_DHA_LINK_BAL", "PT_DHA_STRIPE", "PT_DHA_LINK_STRIPE"):
         k = 3 if mode.startswith("PT") else 1
         plan = dp().plan_generate(cost, mode, k)
         out, pool, st = run_cold(model, plan, ids, dtype, secondaries=[0] * (k - 1))

@@ -95,7 +95,7 @@ def _run(model, plan, ids_np, dtype, k):
 
 @pytest.mark.parametrize("name,B,S", [("tiny_bert", 2, 77), ("tiny_gpt2", 1, 70), ("tiny_roberta", 2, 50),
                                       ("bert_base", 1, 128)])
-@pytest.mark.parametrize("mode,k", [("PT", 2), ("PT_DHA", 3), ("PT_DHA_LINK_BAL", 4)])
+@pytest.mark.parametrize("mode,k", [("PT", 2), ("PT_DHA", 3), ("PT_DHA_LINK_BAL", 4), ("PT_DHA_LINK_STRIPE", 8)])
 @pytest.mark.parametrize("transport", ["sm", "ce"])
 def test_sm_transport_equals_dma_and_oracle(name, B, S, mode, k, transport):
     m = synth.SHAPES[name]
@@ -218,7 +218,8 @@ def _ipc_worker(rank, world, port, name, mode, S, delay_us, transport, q):
 
 
 @pytest.mark.parametrize("name,mode,S,delay", [("tiny_bert", "PT", 32, 0), ("tiny_gpt2", "PT_DHA", 40, 300),
-                                               ("bert_base", "PT_DHA_BAL", 128, 0)])
+                                               ("bert_base", "PT_DHA_BAL", 128, 0),
+                                               ("bert_base", "PT_DHA_LINK_STRIPE", 128, 0)])
 @pytest.mark.parametrize("transport", ["sm", "ce"])
 def test_sm_transport_across_processes(name, mode, S, delay, transport):
     import torch.multiprocessing as mp

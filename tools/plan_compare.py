@@ -38,7 +38,8 @@ for spec in specs:
     out = torch.empty(S, m.hidden, dtype=torch.float16, device="cuda")
     pool = torch.empty(1, m.hidden, dtype=torch.float16, device="cuda") if m.family != "gpt2" else None
     res = {"units": model.n, "bytes": int(model.nbytes), "profile_s": round(prof_s, 2), "plans": {}}
-    for mode in ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "DHA_LINK", "PT", "PT_DHA", "PT_DHA_LINK", "PT_DHA_BAL", "PT_DHA_LINK_BAL"):
+    for mode in ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "DHA_LINK", "PT", "PT_DHA", "PT_DHA_LINK", "PT_DHA_BAL", "PT_DHA_LINK_BAL",
+                 "PT_DHA_STRIPE", "PT_DHA_LINK_STRIPE"):
         for k in ((1, 2, 4, 8) if mode.startswith("PT") else (1,)):
             plan = dp.plan_generate(cost, mode, k)
             lat, _, link = dp.plan_simulate(cost, plan)
