@@ -13,9 +13,12 @@
 //     kernel that reads it.
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <vector>
+
+#include <cuda.h>
 
 #include "engine.h"
 #include "kernels.h"
@@ -417,6 +420,22 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   std::memset(&st, 0, sizeof(st));
   st.n_units = n;
   std::vector<cudaEvent_t> unit_ev(n, nullptr);
+  // Wait points, per link (slot): every piece in the order its link delivers it, with the bytes
+  // its link has carried through its end (the landing-time proxy) and its completion (an event,
+  // or across processes a done word).  Pieces of one link complete in order, so waiting on
+  // piece r covers every earlier piece of that link.
+  struct WaitPt {
+    int64_t proxy = 0;
+    cudaEvent_t ev = nullptr;
+  };
+  std::vector<std::vector<WaitPt>> wp(std::max(1, plan->k));
+  std::vector<std::pair<int, int>> unit_wp(n, {-1, -1});  // (slot, piece) of a loaded unit
+  bool fifo0 = true;                                       // slot 0 on one load stream
+  auto add_wp = [&](int slot, const Piece& p, cudaEvent_t e) {
+    const int64_t prev = wp[slot].empty() ? 0 : wp[slot].back().proxy;
+    wp[slot].push_back({prev + p.bytes, e});
+    for (int u = p.first_unit; u <= p.last_unit; ++u) unit_wp[u] = {slot, (int)wp[slot].size() - 1};
+  };
 
   // fork: side streams start when the execution stream reaches this call
   cudaEvent_t fork = pd.events.get();
@@ -427,6 +446,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   const int64_t cap = std::max<int64_t>(ctx->opts.chunk_bytes, 4096);
   auto pieces0 = slot_pieces(m, plan, 0, cap, opt_tail(ctx));
   const int nh = std::min((int)pd.h2d.size(), std::max(1, ctx->opts.n_h2d_streams));
+  fifo0 = nh == 1;
   for (int i = 0; i < nh; ++i) DP_CUDA(cudaStreamWaitEvent(pd.h2d[i], fork, 0));
   for (size_t c = 0; c < pieces0.size(); ++c) {
     const Piece& p = pieces0[c];
@@ -440,13 +460,13 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     DP_CUDA(cudaEventRecord(e, hs));
     ++st.n_events;
     bind_units(unit_ev, p, e);  // every unit inside this piece completes with it
+    add_wp(0, p, e);
   }
 
   // (2) PT slots
   const bool one_hop = ctx->opts.pt_transport != DP_PT_DMA;  // single hop: SM forwarder or direct DMA
   const bool ce_fwd = ctx->opts.pt_transport == DP_PT_CE;
   // across processes with the SM forwarder: (slot, piece) a loaded unit arrives in
-  std::vector<std::pair<int, int>> unit_piece(n, {-1, -1});
   std::vector<size_t> slot_npieces(plan->k, 0);
   uint32_t epoch = 0;
   if (!ctx->multiproc())
@@ -469,7 +489,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       auto pcs = slot_pieces(m, plan, s, cap, opt_tail(ctx));
       slot_npieces[s] = pcs.size();
       for (size_t r = 0; r < pcs.size(); ++r) {
-        for (int u = pcs[r].first_unit; u <= pcs[r].last_unit; ++u) unit_piece[u] = {s, (int)r};
+        add_wp(s, pcs[r], nullptr);
         st.nvlink_bytes[s] += pcs[r].bytes;
       }
     }
@@ -506,6 +526,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
         DP_CUDA(cudaEventRecord(done, r.h2d));
         ++st.n_events;
         bind_units(unit_ev, p, done);
+        add_wp(s, p, done);
       }
       // the end-of-cold-start join waits on the migration stream: chain it behind the loads
       cudaEvent_t last = sd.events.get();
@@ -539,6 +560,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       st.n_events += 2;
       fwd_done[c] = done;
       bind_units(unit_ev, p, done);
+      add_wp(s, p, done);
     }
   }
 
@@ -556,22 +578,60 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   a.pooled = pooled;
   a.stream = stream;
   a.bn_hint = ctx->opts.gemm_bn;
-  std::pair<int, int> last_piece{-1, -1};
+  // Before a loaded unit's first kernel, wait for its piece -- and, in the same batch,
+  // for every OTHER link's pieces that land no later than it plus kWaitSlack bytes of link
+  // time: with PT the next units come from the other links at about the same time, so one
+  // batch covers a round of them and the execution stream pays one dependency point (and
+  // loses one PDL overlap) per round instead of per unit (a wait costs ~0.6 us in a graph,
+  // ~3.6 us as a kernel outside one: tools/wait_cost.py).  On the unit's own link nothing
+  // later than its piece is waited for, so one link (k = 1) waits exactly as before.
+  static const bool coalesce = std::getenv("DP_NO_WAIT_COALESCE") == nullptr;  // A/B experiments
+  constexpr int64_t kWaitSlack = 2 << 20;
+  std::vector<int> waited(std::max(1, plan->k), -1);
+  std::vector<char> done0(wp[0].size(), 0);
   a.before_unit = [&](int u) {
     if (method[u] == DP_DHA) return;  // DHA layers skip the dependency check
-    if (unit_piece[u].first > 0) {    // across processes: acquire the piece's done word
-      if (unit_piece[u] == last_piece) return;
-      ipc_primary_wait(ctx, unit_piece[u].first, (size_t)unit_piece[u].second, epoch, stream);
+    const int s0 = unit_wp[u].first, r0 = unit_wp[u].second;
+    if (s0 < 0) {  // NCCL rounds (peer.cpp): one event per round, bound per unit
+      cudaEvent_t e = unit_ev[u];
+      DP_CHECK(e != nullptr, DP_ERR_STATE, "internal: loaded unit has no completion event");
+      if (e == last_waited) return;
+      DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
       pdl_state().block_next = true;
-      last_piece = unit_piece[u];
+      last_waited = e;
       return;
     }
-    cudaEvent_t e = unit_ev[u];
-    DP_CHECK(e != nullptr, DP_ERR_STATE, "internal: loaded unit has no completion event");
-    if (e == last_waited) return;
-    DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
+    if (s0 == 0 && !fifo0) {  // several load streams: pieces of link 0 may complete out of order
+      if (done0[r0]) return;
+      done0[r0] = 1;
+    } else if (r0 <= waited[s0]) {
+      return;  // covered by an earlier wait on this link
+    }
+    // candidates: the pieces of the next 2k units (forward order) on the other links, if they
+    // land no later than this one plus the slack -- pieces needed soon, never a later
+    // partition's (with contiguous partitions the next units share this link: no batching)
+    const int64_t horizon = wp[s0][r0].proxy + kWaitSlack;
+    std::vector<int> want(wp.size(), -1);
+    want[s0] = r0;
+    for (int v = u + 1; coalesce && v < n && v <= u + 2 * (int)wp.size(); ++v) {
+      const int s = unit_wp[v].first, r = unit_wp[v].second;
+      if (s < 0 || s == s0 || (s == 0 && !fifo0) || r <= waited[s]) continue;
+      if (wp[s][r].proxy <= horizon) want[s] = std::max(want[s], r);
+    }
+    std::vector<std::pair<int, int>> batch{{s0, r0}};
+    for (int s = 0; s < (int)wp.size(); ++s)
+      if (s != s0 && want[s] > waited[s]) batch.push_back({s, want[s]});
+    std::vector<std::pair<int, size_t>> flags;  // across processes: done words, one wait kernel
+    for (auto& b : batch) {
+      cudaEvent_t e = wp[b.first][b.second].ev;
+      if (e != nullptr)
+        DP_CUDA(cudaStreamWaitEvent(stream, e, 0));
+      else
+        flags.push_back({b.first, (size_t)b.second});
+    }
+    if (!flags.empty()) ipc_primary_wait_many(ctx, flags, epoch, stream);
+    for (auto& b : batch) waited[b.first] = std::max(waited[b.first], b.second);
     pdl_state().block_next = true;  // the next kernel must see the landed weights: no PDL overlap
-    last_waited = e;
   };
   a.pdl = ctx->opts.use_pdl != 0;
   a.fuse_ln = ctx->opts.fuse_ln != 0;
@@ -653,11 +713,55 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.pdl = ctx->opts.use_pdl != 0;
     a.fuse_ln = ctx->opts.fuse_ln != 0;
     a.persistent = ctx->opts.persistent != 0;
+    // Experiment (tools/wait_cost.py): the cost of a dependency wait before every unit on the
+    // execution stream, all already satisfied -- 1: event wait, 2: one-thread acquire-spin
+    // kernel on a device word, 3: cuStreamWaitValue32 (stream memory op)
+    static const int dbg_waits = [] {
+      const char* e = std::getenv("DP_DEBUG_WARM_WAITS");
+      return e ? std::atoi(e) : 0;
+    }();
+    static uint32_t* dbg_word = nullptr;
+    static cudaStream_t dbg_side = nullptr;
+    static cudaEvent_t dbg_fork = nullptr, dbg_ev = nullptr;
+    using WaitValueFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+    static WaitValueFn wait_value = nullptr;
+    if (dbg_waits) {
+      if (!dbg_word) {
+        DP_CUDA(cudaMalloc(&dbg_word, 64));
+        DP_CUDA(cudaMemset(dbg_word, 1, 64));
+        DP_CUDA(cudaStreamCreateWithFlags(&dbg_side, cudaStreamNonBlocking));
+        DP_CUDA(cudaEventCreateWithFlags(&dbg_fork, cudaEventDisableTiming));
+        DP_CUDA(cudaEventCreateWithFlags(&dbg_ev, cudaEventDisableTiming));
+        cudaDriverEntryPointQueryResult q;
+        DP_CUDA(cudaGetDriverEntryPoint("cuStreamWaitValue32", reinterpret_cast<void**>(&wait_value),
+                                        cudaEnableDefault, &q));
+      }
+      a.before_unit = [&](int u) {
+        if (ds.method[u] == DP_DHA) return;
+        if (dbg_waits == 1) {
+          DP_CUDA(cudaStreamWaitEvent(a.stream, dbg_ev, 0));
+        } else if (dbg_waits == 2) {
+          launch_pt_wait(dbg_word, 1, a.stream);
+        } else {
+          DP_CHECK(wait_value(a.stream, (CUdeviceptr)dbg_word, 1, CU_STREAM_WAIT_VALUE_GEQ) == CUDA_SUCCESS,
+                   DP_ERR_CUDA, "cuStreamWaitValue32 failed");
+        }
+        pdl_state().block_next = true;
+      };
+    }
+    auto dbg_fork_side = [&](cudaStream_t st) {
+      if (dbg_waits != 1) return;
+      DP_CUDA(cudaEventRecord(dbg_fork, st));
+      DP_CUDA(cudaStreamWaitEvent(dbg_side, dbg_fork, 0));
+      DP_CUDA(cudaEventRecord(dbg_ev, dbg_side));
+    };
     if (ctx->opts.use_graph) {
       std::string key = "warm|" + std::to_string(a.persistent) + "|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
                         graph_key(ctx, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);
+      if (dbg_waits) key += "|dbgwait" + std::to_string(dbg_waits);
       dp_run_stats gs = run_graph(ds, key, (cudaStream_t)stream, [&](cudaStream_t cs) {
         a.stream = cs;
+        dbg_fork_side(cs);
         run_forward(a);
         dp_run_stats s{};
         s.n_kernels = a.kernels;
@@ -665,6 +769,7 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
       });
       a.kernels = gs.n_kernels;
     } else {
+      dbg_fork_side(a.stream);
       run_forward(a);
     }
     if (stats) {

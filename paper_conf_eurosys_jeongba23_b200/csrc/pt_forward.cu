@@ -202,9 +202,32 @@ void ipc_primary_begin(dp_context* ctx, const dp_plan* plan, int prim_rank, cuda
   DP_CUDA(cudaGetLastError());
 }
 
+void launch_pt_wait(const uint32_t* flag, uint32_t value, cudaStream_t s) {
+  pt_wait_kernel<<<1, 1, 0, s>>>(flag, value);
+  DP_CUDA(cudaGetLastError());
+}
+
 void ipc_primary_wait(dp_context* ctx, int slot, size_t piece, uint32_t epoch, cudaStream_t exec) {
   DP_CHECK(piece < (size_t)kMbMaxPieces, DP_ERR_UNSUPPORTED, "too many PT pieces for the mailbox");
   pt_wait_kernel<<<1, 1, 0, exec>>>(done_word(ctx->mailbox, slot, piece), epoch);
+  DP_CUDA(cudaGetLastError());
+}
+
+__global__ void pt_wait_many_kernel(FlagPtrs f, int n, uint32_t value) {
+  if ((int)threadIdx.x < n) wait_flag(f.p[threadIdx.x], value);
+}
+
+void ipc_primary_wait_many(dp_context* ctx, const std::vector<std::pair<int, size_t>>& pieces, uint32_t epoch,
+                           cudaStream_t exec) {
+  FlagPtrs f{};
+  int n = 0;
+  for (const auto& sp : pieces) {
+    DP_CHECK(sp.second < (size_t)kMbMaxPieces, DP_ERR_UNSUPPORTED, "too many PT pieces for the mailbox");
+    DP_CHECK(n < DP_MAX_DEVICES, DP_ERR_INVALID, "internal: more than one wait per link in a batch");
+    f.p[n++] = done_word(ctx->mailbox, sp.first, sp.second);
+  }
+  if (!n) return;
+  pt_wait_many_kernel<<<1, 32, 0, exec>>>(f, n, epoch);
   DP_CUDA(cudaGetLastError());
 }
 

@@ -31,7 +31,9 @@ stream = torch.cuda.Stream()
 res = []
 ref = None
 bad = []
-for mode, k in (("PIPESWITCH", 1), ("PT", 2), ("PT", 4), ("PT_DHA_LINK_BAL", 4)):
+cases = [tuple(c.split("/")) for c in os.environ.get("DP_PT_CASES", "").split(",") if c] or \
+    [("PIPESWITCH", "1"), ("PT", "2"), ("PT", "4"), ("PT_DHA_LINK_BAL", "4")]
+for mode, k in ((m_, int(k_)) for m_, k_ in cases):
     plan = dp.plan_generate(cost, mode, k)
     for tr in (("dma",) if k == 1 else ("dma", "sm", "ce")):
         ctx.set_opts(pt_transport=tr, use_graph=1)
