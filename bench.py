@@ -251,7 +251,8 @@ def main():
     ids_np = synth.make_ids(m, a.batch, a.seq, seed=1)
     ctx = dp.Context([local])
     ctx.set_opts(chunk_bytes=int(a.chunk_mb * (1 << 20)), n_h2d_streams=a.h2d_streams,
-                 tail_bytes=int(a.tail_mb * (1 << 20)), use_graph=0 if (a.no_graph or world > 1) else 1,
+                 tail_bytes=int(a.tail_mb * (1 << 20)),
+                 use_graph=0 if (a.no_graph or (world > 1 and a.pt_transport == "dma")) else 1,
                  use_pdl=0 if a.no_pdl else 1, fuse_ln=a.fuse_ln, pt_transport=a.pt_transport)
     model = dp.Model(ctx, m, w, dtype)
     if dist_on and a.pt_transport == "dma":

@@ -332,7 +332,7 @@ static std::string graph_key(const dp_context* ctx, const dp_plan* plan, const i
     k.append(reinterpret_cast<const char*>(plan->method), plan->n);
     k.append(reinterpret_cast<const char*>(plan->slot), plan->n);
     k += "|" + std::to_string(plan->k);
-    for (int s = 1; s < plan->k; ++s) k += "," + std::to_string(secondaries[s - 1]);
+    for (int s = 1; s < plan->k; ++s) k += "," + (secondaries ? std::to_string(secondaries[s - 1]) : "r");
   }
   k += "|" + std::to_string((uintptr_t)ids) + "|" + std::to_string((uintptr_t)out) + "|" +
        std::to_string((uintptr_t)pooled) + "|" + std::to_string(batch) + "x" + std::to_string(seq) + "|" +
@@ -391,8 +391,16 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   ensure_slots(m, primary);
   ensure_h2d_streams(ctx, primary);
   ensure_workspace(m, primary, int64_t(batch) * seq);
-  bool graph = ctx->opts.use_graph != 0 && !ctx->multiproc();
-  for (int s = 1; s < plan->k && graph; ++s) graph = secondaries[s - 1] == primary;  // single-device graphs only
+  // across processes: the IPC transports capture (the epoch lives in a device word); the NCCL
+  // gather does not
+  const bool ipc_pt = ctx->multiproc() && ctx->opts.pt_transport != DP_PT_DMA && plan->k > 1;
+  bool graph = ctx->opts.use_graph != 0 && (!ctx->multiproc() || ipc_pt || plan->k == 1);
+  for (int s = 1; s < plan->k && graph && !ctx->multiproc(); ++s)
+    graph = secondaries[s - 1] == primary;  // single-device graphs only
+  if (ipc_pt) {
+    ipc_check_primary(ctx);
+    ipc_set_epoch(ctx, ++ctx->pt_epoch, stream);  // every rank counts the same k > 1 cold starts
+  }
   dp_run_stats st;
   if (graph) {
     st = run_graph(ds, graph_key(ctx, plan, secondaries, ids, batch, seq, out, pooled), stream, [&](cudaStream_t cs) {
@@ -468,7 +476,6 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   const bool ce_fwd = ctx->opts.pt_transport == DP_PT_CE;
   // across processes with the SM forwarder: (slot, piece) a loaded unit arrives in
   std::vector<size_t> slot_npieces(plan->k, 0);
-  uint32_t epoch = 0;
   if (!ctx->multiproc())
     for (int s = 1; s < plan->k; ++s) {
       const int sdev = secondaries[s - 1];
@@ -482,9 +489,8 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   }
   if (ctx->multiproc() && one_hop && plan->k > 1) {
     // go to every secondary; their forwarders store into our slots and release done words
-    ipc_check_primary(ctx);
-    epoch = ++ctx->pt_epoch;
-    ipc_primary_begin(ctx, plan, prim_rank, stream, epoch);
+    ipc_check_primary(ctx);  // the epoch word was set by infer_cold
+    ipc_primary_begin(ctx, plan, prim_rank, stream);
     for (int s = 1; s < plan->k; ++s) {
       auto pcs = slot_pieces(m, plan, s, cap, opt_tail(ctx));
       slot_npieces[s] = pcs.size();
@@ -629,7 +635,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       else
         flags.push_back({b.first, (size_t)b.second});
     }
-    if (!flags.empty()) ipc_primary_wait_many(ctx, flags, epoch, stream);
+    if (!flags.empty()) ipc_primary_wait_many(ctx, flags, stream);
     for (auto& b : batch) waited[b.first] = std::max(waited[b.first], b.second);
     pdl_state().block_next = true;  // the next kernel must see the landed weights: no PDL overlap
   };
@@ -644,7 +650,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     ++st.n_events;
   }
   for (int s = 1; s < plan->k && ctx->multiproc() && one_hop; ++s)  // every piece landed
-    if (slot_npieces[s] > 0) ipc_primary_wait(ctx, s, slot_npieces[s] - 1, epoch, stream);
+    if (slot_npieces[s] > 0) ipc_primary_wait(ctx, s, slot_npieces[s] - 1, stream);
   for (int s = 1; s < plan->k && !ctx->multiproc(); ++s) {
     auto it = ctx->slots.find({s, secondaries[s - 1]});
     if (it == ctx->slots.end()) continue;

@@ -32,11 +32,13 @@ void launch_pt_forward(const void* src, void* dst, int64_t bytes, cudaStream_t s
 // waits on done[slot][piece] before the units of that piece; a secondary forwards its slot.
 void launch_pt_wait(const uint32_t* flag, uint32_t value, cudaStream_t s);  // one-thread acquire-spin
 void ipc_check_primary(dp_context* ctx);
-void ipc_primary_begin(dp_context* ctx, const dp_plan* plan, int prim_rank, cudaStream_t exec, uint32_t epoch);
-void ipc_primary_wait(dp_context* ctx, int slot, size_t piece, uint32_t epoch, cudaStream_t exec);
+// The primary's kernels read the epoch from its mailbox word, set (outside any graph) by
+// ipc_set_epoch before each cold start, so a captured cold-start graph is replayable.
+void ipc_set_epoch(dp_context* ctx, uint32_t epoch, cudaStream_t exec);
+void ipc_primary_begin(dp_context* ctx, const dp_plan* plan, int prim_rank, cudaStream_t exec);
+void ipc_primary_wait(dp_context* ctx, int slot, size_t piece, cudaStream_t exec);
 // One wait kernel for several (slot, piece) done words (at most one per link).
-void ipc_primary_wait_many(dp_context* ctx, const std::vector<std::pair<int, size_t>>& pieces, uint32_t epoch,
-                           cudaStream_t exec);
+void ipc_primary_wait_many(dp_context* ctx, const std::vector<std::pair<int, size_t>>& pieces, cudaStream_t exec);
 void ipc_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, dp_run_stats* stats);
 void ipc_close(dp_context* ctx);
 void ipc_close_model(dp_model* m);

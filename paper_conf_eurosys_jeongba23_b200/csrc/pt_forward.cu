@@ -39,6 +39,7 @@ namespace dp {
 // Mailbox layout (uint32 words).  The primary's done words are written by secondaries; the
 // counters are the forwarding rank's own (last-CTA detection per piece).
 constexpr int kMbGo = 0;
+constexpr int kMbEpoch = 1;  // this rank's current epoch, read by its signal / wait kernels (graph-safe)
 constexpr int kMbMaxPieces = 256;
 constexpr int kMbDone = 64;                                          // [slot][piece]
 constexpr int kMbCount = kMbDone + DP_MAX_DEVICES * kMbMaxPieces;   // [piece]
@@ -127,14 +128,21 @@ struct FlagPtrs {
   uint32_t* p[DP_MAX_DEVICES];
 };
 
-__global__ void pt_signal_kernel(FlagPtrs f, int n, uint32_t value) {
+// value_word != nullptr: the value is read from that device word (the primary's epoch, so a
+// captured CUDA graph stays valid across cold starts)
+__global__ void pt_signal_kernel(FlagPtrs f, int n, uint32_t value, const uint32_t* value_word) {
   if ((int)threadIdx.x < n) {
+    const uint32_t v = value_word ? *value_word : value;
     __threadfence_system();
-    st_release_sys(f.p[threadIdx.x], value);
+    st_release_sys(f.p[threadIdx.x], v);
   }
 }
 
-__global__ void pt_wait_kernel(const uint32_t* flag, uint32_t value) { wait_flag(flag, value); }
+__global__ void pt_set_word_kernel(uint32_t* w, uint32_t v) { *w = v; }
+
+__global__ void pt_wait_kernel(const uint32_t* flag, uint32_t value, const uint32_t* value_word) {
+  wait_flag(flag, value_word ? *value_word : value);
+}
 
 int sm_count(int dev) {
   static int cache[DP_MAX_DEVICES] = {};
@@ -189,7 +197,12 @@ static void ensure_mailbox(dp_context* ctx) {
   ctx->mailbox = static_cast<uint32_t*>(p);
 }
 
-void ipc_primary_begin(dp_context* ctx, const dp_plan* plan, int prim_rank, cudaStream_t exec, uint32_t epoch) {
+void ipc_set_epoch(dp_context* ctx, uint32_t epoch, cudaStream_t exec) {
+  pt_set_word_kernel<<<1, 1, 0, exec>>>(ctx->mailbox + kMbEpoch, epoch);
+  DP_CUDA(cudaGetLastError());
+}
+
+void ipc_primary_begin(dp_context* ctx, const dp_plan* plan, int prim_rank, cudaStream_t exec) {
   FlagPtrs f{};
   int n = 0;
   for (int s = 1; s < plan->k; ++s) {
@@ -198,27 +211,26 @@ void ipc_primary_begin(dp_context* ctx, const dp_plan* plan, int prim_rank, cuda
     f.p[n++] = ctx->peer_mailbox[r] + kMbGo;
   }
   if (!n) return;
-  pt_signal_kernel<<<1, 32, 0, exec>>>(f, n, epoch);
+  pt_signal_kernel<<<1, 32, 0, exec>>>(f, n, 0, ctx->mailbox + kMbEpoch);
   DP_CUDA(cudaGetLastError());
 }
 
 void launch_pt_wait(const uint32_t* flag, uint32_t value, cudaStream_t s) {
-  pt_wait_kernel<<<1, 1, 0, s>>>(flag, value);
+  pt_wait_kernel<<<1, 1, 0, s>>>(flag, value, nullptr);
   DP_CUDA(cudaGetLastError());
 }
 
-void ipc_primary_wait(dp_context* ctx, int slot, size_t piece, uint32_t epoch, cudaStream_t exec) {
+void ipc_primary_wait(dp_context* ctx, int slot, size_t piece, cudaStream_t exec) {
   DP_CHECK(piece < (size_t)kMbMaxPieces, DP_ERR_UNSUPPORTED, "too many PT pieces for the mailbox");
-  pt_wait_kernel<<<1, 1, 0, exec>>>(done_word(ctx->mailbox, slot, piece), epoch);
+  pt_wait_kernel<<<1, 1, 0, exec>>>(done_word(ctx->mailbox, slot, piece), 0, ctx->mailbox + kMbEpoch);
   DP_CUDA(cudaGetLastError());
 }
 
-__global__ void pt_wait_many_kernel(FlagPtrs f, int n, uint32_t value) {
-  if ((int)threadIdx.x < n) wait_flag(f.p[threadIdx.x], value);
+__global__ void pt_wait_many_kernel(FlagPtrs f, int n, const uint32_t* value_word) {
+  if ((int)threadIdx.x < n) wait_flag(f.p[threadIdx.x], *value_word);
 }
 
-void ipc_primary_wait_many(dp_context* ctx, const std::vector<std::pair<int, size_t>>& pieces, uint32_t epoch,
-                           cudaStream_t exec) {
+void ipc_primary_wait_many(dp_context* ctx, const std::vector<std::pair<int, size_t>>& pieces, cudaStream_t exec) {
   FlagPtrs f{};
   int n = 0;
   for (const auto& sp : pieces) {
@@ -227,7 +239,7 @@ void ipc_primary_wait_many(dp_context* ctx, const std::vector<std::pair<int, siz
     f.p[n++] = done_word(ctx->mailbox, sp.first, sp.second);
   }
   if (!n) return;
-  pt_wait_many_kernel<<<1, 32, 0, exec>>>(f, n, epoch);
+  pt_wait_many_kernel<<<1, 32, 0, exec>>>(f, n, ctx->mailbox + kMbEpoch);
   DP_CUDA(cudaGetLastError());
 }
 
@@ -258,7 +270,7 @@ void ipc_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int primar
   uint8_t* dst = static_cast<uint8_t*>(m->peer_dbase[primary]);
   const bool ce = ctx->opts.pt_transport == DP_PT_CE;
   if (ce && !pcs.empty()) {  // the copy engine cannot poll: a one-thread kernel acquires `go`
-    pt_wait_kernel<<<1, 1, 0, ctx->comm_stream>>>(ctx->mailbox + kMbGo, epoch);
+    pt_wait_kernel<<<1, 1, 0, ctx->comm_stream>>>(ctx->mailbox + kMbGo, epoch, nullptr);
     DP_CUDA(cudaGetLastError());
   }
   for (size_t r = 0; r < pcs.size(); ++r) {
@@ -269,7 +281,7 @@ void ipc_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int primar
                               cudaMemcpyDefault, ctx->comm_stream));
       FlagPtrs f{};
       f.p[0] = done_word(ctx->peer_mailbox[primary], slot, r);
-      pt_signal_kernel<<<1, 32, 0, ctx->comm_stream>>>(f, 1, epoch);
+      pt_signal_kernel<<<1, 32, 0, ctx->comm_stream>>>(f, 1, epoch, nullptr);
       DP_CUDA(cudaGetLastError());
       st.h2d_bytes[slot] += pc.bytes;
       st.nvlink_bytes[slot] += pc.bytes;
