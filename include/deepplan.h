@@ -184,6 +184,14 @@ typedef struct {
                              DP_PT_CE = the same single hop driven by the secondary's copy
                              engine: one DMA per piece from the arena straight into the
                              primary's slot through the peer / IPC mapping (no staging ring) */
+  int32_t profile_chain;  /* 1 = dp_profile calibrates the per-unit costs to how the engine runs
+                             them (R23): Exe(InMem) rescaled so that their sum is the
+                             measured chained warm forward (units timed in isolation -- L2
+                             flushed, no PDL overlap -- sum to ~2.6x the real forward on B200;
+                             a DHA unit keeps its absolute extra host-read time), and Load = the
+                             unit's byte share of one whole-arena copy (the engine coalesces
+                             loads, R18; an isolated copy carries ~4 us of per-copy cost) [1] */
+  int32_t reserved[3];
 } dp_engine_opts;
 #define DP_PT_DMA 0
 #define DP_PT_SM 1

@@ -52,7 +52,8 @@ class EngineOpts(C.Structure):
     _fields_ = [("chunk_bytes", C.c_int64), ("n_h2d_streams", C.c_int32), ("use_graph", C.c_int32),
                 ("gemm_bn", C.c_int32), ("debug_delay_us", C.c_int32), ("debug_poison", C.c_int32),
                 ("use_pdl", C.c_int32), ("fuse_ln", C.c_int32), ("tail_bytes", C.c_int64),
-                ("persistent", C.c_int32), ("pt_transport", C.c_int32)]
+                ("persistent", C.c_int32), ("pt_transport", C.c_int32), ("profile_chain", C.c_int32),
+                ("reserved", C.c_int32 * 3)]
 
 
 class ModelConfig(C.Structure):
@@ -280,7 +281,7 @@ class Context:
 
     def set_opts(self, chunk_bytes=None, n_h2d_streams=None, use_graph=None, gemm_bn=None, debug_delay_us=None,
                  debug_poison=None, use_pdl=None, tail_bytes=None, fuse_ln=None, persistent=None,
-                 pt_transport=None):
+                 pt_transport=None, profile_chain=None):
         o = EngineOpts()
         _check(lib.dp_context_get_opts(self.h, C.byref(o)))
         if chunk_bytes is not None:
@@ -303,6 +304,8 @@ class Context:
             o.fuse_ln = 1 if fuse_ln else 0
         if persistent is not None:
             o.persistent = 1 if persistent else 0
+        if profile_chain is not None:
+            o.profile_chain = 1 if profile_chain else 0
         if pt_transport is not None:
             o.pt_transport = PT_TRANSPORTS[pt_transport] if isinstance(pt_transport, str) else int(pt_transport)
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))

@@ -135,6 +135,7 @@ extern "C" dp_status dp_context_create(const int32_t* devs, int32_t ndev, dp_con
     ctx->opts.use_pdl = 1;
     ctx->opts.tail_bytes = 2 << 20;
     ctx->opts.chunk_bytes = 32 << 20;
+    ctx->opts.profile_chain = 1;
     for (int i = 0; i < ndev; ++i) {
       DP_CHECK(devs[i] >= 0 && devs[i] < count && devs[i] < DP_MAX_DEVICES, DP_ERR_INVALID,
                "device " + std::to_string(devs[i]) + " does not exist");
@@ -901,13 +902,13 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
   DP_CUDA(cudaEventCreate(&e1));
   const int warm = 3;
   const int n = (int)m->units.size();
-  auto timed = [&](auto&& body, bool flush) {
+  auto timed = [&](auto&& body, bool flush, long long spin = 60000) {
     std::vector<float> v;
     for (int it = 0; it < warm + iters; ++it) {
       if (flush) launch_l2_flush(d.flush, d.flush_bytes, s);
       // keep the stream busy while the host enqueues the measured work, so the interval
       // e0..e1 holds device time only (not the host's launch latency)
-      launch_spin(60000, s);
+      launch_spin(spin, s);
       DP_CUDA(cudaEventRecord(e0, s));
       body();
       DP_CUDA(cudaEventRecord(e1, s));
@@ -946,6 +947,49 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
     } else {
       out->exe_mem_ns[u] = timed([&] { run_unit(m, dev, u, false, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
       out->exe_dha_ns[u] = timed([&] { run_unit(m, dev, u, true, ids, batch, seq, s, ctx->opts.gemm_bn); }, true);
+    }
+  }
+  // R23: the chained warm forward (every unit resident, PDL chain as the engine runs it, L2
+  // flushed before it) against the sum of the isolated unit times; Exe(InMem) is rescaled to
+  // it, Exe(DHA) keeps its absolute extra (the host reads) over Exe(InMem)
+  if (ctx->opts.profile_chain) {
+    std::vector<int8_t> all_load(n, DP_LOAD);
+    ForwardArgs fa;
+    fa.m = m;
+    fa.dev = dev;
+    fa.method = all_load.data();
+    fa.ids = ids;
+    fa.batch = batch;
+    fa.seq = seq;
+    void* chain_out = nullptr;
+    DP_CUDA(cudaMalloc(&chain_out, size_t(T) * m->cfg.hidden * 4));
+    fa.out = chain_out;
+    fa.pooled = nullptr;
+    fa.stream = s;
+    fa.bn_hint = ctx->opts.gemm_bn;
+    fa.pdl = ctx->opts.use_pdl != 0;
+    fa.fuse_ln = ctx->opts.fuse_ln != 0;
+    // the host enqueues ~100 launches behind a ~1.5 ms spin, so e0..e1 is device time only
+    const int64_t chain = timed([&] { run_forward(fa); }, true, 3000000);
+    DP_CUDA(cudaStreamSynchronize(s));
+    cudaFree(chain_out);
+    int64_t sum = 0;
+    for (int u = 0; u < n; ++u) sum += out->exe_mem_ns[u];
+    // loads: the engine coalesces adjacent loaded units into large DMAs (R18), so a unit's
+    // marginal link time is its share of one copy of the whole arena, not an isolated copy
+    // (which carries ~4 us of per-copy cost: 98 BERT-Base units would add ~0.4 ms)
+    const int64_t all_ns = timed([&] {
+      DP_CUDA(cudaMemcpyAsync(ds.dbase, m->arena, m->arena_bytes, cudaMemcpyHostToDevice, s));
+    }, false);
+    for (int u = 0; u < n; ++u)
+      out->load_ns[u] = (int64_t)llround(double(all_ns) * double(out->bytes[u]) / double(m->arena_bytes));
+    if (chain > 0 && sum > chain) {
+      const double f = double(chain) / double(sum);
+      for (int u = 0; u < n; ++u) {
+        const int64_t mem = (int64_t)llround(double(out->exe_mem_ns[u]) * f);
+        if (out->exe_dha_ns[u] < DP_INF_NS) out->exe_dha_ns[u] = std::max<int64_t>(0, mem + out->exe_dha_ns[u] - out->exe_mem_ns[u]);
+        out->exe_mem_ns[u] = mem;
+      }
     }
   }
   // link time of each unit's DHA reads (link-aware modes): the unit's own measured load time
