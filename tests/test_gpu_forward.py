@@ -316,10 +316,12 @@ def test_bert_base_batched_cold_start():
     model.close()
 
 
-@pytest.mark.parametrize("name,S,mode,k", [("bert_large", 384, "PT_DHA_LINK_BAL", 2),
-                                           ("roberta_large", 384, "DHA_LINK", 1),
-                                           ("bert_large", 384, "PT_DHA", 4)])
-def test_large_models_full_size(name, S, mode, k):
+@pytest.mark.parametrize("name,S,mode,k,transport", [("bert_large", 384, "PT_DHA_LINK_BAL", 2, "dma"),
+                                                     ("roberta_large", 384, "DHA_LINK", 1, "dma"),
+                                                     ("bert_large", 384, "PT_DHA", 4, "dma"),
+                                                     ("bert_large", 384, "PT_DHA_LINK_STRIPE", 8, "ce"),
+                                                     ("roberta_large", 384, "PT_DHA_STRIPE", 4, "sm")])
+def test_large_models_full_size(name, S, mode, k, transport):
     """BASELINE.json configs[2]/[3] at full size: BERT-Large / RoBERTa-Large fp16, batch 1, seq
     384, a live profile -> the plan -> cold start (PT slots served in loopback on this one GPU:
     the event / ring logic of the multi-GPU path, not its bandwidth), vs the fp64 oracle at the
@@ -329,7 +331,9 @@ def test_large_models_full_size(name, S, mode, k):
     w = synth.make_weights(m, seed=7, dtype=dtype)
     ids = synth.make_ids(m, 1, S, seed=8)
     ref, ref_pool = F.forward(m, w, ids, dtype)
-    model = dp().Model(ctx(), m, w, dtype)
+    c = dp().Context([0])
+    c.set_opts(pt_transport=transport)
+    model = dp().Model(c, m, w, dtype)
     cost = model.profile(0, 1, S, iters=2)
     plan = dp().plan_generate(cost, mode, k)
     om, osl, ser = OP.plan(cost, mode, k)
@@ -341,3 +345,4 @@ def test_large_models_full_size(name, S, mode, k):
     link = OP.simulate(cost, om, osl, k, ser)["link_bytes"]
     assert st["h2d_bytes"][:len(link)] == link
     model.close()
+    c.close()

@@ -39,13 +39,13 @@ def _cost(name):
                "exe_dha_ns": exe + rng.integers(0, 3000, n)}
 
 
-def _worker(rank, world, port, name, chunk, q):
+def _worker(rank, world, port, name, chunk, q, mode="PT_DHA"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         import paper_conf_eurosys_jeongba23_b200._lib as L
         m, cost = _cost(name)
-        plan = L.plan_generate(cost, "PT_DHA", world)
+        plan = L.plan_generate(cost, mode, world)
         # every rank derives the identical plan
         mine = torch.from_numpy(plan.method.astype(np.int64))
         other = mine.clone()
@@ -74,14 +74,17 @@ def _worker(rank, world, port, name, chunk, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("name,chunk", [("tiny_bert", 4096), ("tiny_gpt2", 1 << 20), ("bert_base", 4 << 20)])
-def test_pt_gather_schedule_gloo(name, chunk):
+@pytest.mark.parametrize("name,chunk,mode", [("tiny_bert", 4096, "PT_DHA"), ("tiny_gpt2", 1 << 20, "PT_DHA"),
+                                             ("bert_base", 4 << 20, "PT_DHA"),
+                                             ("bert_base", 4 << 20, "PT_DHA_LINK_STRIPE"),
+                                             ("tiny_gpt2", 1 << 20, "PT_DHA_STRIPE")])
+def test_pt_gather_schedule_gloo(name, chunk, mode):
     from oracle import planner as OP
     from oracle import units as OU
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, name, chunk, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, name, chunk, q, mode)) for r in range(2)]
     for p in procs:
         p.start()
     res = q.get(timeout=300)
@@ -90,9 +93,9 @@ def test_pt_gather_schedule_gloo(name, chunk):
     assert res[0] == "ok", res
     _, got, dest, method, slot = res
     m, cost = _cost(name)
-    om, osl, _ = OP.plan(cost, "PT_DHA", 2)
+    om, osl, _ = OP.plan(cost, mode, 2)
     assert method == om and slot == osl
-    link = OP.simulate(cost, om, osl, 2)["link_bytes"]
+    link = OP.simulate(cost, om, osl, 2, link_aware=mode in OP.LINK_AWARE)["link_bytes"]
     assert got == link[1]
     # the bytes of every slot-1 unit arrived at its arena offset, nothing else was written
     import paper_conf_eurosys_jeongba23_b200._lib as L
