@@ -564,11 +564,13 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
 void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
                           const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
                           int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
+  if (ablate_mask() & 4) return;
   gemm_impl(dtype, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, bn_hint, s);
 }
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
+  if (ablate_mask() & 4) return;
   launch_gemm_tc_group(dtype, x, ldx, 1, &w, &bias, nullptr, res, ldr, y, ldy, M, N, K, act, io, bn_hint, s);
 }
 

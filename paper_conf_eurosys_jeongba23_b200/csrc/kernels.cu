@@ -222,6 +222,7 @@ static void layernorm_t(const void* x, const void* r, const void* g, const void*
 
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
                       int n, float eps, bool in_f32, cudaStream_t s, void* y32) {
+  if (ablate_mask() & 2) return;
   DP_CHECK(n % 8 == 0 && n > 0, DP_ERR_INVALID, "LN width must be a multiple of 8");
   if (rows <= 0) return;
   if (dtype == DP_BF16)
@@ -450,6 +451,7 @@ int skinny_cluster(int K);
 // weight staging with the per-CTA products on mma.sync (the link stays the bound).
 void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
                           int ldr, void* y, int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
+  if (ablate_mask() & 8) return;
   DP_CHECK(K % 8 == 0 && K > 0 && N > 0, DP_ERR_INVALID, "skinny linear needs K % 8 == 0");
   if (M <= 0) return;
   const bool mma = M > 16 && N % 16 == 0 && K % 16 == 0 && ldx % 8 == 0 && ((uintptr_t)x % 16) == 0 &&
@@ -492,6 +494,7 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
 
 void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
                       bool causal, cudaStream_t s) {
+  if (ablate_mask() & 1) return;
   DP_CHECK(heads > 0 && H % heads == 0 && H / heads == ATT_D, DP_ERR_UNSUPPORTED, "attention needs head dim 64");
   DP_CHECK(ldqkv % 8 == 0, DP_ERR_INVALID, "ldqkv must be a multiple of 8");
   if (batch <= 0 || seq <= 0) return;

@@ -8,6 +8,8 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <cstdlib>
+
 #include "common.h"
 
 namespace dp {
@@ -68,6 +70,18 @@ inline void launch_kernel_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block,
   cfg.attrs = n ? at : nullptr;
   cfg.numAttrs = n;
   DP_CUDA(cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...));
+}
+
+// Timing ablation (tools/ablate.py only): DP_ABLATE is a bit mask of kernel families whose
+// launches are skipped -- 1 attention, 2 LayerNorm, 4 resident GEMM (query, key and value
+// grouped or not), 8 skinny linear / GEMV.  Outputs are garbage; the warm forward's time
+// without a family is what its share of the chain is.
+inline int ablate_mask() {
+  static const int m = [] {
+    const char* e = std::getenv("DP_ABLATE");
+    return e ? std::atoi(e) : 0;
+  }();
+  return m;
 }
 
 // Device side: no-ops when the grid was not launched with PDL.
