@@ -72,6 +72,15 @@ for spec in specs:
         res["plans"][f"EXHAUSTIVE_w{len(free)}/k{k}"] = {"sim_ms": round(lat / 1e6, 4),
                                                       "dha_units": int(p.method.sum()),
                                                       "search_s": round(time.perf_counter() - t0, 2)}
+    # windowed exhaustive over the striped split (R22) at k = 8: the first `window` slot-0
+    # units free (the striped plan's own partition kept)
+    base = dp.plan_generate(cost, "PT_DHA_STRIPE", 8)
+    free = [i for i in range(model.n) if base.slot[i] == 0][:window]
+    t0 = time.perf_counter()
+    lat, p = dp.plan_exhaustive(cost, base, free)
+    res["plans"][f"EXHAUSTIVE_STRIPE_w{len(free)}/k8"] = {"sim_ms": round(lat / 1e6, 4),
+                                                         "dha_units": int(p.method.sum()),
+                                                         "search_s": round(time.perf_counter() - t0, 2)}
     model.close()
     report[spec] = res
 print(json.dumps(report, indent=1))
