@@ -70,64 +70,12 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t* r, const void* p) {
 
 constexpr int ATT_D = 64, ATT_BQ = 64, ATT_BK = 64, ATT_LD = 72;  // padded row (144 B): no ldmatrix conflicts
 
-template <class T, class Sync>
-__device__ __forceinline__ void attention_tile(const T* __restrict__ qkv, int ldqkv, T* __restrict__ ctx, int seq,
-                                               int H, int causal, float scale_log2, int qt, int head, int bidx,
-                                               T* sq, T* sk_, T* sv_, int tid, Sync sync) {
-  // Q tile + a 2-deep ring of (K, V) tiles, all filled with cp.async: the Q tile and the
-  // first two key tiles are in flight together (one L2 round trip, not one per tile), and
-  // tile kt+2 streams in while tile kt is computed.  Rows past `seq` are zero-filled.
-  T* sk[2] = {sk_, sk_ + ATT_BK * ATT_LD};
-  T* sv[2] = {sv_, sv_ + ATT_BK * ATT_LD};
-  const int lane = tid & 31, warp = tid >> 5;
-  sync();  // the previous tile's readers are done with the buffers
-  const size_t tok0 = (size_t)bidx * seq;
-  const int q0 = qt * ATT_BQ;
-  const T* qbase = qkv + tok0 * ldqkv + head * ATT_D;
-  const T* kbase = qbase + H;
-  const T* vbase = qbase + 2 * H;
-  int nkt = (seq + ATT_BK - 1) / ATT_BK;
-  if (causal) nkt = min(nkt, (q0 + ATT_BQ - 1) / ATT_BK + 1);
-  auto load_kv = [&](int kt) {
-    const int k0 = kt * ATT_BK;
-    for (int i = tid; i < ATT_BK * 8; i += 128) {
-      const int r = i >> 3, c = i & 7;
-      const bool ok = k0 + r < seq;
-      const size_t off = (size_t)(ok ? k0 + r : 0) * ldqkv + c * 8;
-      cp_async16_zfill(&sk[kt & 1][r * ATT_LD + c * 8], kbase + off, ok);
-      cp_async16_zfill(&sv[kt & 1][r * ATT_LD + c * 8], vbase + off, ok);
-    }
-  };
-  for (int i = tid; i < ATT_BQ * 8; i += 128) {  // Q: 64 rows x 64 d = 512 vectors of 16 B
-    const int r = i >> 3, c = i & 7;
-    const bool ok = q0 + r < seq;
-    cp_async16_zfill(&sq[r * ATT_LD + c * 8], qbase + (size_t)(ok ? q0 + r : 0) * ldqkv + c * 8, ok);
-  }
-  load_kv(0);
-  cp_async_commit();
-  if (nkt > 1) load_kv(1);
-  cp_async_commit();
-  cp_async_wait<1>();
-  sync();
-  uint32_t qa[4][4];  // A fragments: 16 rows of this warp x 64 d (4 k-steps)
-  {
-    const int r = warp * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
-#pragma unroll
-    for (int kk = 0; kk < 4; ++kk) ldsm_x4(qa[kk], &sq[r * ATT_LD + kk * 16 + (lane >> 4) * 8]);
-  }
-  float o[8][4];
-#pragma unroll
-  for (int i = 0; i < 8; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
-  float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
-  const int qrow0 = q0 + warp * 16 + (lane >> 2);  // rows qrow0 and qrow0 + 8
-  for (int kt = 0; kt < nkt; ++kt) {
-    const int k0 = kt * ATT_BK;
-    if (kt > 0) {
-      cp_async_wait<1>();  // tile kt landed (tile kt+1 may still be in flight)
-      sync();
-    }
-    const T* skt = sk[kt & 1];
-    const T* svt = sv[kt & 1];
+// One key tile of the online-softmax flash step for one warp's 16 query rows (rows qrow0 and
+// qrow0 + 8 per lane): S = Q K^T, mask, running max / sum, O = O * corr + P V.
+template <class T>
+__device__ __forceinline__ void attention_key_tile(const T* skt, const T* svt, const uint32_t (&qa)[4][4],
+                                                   float (&o)[8][4], float (&mrow)[2], float (&lrow)[2], int k0,
+                                                   int qrow0, int seq, int causal, float scale_log2, int lane) {
     float s[8][4];
 #pragma unroll
     for (int nb = 0; nb < 8; ++nb) s[nb][0] = s[nb][1] = s[nb][2] = s[nb][3] = 0.f;
@@ -202,6 +150,65 @@ __device__ __forceinline__ void attention_tile(const T* __restrict__ qkv, int ld
         MmaOp<T>::mma(o[db + 1], pa, bfr + 2);
       }
     }
+}
+
+template <class T, class Sync>
+__device__ __forceinline__ void attention_tile(const T* __restrict__ qkv, int ldqkv, T* __restrict__ ctx, int seq,
+                                               int H, int causal, float scale_log2, int qt, int head, int bidx,
+                                               T* sq, T* sk_, T* sv_, int tid, Sync sync) {
+  // Q tile + a 2-deep ring of (K, V) tiles, all filled with cp.async: the Q tile and the
+  // first two key tiles are in flight together (one L2 round trip, not one per tile), and
+  // tile kt+2 streams in while tile kt is computed.  Rows past `seq` are zero-filled.
+  T* sk[2] = {sk_, sk_ + ATT_BK * ATT_LD};
+  T* sv[2] = {sv_, sv_ + ATT_BK * ATT_LD};
+  const int lane = tid & 31, warp = tid >> 5;
+  sync();  // the previous tile's readers are done with the buffers
+  const size_t tok0 = (size_t)bidx * seq;
+  const int q0 = qt * ATT_BQ;
+  const T* qbase = qkv + tok0 * ldqkv + head * ATT_D;
+  const T* kbase = qbase + H;
+  const T* vbase = qbase + 2 * H;
+  int nkt = (seq + ATT_BK - 1) / ATT_BK;
+  if (causal) nkt = min(nkt, (q0 + ATT_BQ - 1) / ATT_BK + 1);
+  auto load_kv = [&](int kt) {
+    const int k0 = kt * ATT_BK;
+    for (int i = tid; i < ATT_BK * 8; i += 128) {
+      const int r = i >> 3, c = i & 7;
+      const bool ok = k0 + r < seq;
+      const size_t off = (size_t)(ok ? k0 + r : 0) * ldqkv + c * 8;
+      cp_async16_zfill(&sk[kt & 1][r * ATT_LD + c * 8], kbase + off, ok);
+      cp_async16_zfill(&sv[kt & 1][r * ATT_LD + c * 8], vbase + off, ok);
+    }
+  };
+  for (int i = tid; i < ATT_BQ * 8; i += 128) {  // Q: 64 rows x 64 d = 512 vectors of 16 B
+    const int r = i >> 3, c = i & 7;
+    const bool ok = q0 + r < seq;
+    cp_async16_zfill(&sq[r * ATT_LD + c * 8], qbase + (size_t)(ok ? q0 + r : 0) * ldqkv + c * 8, ok);
+  }
+  load_kv(0);
+  cp_async_commit();
+  if (nkt > 1) load_kv(1);
+  cp_async_commit();
+  cp_async_wait<1>();
+  sync();
+  uint32_t qa[4][4];  // A fragments: 16 rows of this warp x 64 d (4 k-steps)
+  {
+    const int r = warp * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
+#pragma unroll
+    for (int kk = 0; kk < 4; ++kk) ldsm_x4(qa[kk], &sq[r * ATT_LD + kk * 16 + (lane >> 4) * 8]);
+  }
+  float o[8][4];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
+  float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
+  const int qrow0 = q0 + warp * 16 + (lane >> 2);  // rows qrow0 and qrow0 + 8
+  for (int kt = 0; kt < nkt; ++kt) {
+    const int k0 = kt * ATT_BK;
+    if (kt > 0) {
+      cp_async_wait<1>();  // tile kt landed (tile kt+1 may still be in flight)
+      sync();
+    }
+    attention_key_tile<T>(sk[kt & 1], sv[kt & 1], qa, o, mrow, lrow, k0, qrow0, seq, causal, scale_log2, lane);
     if (kt + 2 < nkt) {
       sync();  // every warp is done with slot kt & 1
       load_kv(kt + 2);

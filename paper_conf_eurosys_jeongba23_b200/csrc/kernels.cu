@@ -11,6 +11,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 
 #include "common.h"
 #include "dtype.cuh"
@@ -492,6 +493,128 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
                     threadIdx.x, [] { __syncthreads(); });
 }
 
+// K5b: the same tile on 8 warps in two groups that split the key tiles (group g takes tiles
+// g, g+2, ...) for the same 64 query rows, each with its own 2-deep K/V ring; the two partial
+// online-softmax states (running max, sum, unnormalised O) are merged through shared memory at
+// the end.  Halves the dependent chain of key tiles per query tile (the causal S = 1024 tiles
+// near the diagonal walk 16 of them) and doubles the warps feeding the SM's tensor pipes.
+constexpr int ATT2_SMEM = (ATT_BQ * ATT_LD + 8 * ATT_BK * ATT_LD) * 2;  // Q + 2 stages x 2 groups x (K, V)
+
+template <class T>
+__global__ void __launch_bounds__(256) attention2_kernel(const T* __restrict__ qkv, int ldqkv, T* __restrict__ ctx,
+                                                         int seq, int H, int causal, float scale_log2) {
+  extern __shared__ __align__(16) uint8_t att2_smem[];
+  T* sq = reinterpret_cast<T*>(att2_smem);
+  T* kv = sq + ATT_BQ * ATT_LD;
+  auto ktile = [&](int stage, int g) { return kv + ((stage * 2 + g) * 2 + 0) * ATT_BK * ATT_LD; };
+  auto vtile = [&](int stage, int g) { return kv + ((stage * 2 + g) * 2 + 1) * ATT_BK * ATT_LD; };
+  pdl_trigger();
+  pdl_wait();  // q, k, v come from the previous kernels
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, grp = warp >> 2, wq = warp & 3;
+  const int qt = blockIdx.x, head = blockIdx.y, bidx = blockIdx.z;
+  const size_t tok0 = (size_t)bidx * seq;
+  const int q0 = qt * ATT_BQ;
+  const T* qbase = qkv + tok0 * ldqkv + head * ATT_D;
+  const T* kbase = qbase + H;
+  const T* vbase = qbase + 2 * H;
+  int nkt = (seq + ATT_BK - 1) / ATT_BK;
+  if (causal) nkt = min(nkt, (q0 + ATT_BQ - 1) / ATT_BK + 1);
+  const int npair = (nkt + 1) / 2;
+  auto load_pair = [&](int j) {  // key tiles 2j (group 0) and 2j + 1 (group 1) into stage j & 1
+    for (int i = tid; i < 2 * ATT_BK * 8; i += 256) {
+      const int g = i / (ATT_BK * 8), r = (i >> 3) & (ATT_BK - 1), c = i & 7;
+      const int kt = 2 * j + g;
+      if (kt >= nkt) continue;
+      const int k0 = kt * ATT_BK;
+      const bool ok = k0 + r < seq;
+      const size_t off = (size_t)(ok ? k0 + r : 0) * ldqkv + c * 8;
+      cp_async16_zfill(&ktile(j & 1, g)[r * ATT_LD + c * 8], kbase + off, ok);
+      cp_async16_zfill(&vtile(j & 1, g)[r * ATT_LD + c * 8], vbase + off, ok);
+    }
+  };
+  for (int i = tid; i < ATT_BQ * 8; i += 256) {
+    const int r = i >> 3, c = i & 7;
+    const bool ok = q0 + r < seq;
+    cp_async16_zfill(&sq[r * ATT_LD + c * 8], qbase + (size_t)(ok ? q0 + r : 0) * ldqkv + c * 8, ok);
+  }
+  load_pair(0);
+  cp_async_commit();
+  if (npair > 1) load_pair(1);
+  cp_async_commit();
+  cp_async_wait<1>();
+  __syncthreads();
+  uint32_t qa[4][4];
+  {
+    const int r = wq * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
+#pragma unroll
+    for (int kk = 0; kk < 4; ++kk) ldsm_x4(qa[kk], &sq[r * ATT_LD + kk * 16 + (lane >> 4) * 8]);
+  }
+  float o[8][4];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) o[i][0] = o[i][1] = o[i][2] = o[i][3] = 0.f;
+  float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
+  const int qrow0 = q0 + wq * 16 + (lane >> 2);
+  for (int j = 0; j < npair; ++j) {
+    if (j > 0) {
+      cp_async_wait<1>();
+      __syncthreads();
+    }
+    const int kt = 2 * j + grp;
+    if (kt < nkt)
+      attention_key_tile<T>(ktile(j & 1, grp), vtile(j & 1, grp), qa, o, mrow, lrow, kt * ATT_BK, qrow0, seq, causal,
+                            scale_log2, lane);
+    if (j + 2 < npair) {
+      __syncthreads();  // both groups are done with stage j & 1
+      load_pair(j + 2);
+    }
+    cp_async_commit();
+  }
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {  // full row sums across the 4 lanes of a row
+    lrow[h] += __shfl_xor_sync(0xffffffffu, lrow[h], 1);
+    lrow[h] += __shfl_xor_sync(0xffffffffu, lrow[h], 2);
+  }
+  // merge: group 1 publishes its state per (warp, lane) -- the same fragment elements as the
+  // group-0 lane that merges it
+  cp_async_wait<0>();
+  __syncthreads();
+  float* xs = reinterpret_cast<float*>(kv);  // [4 warps][32 lanes][36]
+  float* mine = xs + (wq * 32 + lane) * 36;
+  if (grp == 1) {
+#pragma unroll
+    for (int db = 0; db < 8; ++db)
+#pragma unroll
+      for (int e = 0; e < 4; ++e) mine[db * 4 + e] = o[db][e];
+    mine[32] = mrow[0], mine[33] = mrow[1], mine[34] = lrow[0], mine[35] = lrow[1];
+  }
+  __syncthreads();
+  if (grp == 1) return;
+  float a0[2], a1[2], inv[2];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const float m1 = mine[32 + h], l1 = mine[34 + h];
+    const float m = fmaxf(mrow[h], m1);
+    a0[h] = (mrow[h] == -INFINITY) ? 0.f : exp2f(mrow[h] - m);
+    a1[h] = (m1 == -INFINITY) ? 0.f : exp2f(m1 - m);
+    const float l = lrow[h] * a0[h] + l1 * a1[h];
+    inv[h] = l > 0.f ? 1.f / l : 0.f;
+  }
+  T* cbase = ctx + tok0 * H + head * ATT_D;
+#pragma unroll
+  for (int db = 0; db < 8; ++db) {
+    const int col = db * 8 + (lane & 3) * 2;
+    float v[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int h = e >> 1;
+      v[e] = (o[db][e] * a0[h] + mine[db * 4 + e] * a1[h]) * inv[h];
+    }
+    if (qrow0 < seq) *reinterpret_cast<uint32_t*>(cbase + (size_t)qrow0 * H + col) = Cvt<T>::from2(v[0], v[1]);
+    if (qrow0 + 8 < seq)
+      *reinterpret_cast<uint32_t*>(cbase + (size_t)(qrow0 + 8) * H + col) = Cvt<T>::from2(v[2], v[3]);
+  }
+}
+
 void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
                       bool causal, cudaStream_t s) {
   if (ablate_mask() & 1) return;
@@ -500,6 +623,26 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   if (batch <= 0 || seq <= 0) return;
   dim3 grid((seq + ATT_BQ - 1) / ATT_BQ, heads, batch);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)ATT_D);
+  static const int env_att = getenv("DP_ATT_GROUPS") ? atoi(getenv("DP_ATT_GROUPS")) : 2;  // experiments
+  // >= 3 key tiles: two key groups per query tile (K5b).  At 2 tiles (BERT-Base S = 128) the
+  // merge and the larger footprint cost more than the shorter chain saves (warm forward 0.480
+  // vs 0.472 ms); BERT-Large S = 384 1.78 -> 1.58 ms, GPT-2 Medium S = 1024 2.81 -> 2.47 ms
+  if (env_att == 2 && seq > 2 * ATT_BK) {
+    static bool attr = false;
+    if (!attr) {
+      DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__half>, cudaFuncAttributeMaxDynamicSharedMemorySize, ATT2_SMEM));
+      DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   ATT2_SMEM));
+      attr = true;
+    }
+    if (dtype == DP_BF16)
+      launch_kernel(attention2_kernel<__nv_bfloat16>, grid, dim3(256), ATT2_SMEM, s, (const __nv_bfloat16*)qkv, ldqkv,
+                    (__nv_bfloat16*)ctx, seq, H, causal ? 1 : 0, scale_log2);
+    else
+      launch_kernel(attention2_kernel<__half>, grid, dim3(256), ATT2_SMEM, s, (const __half*)qkv, ldqkv, (__half*)ctx,
+                    seq, H, causal ? 1 : 0, scale_log2);
+    return;
+  }
   if (dtype == DP_BF16)
     launch_kernel(attention_kernel<__nv_bfloat16>, grid, dim3(128), 0, s, (const __nv_bfloat16*)qkv, ldqkv,
                   (__nv_bfloat16*)ctx, seq, H, causal ? 1 : 0, scale_log2);
