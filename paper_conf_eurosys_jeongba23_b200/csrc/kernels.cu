@@ -12,6 +12,7 @@
 
 #include <cstdint>
 #include <cstdlib>
+#include <type_traits>
 
 #include "common.h"
 #include "dtype.cuh"
@@ -498,16 +499,19 @@ __global__ void __launch_bounds__(128) attention_kernel(const T* __restrict__ qk
 // online-softmax states (running max, sum, unnormalised O) are merged through shared memory at
 // the end.  Halves the dependent chain of key tiles per query tile (the causal S = 1024 tiles
 // near the diagonal walk 16 of them) and doubles the warps feeding the SM's tensor pipes.
-constexpr int ATT2_SMEM = (ATT_BQ * ATT_LD + 8 * ATT_BK * ATT_LD) * 2;  // Q + 2 stages x 2 groups x (K, V)
+// Q + 2 stages x G groups x (K, V)
+template <int G>
+constexpr int att_groups_smem() { return (ATT_BQ * ATT_LD + 4 * G * ATT_BK * ATT_LD) * 2; }
 
-template <class T>
-__global__ void __launch_bounds__(256) attention2_kernel(const T* __restrict__ qkv, int ldqkv, T* __restrict__ ctx,
-                                                         int seq, int H, int causal, float scale_log2) {
+template <class T, int G>
+__global__ void __launch_bounds__(128 * G) attention2_kernel(const T* __restrict__ qkv, int ldqkv, T* __restrict__ ctx,
+                                                             int seq, int H, int causal, float scale_log2) {
   extern __shared__ __align__(16) uint8_t att2_smem[];
   T* sq = reinterpret_cast<T*>(att2_smem);
   T* kv = sq + ATT_BQ * ATT_LD;
-  auto ktile = [&](int stage, int g) { return kv + ((stage * 2 + g) * 2 + 0) * ATT_BK * ATT_LD; };
-  auto vtile = [&](int stage, int g) { return kv + ((stage * 2 + g) * 2 + 1) * ATT_BK * ATT_LD; };
+  auto ktile = [&](int stage, int g) { return kv + ((stage * G + g) * 2 + 0) * ATT_BK * ATT_LD; };
+  auto vtile = [&](int stage, int g) { return kv + ((stage * G + g) * 2 + 1) * ATT_BK * ATT_LD; };
+  constexpr int NT = 128 * G;
   pdl_trigger();
   pdl_wait();  // q, k, v come from the previous kernels
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, grp = warp >> 2, wq = warp & 3;
@@ -519,11 +523,11 @@ __global__ void __launch_bounds__(256) attention2_kernel(const T* __restrict__ q
   const T* vbase = qbase + 2 * H;
   int nkt = (seq + ATT_BK - 1) / ATT_BK;
   if (causal) nkt = min(nkt, (q0 + ATT_BQ - 1) / ATT_BK + 1);
-  const int npair = (nkt + 1) / 2;
-  auto load_pair = [&](int j) {  // key tiles 2j (group 0) and 2j + 1 (group 1) into stage j & 1
-    for (int i = tid; i < 2 * ATT_BK * 8; i += 256) {
+  const int npair = (nkt + G - 1) / G;
+  auto load_pair = [&](int j) {  // key tiles G*j + g (group g) into stage j & 1
+    for (int i = tid; i < G * ATT_BK * 8; i += NT) {
       const int g = i / (ATT_BK * 8), r = (i >> 3) & (ATT_BK - 1), c = i & 7;
-      const int kt = 2 * j + g;
+      const int kt = G * j + g;
       if (kt >= nkt) continue;
       const int k0 = kt * ATT_BK;
       const bool ok = k0 + r < seq;
@@ -532,7 +536,7 @@ __global__ void __launch_bounds__(256) attention2_kernel(const T* __restrict__ q
       cp_async16_zfill(&vtile(j & 1, g)[r * ATT_LD + c * 8], vbase + off, ok);
     }
   };
-  for (int i = tid; i < ATT_BQ * 8; i += 256) {
+  for (int i = tid; i < ATT_BQ * 8; i += NT) {
     const int r = i >> 3, c = i & 7;
     const bool ok = q0 + r < seq;
     cp_async16_zfill(&sq[r * ATT_LD + c * 8], qbase + (size_t)(ok ? q0 + r : 0) * ldqkv + c * 8, ok);
@@ -559,7 +563,7 @@ __global__ void __launch_bounds__(256) attention2_kernel(const T* __restrict__ q
       cp_async_wait<1>();
       __syncthreads();
     }
-    const int kt = 2 * j + grp;
+    const int kt = G * j + grp;
     if (kt < nkt)
       attention_key_tile<T>(ktile(j & 1, grp), vtile(j & 1, grp), qa, o, mrow, lrow, kt * ATT_BK, qrow0, seq, causal,
                             scale_log2, lane);
@@ -578,9 +582,9 @@ __global__ void __launch_bounds__(256) attention2_kernel(const T* __restrict__ q
   // group-0 lane that merges it
   cp_async_wait<0>();
   __syncthreads();
-  float* xs = reinterpret_cast<float*>(kv);  // [4 warps][32 lanes][36]
-  float* mine = xs + (wq * 32 + lane) * 36;
-  if (grp == 1) {
+  float* xs = reinterpret_cast<float*>(kv);  // [G-1 groups][4 warps][32 lanes][36]
+  if (grp > 0) {
+    float* mine = xs + (((grp - 1) * 4 + wq) * 32 + lane) * 36;
 #pragma unroll
     for (int db = 0; db < 8; ++db)
 #pragma unroll
@@ -588,27 +592,36 @@ __global__ void __launch_bounds__(256) attention2_kernel(const T* __restrict__ q
     mine[32] = mrow[0], mine[33] = mrow[1], mine[34] = lrow[0], mine[35] = lrow[1];
   }
   __syncthreads();
-  if (grp == 1) return;
-  float a0[2], a1[2], inv[2];
+  if (grp > 0) return;
+  // group 0 merges the groups in order 1..G-1 (deterministic)
+  float inv[2];
 #pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    const float m1 = mine[32 + h], l1 = mine[34 + h];
-    const float m = fmaxf(mrow[h], m1);
-    a0[h] = (mrow[h] == -INFINITY) ? 0.f : exp2f(mrow[h] - m);
-    a1[h] = (m1 == -INFINITY) ? 0.f : exp2f(m1 - m);
-    const float l = lrow[h] * a0[h] + l1 * a1[h];
-    inv[h] = l > 0.f ? 1.f / l : 0.f;
+  for (int g = 1; g < G; ++g) {
+    const float* ot = xs + (((g - 1) * 4 + wq) * 32 + lane) * 36;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const float m1 = ot[32 + h], l1 = ot[34 + h];
+      const float m = fmaxf(mrow[h], m1);
+      const float a0 = (mrow[h] == -INFINITY) ? 0.f : exp2f(mrow[h] - m);
+      const float a1 = (m1 == -INFINITY) ? 0.f : exp2f(m1 - m);
+      lrow[h] = lrow[h] * a0 + l1 * a1;
+      mrow[h] = m;
+#pragma unroll
+      for (int db = 0; db < 8; ++db) {
+        o[db][2 * h] = o[db][2 * h] * a0 + ot[db * 4 + 2 * h] * a1;
+        o[db][2 * h + 1] = o[db][2 * h + 1] * a0 + ot[db * 4 + 2 * h + 1] * a1;
+      }
+    }
   }
+#pragma unroll
+  for (int h = 0; h < 2; ++h) inv[h] = lrow[h] > 0.f ? 1.f / lrow[h] : 0.f;
   T* cbase = ctx + tok0 * H + head * ATT_D;
 #pragma unroll
   for (int db = 0; db < 8; ++db) {
     const int col = db * 8 + (lane & 3) * 2;
     float v[4];
 #pragma unroll
-    for (int e = 0; e < 4; ++e) {
-      const int h = e >> 1;
-      v[e] = (o[db][e] * a0[h] + mine[db * 4 + e] * a1[h]) * inv[h];
-    }
+    for (int e = 0; e < 4; ++e) v[e] = o[db][e] * inv[e >> 1];
     if (qrow0 < seq) *reinterpret_cast<uint32_t*>(cbase + (size_t)qrow0 * H + col) = Cvt<T>::from2(v[0], v[1]);
     if (qrow0 + 8 < seq)
       *reinterpret_cast<uint32_t*>(cbase + (size_t)(qrow0 + 8) * H + col) = Cvt<T>::from2(v[2], v[3]);
@@ -623,24 +636,38 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   if (batch <= 0 || seq <= 0) return;
   dim3 grid((seq + ATT_BQ - 1) / ATT_BQ, heads, batch);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)ATT_D);
-  static const int env_att = getenv("DP_ATT_GROUPS") ? atoi(getenv("DP_ATT_GROUPS")) : 2;  // experiments
-  // >= 3 key tiles: two key groups per query tile (K5b).  At 2 tiles (BERT-Base S = 128) the
-  // merge and the larger footprint cost more than the shorter chain saves (warm forward 0.480
-  // vs 0.472 ms); BERT-Large S = 384 1.78 -> 1.58 ms, GPT-2 Medium S = 1024 2.81 -> 2.47 ms
-  if (env_att == 2 && seq > 2 * ATT_BK) {
+  static const int env_att = getenv("DP_ATT_GROUPS") ? atoi(getenv("DP_ATT_GROUPS")) : 0;  // experiments
+  // >= 3 key tiles: 2 or 4 key-tile groups per query tile (K5b).  At 2 tiles (BERT-Base
+  // S = 128) the merge and the larger footprint cost more than the shorter chain saves (warm
+  // forward 0.480 vs 0.472 ms); with 2 groups BERT-Large S = 384 1.78 -> 1.58 ms, GPT-2 Medium
+  // S = 1024 2.81 -> 2.47 ms
+  auto run_groups = [&](auto gtag) {
+    constexpr int G = decltype(gtag)::value;
+    constexpr int smem = att_groups_smem<G>();
     static bool attr = false;
     if (!attr) {
-      DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__half>, cudaFuncAttributeMaxDynamicSharedMemorySize, ATT2_SMEM));
-      DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   ATT2_SMEM));
+      DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__half, G>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+      DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__nv_bfloat16, G>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   smem));
       attr = true;
     }
     if (dtype == DP_BF16)
-      launch_kernel(attention2_kernel<__nv_bfloat16>, grid, dim3(256), ATT2_SMEM, s, (const __nv_bfloat16*)qkv, ldqkv,
-                    (__nv_bfloat16*)ctx, seq, H, causal ? 1 : 0, scale_log2);
+      launch_kernel(attention2_kernel<__nv_bfloat16, G>, grid, dim3(128 * G), smem, s, (const __nv_bfloat16*)qkv,
+                    ldqkv, (__nv_bfloat16*)ctx, seq, H, causal ? 1 : 0, scale_log2);
     else
-      launch_kernel(attention2_kernel<__half>, grid, dim3(256), ATT2_SMEM, s, (const __half*)qkv, ldqkv, (__half*)ctx,
-                    seq, H, causal ? 1 : 0, scale_log2);
+      launch_kernel(attention2_kernel<__half, G>, grid, dim3(128 * G), smem, s, (const __half*)qkv, ldqkv,
+                    (__half*)ctx, seq, H, causal ? 1 : 0, scale_log2);
+  };
+  // groups by key tiles (DP_ATT_GROUPS forces 1 / 2 / 4 for experiments): >= 4 tiles -> 4
+  // groups (BERT-Large S384 warm 1.58 -> 1.48 ms; GPT-2 Medium S1024 unchanged), 3 -> 2
+  const int nkt = (seq + ATT_BK - 1) / ATT_BK;
+  const int groups = env_att > 0 ? env_att : (nkt >= 4 ? 4 : nkt == 3 ? 2 : 1);
+  if (groups == 4 && nkt >= 3) {
+    run_groups(std::integral_constant<int, 4>{});
+    return;
+  }
+  if (groups == 2 && nkt >= 3) {
+    run_groups(std::integral_constant<int, 2>{});
     return;
   }
   if (dtype == DP_BF16)
