@@ -27,7 +27,12 @@ full embed_dha embed embed 3
 full attention attn attention 3
 full layernorm ln layernorm 3
 full lmhead_hbm lmhead gemv 16
-timeout 900 python tools/plan_compare.py > $o/plan_compare.json 2> $o/plan_compare.err
+full attention_k5b attn attention2 3
+full pt_forward ptfwd pt_forward 12
+timeout 1500 python tools/plan_compare.py > $o/plan_compare.json 2> $o/plan_compare.err
+timeout 600 python tools/dump_costs.py > $o/cost_tables.json 2> $o/cost_tables.err
+timeout 300 python tools/torch_warm_baseline.py bert_base:128 bert_large:384 gpt2:256 gpt2_medium:1024 > $o/warm_vs_torch.jsonl 2>&1
+python bench.py > $o/bench.log 2>&1
 timeout 600 python tools/serve_bench.py --mix bert_base:128:4,roberta_base:384:4,gpt2:1024:1 --instances 45 \
   --fit 8 --rate 200 --requests 600 --slo-ms 20 > $o/serve_mix.json 2> $o/serve_mix.err
 echo evidence-done

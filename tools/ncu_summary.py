@@ -82,6 +82,8 @@ ALGO = {
     "layernorm": {"shape": "128 x 768", "bytes": 2 * 2 * 128 * 768},
     "lmhead_hbm": {"shape": "GPT-2 tied LM head, 1 row, V50257 H768, wte in HBM (streaming GEMV)",
                    "bytes": 2 * 50257 * 768},
+    "attention_k5b": {"shape": "B1 S384 H1024 16 heads, 4 key-tile groups (K5b)", "flops": 4 * 384 * 384 * 1024},
+    "pt_forward": {"shape": "32 MiB pinned host -> HBM, SM forwarder (K7)", "host_bytes": 32 << 20},
 }
 
 
