@@ -515,7 +515,11 @@ __global__ void __launch_bounds__(128 * G) attention2_kernel(const T* __restrict
   pdl_trigger();
   pdl_wait();  // q, k, v come from the previous kernels
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, grp = warp >> 2, wq = warp & 3;
-  const int qt = blockIdx.x, head = blockIdx.y, bidx = blockIdx.z;
+  // grid (heads, query tiles, batch): CTAs start in linear order, so with causal masking the
+  // query tiles are visited last-first -- the longest key chains go out in the first wave and
+  // the short ones fill in behind them (longest-processing-time-first)
+  const int head = blockIdx.x, bidx = blockIdx.z;
+  const int qt = causal > 1 ? (int)gridDim.y - 1 - (int)blockIdx.y : (int)blockIdx.y;
   const size_t tok0 = (size_t)bidx * seq;
   const int q0 = qt * ATT_BQ;
   const T* qbase = qkv + tok0 * ldqkv + head * ATT_D;
@@ -651,12 +655,15 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
                                    smem));
       attr = true;
     }
+    const dim3 g2(heads, grid.x, batch);
+    static const int env_lpt = getenv("DP_ATT_LPT") ? atoi(getenv("DP_ATT_LPT")) : 1;  // experiments
+    const int cmode = causal ? (env_lpt ? 2 : 1) : 0;  // 2: causal, longest query tiles first
     if (dtype == DP_BF16)
-      launch_kernel(attention2_kernel<__nv_bfloat16, G>, grid, dim3(128 * G), smem, s, (const __nv_bfloat16*)qkv,
-                    ldqkv, (__nv_bfloat16*)ctx, seq, H, causal ? 1 : 0, scale_log2);
+      launch_kernel(attention2_kernel<__nv_bfloat16, G>, g2, dim3(128 * G), smem, s, (const __nv_bfloat16*)qkv,
+                    ldqkv, (__nv_bfloat16*)ctx, seq, H, cmode, scale_log2);
     else
-      launch_kernel(attention2_kernel<__half, G>, grid, dim3(128 * G), smem, s, (const __half*)qkv, ldqkv,
-                    (__half*)ctx, seq, H, causal ? 1 : 0, scale_log2);
+      launch_kernel(attention2_kernel<__half, G>, g2, dim3(128 * G), smem, s, (const __half*)qkv, ldqkv,
+                    (__half*)ctx, seq, H, cmode, scale_log2);
   };
   // groups by key tiles (DP_ATT_GROUPS forces 1 / 2 / 4 for experiments): >= 4 tiles -> 4
   // groups (BERT-Large S384 warm 1.58 -> 1.48 ms; GPT-2 Medium S1024 unchanged), 3 -> 2
