@@ -668,7 +668,8 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   // groups by key tiles (DP_ATT_GROUPS forces 1 / 2 / 4 for experiments): >= 4 tiles -> 4
   // groups (BERT-Large S384 warm 1.58 -> 1.48 ms; GPT-2 Medium S1024 unchanged), 3 -> 2
   const int nkt = (seq + ATT_BK - 1) / ATT_BK;
-  const int groups = env_att > 0 ? env_att : (nkt >= 4 ? 4 : nkt == 3 ? 2 : 1);
+  // causal: 2 groups (2 CTAs per SM fit; GPT-2 S256 0.542 vs 0.554 ms with 4, S1024 equal)
+  const int groups = env_att > 0 ? env_att : causal ? (nkt >= 3 ? 2 : 1) : (nkt >= 4 ? 4 : nkt == 3 ? 2 : 1);
   if (groups == 4 && nkt >= 3) {
     run_groups(std::integral_constant<int, 4>{});
     return;
