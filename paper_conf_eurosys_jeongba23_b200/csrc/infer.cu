@@ -6,11 +6,15 @@
 //   * slot-s LOAD units (PT): H2D over the link of the slot's GPU into a staging
 //     ring, then forwarded into the primary's HBM slot by that GPU's migration stream
 //     (cudaMemcpyPeerAsync over NVLink; a D2D copy in loopback; NCCL send/recv across
-//     processes -- peer.cpp), one event per forwarded piece;
+//     processes -- peer.cpp), one event per forwarded piece; or, with opts.pt_transport =
+//     DP_PT_SM / DP_PT_CE (pt_forward.cu), in ONE hop by a forwarder kernel or a
+//     DMA on the secondary straight into the primary's slot (across processes over CUDA IPC,
+//     with release/acquire mailbox words instead of events);
 //   * DHA units: no transfer; their kernels read the arena in place ("we can skip
 //     the dependency check");
-//   * the execution stream (the caller's) waits on a unit's event right before the first
-//     kernel that reads it.
+//   * the execution stream (the caller's) waits on a unit's piece right before the first
+//     kernel that reads it, batched per round of links (the pieces of the next units on the
+//     other links that land no later are waited for in the same batch).
 #include <algorithm>
 #include <chrono>
 #include <cstdlib>
