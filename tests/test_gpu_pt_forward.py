@@ -249,3 +249,28 @@ def test_sm_transport_across_processes(name, mode, S, delay, transport, graph):
         assert h2d[1] == link[1] and nvl[1] == link[1]
     for h2d, nvl in r0["stats"]:
         assert h2d[0] == link[0] and nvl[1] == link[1]
+
+
+@pytest.mark.parametrize("name,S", [("tiny_bert", 77), ("tiny_gpt2", 70), ("bert_base", 128)])
+@pytest.mark.parametrize("transport", ["sm", "ce"])
+def test_one_hop_transports_bf16_striped(name, S, transport):
+    """bf16 storage, the striped plan (R22) over 4 loopback links: one-hop transports equal the
+    DMA path bit for bit and stay within the bf16 tolerance (R15) of the oracle."""
+    m = synth.SHAPES[name]
+    dtype = "bf16"
+    w = synth.make_weights(m, seed=61, dtype=dtype)
+    ids = synth.make_ids(m, 1, S, seed=62)
+    ref, _ = F.forward(m, w, ids, dtype)
+    c = dp().Context([0])
+    model = dp().Model(c, m, w, dtype)
+    plan = dp().plan_generate(fake_cost(m, dtype, seed=9), "PT_DHA_LINK_STRIPE", 4)
+    c.set_opts(pt_transport="dma")
+    a, _, sa = _run(model, plan, ids, dtype, 4)
+    c.set_opts(pt_transport=transport)
+    b, _, sb = _run(model, plan, ids, dtype, 4)
+    assert torch.equal(a, b)
+    r = ref.reshape(S, -1)
+    assert np.all(np.abs(f64(b) - r) <= 2.0 ** -5 * np.maximum(1.0, np.abs(r)))
+    assert sa["h2d_bytes"] == sb["h2d_bytes"] and sa["nvlink_bytes"] == sb["nvlink_bytes"]
+    model.close()
+    c.close()
