@@ -131,7 +131,8 @@ dp_status dp_plan_partition(const int64_t* bytes, int32_t n, int32_t k, int8_t* 
 
 /* Exhaustive search (optimal under the cost model) over the methods of the `nfree` units
  * listed in free_idx (<= 30), all other units keep base->method; PT partition fixed as in
- * DP_MODE_PT_DHA when base->k > 1.  Ties -> lexicographically smallest method vector.
+ * DP_MODE_PT_DHA when base->k > 1 (DP_ERR_INVALID if a free index names a unit of a
+ * partition >= 1: those must stay LOAD).  Ties -> lexicographically smallest method vector.
  * out gets the best plan, *latency_ns its latency. */
 dp_status dp_plan_exhaustive(const dp_cost_table* cost, const dp_plan* base, const int32_t* free_idx,
                              int32_t nfree, dp_plan* out, int64_t* latency_ns);
@@ -329,7 +330,8 @@ typedef struct {
  * (device ordinals in a single-process context, or NCCL ranks after dp_peer_init; a
  * secondary equal to the primary means loopback: staged and forwarded on one GPU).
  * Execution is enqueued on `stream` (the execution stream); every non-DHA unit's first
- * kernel waits on its load event.  d_ids: int32 [batch*seq] on the primary;
+ * kernel waits on its load event.  d_ids: int32 [batch*seq] on the primary (ids
+ * outside [0, vocab) are clamped, so a bad id never reads past a table in the arena);
  * d_out: [batch*seq*hidden] storage dtype; d_pooled: [batch*hidden] or NULL (BERT/
  * RoBERTa pooler).  On return the work is enqueued (asynchronous); the model is then
  * resident on the primary with the plan's DHA units left in host memory.

@@ -390,6 +390,9 @@ def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 
     slot = list(part)
     if free is None:
         free = [i for i in range(n) if part[i] == 0]
+    if any(part[u] >= 1 for u in free):
+        # a unit of a PT partition must stay LOAD (the secondaries only transmit)
+        raise ValueError("free index names a unit of a PT partition (slot >= 1)")
     base = np.array([LOAD] * n if base_method is None else base_method, dtype=np.int8)
     for i in range(n):
         if part[i] >= 1:

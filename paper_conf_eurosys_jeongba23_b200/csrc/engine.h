@@ -63,6 +63,8 @@ struct ForwardArgs {
 };
 
 void ensure_workspace(dp_model* m, int dev, int64_t tokens);
+// Destroy every captured graph / K6 program of a device state (their buffers are going away).
+void drop_graphs(DevState& ds);
 void run_forward(ForwardArgs& a);
 
 // Execute one unit's ops in isolation (profiling): inputs are the workspace buffers.
@@ -83,6 +85,7 @@ struct dp_context {
   uint32_t* mailbox = nullptr;                    // this rank's (pt_forward.cu layout)
   uint32_t* peer_mailbox[DP_MAX_DEVICES] = {};     // other ranks' (IPC-mapped), by rank
   uint32_t pt_epoch = 0;                          // cold starts run in SM/IPC mode so far
+  uint64_t ring_gen = 0;  // bumped whenever a staging ring is reallocated (part of graph keys)
   bool multiproc() const { return nranks > 0; }
   dp::DevCtx& on(int dev);
 };

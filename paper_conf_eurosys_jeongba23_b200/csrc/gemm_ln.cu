@@ -319,11 +319,10 @@ void run_ln(const void* x, int ldx, const void* w, const void* bias, int M, int 
   constexpr size_t STAGE_BYTES = LBM * LBK * 2 + BN * LBK * 2;
   constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
   static_assert(size_t(LBM) * (BN + 1) * 4 + 1024 <= smem_max, "fp32 tile must fit the ring");
-  static bool attr = false;
-  if (!attr) {
+  static std::atomic<unsigned> attr{0};
+  if (first_on_device(attr)) {
     DP_CUDA(cudaFuncSetAttribute(gemm_ln_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max));
     DP_CUDA(cudaFuncSetAttribute(gemm_ln_kernel<T, BN>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
-    attr = true;
   }
   const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
   const CUtensorMap mw = make_kmajor_map(w, dtype, N, K, K, LBM);

@@ -446,12 +446,10 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   nst = std::max(nst, std::max(min_st, 1));
   DP_CHECK(nst <= STAGES, DP_ERR_INVALID, "gemm: epilogue buffers do not fit this tile width");
   const size_t smem = size_t(nst) * STAGE_BYTES + 1024;
-  static bool attr = false;
-  if (!attr) {
+  static std::atomic<unsigned> attr{0};
+  if (first_on_device(attr))
     DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN, ACT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)smem_max));
-    attr = true;
-  }
   const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
   GemmGroup g;
   std::memset(&g, 0, sizeof(g));

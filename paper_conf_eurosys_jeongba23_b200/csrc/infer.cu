@@ -77,6 +77,8 @@ static void ensure_h2d_streams(dp_context* ctx, int dev) {
   }
 }
 
+constexpr int64_t kRingSlots = 3;  // staging ring depth of a two-hop PT slot
+
 static SlotRes& slot_res(dp_context* ctx, int slot, int dev, int64_t ring_bytes) {
   auto& r = ctx->slots[{slot, dev}];
   DeviceGuard g(dev);
@@ -86,7 +88,13 @@ static SlotRes& slot_res(dp_context* ctx, int slot, int dev, int64_t ring_bytes)
     DP_CUDA(cudaStreamCreateWithFlags(&r.mig, cudaStreamNonBlocking));
   }
   if (r.ring_bytes < ring_bytes) {
-    if (r.ring) DP_CUDA(cudaFree(r.ring));
+    // a captured graph may reference the old ring: synchronise before freeing it, and make
+    // every graph key that named it unreachable (stale-pointer replay)
+    ++ctx->ring_gen;
+    if (r.ring) {
+      DP_CUDA(cudaDeviceSynchronize());
+      DP_CUDA(cudaFree(r.ring));
+    }
     r.ring = nullptr;
     if (cudaMalloc(&r.ring, ring_bytes) != cudaSuccess) fail(DP_ERR_OOM, "staging ring cudaMalloc failed");
     r.ring_bytes = ring_bytes;
@@ -330,9 +338,13 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
                                  void* pooled, cudaStream_t stream);
 
 // Key of a captured cold-start / warm graph: everything the enqueued work depends on.
-static std::string graph_key(const dp_context* ctx, const dp_plan* plan, const int32_t* secondaries, const void* ids,
-                             int batch, int seq, const void* out, const void* pooled) {
-  std::string k;
+static std::string graph_key(const dp_context* ctx, const DevState& ds, const dp_plan* plan,
+                             const int32_t* secondaries, const void* ids, int batch, int seq, const void* out,
+                             const void* pooled) {
+  // every device buffer the captured work touches: the HBM slots, the workspace, the staging
+  // rings (by generation) -- a graph is never replayed on memory that was reallocated
+  std::string k = std::to_string((uintptr_t)ds.dbase) + "/" + std::to_string((uintptr_t)ds.ws.base) + "/" +
+                  std::to_string(ds.ws.tokens) + "/" + std::to_string(ctx->ring_gen) + "|";
   if (plan) {
     k.append(reinterpret_cast<const char*>(plan->method), plan->n);
     k.append(reinterpret_cast<const char*>(plan->slot), plan->n);
@@ -402,13 +414,27 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   bool graph = ctx->opts.use_graph != 0 && (!ctx->multiproc() || ipc_pt || plan->k == 1);
   for (int s = 1; s < plan->k && graph && !ctx->multiproc(); ++s)
     graph = secondaries[s - 1] == primary;  // single-device graphs only
+  // staging rings of the two-hop PT slots are sized before any capture (their pointers are
+  // part of the graph key)
+  if (!ctx->multiproc() && ctx->opts.pt_transport == DP_PT_DMA) {
+    const int64_t cap = std::max<int64_t>(ctx->opts.chunk_bytes, 4096);
+    for (int s = 1; s < plan->k; ++s) {
+      auto pcs = slot_pieces(m, plan, s, cap, opt_tail(ctx));
+      int64_t slot_bytes = 0;
+      for (const auto& p : pcs) slot_bytes = std::max(slot_bytes, p.bytes);
+      const int sdev = secondaries[s - 1];
+      DP_CHECK(sdev >= 0 && sdev < DP_MAX_DEVICES && ctx->dc[sdev].ready, DP_ERR_INVALID,
+               "secondary device not in the context");
+      if (slot_bytes > 0) slot_res(ctx, s, sdev, kRingSlots * slot_bytes);
+    }
+  }
   if (ipc_pt) {
     ipc_check_primary(ctx);
     ipc_set_epoch(ctx, ++ctx->pt_epoch, stream);  // every rank counts the same k > 1 cold starts
   }
   dp_run_stats st;
   if (graph) {
-    st = run_graph(ds, graph_key(ctx, plan, secondaries, ids, batch, seq, out, pooled), stream, [&](cudaStream_t cs) {
+    st = run_graph(ds, graph_key(ctx, ds, plan, secondaries, ids, batch, seq, out, pooled), stream, [&](cudaStream_t cs) {
       return enqueue_cold(ctx, m, plan, primary, prim_rank, secondaries, ids, batch, seq, out, pooled, cs);
     });
   } else {
@@ -509,7 +535,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     auto pcs = slot_pieces(m, plan, s, cap, opt_tail(ctx));
     if (pcs.empty()) continue;
     const int sdev = secondaries[s - 1];
-    const int64_t ring_slots = 3;
+    const int64_t ring_slots = kRingSlots;
     int64_t slot_bytes = 0;
     for (const auto& p : pcs) slot_bytes = std::max(slot_bytes, p.bytes);
     SlotRes& r = slot_res(ctx, s, sdev, one_hop ? 0 : ring_slots * slot_bytes);
@@ -768,7 +794,7 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     };
     if (ctx->opts.use_graph) {
       std::string key = "warm|" + std::to_string(a.persistent) + "|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
-                        graph_key(ctx, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);
+                        graph_key(ctx, ds, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);
       if (dbg_waits) key += "|dbgwait" + std::to_string(dbg_waits);
       dp_run_stats gs = run_graph(ds, key, (cudaStream_t)stream, [&](cudaStream_t cs) {
         a.stream = cs;

@@ -35,7 +35,7 @@ template <class T, int VPL>
 __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ ids, int ntok, int seq, int pos_off,
                                                     const T* word, const T* pos, const T* type, const T* g,
                                                     const T* b, int H, float eps, void* __restrict__ out_,
-                                                    int out_f32, float* __restrict__ out32) {
+                                                    int out_f32, float* __restrict__ out32, int vocab) {
   extern __shared__ uint4 sm[];  // [type0 | gamma | beta] as 16-byte vectors
   pdl_trigger();
   const int nv = H / 8;
@@ -57,7 +57,10 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
   const int lane = threadIdx.x & 31;
   const int t = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const bool live = t < ntok;
-  const int id = live ? ids[t] : 0;
+  // ids outside [0, vocab) are clamped: a bad id must never make a DHA gather read past the
+  // table in the pinned arena (vocab <= 0: unchecked, the caller's tables)
+  int id = live ? ids[t] : 0;
+  if (vocab > 0) id = min(max(id, 0), vocab - 1);
   const int p = pos_off + (live ? t % seq : 0);
   uint4 wv[VPL], pv[VPL];
 #pragma unroll
@@ -141,14 +144,14 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
 template <class T>
 static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                     const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
-                    float* out32, cudaStream_t s) {
+                    float* out32, int vocab, cudaStream_t s) {
   const int warps = 8;
   dim3 grid((ntok + warps - 1) / warps);
   const size_t sm = size_t(3) * (H / 8) * 16;
   const int vpl = (H / 8 + 31) / 32;
 #define DP_EMB(V)                                                                                      \
   launch_kernel(embed_kernel<T, V>, grid, dim3(warps * 32), sm, s, ids, ntok, seq, pos_off, (const T*)word, \
-                (const T*)pos, (const T*)type, (const T*)g, (const T*)b, H, eps, out, (int)out_f32, out32)
+                (const T*)pos, (const T*)type, (const T*)g, (const T*)b, H, eps, out, (int)out_f32, out32, vocab)
   switch (vpl) {
     case 1: DP_EMB(1); break;
     case 2: DP_EMB(2); break;
@@ -164,16 +167,16 @@ static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const vo
 
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                   const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
-                  cudaStream_t s, void* out32) {
+                  cudaStream_t s, void* out32, int vocab) {
   DP_CHECK(H % 8 == 0 && H > 0, DP_ERR_INVALID, "hidden must be a multiple of 8");
   DP_CHECK(seq > 0 && ntok >= 0, DP_ERR_INVALID, "bad token counts");
   if (ntok == 0) return;
   if (dtype == DP_BF16)
     embed_t<__nv_bfloat16>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32,
-                           static_cast<float*>(out32), s);
+                           static_cast<float*>(out32), vocab, s);
   else
     embed_t<__half>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, static_cast<float*>(out32),
-                    s);
+                    vocab, s);
 }
 
 // -------------------------------------------------------------------------------------
@@ -435,11 +438,9 @@ static void skinny_t(const void* x, int ldx, const void* w, const void* bias, co
                      int ldy, int M, int N, int K, int act, int io, cudaStream_t s) {
   constexpr int R = 8;
   const size_t sm = size_t(R) * K * sizeof(float);
-  static bool attr_set = false;  // one per template instantiation
-  if (!attr_set) {
+  static std::atomic<unsigned> attr_set{0};  // one per template instantiation
+  if (first_on_device(attr_set))
     DP_CUDA(cudaFuncSetAttribute(skinny_linear_kernel<T, R>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
-    attr_set = true;
-  }
   launch_kernel(skinny_linear_kernel<T, R>, dim3((N + R - 1) / R), dim3(256), sm, s, (const T*)x, ldx, (const T*)w,
                 (const T*)bias, res, ldr, y, ldy, M, N, K, act, io);
 }
@@ -648,12 +649,11 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   auto run_groups = [&](auto gtag) {
     constexpr int G = decltype(gtag)::value;
     constexpr int smem = att_groups_smem<G>();
-    static bool attr = false;
-    if (!attr) {
+    static std::atomic<unsigned> attr{0};
+    if (first_on_device(attr)) {
       DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__half, G>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
       DP_CUDA(cudaFuncSetAttribute(attention2_kernel<__nv_bfloat16, G>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    smem));
-      attr = true;
     }
     const dim3 g2(heads, grid.x, batch);
     static const int env_lpt = getenv("DP_ATT_LPT") ? atoi(getenv("DP_ATT_LPT")) : 1;  // experiments
@@ -864,11 +864,10 @@ void skinny_mma_t(const void* x, int ldx, const void* w, const void* bias, const
   DP_CHECK(cs > 0, DP_ERR_UNSUPPORTED, "skinny linear: K must split into <= 8 slices of <= 768 (multiples of 16)");
   const int KS = K / cs;
   const size_t sm = (size_t(16) * (KS + 8) + size_t(SK_STG) * SK_TOK * SK_XP) * sizeof(T);
-  static bool attr_set = false;  // one per template instantiation
-  if (!attr_set) {
+  static std::atomic<unsigned> attr_set{0};  // one per template instantiation
+  if (first_on_device(attr_set)) {
     DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024));
     DP_CUDA(cudaFuncSetAttribute(skinny_mma_kernel<T>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
-    attr_set = true;
   }
   launch_kernel_cluster(skinny_mma_kernel<T>, dim3((N / 16) * cs), dim3(256), sm, dim3(cs, 1, 1), s, (const T*)x, ldx,
                         (const T*)w, (const T*)bias, res, ldr, y, ldy, M, N, K, KS, cs, act, io);

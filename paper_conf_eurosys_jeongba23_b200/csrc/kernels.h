@@ -14,7 +14,8 @@ enum Io { IO_RES_F32 = 1, IO_OUT_F32 = 2 };
 // host-mapped (direct-host-access).  ln_g == nullptr -> no LN (GPT-2).
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                   const void* type, const void* ln_g, const void* ln_b, int H, float eps, void* out, bool out_f32,
-                  cudaStream_t s, void* out32 = nullptr);  // out32: optional fp32 copy of the LN output
+                  cudaStream_t s, void* out32 = nullptr,  // out32: optional fp32 copy of the LN output
+                  int vocab = 0);  // > 0: ids are clamped to [0, vocab) (engine path)
 
 // K4: y = LN(x (+ r)) * g + b; g/b may be host-mapped.
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,

@@ -8,6 +8,7 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdlib>
 
 #include "common.h"
@@ -72,16 +73,31 @@ inline void launch_kernel_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block,
   DP_CUDA(cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...));
 }
 
-// Timing ablation (tools/ablate.py only): DP_ABLATE is a bit mask of kernel families whose
-// launches are skipped -- 1 attention, 2 LayerNorm, 4 resident GEMM (query, key and value
-// grouped or not), 8 skinny linear / GEMV.  Outputs are garbage; the warm forward's time
-// without a family is what its share of the chain is.
+// Function attributes (dynamic shared memory size, non-portable clusters) are per device: a
+// call site sets them the first time it runs on each device.  `seen` is the call site's
+// static bit mask of devices (atomic: the serving harness drives devices from several threads).
+inline bool first_on_device(std::atomic<unsigned>& seen) {
+  int d = 0;
+  DP_CUDA(cudaGetDevice(&d));
+  const unsigned bit = 1u << d;
+  return (seen.fetch_or(bit) & bit) == 0;
+}
+
+// Timing ablation (tools/ablate.py only, instrumented builds: DP_NVCC_EXTRA=-DDP_INSTRUMENT):
+// DP_ABLATE is a bit mask of kernel families whose launches are skipped -- 1 attention,
+// 2 LayerNorm, 4 resident GEMM (query, key and value grouped or not), 8 skinny linear / GEMV.
+// Outputs are garbage; the warm forward's time without a family is what its share of the
+// chain is.  The release library compiles it to 0 (no environment variable can drop kernels).
 inline int ablate_mask() {
+#ifdef DP_INSTRUMENT
   static const int m = [] {
     const char* e = std::getenv("DP_ABLATE");
     return e ? std::atoi(e) : 0;
   }();
   return m;
+#else
+  return 0;
+#endif
 }
 
 // Device side: no-ops when the grid was not launched with PDL.

@@ -69,6 +69,11 @@ struct PeerState {
   std::vector<cudaEvent_t> ev;  // recycled
   size_t used = 0;
   cudaEvent_t last = nullptr;   // primary: last recv round
+  // secondary: the previous cold start's last send (its ring slots are free only after it);
+  // the next call's first H2D into the ring waits on it (ncclSend blocks until the
+  // primary posts its recv, so the previous call's sends may still be reading the ring)
+  cudaEvent_t sends_done = nullptr;
+  bool sends_pending = false;
   cudaEvent_t get() {
     if (used == ev.size()) {
       cudaEvent_t e;
@@ -148,8 +153,13 @@ void peer_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int prima
   int64_t big = 0;
   for (auto& pc : pcs) big = std::max(big, pc.bytes);
   if (!p.h2d) DP_CUDA(cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking));
+  if (!p.sends_done) DP_CUDA(cudaEventCreateWithFlags(&p.sends_done, cudaEventDisableTiming));
+  if (p.sends_pending) DP_CUDA(cudaStreamWaitEvent(p.h2d, p.sends_done, 0));
   if (p.ring_bytes < kRing * big) {
-    if (p.ring) DP_CUDA(cudaFree(p.ring));
+    if (p.ring) {
+      DP_CUDA(cudaStreamSynchronize(ctx->comm_stream));  // earlier sends still read the old ring
+      DP_CUDA(cudaFree(p.ring));
+    }
     p.ring = nullptr;
     if (cudaMalloc(&p.ring, kRing * big) != cudaSuccess) fail(DP_ERR_OOM, "staging ring cudaMalloc failed");
     p.ring_bytes = kRing * big;
@@ -174,6 +184,8 @@ void peer_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int prima
     sent[r] = done;
     st.n_events += 2;
   }
+  DP_CUDA(cudaEventRecord(p.sends_done, ctx->comm_stream));
+  p.sends_pending = true;
   if (stats) *stats = st;
 }
 

@@ -37,6 +37,7 @@
 #include "dtype.cuh"
 #include "engine.h"
 #include "kernels.h"
+#include "launch.cuh"
 #include "persist.h"
 #include "tc.cuh"
 
@@ -813,14 +814,12 @@ int persist_num_ops(const PersistProgram& p) { return p.nops; }
 
 void launch_persist(const PersistProgram& p, void* final_out, cudaStream_t s) {
   const size_t smem = persist_smem_bytes();
-  static bool attr[2] = {false, false};
+  static std::atomic<unsigned> attr[2];
   const bool bf = p.dtype == DP_BF16;
   auto kern = bf ? persist_kernel<__nv_bfloat16> : persist_kernel<__half>;
-  if (!attr[bf]) {
+  if (first_on_device(attr[bf]))
     DP_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void*>(kern), cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)smem));
-    attr[bf] = true;
-  }
   DP_CUDA(cudaMemsetAsync(p.d_bar, 0, sizeof(unsigned), s));
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(p.G);

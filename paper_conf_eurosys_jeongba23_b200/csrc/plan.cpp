@@ -332,8 +332,12 @@ extern "C" dp_status dp_plan_exhaustive(const dp_cost_table* cost, const dp_plan
     }
     for (int i = 0; i < n; ++i)
       if (part[i] >= 1) m[i] = DP_LOAD;
-    for (int b = 0; b < nfree; ++b)
+    for (int b = 0; b < nfree; ++b) {
       DP_CHECK(free_idx[b] >= 0 && free_idx[b] < n, DP_ERR_INVALID, "free index out of range");
+      // a unit of a PT partition (slot >= 1) must stay LOAD: freeing it could put DHA on a
+      // secondary's slot, an infeasible plan whose under-counted latency would win
+      DP_CHECK(part[free_idx[b]] == 0, DP_ERR_INVALID, "free index names a unit of a PT partition (slot >= 1)");
+    }
     int64_t best = INT64_MAX;
     uint64_t best_v = 0;
     const uint64_t total = uint64_t(1) << nfree;

@@ -346,3 +346,29 @@ def test_large_models_full_size(name, S, mode, k, transport):
     assert st["h2d_bytes"][:len(link)] == link
     model.close()
     c.close()
+
+
+def test_graph_replay_after_workspace_regrowth():
+    """with use_graph, batch 1 -> batch 4 (the workspace is reallocated) ->
+    batch 1 again must not replay the first batch-1 graph on freed memory.  Every replay equals
+    the eager run of the same shape, bit for bit."""
+    m = synth.SHAPES["tiny_bert"]
+    dtype = "fp16"
+    w = synth.make_weights(m, seed=31, dtype=dtype)
+    c = dp().Context([0])
+    model = dp().Model(c, m, w, dtype)
+    plan = dp().plan_generate(fake_cost(m, dtype), "DHA", 1)
+    eager = {}
+    for B in (1, 4):
+        ids = synth.make_ids(m, B, 48, seed=32 + B)
+        o, p, _ = run_cold(model, plan, ids, dtype)
+        eager[B] = (ids, o.clone(), p.clone())
+        model.evict(0)
+    c.set_opts(use_graph=1, debug_poison=1)
+    for B in (1, 4, 1, 4, 1):
+        ids, ref, ref_pool = eager[B]
+        out, pool, _ = run_cold(model, plan, ids, dtype)
+        assert torch.equal(out, ref) and torch.equal(pool, ref_pool), B
+        model.evict(0)
+    model.close()
+    c.close()

@@ -83,3 +83,19 @@ def test_exhaustive_matches(seed):
     free = [i for i in range(n) if part[i] == 0]
     lat, p = dp.plan_exhaustive(c, base, free)
     assert lat == lat_o and list(p.method) == m_o and list(p.slot) == slot_o
+
+
+def test_exhaustive_rejects_pt_partition_units():
+    """A unit of a PT partition (slot >= 1) must stay LOAD: freeing it in the
+    exhaustive search is rejected by both planners instead of returning an infeasible plan
+    whose under-counted latency wins."""
+    c = synth.make_cost_table(8, 77)
+    k = 3
+    part = P.partition(list(c["bytes"]), k)
+    bad = [i for i in range(8) if part[i] >= 1][:1]
+    assert bad
+    base = dp.plan_generate(c, "PT", k)
+    with pytest.raises(dp.DeepPlanError):
+        dp.plan_exhaustive(c, base, bad)
+    with pytest.raises(ValueError):
+        P.exhaustive(c, k=k, free=bad)

@@ -2,7 +2,10 @@
 flushed) with whole kernel families skipped (DP_ABLATE bit mask: 1 attention, 2 LayerNorm,
 4 resident GEMM, 8 skinny/GEMV), each in its own process.  Outputs are garbage; the time a
 family's removal saves is its share of the chained forward (PDL overlap included).
-python tools/ablate.py [model:seq ...]"""
+python tools/ablate.py [model:seq ...]
+
+Needs the instrumented library (the release build compiles DP_ABLATE out):
+    DP_NVCC_EXTRA=-DDP_INSTRUMENT python paper_conf_eurosys_jeongba23_b200/build.py"""
 import json
 import os
 import subprocess
