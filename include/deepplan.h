@@ -49,8 +49,10 @@ typedef int32_t dp_status;
 
 /* Model families of the paper's transformer workloads. */
 enum { DP_FAMILY_BERT = 0, DP_FAMILY_ROBERTA = 1, DP_FAMILY_GPT2 = 2 };
-/* Weight storage dtypes (the paper never states one; fp16 is the default). */
-enum { DP_FP16 = 0, DP_BF16 = 1 };
+/* Weight storage dtypes (the paper never states one; fp16 is the default).  DP_FP32
+ * is the paper's own precision (Table 1's byte counts are fp32): every kernel then
+ * reads and writes fp32 and the linears run on CUDA cores (there is no fp32 tcgen05 kind). */
+enum { DP_FP16 = 0, DP_BF16 = 1, DP_FP32 = 2 };
 /* Planning-unit kinds (Table 3: Emb, LN, FC). */
 enum { DP_UNIT_EMB = 0, DP_UNIT_LN = 1, DP_UNIT_LINEAR = 2 };
 /* Engine options + the "initial approach" of P:41 (GREEDY). */
@@ -192,7 +194,12 @@ typedef struct {
                              a DHA unit keeps its absolute extra host-read time), and Load = the
                              unit's byte share of one whole-arena copy (the engine coalesces
                              loads, R18; an isolated copy carries ~4 us of per-copy cost) [1] */
-  int32_t reserved[3];
+  int32_t trace_units;    /* 1 = dp_infer_cold records per-unit timestamps (read back with
+                             dp_run_timeline): timing events after every transfer piece and around
+                             every unit's dependency wait on the execution stream.  Costs event
+                             records between kernels (no PDL overlap) and forces eager enqueue (no
+                             graph): a measurement mode [0] */
+  int32_t reserved[2];
 } dp_engine_opts;
 #define DP_PT_DMA 0
 #define DP_PT_SM 1
@@ -341,6 +348,26 @@ dp_status dp_infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int32
                         const int32_t* secondaries, int32_t nsec, const int32_t* d_ids, int32_t batch,
                         int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats);
 
+/* Per-unit timeline of the last cold start of m on `dev` run with opts.trace_units = 1 (SURVEY
+ * §8(b) "per-unit ready/start/end ns"; dp_run_stats is filled at enqueue time, before any of it
+ * happened, so the times are read back here).  Synchronises on that cold start.  All times are ns
+ * since the cold start's first event on the execution stream; arrays of n = unit count
+ * (caller-owned, each nullable):
+ *   ready_ns  when the unit's bytes had landed in HBM (the end of its DMA / forwarded piece; 0 for
+ *             a DHA unit, which is read in place; -1 if not observable, e.g. another process's IPC
+ *             transfer)
+ *   start_ns  when the execution stream passed the unit's dependency wait -- its first
+ *             kernel can start
+ *   end_ns    when the execution stream reached the next unit (its kernels -- and the
+ *             parameterless ops charged to it, SURVEY G1 -- are done); units whose kernels are
+ *             grouped (BERT's q/k/v: one launch) end when the group's first kernel starts
+ *   stall_ns  start_ns minus when the stream reached the wait: the pipeline stall of P:162-170,
+ *             the quantity the simulator (dp_plan_simulate) predicts per unit
+ * Units the forward never reached (e.g. the pooler without a pooled output) get -1.
+ * DP_ERR_STATE if no traced cold start of m ran on dev. */
+dp_status dp_run_timeline(dp_context* ctx, dp_model* m, int32_t dev, int32_t n, int64_t* ready_ns, int64_t* start_ns,
+                          int64_t* end_ns, int64_t* stall_ns);
+
 /* Warm inference: the model is resident on dev (DP_ERR_STATE otherwise). */
 dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, const int32_t* d_ids, int32_t batch,
                         int32_t seq, void* d_out, void* d_pooled, void* stream, dp_run_stats* stats);
@@ -356,10 +383,20 @@ dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, const int32_t
 dp_status dp_lm_head(dp_context* ctx, dp_model* m, int32_t dev, const void* d_hidden, int32_t ld_hidden,
                      int32_t rows, float* d_logits, void* stream);
 
-/* Residency: make the model non-resident on dev (its HBM slots return to the pool).
- * Synchronises the device's streams first. */
+/* Residency: make the model non-resident on dev.  Synchronises the device first; its HBM slot
+ * block returns to the context's per-device pool (reused by the next cold start of any model;
+ * dp_pool_trim hands free blocks back to the driver).  A model exported with dp_peer_ipc_export
+ * keeps its full-arena slots (peers hold IPC mappings of them). */
 dp_status dp_model_evict(dp_context* ctx, dp_model* m, int32_t dev);
 int32_t dp_model_is_resident(const dp_model* m, int32_t dev);
+/* HBM bytes the resident model holds on dev (0 if not resident): only the LOADED units take
+ * slots -- a cold start lays the block out like the arena with every DHA unit's range left out,
+ * so DHA layers cost no GPU memory ("DeepPlan can serve more instances"). */
+int64_t dp_model_resident_bytes(const dp_model* m, int32_t dev);
+/* The per-device slot pool: bytes reserved from the driver and bytes held by resident models. */
+dp_status dp_pool_stats(dp_context* ctx, int32_t dev, int64_t* reserved, int64_t* in_use);
+/* Release the pool's free blocks to the driver (cudaFree); *freed (nullable) gets the bytes. */
+dp_status dp_pool_trim(dp_context* ctx, int32_t dev, int64_t* freed);
 
 /* ---------------------------------------------------------------------------------
  * Kernel entry points (parity-test hooks; same kernels the executor launches).

@@ -17,7 +17,10 @@ GPT-2 (pre-LN, Conv1D weights are [in, out])
   per block: x += c_proj(attn_causal(c_attn(LN1(x)))); x += proj2(gelu_tanh(fc(LN2(x))))
   x = ln_f(x)
 
-All arithmetic is float64 on the storage-rounded weights (fp16/bf16/fp32 -> f64).
+All arithmetic is float64 on the storage-rounded weights (fp16/bf16/fp32 -> f64).  The one
+exception is `forward(..., compute="f32")`: the same definition evaluated in numpy float32, the
+"numpy fp32 forward" SURVEY §8(d) times as the CPU baseline beside the GPU (never a parity
+reference).
 """
 from __future__ import annotations
 
@@ -72,11 +75,18 @@ def _w(weights, name, dtype):
     return storage_to_f64(weights[name], dtype)
 
 
-def forward(m: ModelShape, weights, ids: np.ndarray, dtype: str = "fp16"):
-    """Returns (last_hidden_state [B,S,H] f64, pooled [B,H] f64 or None)."""
+def forward(m: ModelShape, weights, ids: np.ndarray, dtype: str = "fp16", compute: str = "f64"):
+    """Returns (last_hidden_state [B,S,H], pooled [B,H] or None) in float64 (compute="f64", the
+    oracle) or float32 (compute="f32", the CPU-baseline timing variant)."""
     ids = np.asarray(ids)
     B, S = ids.shape
-    W = lambda n: _w(weights, n, dtype)  # noqa: E731
+    cdt = {"f64": np.float64, "f32": np.float32}[compute]
+    cache = {}
+
+    def W(n):
+        if n not in cache:
+            cache[n] = _w(weights, n, dtype).astype(cdt, copy=False)
+        return cache[n]
     if m.family in ("bert", "roberta"):
         if m.family == "bert":
             pos = np.arange(S)

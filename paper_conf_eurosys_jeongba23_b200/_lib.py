@@ -14,7 +14,7 @@ MODES = {"BASELINE": 0, "PIPESWITCH": 1, "GREEDY": 2, "DHA": 3, "PT": 4, "PT_DHA
          "PT_DHA_LINK": 7, "PT_DHA_BAL": 8, "PT_DHA_LINK_BAL": 9, "PT_DHA_STRIPE": 10, "PT_DHA_LINK_STRIPE": 11}
 UNIT_KINDS = {0: "emb", 1: "ln", 2: "linear"}
 FAMILIES = {"bert": 0, "roberta": 1, "gpt2": 2}
-DTYPES = {"fp16": 0, "bf16": 1}
+DTYPES = {"fp16": 0, "bf16": 1, "fp32": 2}
 ACTS = {"none": 0, "gelu_erf": 1, "gelu_tanh": 2, "tanh": 3}
 PT_TRANSPORTS = {"dma": 0, "sm": 1, "ce": 2}  # dp_engine_opts.pt_transport: DP_PT_DMA / _SM / _CE
 DP_MAX_DEVICES = 8
@@ -53,7 +53,7 @@ class EngineOpts(C.Structure):
                 ("gemm_bn", C.c_int32), ("debug_delay_us", C.c_int32), ("debug_poison", C.c_int32),
                 ("use_pdl", C.c_int32), ("fuse_ln", C.c_int32), ("tail_bytes", C.c_int64),
                 ("persistent", C.c_int32), ("pt_transport", C.c_int32), ("profile_chain", C.c_int32),
-                ("reserved", C.c_int32 * 3)]
+                ("trace_units", C.c_int32), ("reserved", C.c_int32 * 2)]
 
 
 class ModelConfig(C.Structure):
@@ -137,10 +137,14 @@ _sig("dp_measure_h2d", [C.c_int32, C.c_int64, C.c_int32, C.POINTER(C.c_double)])
 _sig("dp_profile",[vp, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.POINTER(CostTable)])
 _sig("dp_infer_cold", [vp, vp, C.POINTER(Plan), C.c_int32, i32p, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp, vp,
                        C.POINTER(RunStats)])
+_sig("dp_run_timeline", [vp, vp, C.c_int32, C.c_int32, i64p, i64p, i64p, i64p])
 _sig("dp_infer_warm", [vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp, vp, C.POINTER(RunStats)])
 _sig("dp_model_evict", [vp, vp, C.c_int32])
 _sig("dp_lm_head", [vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, vp, vp])
 _sig("dp_model_is_resident", [vp, C.c_int32])
+_sig("dp_model_resident_bytes", [vp, C.c_int32], C.c_int64)
+_sig("dp_pool_stats", [vp, C.c_int32, i64p, i64p])
+_sig("dp_pool_trim", [vp, C.c_int32, i64p])
 _sig("dp_host_alloc", [C.c_int64, C.POINTER(vp)])
 _sig("dp_host_free", [vp])
 _sig("dp_embed", [vp, C.c_int32, C.c_int32, C.c_int32, vp, vp, vp, vp, vp, C.c_int32, C.c_double, C.c_int32,
@@ -281,7 +285,7 @@ class Context:
 
     def set_opts(self, chunk_bytes=None, n_h2d_streams=None, use_graph=None, gemm_bn=None, debug_delay_us=None,
                  debug_poison=None, use_pdl=None, tail_bytes=None, fuse_ln=None, persistent=None,
-                 pt_transport=None, profile_chain=None):
+                 pt_transport=None, profile_chain=None, trace_units=None):
         o = EngineOpts()
         _check(lib.dp_context_get_opts(self.h, C.byref(o)))
         if chunk_bytes is not None:
@@ -306,9 +310,22 @@ class Context:
             o.persistent = 1 if persistent else 0
         if profile_chain is not None:
             o.profile_chain = 1 if profile_chain else 0
+        if trace_units is not None:
+            o.trace_units = 1 if trace_units else 0
         if pt_transport is not None:
             o.pt_transport = PT_TRANSPORTS[pt_transport] if isinstance(pt_transport, str) else int(pt_transport)
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))
+
+    def pool_stats(self, dev: int = 0):
+        """(reserved, in_use) bytes of the device's HBM slot pool."""
+        r, u = C.c_int64(), C.c_int64()
+        _check(lib.dp_pool_stats(self.h, int(dev), C.byref(r), C.byref(u)))
+        return int(r.value), int(u.value)
+
+    def pool_trim(self, dev: int = 0) -> int:
+        f = C.c_int64()
+        _check(lib.dp_pool_trim(self.h, int(dev), C.byref(f)))
+        return int(f.value)
 
     def peer_init(self, uid: bytes, rank: int, nranks: int):
         buf = C.create_string_buffer(uid, 128)
@@ -445,6 +462,14 @@ class Model:
                                  C.byref(st)))
         return _stats(st)
 
+    def timeline(self, dev: int) -> dict:
+        """Per-unit ready / start / end / stall ns of the last traced cold start (opts.trace_units)."""
+        arrs = {k: np.zeros(self.n, dtype=np.int64) for k in ("ready_ns", "start_ns", "end_ns", "stall_ns")}
+        _check(lib.dp_run_timeline(self.ctx.h, self.h, int(dev), self.n, *[_ptr(arrs[k], i64p) for k in
+                                                                           ("ready_ns", "start_ns", "end_ns",
+                                                                            "stall_ns")]))
+        return arrs
+
     def infer_warm(self, dev: int, ids, out, pooled=None, stream=None) -> dict:
         st = RunStats()
         B, S = ids.shape
@@ -478,6 +503,10 @@ class Model:
 
     def is_resident(self, dev: int) -> bool:
         return bool(lib.dp_model_is_resident(self.h, int(dev)))
+
+    def resident_bytes(self, dev: int) -> int:
+        """HBM bytes held while resident (loaded units only; DHA units stay in host memory)."""
+        return int(lib.dp_model_resident_bytes(self.h, int(dev)))
 
     def close(self):
         if self.h:

@@ -22,7 +22,8 @@ extern "C" dp_status dp_host_free(void* p) {
 }
 
 static void check_dtype(int32_t dtype) {
-  DP_CHECK(dtype == DP_FP16 || dtype == DP_BF16, DP_ERR_UNSUPPORTED, "dtype must be DP_FP16 or DP_BF16");
+  DP_CHECK(dtype == DP_FP16 || dtype == DP_BF16 || dtype == DP_FP32, DP_ERR_UNSUPPORTED,
+           "dtype must be DP_FP16, DP_BF16 or DP_FP32");
 }
 
 extern "C" dp_status dp_embed(const int32_t* d_ids, int32_t ntok, int32_t seq, int32_t pos_offset, const void* word,
@@ -47,6 +48,7 @@ extern "C" dp_status dp_linear(const void* x, int32_t ldx, const void* w, const 
              "bad shapes / strides");
     DP_CHECK(act >= 0 && act <= 3, DP_ERR_INVALID, "act must be 0..3");
     if (path == 0) {
+      DP_CHECK(dtype != DP_FP32, DP_ERR_UNSUPPORTED, "the tcgen05 path has no fp32 kind: use path 1 for fp32");
       cudaPointerAttributes at;
       DP_CUDA(cudaPointerGetAttributes(&at, w));
       DP_CHECK(at.type == cudaMemoryTypeDevice, DP_ERR_INVALID, "the tcgen05 path needs W in device memory");

@@ -51,6 +51,6 @@ dp_status guard(F&& body) {
   }
 }
 
-inline int dtype_bytes(int dtype) { return 2; }  // fp16 / bf16 storage
+inline int dtype_bytes(int dtype) { return dtype == DP_FP32 ? 4 : 2; }  // storage element bytes
 
 }  // namespace dp

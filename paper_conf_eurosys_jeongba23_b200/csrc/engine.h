@@ -36,8 +36,18 @@ struct Piece {
   int first_unit = -1, last_unit = -1;
 };
 
+// Device-memory pool of one device (infer.cu): the HBM slot blocks of the models.  Evicting a
+// model returns its block here (not to the driver), so the next cold start of any model reuses
+// it; dp_pool_trim releases the free blocks to the driver.
+struct HbmPool {
+  std::multimap<int64_t, void*> free_;  // free blocks by size
+  std::map<void*, int64_t> size_;       // every block the pool owns -> its size
+  int64_t reserved = 0, in_use = 0;
+};
+
 struct DevCtx {
   int ord = -1;
+  HbmPool pool;
   bool ready = false;
   std::vector<cudaStream_t> h2d;  // load streams ("load stream")
   EventPool events;
@@ -63,6 +73,11 @@ struct ForwardArgs {
 };
 
 void ensure_workspace(dp_model* m, int dev, int64_t tokens);
+// HBM slots of the units `method` loads (compact layout, from the pool; infer.cu), their release,
+// and the full-arena slots of an IPC-exported model.
+void acquire_slots(dp_context* ctx, dp_model* m, int dev, const int8_t* method);
+void release_slots(dp_context* ctx, dp_model* m, int dev);
+void pin_full_slots(dp_model* m, int dev);
 // Destroy every captured graph / K6 program of a device state (their buffers are going away).
 void drop_graphs(DevState& ds);
 void run_forward(ForwardArgs& a);

@@ -102,15 +102,126 @@ static SlotRes& slot_res(dp_context* ctx, int slot, int dev, int64_t ring_bytes)
   return r;
 }
 
-void dp::ensure_slots(dp_model* m, int dev) {
+// ---------------------------------------------------------------------------------------
+// HBM slots: a per-device pool of blocks; a model holds one block while resident, laid out
+// like the arena minus the DHA units' ranges (DHA layers occupy no GPU memory).
+// ---------------------------------------------------------------------------------------
+
+namespace dp {
+
+constexpr int64_t kPoolGrain = 2 << 20;  // block sizes are rounded to 2 MiB (easier reuse)
+
+// Free every unused block of the pool (back to the driver); returns the bytes released.
+static int64_t pool_trim(HbmPool& p, int dev) {
+  DeviceGuard g(dev);
+  int64_t freed = 0;
+  for (auto& kv : p.free_) {
+    DP_CUDA(cudaFree(kv.second));
+    p.size_.erase(kv.second);
+    freed += kv.first;
+  }
+  p.free_.clear();
+  p.reserved -= freed;
+  return freed;
+}
+
+// A block of >= bytes: `prefer` if it is free and fits (a model re-acquiring its last block keeps
+// its captured graphs valid), else the best fit among the free blocks not more than 2x too large,
+// else a new cudaMalloc (trimming the free blocks and retrying once if HBM is exhausted).
+static void* pool_alloc(HbmPool& p, int dev, int64_t bytes, void* prefer) {
+  bytes = (bytes + kPoolGrain - 1) / kPoolGrain * kPoolGrain;
+  auto take = [&](std::multimap<int64_t, void*>::iterator it) {
+    void* b = it->second;
+    p.in_use += it->first;
+    p.free_.erase(it);
+    return b;
+  };
+  if (prefer) {
+    for (auto it = p.free_.begin(); it != p.free_.end(); ++it)
+      if (it->second == prefer && it->first >= bytes && it->first <= 2 * bytes) return take(it);
+  }
+  auto it = p.free_.lower_bound(bytes);
+  if (it != p.free_.end() && it->first <= 2 * bytes) return take(it);
+  DeviceGuard g(dev);
+  void* b = nullptr;
+  if (cudaMalloc(&b, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    pool_trim(p, dev);
+    if (cudaMalloc(&b, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      fail(DP_ERR_OOM, "HBM slot allocation for the model failed");
+    }
+  }
+  p.size_[b] = bytes;
+  p.reserved += bytes;
+  p.in_use += bytes;
+  return b;
+}
+
+static void pool_free(HbmPool& p, void* b) {
+  auto it = p.size_.find(b);
+  DP_CHECK(it != p.size_.end(), DP_ERR_STATE, "internal: block not owned by this pool");
+  p.in_use -= it->second;
+  p.free_.emplace(it->second, b);
+}
+
+// Compact layout: loaded units keep the arena's relative offsets; each DHA unit's arena span
+// (its bytes plus alignment padding up to the next unit) is left out.  Units between which no DHA
+// unit lies stay contiguous, so every DMA piece (consecutive loaded units) is one contiguous
+// destination range.
+static int64_t compact_layout(const dp_model* m, const int8_t* method, std::vector<int64_t>& doff) {
+  const int n = (int)m->units.size();
+  doff.assign(n, -1);
+  int64_t removed = 0;
+  for (int u = 0; u < n; ++u) {
+    const int64_t end = u + 1 < n ? m->units[u + 1].off : m->arena_bytes;
+    if (method && method[u] == DP_DHA) {
+      removed += end - m->units[u].off;
+      continue;
+    }
+    doff[u] = m->units[u].off - removed;
+  }
+  return m->arena_bytes - removed;
+}
+
+void acquire_slots(dp_context* ctx, dp_model* m, int dev, const int8_t* method) {
   DevState& ds = m->dev[dev];
-  if (ds.dbase) return;
+  if (ds.pinned_full) {  // IPC-exported: the peers write into the full arena layout
+    compact_layout(m, nullptr, ds.doff);
+    return;
+  }
+  DP_CHECK(!ds.dbase, DP_ERR_STATE, "internal: HBM slots already held");
+  std::vector<int64_t> doff;
+  const int64_t bytes = std::max<int64_t>(compact_layout(m, method, doff), 256);
+  ds.dbase = pool_alloc(ctx->on(dev).pool, dev, bytes, ds.last_block);
+  ds.dbytes = bytes;
+  ds.doff.swap(doff);
+}
+
+void release_slots(dp_context* ctx, dp_model* m, int dev) {
+  DevState& ds = m->dev[dev];
+  if (ds.pinned_full || !ds.dbase) return;
+  pool_free(ctx->on(dev).pool, ds.dbase);
+  ds.last_block = ds.dbase;
+  ds.dbase = nullptr;
+  ds.dbytes = 0;
+}
+
+void pin_full_slots(dp_model* m, int dev) {
+  DevState& ds = m->dev[dev];
+  if (ds.pinned_full) return;
+  DP_CHECK(!ds.resident && !ds.dbase, DP_ERR_STATE, "export the model's slots before its first cold start");
   DeviceGuard g(dev);
   if (cudaMalloc(&ds.dbase, m->arena_bytes) != cudaSuccess) {
     ds.dbase = nullptr;
     fail(DP_ERR_OOM, "HBM slot allocation for the model failed");
   }
+  ds.dbytes = m->arena_bytes;
+  ds.pinned_full = true;
+  compact_layout(m, nullptr, ds.doff);
 }
+
+}  // namespace dp
 
 // Single-process SM forwarding to another GPU stores through the peer mapping.
 static void ensure_peer_access(int from, int to) {
@@ -167,6 +278,8 @@ extern "C" dp_status dp_context_destroy(dp_context* ctx) {
       DeviceGuard g(d);
       cudaDeviceSynchronize();
       DevCtx& dc = ctx->dc[d];
+      for (auto& kv : dc.pool.size_) cudaFree(kv.first);  // models must be destroyed first
+      dc.pool = HbmPool();
       for (auto s : dc.h2d) cudaStreamDestroy(s);
       dc.events.destroy();
       if (dc.flush) cudaFree(dc.flush);
@@ -315,7 +428,7 @@ static void validate_plan(const dp_model* m, const dp_plan* p) {
 
 // Host-link bytes a unit's DHA kernels must read (algorithmic; Table 1's closed forms).
 static int64_t unit_dha_bytes(const dp_model* m, int u, int T, int seq) {
-  const int64_t row = int64_t(m->cfg.hidden) * 2;
+  const int64_t row = int64_t(m->cfg.hidden) * dtype_bytes(m->cfg.dtype);
   switch (m->units[u].role) {
     case R_WORD: case R_WTE: return int64_t(T) * row;  // one row per token
     case R_POS: case R_WPE: return int64_t(std::min<int64_t>(seq, m->cfg.max_pos)) * row;
@@ -405,13 +518,13 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
   DP_CHECK(seq + (m->cfg.family == DP_FAMILY_ROBERTA ? m->cfg.pad_idx + 1 : 0) <= m->cfg.max_pos, DP_ERR_INVALID,
            "sequence longer than the position table");
   DeviceGuard g(primary);
-  ensure_slots(m, primary);
+  acquire_slots(ctx, m, primary, plan->method);
   ensure_h2d_streams(ctx, primary);
   ensure_workspace(m, primary, int64_t(batch) * seq);
   // across processes: the IPC transports capture (the epoch lives in a device word); the NCCL
   // gather does not
   const bool ipc_pt = ctx->multiproc() && ctx->opts.pt_transport != DP_PT_DMA && plan->k > 1;
-  bool graph = ctx->opts.use_graph != 0 && (!ctx->multiproc() || ipc_pt || plan->k == 1);
+  bool graph = ctx->opts.use_graph != 0 && !ctx->opts.trace_units && (!ctx->multiproc() || ipc_pt || plan->k == 1);
   for (int s = 1; s < plan->k && graph && !ctx->multiproc(); ++s)
     graph = secondaries[s - 1] == primary;  // single-device graphs only
   // staging rings of the two-hop PT slots are sized before any capture (their pointers are
@@ -480,6 +593,24 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   cudaEvent_t fork = pd.events.get();
   DP_CUDA(cudaEventRecord(fork, stream));
   ++st.n_events;
+  // opts.trace_units: timing events for dp_run_timeline (eager only: graphs are off)
+  const bool trace = ctx->opts.trace_units != 0;
+  UnitTrace& tr = ds.trace;
+  if (trace) {
+    tr.valid = false;
+    tr.used = 0;
+    tr.ready.assign(n, nullptr);
+    tr.pre.assign(n, nullptr);
+    tr.start.assign(n, nullptr);
+    tr.t0 = tr.get();
+    DP_CUDA(cudaEventRecord(tr.t0, stream));
+  }
+  auto trace_piece = [&](const Piece& p, cudaStream_t on) {  // the piece's bytes have landed
+    if (!trace) return;
+    cudaEvent_t e = tr.get();
+    DP_CUDA(cudaEventRecord(e, on));
+    for (int u = p.first_unit; u <= p.last_unit; ++u) tr.ready[u] = e;
+  };
 
   // (1) slot-0 loads on the primary's link
   const int64_t cap = std::max<int64_t>(ctx->opts.chunk_bytes, 4096);
@@ -491,8 +622,8 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     const Piece& p = pieces0[c];
     cudaStream_t hs = pd.h2d[c % nh];
     if (ctx->opts.debug_delay_us > 0) launch_spin((long long)ctx->opts.debug_delay_us * 2000, hs);
-    DP_CUDA(cudaMemcpyAsync(static_cast<uint8_t*>(ds.dbase) + p.off, static_cast<const uint8_t*>(m->arena) + p.off,
-                            p.bytes, cudaMemcpyHostToDevice, hs));
+    DP_CUDA(cudaMemcpyAsync(m->device(primary, p.first_unit), static_cast<const uint8_t*>(m->arena) + p.off, p.bytes,
+                            cudaMemcpyHostToDevice, hs));
     ++st.n_copies;
     st.h2d_bytes[0] += p.bytes;
     cudaEvent_t e = pd.events.get();
@@ -500,6 +631,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     ++st.n_events;
     bind_units(unit_ev, p, e);  // every unit inside this piece completes with it
     add_wp(0, p, e);
+    trace_piece(p, hs);
   }
 
   // (2) PT slots
@@ -550,12 +682,12 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       for (const Piece& p : pcs) {
         if (ctx->opts.debug_delay_us > 0) launch_spin((long long)ctx->opts.debug_delay_us * 2000, r.h2d);
         if (ce_fwd) {
-          DP_CUDA(cudaMemcpyAsync(static_cast<uint8_t*>(ds.dbase) + p.off, static_cast<const uint8_t*>(m->arena) + p.off,
+          DP_CUDA(cudaMemcpyAsync(m->device(primary, p.first_unit), static_cast<const uint8_t*>(m->arena) + p.off,
                                   p.bytes, cudaMemcpyDefault, r.h2d));
           ++st.n_copies;
         } else {
-          launch_pt_forward(static_cast<const uint8_t*>(m->arena) + p.off, static_cast<uint8_t*>(ds.dbase) + p.off,
-                            p.bytes, r.h2d, nullptr, 0, nullptr, nullptr);
+          launch_pt_forward(static_cast<const uint8_t*>(m->arena) + p.off, m->device(primary, p.first_unit), p.bytes,
+                            r.h2d, nullptr, 0, nullptr, nullptr);
         }
         st.h2d_bytes[s] += p.bytes;
         st.nvlink_bytes[s] += p.bytes;
@@ -564,6 +696,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
         ++st.n_events;
         bind_units(unit_ev, p, done);
         add_wp(s, p, done);
+        if (sdev == primary) trace_piece(p, r.h2d);  // timing events only within one device
       }
       // the end-of-cold-start join waits on the migration stream: chain it behind the loads
       cudaEvent_t last = sd.events.get();
@@ -586,7 +719,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       DP_CUDA(cudaEventRecord(landed, r.h2d));
       DP_CUDA(cudaStreamWaitEvent(r.mig, landed, 0));
       if (ctx->opts.debug_delay_us > 0) launch_spin((long long)ctx->opts.debug_delay_us * 2000, r.mig);
-      uint8_t* dst = static_cast<uint8_t*>(ds.dbase) + p.off;
+      uint8_t* dst = m->device(primary, p.first_unit);
       if (sdev == primary)
         DP_CUDA(cudaMemcpyAsync(dst, stage, p.bytes, cudaMemcpyDeviceToDevice, r.mig));
       else
@@ -598,6 +731,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       fwd_done[c] = done;
       bind_units(unit_ev, p, done);
       add_wp(s, p, done);
+      if (sdev == primary) trace_piece(p, r.mig);
     }
   }
 
@@ -672,7 +806,22 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   };
   a.pdl = ctx->opts.use_pdl != 0;
   a.fuse_ln = ctx->opts.fuse_ln != 0;
+  if (trace) {  // an event on each side of the unit's dependency wait
+    auto gate = a.before_unit;
+    a.before_unit = [&, gate](int u) {
+      tr.pre[u] = tr.get();
+      DP_CUDA(cudaEventRecord(tr.pre[u], stream));
+      gate(u);
+      tr.start[u] = tr.get();
+      DP_CUDA(cudaEventRecord(tr.start[u], stream));
+    };
+  }
   run_forward(a);
+  if (trace) {
+    tr.fin = tr.get();
+    DP_CUDA(cudaEventRecord(tr.fin, stream));
+    tr.valid = true;
+  }
   // join every side stream (units never read, e.g. an unused pooler, still finish loading)
   for (int i = 0; i < nh; ++i) {
     cudaEvent_t e = pd.events.get();
@@ -723,6 +872,41 @@ extern "C" dp_status dp_infer_cold(dp_context* ctx, dp_model* m, const dp_plan* 
     }
     infer_cold(ctx, m, plan, primary, -1, secondaries, nsec, d_ids, batch, seq, d_out, d_pooled, (cudaStream_t)stream,
                stats);
+  });
+}
+
+extern "C" dp_status dp_run_timeline(dp_context* ctx, dp_model* m, int32_t dev, int32_t n, int64_t* ready_ns,
+                                     int64_t* start_ns, int64_t* end_ns, int64_t* stall_ns) {
+  return guard([&] {
+    DP_CHECK(ctx && m, DP_ERR_INVALID, "NULL context/model");
+    ctx->on(dev);
+    UnitTrace& tr = m->dev[dev].trace;
+    DP_CHECK(tr.valid, DP_ERR_STATE, "no traced cold start (set opts.trace_units) of this model on this device");
+    DP_CHECK(n == (int)m->units.size() && (int)tr.pre.size() == n, DP_ERR_INVALID, "n must be the unit count");
+    DeviceGuard g(dev);
+    DP_CUDA(cudaEventSynchronize(tr.fin));
+    for (cudaEvent_t e : tr.ready)  // a piece on a side stream may land after the forward's end
+      if (e) DP_CUDA(cudaEventSynchronize(e));
+    auto ns = [&](cudaEvent_t e) -> int64_t {
+      if (!e) return -1;
+      float ms = 0.f;
+      DP_CUDA(cudaEventElapsedTime(&ms, tr.t0, e));
+      return (int64_t)llround(double(ms) * 1e6);
+    };
+    const int8_t* method = m->dev[dev].method.data();
+    for (int u = 0; u < n; ++u) {
+      const int64_t pre = ns(tr.pre[u]), start = ns(tr.start[u]);
+      int64_t end = -1;
+      if (start >= 0) {
+        int v = u + 1;
+        while (v < n && !tr.pre[v]) ++v;
+        end = v < n ? ns(tr.pre[v]) : ns(tr.fin);
+      }
+      if (ready_ns) ready_ns[u] = method[u] == DP_DHA ? 0 : ns(tr.ready[u]);
+      if (start_ns) start_ns[u] = start;
+      if (end_ns) end_ns[u] = end;
+      if (stall_ns) stall_ns[u] = (start >= 0 && pre >= 0) ? std::max<int64_t>(0, start - pre) : -1;
+    }
   });
 }
 
@@ -844,10 +1028,33 @@ extern "C" dp_status dp_model_evict(dp_context* ctx, dp_model* m, int32_t dev) {
     DeviceGuard g(dev);
     DP_CUDA(cudaDeviceSynchronize());
     if (ctx->opts.debug_poison && m->dev[dev].dbase) {
-      DP_CUDA(cudaMemset(m->dev[dev].dbase, 0xFF, m->arena_bytes));
+      DP_CUDA(cudaMemset(m->dev[dev].dbase, 0xFF, m->dev[dev].dbytes));
       DP_CUDA(cudaDeviceSynchronize());
     }
     m->dev[dev].resident = false;
+    release_slots(ctx, m, dev);  // the block returns to the device's pool
+  });
+}
+
+extern "C" int64_t dp_model_resident_bytes(const dp_model* m, int32_t dev) {
+  if (!m || dev < 0 || dev >= DP_MAX_DEVICES || !m->dev[dev].resident) return 0;
+  return m->dev[dev].dbytes;
+}
+
+extern "C" dp_status dp_pool_stats(dp_context* ctx, int32_t dev, int64_t* reserved, int64_t* in_use) {
+  return guard([&] {
+    DP_CHECK(ctx && reserved && in_use, DP_ERR_INVALID, "NULL argument");
+    const HbmPool& p = ctx->on(dev).pool;
+    *reserved = p.reserved;
+    *in_use = p.in_use;
+  });
+}
+
+extern "C" dp_status dp_pool_trim(dp_context* ctx, int32_t dev, int64_t* freed) {
+  return guard([&] {
+    DP_CHECK(ctx, DP_ERR_INVALID, "NULL context");
+    const int64_t f = pool_trim(ctx->on(dev).pool, dev);
+    if (freed) *freed = f;
   });
 }
 
@@ -868,7 +1075,11 @@ extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
         ds.graphs.clear();
         ds.persist.clear();
         if (ds.capture) cudaStreamDestroy(ds.capture);
-        if (ds.dbase) cudaFree(ds.dbase);
+        if (ds.pinned_full) {
+          cudaFree(ds.dbase);
+        } else if (ds.dbase && ctx) {
+          release_slots(ctx, m, d);
+        }
         if (ds.ws.base) cudaFree(ds.ws.base);
       }
     }
@@ -907,7 +1118,19 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
   DevState& ds = m->dev[dev];
   DP_CHECK(!ds.resident, DP_ERR_STATE, "evict the model before profiling");
   DeviceGuard g(dev);
-  ensure_slots(m, dev);
+  acquire_slots(ctx, m, dev, nullptr);  // every unit resident for the in-memory runs (full layout)
+  struct Release {
+    dp_context* c;
+    dp_model* mm;
+    int d;
+    ~Release() {
+      try {
+        cudaDeviceSynchronize();
+        release_slots(c, mm, d);
+      } catch (...) {
+      }
+    }
+  } release_at_exit{ctx, m, dev};
   const int T = batch * seq;
   ensure_workspace(m, dev, T);
   if (!d.flush) {
@@ -926,7 +1149,7 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
   }
   DP_CUDA(cudaMemset(m->dev[dev].ws.base, 0, 1));
   // all weights resident for the in-memory runs
-  DP_CUDA(cudaMemcpy(ds.dbase, m->arena, m->arena_bytes, cudaMemcpyHostToDevice));
+  DP_CUDA(cudaMemcpy(ds.dbase, m->arena, m->arena_bytes, cudaMemcpyHostToDevice));  // full layout
   cudaEvent_t e0, e1;
   DP_CUDA(cudaEventCreate(&e0));
   DP_CUDA(cudaEventCreate(&e1));
@@ -962,7 +1185,7 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
   for (int u = 0; u < n; ++u) {
     const auto& un = m->units[u];
     out->bytes[u] = un.bytes;
-    uint8_t* dst = static_cast<uint8_t*>(ds.dbase) + un.off;
+    uint8_t* dst = m->device(dev, u);
     const uint8_t* src = static_cast<const uint8_t*>(m->arena) + un.off;
     out->load_ns[u] = timed([&] { DP_CUDA(cudaMemcpyAsync(dst, src, un.bytes, cudaMemcpyHostToDevice, s)); }, false);
     uint8_t* scratch = static_cast<uint8_t*>(d.flush);

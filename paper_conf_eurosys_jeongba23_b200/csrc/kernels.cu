@@ -171,6 +171,10 @@ void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off,
   DP_CHECK(H % 8 == 0 && H > 0, DP_ERR_INVALID, "hidden must be a multiple of 8");
   DP_CHECK(seq > 0 && ntok >= 0, DP_ERR_INVALID, "bad token counts");
   if (ntok == 0) return;
+  if (dtype == DP_FP32) {
+    launch_embed_f32(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out32, vocab, s);
+    return;
+  }
   if (dtype == DP_BF16)
     embed_t<__nv_bfloat16>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32,
                            static_cast<float*>(out32), vocab, s);
@@ -230,6 +234,10 @@ void launch_layernorm(int dtype, const void* x, const void* r, const void* g, co
   if (ablate_mask() & 2) return;
   DP_CHECK(n % 8 == 0 && n > 0, DP_ERR_INVALID, "LN width must be a multiple of 8");
   if (rows <= 0) return;
+  if (dtype == DP_FP32) {
+    launch_layernorm_f32(x, r, g, b, y, rows, n, eps, s, y32);
+    return;
+  }
   if (dtype == DP_BF16)
     layernorm_t<__nv_bfloat16>(x, r, g, b, y, rows, n, eps, in_f32, static_cast<float*>(y32), s);
   else
@@ -457,6 +465,10 @@ void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, cons
   if (ablate_mask() & 8) return;
   DP_CHECK(K % 8 == 0 && K > 0 && N > 0, DP_ERR_INVALID, "skinny linear needs K % 8 == 0");
   if (M <= 0) return;
+  if (dtype == DP_FP32) {  // W read once, as below; fp32 in / out (io flags are implied)
+    launch_linear_f32(x, ldx, w, bias, res, ldr, y, ldy, M, N, K, act, s);
+    return;
+  }
   const bool mma = M > 16 && N % 16 == 0 && K % 16 == 0 && ldx % 8 == 0 && ((uintptr_t)x % 16) == 0 &&
                    skinny_cluster(K) > 0;
   if (mma) {
@@ -639,6 +651,10 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   DP_CHECK(heads > 0 && H % heads == 0 && H / heads == ATT_D, DP_ERR_UNSUPPORTED, "attention needs head dim 64");
   DP_CHECK(ldqkv % 8 == 0, DP_ERR_INVALID, "ldqkv must be a multiple of 8");
   if (batch <= 0 || seq <= 0) return;
+  if (dtype == DP_FP32) {
+    launch_attention_f32(qkv, ldqkv, ctx, batch, seq, H, heads, causal, s);
+    return;
+  }
   dim3 grid((seq + ATT_BQ - 1) / ATT_BQ, heads, batch);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)ATT_D);
   static const int env_att = getenv("DP_ATT_GROUPS") ? atoi(getenv("DP_ATT_GROUPS")) : 0;  // experiments

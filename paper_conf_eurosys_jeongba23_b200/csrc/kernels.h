@@ -46,6 +46,18 @@ void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const 
                           const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
                           int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);
 
+// fp32 storage (DP_FP32, kernels_f32.cu): CUDA-core kernels with the same contracts; the
+// launchers above dispatch to them when dtype == DP_FP32 (all activations are then fp32).
+void launch_embed_f32(const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
+                      const void* type, const void* g, const void* b, int H, float eps, void* out, void* out32,
+                      int vocab, cudaStream_t s);
+void launch_layernorm_f32(const void* x, const void* r, const void* g, const void* b, void* y, int rows, int n,
+                          float eps, cudaStream_t s, void* y32);
+void launch_linear_f32(const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr, void* y,
+                       int ldy, int M, int N, int K, int act, cudaStream_t s);
+void launch_attention_f32(const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads, bool causal,
+                          cudaStream_t s);
+
 // Scratch kernels
 void launch_l2_flush(void* buf, size_t bytes, cudaStream_t s);
 void launch_spin(long long cycles, cudaStream_t s);

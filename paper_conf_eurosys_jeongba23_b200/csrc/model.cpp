@@ -16,7 +16,8 @@ namespace dp {
 void validate_config(const dp_model_config& c) {
   DP_CHECK(c.family == DP_FAMILY_BERT || c.family == DP_FAMILY_ROBERTA || c.family == DP_FAMILY_GPT2,
            DP_ERR_INVALID, "unknown model family");
-  DP_CHECK(c.dtype == DP_FP16 || c.dtype == DP_BF16, DP_ERR_UNSUPPORTED, "dtype must be fp16 or bf16");
+  DP_CHECK(c.dtype == DP_FP16 || c.dtype == DP_BF16 || c.dtype == DP_FP32, DP_ERR_UNSUPPORTED,
+           "dtype must be fp16, bf16 or fp32");
   DP_CHECK(c.hidden > 0 && c.hidden % 64 == 0, DP_ERR_INVALID, "hidden must be a positive multiple of 64");
   DP_CHECK(c.heads > 0 && c.hidden % c.heads == 0, DP_ERR_INVALID, "hidden % heads != 0");
   DP_CHECK(c.ffn > 0 && c.ffn % 64 == 0, DP_ERR_INVALID, "ffn must be a positive multiple of 64");
@@ -35,7 +36,7 @@ std::vector<ParamDesc> config_params(const dp_model_config& c) {
     p.ndim = b < 0 ? 1 : 2;
     p.shape[0] = a;
     p.shape[1] = b < 0 ? 0 : b;
-    p.bytes = a * (b < 0 ? 1 : b) * 2;
+    p.bytes = a * (b < 0 ? 1 : b) * dtype_bytes(c.dtype);
     p.transpose = tr;
     ps.push_back(p);
   };
@@ -206,11 +207,18 @@ extern "C" dp_status dp_model_create(dp_context* ctx, const dp_model_config* cfg
       if (!p.transpose) {
         std::memcpy(base + p.off, host_params[i], p.bytes);
       } else {  // [in=a, out=b] -> [out, in]
-        const uint16_t* src = static_cast<const uint16_t*>(host_params[i]);
-        uint16_t* dst = reinterpret_cast<uint16_t*>(base + p.off);
         const int64_t a = p.shape[0], b = p.shape[1];
-        for (int64_t r = 0; r < a; ++r)
-          for (int64_t c = 0; c < b; ++c) dst[c * a + r] = src[r * b + c];
+        if (dtype_bytes(cfg->dtype) == 4) {
+          const uint32_t* src = static_cast<const uint32_t*>(host_params[i]);
+          uint32_t* dst = reinterpret_cast<uint32_t*>(base + p.off);
+          for (int64_t r = 0; r < a; ++r)
+            for (int64_t c = 0; c < b; ++c) dst[c * a + r] = src[r * b + c];
+        } else {
+          const uint16_t* src = static_cast<const uint16_t*>(host_params[i]);
+          uint16_t* dst = reinterpret_cast<uint16_t*>(base + p.off);
+          for (int64_t r = 0; r < a; ++r)
+            for (int64_t c = 0; c < b; ++c) dst[c * a + r] = src[r * b + c];
+        }
       }
     }
     *out = m;

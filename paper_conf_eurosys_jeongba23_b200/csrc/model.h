@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <map>
+#include <stdexcept>
 #include <memory>
 #include <string>
 #include <vector>
@@ -35,7 +36,7 @@ struct UnitDesc {
   int layer = -1;
   int first_param = 0, nparams = 0;
   int64_t off = 0, bytes = 0;
-  int64_t N = 0, K = 0;  // linear: W [N, K] at off, bias [N] at off + N*K*2
+  int64_t N = 0, K = 0;  // linear: W [N, K] at off, bias [N] at off + N*K*(element bytes)
 };
 
 // Activation workspace on one device for T tokens.
@@ -59,12 +60,37 @@ struct GraphEntry {
   dp_run_stats stats{};
 };
 
+// Per-unit timestamps of a traced cold start (opts.trace_units; dp_run_timeline).
+struct UnitTrace {
+  bool valid = false;
+  std::vector<cudaEvent_t> pool;  // timing-enabled events, recycled
+  size_t used = 0;
+  cudaEvent_t t0 = nullptr, fin = nullptr;
+  std::vector<cudaEvent_t> ready, pre, start;  // per unit (nullptr: not observed)
+  cudaEvent_t get() {
+    if (used == pool.size()) {
+      cudaEvent_t e;
+      if (cudaEventCreate(&e) != cudaSuccess) throw std::runtime_error("cudaEventCreate failed");
+      pool.push_back(e);
+    }
+    return pool[used++];
+  }
+};
+
 struct DevState {
-  void* dbase = nullptr;  // HBM copy of the arena layout (slots for loaded units)
+  // HBM slots of the loaded units: one block from the context's pool (infer.cu), laid out like
+  // the arena with the DHA units' ranges left out (they stay in host memory: DeepPlan
+  // "serves more instances" because DHA layers take no GPU memory)
+  void* dbase = nullptr;
+  int64_t dbytes = 0;          // bytes of the block
+  std::vector<int64_t> doff;   // per unit: offset in the block, -1 for a DHA unit (read in place)
+  bool pinned_full = false;    // IPC-exported slots: full arena layout, outside the pool, kept
+  void* last_block = nullptr;  // the block released by the last eviction (reacquired if free)
   bool resident = false;
   std::vector<int8_t> method;  // per unit, fixed when the model became resident
   Workspace ws;
   std::map<std::string, GraphEntry> graphs;  // captured cold / warm runs (opts.use_graph)
+  UnitTrace trace;                           // last traced cold start
   cudaStream_t capture = nullptr;            // private stream the graphs are captured on
   // K6 programs per (batch, seq, workspace): their tensor maps point into dbase and ws
   std::map<std::string, std::shared_ptr<PersistProgram>> persist;
@@ -92,5 +118,5 @@ struct dp_model {
   void* peer_dbase[DP_MAX_DEVICES] = {};  // other ranks' HBM slots, IPC-mapped (by rank)
 
   const uint8_t* host(int u) const { return static_cast<const uint8_t*>(arena) + units[u].off; }
-  uint8_t* device(int d, int u) const { return static_cast<uint8_t*>(dev[d].dbase) + units[u].off; }
+  uint8_t* device(int d, int u) const { return static_cast<uint8_t*>(dev[d].dbase) + dev[d].doff[u]; }
 };

@@ -110,13 +110,12 @@ void peer_recv_all(dp_context* ctx, dp_model* m, const dp_plan* plan, int primar
   }
   DP_CUDA(cudaStreamWaitEvent(ctx->comm_stream, fork, 0));
   auto* comm = static_cast<ncclComm_t>(ctx->comm);
-  uint8_t* dbase = static_cast<uint8_t*>(m->dev[dev].dbase);
   for (size_t r = 0; r < rounds; ++r) {
     DP_NCCL(nccl().groupStart());
     for (int s = 1; s < plan->k; ++s) {
       if (r >= pcs[s].size()) continue;
       const Piece& pc = pcs[s][r];
-      DP_NCCL(nccl().recv(dbase + pc.off, pc.bytes, ncclUint8, peer_rank_of_slot(ctx, primary, s), comm,
+      DP_NCCL(nccl().recv(m->device(dev, pc.first_unit), pc.bytes, ncclUint8, peer_rank_of_slot(ctx, primary, s), comm,
                           ctx->comm_stream));
       st.nvlink_bytes[s] += pc.bytes;
     }

@@ -43,6 +43,6 @@ void ipc_send_rank(dp_context* ctx, dp_model* m, const dp_plan* plan, int primar
 void ipc_close(dp_context* ctx);
 void ipc_close_model(dp_model* m);
 // The model's HBM slots on dev (infer.cu).
-void ensure_slots(dp_model* m, int dev);
+void acquire_slots(dp_context* ctx, dp_model* m, int dev, const int8_t* method);
 
 }  // namespace dp

@@ -349,7 +349,7 @@ extern "C" dp_status dp_peer_ipc_export(dp_context* ctx, dp_model* m, void* out)
     DP_CUDA(cudaGetDevice(&prev));
     DP_CUDA(cudaSetDevice(dev));
     try {
-      ensure_slots(m, dev);
+      pin_full_slots(m, dev);
       ensure_mailbox(ctx);
       cudaIpcMemHandle_t h[2];
       DP_CUDA(cudaIpcGetMemHandle(&h[0], m->dev[dev].dbase));

@@ -82,8 +82,8 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
         int32_t* ids;
         void *y, *pooled;
         DP_CUDA(cudaMalloc(&ids, sizeof(int32_t) * T));
-        DP_CUDA(cudaMalloc(&y, size_t(T) * maxH * 2));
-        DP_CUDA(cudaMalloc(&pooled, size_t(o.batch) * maxH * 2));
+        DP_CUDA(cudaMalloc(&y, size_t(T) * maxH * 4));  // room for any storage dtype
+        DP_CUDA(cudaMalloc(&pooled, size_t(o.batch) * maxH * 4));
         std::vector<int32_t> h(T);
         for (int t = 0; t < T; ++t) h[t] = 3 + (t * 7919) % 997;
         DP_CUDA(cudaMemcpy(ids, h.data(), sizeof(int32_t) * T, cudaMemcpyHostToDevice));

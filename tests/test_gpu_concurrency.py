@@ -24,6 +24,10 @@ def dp():
 
 
 def _stress(fn, out, reps, noise_src, noise_dst, side, main):
+    # the inputs were written on the default stream: `main` must not read them before that
+    # finished (without this the quiet reference itself could read unwritten inputs -- seen once
+    # as 600/600 "mismatches" of a correct kernel against a garbage reference)
+    torch.cuda.synchronize()
     with torch.cuda.stream(main):
         fn()
     torch.cuda.synchronize()

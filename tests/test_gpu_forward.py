@@ -213,19 +213,21 @@ def test_bert_base_cold_start_bench_configuration():
     model.close()
 
 
-def test_gpt2_medium_causal_prefix_full_size():
-    """GPT-2 Medium at S=1024 (the full config): causal attention means the first r
-    outputs depend only on the first r tokens, so the oracle checks a 48-token prefix."""
+def test_gpt2_medium_full_size_every_row():
+    """BASELINE.json configs[3]: GPT-2 Medium fp16 at S=1024, PT_DHA over two slots (loopback),
+    compared with the fp64 oracle element by element on ALL 1024 x 1024 outputs (the oracle's
+    full forward takes ~15 s on the host) at the north_star's max-abs 1e-2."""
     m = synth.SHAPES["gpt2_medium"]
     dtype = "fp16"
     w = synth.make_weights(m, seed=5, dtype=dtype)
     ids = synth.make_ids(m, 1, 1024, seed=6)
-    ref, _ = F.forward(m, w, ids[:, :48], dtype)
+    ref, _ = F.forward(m, w, ids, dtype)
     model = dp().Model(ctx(), m, w, dtype)
     plan = dp().plan_generate(fake_cost(m, dtype), "PT_DHA", 2)
     out, _, _ = run_cold(model, plan, ids, dtype, secondaries=[0])
     model.evict(0)
-    assert np.abs(f64(out[:48]) - ref.reshape(48, -1)).max() <= 1e-2
+    err = np.abs(f64(out) - ref.reshape(1024, -1))
+    assert err.max() <= 1e-2, err.max()
     model.close()
 
 
