@@ -49,7 +49,6 @@ def parse():
     ap.add_argument("--h2d-streams", type=int, default=1)
     ap.add_argument("--no-graph", action="store_true", help="eager enqueue instead of CUDA-graph replay")
     ap.add_argument("--no-pdl", action="store_true")
-    ap.add_argument("--fuse-ln", action="store_true", help="LayerNorm in the preceding GEMM's epilogue")
     ap.add_argument("--profile-iters", type=int, default=10)
     ap.add_argument("--pt-transport", default="ce", choices=["dma", "sm", "ce"],
                     help="PT slots at N>1: dma = copy engine into a staging ring + NCCL send/recv (the paper's "
@@ -343,7 +342,7 @@ def main():
     ctx.set_opts(chunk_bytes=int(a.chunk_mb * (1 << 20)), n_h2d_streams=a.h2d_streams,
                  tail_bytes=int(a.tail_mb * (1 << 20)),
                  use_graph=0 if (a.no_graph or (world > 1 and a.pt_transport == "dma")) else 1,
-                 use_pdl=0 if a.no_pdl else 1, fuse_ln=a.fuse_ln, pt_transport=a.pt_transport)
+                 use_pdl=0 if a.no_pdl else 1, pt_transport=a.pt_transport)
     model = dp.Model(ctx, m, w, dtype)
     if dist_on and a.pt_transport == "dma":
         uid = dp.peer_unique_id() if rank == 0 else None

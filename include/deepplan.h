@@ -393,6 +393,9 @@ int32_t dp_model_is_resident(const dp_model* m, int32_t dev);
  * slots -- a cold start lays the block out like the arena with every DHA unit's range left out,
  * so DHA layers cost no GPU memory ("DeepPlan can serve more instances"). */
 int64_t dp_model_resident_bytes(const dp_model* m, int32_t dev);
+/* HBM bytes a cold start under `plan` will hold (the compact layout; what the serving harness
+ * budgets per instance); -1 on a NULL / mismatched plan. */
+int64_t dp_plan_resident_bytes(const dp_model* m, const dp_plan* plan);
 /* The per-device slot pool: bytes reserved from the driver and bytes held by resident models. */
 dp_status dp_pool_stats(dp_context* ctx, int32_t dev, int64_t* reserved, int64_t* in_use);
 /* Release the pool's free blocks to the driver (cudaFree); *freed (nullable) gets the bytes. */
@@ -461,7 +464,7 @@ typedef struct {
   int64_t slo_ns;                /* goodput threshold (100 ms) */
   /* dry-run latency table, per MODEL index: cold / warm ns, resident bytes */
   int32_t nmodels;
-  int32_t reserved0;
+  int32_t no_prewarm;            /* live: 1 = skip the pre-warm pass (every instance once per GPU) */
   const int64_t* cold_ns;
   const int64_t* warm_ns;
   const int64_t* resident_bytes;
@@ -470,19 +473,25 @@ typedef struct {
   int32_t batch, seq;
   int32_t reserved1;
   /* live mode: models[i] is instance i's dp_model (nmodels == ninstances) and plans[i]
-   * its cold-start plan; a plan with k > 1 uses the next k-1 GPUs of the context as
-   * secondaries (their PCIe links and copy engines, not their compute) */
+   * its cold-start plan; a plan with k > 1 borrows k-1 other GPUs of the context as
+   * secondaries (their PCIe links and copy engines, not their compute): idle ones first.
+   * Live decisions are made online on the observed state (R11-live): warm on the
+   * GPU holding the instance, else cold on the GPU with the fewest outstanding requests,
+   * evicting LRU instances without outstanding requests (dp_model_evict: HBM back to the
+   * pool) until the instance's LOADED bytes fit the budget (cold_ns / warm_ns /
+   * resident_bytes are not used).  Token ids are 3 + (t * 7919) % 997. */
   const dp_plan* const* plans;
   const int32_t* seq_of_model; /* nullable: per model index sequence length (else `seq`) */
 } dp_serve_opts;
 
 typedef struct {
   int64_t start_ns;    /* when the request began executing */
-  int64_t finish_ns;   /* completion time */
+  int64_t finish_ns;   /* completion time (live: when the dispatcher observed it) */
   int32_t gpu;         /* GPU that ran it */
   int32_t cold;        /* 1 = cold start */
   int32_t nevicted;    /* instances evicted to make room */
-  int32_t reserved;
+  int32_t sec_mask;    /* live PT cold start: bit g set = GPU g lent its link (0 otherwise) */
+  int64_t decide_ns;   /* live: when the dispatcher decided it (dry run: its arrival) */
 } dp_serve_result;
 
 /* Replay (dry_run=1) or run live (dry_run=0: models[] are real dp_models, one per

@@ -20,7 +20,11 @@ GPT-2 (pre-LN, Conv1D weights are [in, out])
 All arithmetic is float64 on the storage-rounded weights (fp16/bf16/fp32 -> f64).  The one
 exception is `forward(..., compute="f32")`: the same definition evaluated in numpy float32, the
 "numpy fp32 forward" SURVEY §8(d) times as the CPU baseline beside the GPU (never a parity
-reference).
+reference).  And `forward(..., act_round="bf16")`: the same definition with the activations
+rounded to a 16-bit type exactly where a pipeline that stores them in that type must round them
+(every linear's input operand, the attention inputs q / k / v, the softmax numerators before P.V,
+the output) and nothing else (residual sums stay exact).  It measures the REPRESENTATION error
+of storing activations in that type -- the bf16 tolerance is set from it (R15).
 """
 from __future__ import annotations
 
@@ -29,7 +33,7 @@ import math
 import numpy as np
 from scipy.special import erf
 
-from synth import ModelShape, storage_to_f64
+from synth import ModelShape, round_to, storage_to_f64
 
 
 def layer_norm(x: np.ndarray, gamma: np.ndarray, beta: np.ndarray, eps: float) -> np.ndarray:
@@ -55,8 +59,16 @@ def softmax(z: np.ndarray) -> np.ndarray:
     return e / e.sum(axis=-1, keepdims=True)
 
 
-def attention(q: np.ndarray, k: np.ndarray, v: np.ndarray, heads: int, causal: bool) -> np.ndarray:
-    """Multi-head scaled dot-product attention. q,k,v: [B,S,H] -> [B,S,H]."""
+def _rnd(x: np.ndarray, dtype) -> np.ndarray:
+    """Round to a 16-bit storage type (RNE) and back; identity when dtype is None."""
+    if dtype is None:
+        return x
+    return storage_to_f64(round_to(np.asarray(x, dtype=np.float32), dtype), dtype).astype(x.dtype, copy=False)
+
+
+def attention(q: np.ndarray, k: np.ndarray, v: np.ndarray, heads: int, causal: bool, p_round=None) -> np.ndarray:
+    """Multi-head scaled dot-product attention. q,k,v: [B,S,H] -> [B,S,H].  p_round: the storage
+    type the softmax numerators exp(s - max) are rounded to before P.V (the row sums are not)."""
     B, S, H = q.shape
     d = H // heads
     qh = q.reshape(B, S, heads, d).transpose(0, 2, 1, 3)
@@ -66,8 +78,12 @@ def attention(q: np.ndarray, k: np.ndarray, v: np.ndarray, heads: int, causal: b
     if causal:
         mask = np.triu(np.ones((S, S), dtype=bool), k=1)
         scores = np.where(mask, -np.inf, scores)
-    p = softmax(scores)
-    ctx = p @ vh
+    if p_round is None:
+        p = softmax(scores)
+        ctx = p @ vh
+    else:
+        e = np.exp(scores - scores.max(axis=-1, keepdims=True))
+        ctx = (_rnd(e, p_round) @ vh) / e.sum(axis=-1, keepdims=True)
     return ctx.transpose(0, 2, 1, 3).reshape(B, S, H)
 
 
@@ -75,9 +91,12 @@ def _w(weights, name, dtype):
     return storage_to_f64(weights[name], dtype)
 
 
-def forward(m: ModelShape, weights, ids: np.ndarray, dtype: str = "fp16", compute: str = "f64"):
+def forward(m: ModelShape, weights, ids: np.ndarray, dtype: str = "fp16", compute: str = "f64",
+            act_round: str | None = None):
     """Returns (last_hidden_state [B,S,H], pooled [B,H] or None) in float64 (compute="f64", the
-    oracle) or float32 (compute="f32", the CPU-baseline timing variant)."""
+    oracle) or float32 (compute="f32", the CPU-baseline timing variant).  act_round: see the
+    module docstring (None = exact)."""
+    R = lambda t: _rnd(t, act_round)  # noqa: E731
     ids = np.asarray(ids)
     B, S = ids.shape
     cdt = {"f64": np.float64, "f32": np.float32}[compute]
@@ -98,32 +117,34 @@ def forward(m: ModelShape, weights, ids: np.ndarray, dtype: str = "fp16", comput
         x = layer_norm(e, W("embeddings.LayerNorm.weight"), W("embeddings.LayerNorm.bias"), m.ln_eps)
         for i in range(m.layers):
             p = f"encoder.layer.{i}."
-            lin = lambda t, n: t @ W(p + n + ".weight").T + W(p + n + ".bias")  # noqa: E731
-            q = lin(x, "attention.self.query")
-            k = lin(x, "attention.self.key")
-            v = lin(x, "attention.self.value")
-            c = attention(q, k, v, m.heads, causal=False)
+            lin = lambda t, n: R(t) @ W(p + n + ".weight").T + W(p + n + ".bias")  # noqa: E731
+            q = R(lin(x, "attention.self.query"))
+            k = R(lin(x, "attention.self.key"))
+            v = R(lin(x, "attention.self.value"))
+            c = attention(q, k, v, m.heads, causal=False, p_round=act_round)
             x1 = layer_norm(x + lin(c, "attention.output.dense"),
                             W(p + "attention.output.LayerNorm.weight"),
                             W(p + "attention.output.LayerNorm.bias"), m.ln_eps)
             h = gelu_erf(lin(x1, "intermediate.dense"))
             x = layer_norm(x1 + lin(h, "output.dense"), W(p + "output.LayerNorm.weight"),
                            W(p + "output.LayerNorm.bias"), m.ln_eps)
-        pooled = np.tanh(x[:, 0] @ W("pooler.dense.weight").T + W("pooler.dense.bias"))
+        x = R(x)  # the output itself is stored in the type
+        pooled = R(np.tanh(x[:, 0] @ W("pooler.dense.weight").T + W("pooler.dense.bias")))
         return x, pooled
     if m.family == "gpt2":
         x = W("wte.weight")[ids] + W("wpe.weight")[np.arange(S)][None]
         H = m.hidden
         for i in range(m.layers):
             p = f"h.{i}."
-            conv = lambda t, n: t @ W(p + n + ".weight") + W(p + n + ".bias")  # noqa: E731
+            conv = lambda t, n: R(t) @ W(p + n + ".weight") + W(p + n + ".bias")  # noqa: E731
             a = layer_norm(x, W(p + "ln_1.weight"), W(p + "ln_1.bias"), m.ln_eps)
-            qkv = conv(a, "attn.c_attn")
-            c = attention(qkv[..., :H], qkv[..., H:2 * H], qkv[..., 2 * H:], m.heads, causal=True)
+            qkv = R(conv(a, "attn.c_attn"))
+            c = attention(qkv[..., :H], qkv[..., H:2 * H], qkv[..., 2 * H:], m.heads, causal=True,
+                          p_round=act_round)
             x = x + conv(c, "attn.c_proj")
             a = layer_norm(x, W(p + "ln_2.weight"), W(p + "ln_2.bias"), m.ln_eps)
             x = x + conv(gelu_tanh(conv(a, "mlp.c_fc")), "mlp.c_proj")
-        x = layer_norm(x, W("ln_f.weight"), W("ln_f.bias"), m.ln_eps)
+        x = R(layer_norm(x, W("ln_f.weight"), W("ln_f.bias"), m.ln_eps))
         return x, None
     raise ValueError(m.family)
 

@@ -62,3 +62,48 @@ def metrics(arrival_ns, res, slo_ns):
     lat = (res["finish_ns"] - np.asarray(arrival_ns)).astype(np.float64)
     return {"p99_ms": float(np.percentile(lat, 99) / 1e6), "mean_ms": float(lat.mean() / 1e6),
             "goodput": float(np.mean(lat <= slo_ns)), "cold_rate": float(np.mean(res["cold"]))}
+
+
+def replay_online(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, resident_bytes, decide_ns, finish_ns):
+    """The live (online) policy, R11-live, re-derived from what the live dispatcher had
+    observed when it decided each request -- its decision time decide_ns[r] and the time it saw
+    each request complete, finish_ns[q]: request q is complete at r's decision iff
+    finish_ns[q] <= decide_ns[r].  In arrival order:
+      * instance resident (or becoming resident) on g  -> warm on g;
+      * else cold on the GPU with the fewest outstanding (decided, not complete) requests, lowest
+        index on ties; there, least recently used resident instances with no outstanding request
+        are evicted until the instance's resident bytes fit the budget (if none can go,
+        the GPU runs over budget until they finish).
+    resident_bytes is per INSTANCE (its plan's loaded units).  Returns gpu, cold, nevicted."""
+    n = len(arrival_ns)
+    gpu = np.full(n, -1, dtype=np.int64)
+    cold = np.zeros(n, dtype=np.int64)
+    nev = np.zeros(n, dtype=np.int64)
+    home = {}
+    lru = [OrderedDict() for _ in range(ngpu)]  # instance -> bytes, least recently used first
+    used = [0] * ngpu
+    for r in range(n):
+        t = decide_ns[r]
+        live = [q for q in range(r) if finish_ns[q] > t]  # decided earlier, not observed complete
+        i = int(instance[r])
+        if i in home:
+            g = home[i]
+            lru[g].move_to_end(i)
+        else:
+            busy = [sum(1 for q in live if gpu[q] == x) for x in range(ngpu)]
+            g = min(range(ngpu), key=lambda x: (busy[x], x))
+            pend = {int(instance[q]) for q in live}
+            for v in list(lru[g].keys()):
+                if used[g] + int(resident_bytes[i]) <= per_gpu_budget_bytes:
+                    break
+                if v in pend:
+                    continue
+                used[g] -= lru[g].pop(v)
+                del home[v]
+                nev[r] += 1
+            lru[g][i] = int(resident_bytes[i])
+            used[g] += int(resident_bytes[i])
+            home[i] = g
+            cold[r] = 1
+        gpu[r] = g
+    return {"gpu": gpu, "cold": cold, "nevicted": nev}

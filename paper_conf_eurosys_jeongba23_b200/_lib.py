@@ -88,7 +88,7 @@ class TraceEvent(C.Structure):
 class ServeOpts(C.Structure):
     _fields_ = [("plan_mode", C.c_int32), ("k_max", C.c_int32), ("ngpu", C.c_int32), ("dry_run", C.c_int32),
                 ("per_gpu_budget_bytes", C.c_int64), ("slo_ns", C.c_int64), ("nmodels", C.c_int32),
-                ("reserved0", C.c_int32), ("cold_ns", i64p), ("warm_ns", i64p), ("resident_bytes", i64p),
+                ("no_prewarm", C.c_int32), ("cold_ns", i64p), ("warm_ns", i64p), ("resident_bytes", i64p),
                 ("model_of_instance", i32p), ("ninstances", C.c_int32), ("batch", C.c_int32),
                 ("seq", C.c_int32), ("reserved1", C.c_int32), ("plans", C.POINTER(C.POINTER(Plan))),
                 ("seq_of_model", i32p)]
@@ -96,7 +96,7 @@ class ServeOpts(C.Structure):
 
 class ServeResult(C.Structure):
     _fields_ = [("start_ns", C.c_int64), ("finish_ns", C.c_int64), ("gpu", C.c_int32), ("cold", C.c_int32),
-                ("nevicted", C.c_int32), ("reserved", C.c_int32)]
+                ("nevicted", C.c_int32), ("sec_mask", C.c_int32), ("decide_ns", C.c_int64)]
 
 
 def _sig(name, args, res=C.c_int32):
@@ -145,6 +145,7 @@ _sig("dp_model_is_resident", [vp, C.c_int32])
 _sig("dp_model_resident_bytes", [vp, C.c_int32], C.c_int64)
 _sig("dp_pool_stats", [vp, C.c_int32, i64p, i64p])
 _sig("dp_pool_trim", [vp, C.c_int32, i64p])
+_sig("dp_plan_resident_bytes", [vp, C.POINTER(Plan)], C.c_int64)
 _sig("dp_host_alloc", [C.c_int64, C.POINTER(vp)])
 _sig("dp_host_free", [vp])
 _sig("dp_embed", [vp, C.c_int32, C.c_int32, C.c_int32, vp, vp, vp, vp, vp, C.c_int32, C.c_double, C.c_int32,
@@ -574,9 +575,14 @@ def attention(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp1
 # Serving harness
 # --------------------------------------------------------------------------------------
 
+def plan_resident_bytes(model: "Model", plan: "PlanArrays") -> int:
+    """HBM bytes the model holds when resident under `plan` (loaded units only)."""
+    return int(lib.dp_plan_resident_bytes(model.h, C.byref(plan.s)))
+
+
 def serve_run(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, cold_ns, warm_ns, resident_bytes,
               model_of_instance, slo_ns=100_000_000, dry_run=True, ctx: Context | None = None, models=None,
-              plans=None, batch=1, seq=128, plan_mode="DHA", k_max=1, seq_of_model=None):
+              plans=None, batch=1, seq=128, plan_mode="DHA", k_max=1, seq_of_model=None, prewarm=True):
     arrival_ns = _i64(arrival_ns)
     instance = np.ascontiguousarray(instance, dtype=np.int32)
     n = len(arrival_ns)
@@ -593,6 +599,7 @@ def serve_run(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, cold_ns, warm
     o.k_max = int(k_max)
     o.ngpu = int(ngpu)
     o.dry_run = int(bool(dry_run))
+    o.no_prewarm = 0 if prewarm else 1
     o.per_gpu_budget_bytes = int(per_gpu_budget_bytes)
     o.slo_ns = int(slo_ns)
     o.nmodels = len(cold)
@@ -615,5 +622,5 @@ def serve_run(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, cold_ns, warm
     res = (ServeResult * max(n, 1))()
     _check(lib.dp_serve_run(ctx.h if ctx else None, mh, len(models) if models else 0, trace, n, C.byref(o), res))
     out = {k: np.array([getattr(res[i], k) for i in range(n)], dtype=np.int64)
-           for k in ("start_ns", "finish_ns", "gpu", "cold", "nevicted")}
+           for k in ("start_ns", "finish_ns", "gpu", "cold", "nevicted", "sec_mask", "decide_ns")}
     return out

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <stdexcept>
 #include <string>
 
@@ -49,6 +50,19 @@ dp_status guard(F&& body) {
     set_last_error(e.what());
     return DP_ERR_INVALID;
   }
+}
+
+// Experiment knobs (tools/ sweeps and A/B runs) read from the environment ONLY in instrumented
+// builds (DP_NVCC_EXTRA=-DDP_INSTRUMENT); the release library always uses `dflt`, so no
+// environment variable can change what it computes or launches.
+inline int experiment_env(const char* name, int dflt) {
+#ifdef DP_INSTRUMENT
+  const char* e = std::getenv(name);
+  return e ? std::atoi(e) : dflt;
+#else
+  (void)name;
+  return dflt;
+#endif
 }
 
 inline int dtype_bytes(int dtype) { return dtype == DP_FP32 ? 4 : 2; }  // storage element bytes

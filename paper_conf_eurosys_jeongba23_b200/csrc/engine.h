@@ -27,6 +27,11 @@ struct SlotRes {
   cudaStream_t h2d = nullptr, mig = nullptr;
   void* ring = nullptr;
   int64_t ring_bytes = 0;
+  // the last cold start's final forward out of the ring: the next cold start using this slot
+  // resource (e.g. a concurrent one on another primary, in serving) waits for it before its first
+  // H2D into the ring
+  cudaEvent_t tail = nullptr;
+  bool tail_set = false;
 };
 
 // A contiguous byte range of the arena moved by one DMA (and one forward for PT): the
@@ -68,8 +73,6 @@ struct ForwardArgs {
   int kernels = 0;
   int bn_hint = 0;
   bool pdl = false;  // chain kernels with programmatic dependent launch (opts.use_pdl)
-  bool fuse_ln = false;  // LayerNorm in the preceding GEMM's epilogue (opts.fuse_ln)
-  bool persistent = false;  // all layers in one K6 launch when every layer unit is resident
 };
 
 void ensure_workspace(dp_model* m, int dev, int64_t tokens);

@@ -441,7 +441,7 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   const int min_st = int((need + STAGE_BYTES - 1) / STAGE_BYTES);
   // ring depth: the full ring unless DP_GEMM_STAGES caps it (experiments), and never deeper
   // than the K blocks a CTA streams
-  static const int env_st = getenv("DP_GEMM_STAGES") ? atoi(getenv("DP_GEMM_STAGES")) : 0;
+  static const int env_st = experiment_env("DP_GEMM_STAGES", 0);
   int nst = env_st > 0 ? std::min(env_st, STAGES) : STAGES;
   nst = std::max(nst, std::max(min_st, 1));
   DP_CHECK(nst <= STAGES, DP_ERR_INVALID, "gemm: epilogue buffers do not fit this tile width");
@@ -545,8 +545,8 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
   DP_CHECK(ldy % 8 == 0 && (!res || ldr % 8 == 0), DP_ERR_INVALID, "GEMM output rows must be 16-byte aligned");
   if (M <= 0) return;
   // tuning override for experiments (DP_GEMM_BN), read once
-  static const int env_bn = getenv("DP_GEMM_BN") ? atoi(getenv("DP_GEMM_BN")) : 0;
-  static const int env_sp = getenv("DP_GEMM_SPLIT") ? atoi(getenv("DP_GEMM_SPLIT")) : 0;
+  static const int env_bn = experiment_env("DP_GEMM_BN", 0);
+  static const int env_sp = experiment_env("DP_GEMM_SPLIT", 0);
   const GemmCfg cfg = pick_cfg(M, N * ngroups, K);
   const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : cfg.bn);
   int sp = env_sp > 0 ? env_sp : (bn_hint > 0 || env_bn > 0 ? 1 : cfg.sp);

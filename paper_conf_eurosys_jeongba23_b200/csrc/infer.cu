@@ -184,6 +184,12 @@ static int64_t compact_layout(const dp_model* m, const int8_t* method, std::vect
   return m->arena_bytes - removed;
 }
 
+// HBM bytes a cold start under `method` holds while resident (the compact layout's size).
+int64_t plan_resident_bytes(const dp_model* m, const int8_t* method) {
+  std::vector<int64_t> doff;
+  return compact_layout(m, method, doff);
+}
+
 void acquire_slots(dp_context* ctx, dp_model* m, int dev, const int8_t* method) {
   DevState& ds = m->dev[dev];
   if (ds.pinned_full) {  // IPC-exported: the peers write into the full arena layout
@@ -289,6 +295,7 @@ extern "C" dp_status dp_context_destroy(dp_context* ctx) {
       if (kv.second.h2d) cudaStreamDestroy(kv.second.h2d);
       if (kv.second.mig) cudaStreamDestroy(kv.second.mig);
       if (kv.second.ring) cudaFree(kv.second.ring);
+      if (kv.second.tail) cudaEventDestroy(kv.second.tail);
     }
     if (!ctx->devs.empty()) {
       DeviceGuard g(ctx->devs[0]);
@@ -308,6 +315,9 @@ extern "C" dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* 
              DP_ERR_INVALID, "gemm_bn must be 0/32/64/128/256");
     DP_CHECK(o->pt_transport == DP_PT_DMA || o->pt_transport == DP_PT_SM || o->pt_transport == DP_PT_CE,
              DP_ERR_INVALID, "pt_transport must be DP_PT_DMA, DP_PT_SM or DP_PT_CE");
+    // measured slower and moved out of the library (tools/experiments)
+    DP_CHECK(!o->fuse_ln && !o->persistent, DP_ERR_UNSUPPORTED,
+             "fuse_ln / persistent: experiments kept in tools/experiments, not built into the library");
     ctx->opts = *o;
   });
 }
@@ -468,7 +478,7 @@ static std::string graph_key(const dp_context* ctx, const DevState& ds, const dp
        std::to_string((uintptr_t)pooled) + "|" + std::to_string(batch) + "x" + std::to_string(seq) + "|" +
        std::to_string(ctx->opts.chunk_bytes) + "," + std::to_string(ctx->opts.n_h2d_streams) + "," +
        std::to_string(ctx->opts.gemm_bn) + "," + std::to_string(ctx->opts.debug_delay_us) + "," +
-       std::to_string(ctx->opts.use_pdl) + "," + std::to_string(ctx->opts.fuse_ln) + "," +
+       std::to_string(ctx->opts.use_pdl) + "," +
        std::to_string(ctx->opts.pt_transport);
   return k;
 }
@@ -705,6 +715,11 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       continue;
     }
     std::vector<cudaEvent_t> fwd_done(pcs.size(), nullptr);
+    {
+      DeviceGuard gs(sdev);
+      if (!r.tail) DP_CUDA(cudaEventCreateWithFlags(&r.tail, cudaEventDisableTiming));
+      if (r.tail_set) DP_CUDA(cudaStreamWaitEvent(r.h2d, r.tail, 0));
+    }
     for (size_t c = 0; c < pcs.size(); ++c) {
       const Piece& p = pcs[c];
       uint8_t* stage = static_cast<uint8_t*>(r.ring) + (c % ring_slots) * slot_bytes;
@@ -733,6 +748,11 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       add_wp(s, p, done);
       if (sdev == primary) trace_piece(p, r.mig);
     }
+    {
+      DeviceGuard gs(sdev);
+      DP_CUDA(cudaEventRecord(r.tail, r.mig));
+      r.tail_set = true;
+    }
   }
 
   // (3) execution stream: wait per unit, then its kernels
@@ -756,7 +776,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   // loses one PDL overlap) per round instead of per unit (a wait costs ~0.6 us in a graph,
   // ~3.6 us as a kernel outside one: tools/wait_cost.py).  On the unit's own link nothing
   // later than its piece is waited for, so one link (k = 1) waits exactly as before.
-  static const bool coalesce = std::getenv("DP_NO_WAIT_COALESCE") == nullptr;  // A/B experiments
+  static const bool coalesce = experiment_env("DP_NO_WAIT_COALESCE", 0) == 0;  // A/B experiments
   constexpr int64_t kWaitSlack = 2 << 20;
   std::vector<int> waited(std::max(1, plan->k), -1);
   std::vector<char> done0(wp[0].size(), 0);
@@ -805,7 +825,6 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     pdl_state().block_next = true;  // the next kernel must see the landed weights: no PDL overlap
   };
   a.pdl = ctx->opts.use_pdl != 0;
-  a.fuse_ln = ctx->opts.fuse_ln != 0;
   if (trace) {  // an event on each side of the unit's dependency wait
     auto gate = a.before_unit;
     a.before_unit = [&, gate](int u) {
@@ -932,15 +951,10 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.stream = (cudaStream_t)stream;
     a.bn_hint = ctx->opts.gemm_bn;
     a.pdl = ctx->opts.use_pdl != 0;
-    a.fuse_ln = ctx->opts.fuse_ln != 0;
-    a.persistent = ctx->opts.persistent != 0;
     // Experiment (tools/wait_cost.py): the cost of a dependency wait before every unit on the
     // execution stream, all already satisfied -- 1: event wait, 2: one-thread acquire-spin
     // kernel on a device word, 3: cuStreamWaitValue32 (stream memory op)
-    static const int dbg_waits = [] {
-      const char* e = std::getenv("DP_DEBUG_WARM_WAITS");
-      return e ? std::atoi(e) : 0;
-    }();
+    static const int dbg_waits = experiment_env("DP_DEBUG_WARM_WAITS", 0);
     static uint32_t* dbg_word = nullptr;
     static cudaStream_t dbg_side = nullptr;
     static cudaEvent_t dbg_fork = nullptr, dbg_ev = nullptr;
@@ -977,7 +991,7 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
       DP_CUDA(cudaEventRecord(dbg_ev, dbg_side));
     };
     if (ctx->opts.use_graph) {
-      std::string key = "warm|" + std::to_string(a.persistent) + "|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
+      std::string key = "warm|" + std::string(reinterpret_cast<const char*>(ds.method.data()), ds.method.size()) +
                         graph_key(ctx, ds, nullptr, nullptr, d_ids, batch, seq, d_out, d_pooled);
       if (dbg_waits) key += "|dbgwait" + std::to_string(dbg_waits);
       dp_run_stats gs = run_graph(ds, key, (cudaStream_t)stream, [&](cudaStream_t cs) {
@@ -1041,6 +1055,11 @@ extern "C" int64_t dp_model_resident_bytes(const dp_model* m, int32_t dev) {
   return m->dev[dev].dbytes;
 }
 
+extern "C" int64_t dp_plan_resident_bytes(const dp_model* m, const dp_plan* plan) {
+  if (!m || !plan || !plan->method || plan->n != (int)m->units.size()) return -1;
+  return plan_resident_bytes(m, plan->method);
+}
+
 extern "C" dp_status dp_pool_stats(dp_context* ctx, int32_t dev, int64_t* reserved, int64_t* in_use) {
   return guard([&] {
     DP_CHECK(ctx && reserved && in_use, DP_ERR_INVALID, "NULL argument");
@@ -1073,7 +1092,6 @@ extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
         cudaDeviceSynchronize();
         for (auto& kv : ds.graphs) cudaGraphExecDestroy(kv.second.exec);
         ds.graphs.clear();
-        ds.persist.clear();
         if (ds.capture) cudaStreamDestroy(ds.capture);
         if (ds.pinned_full) {
           cudaFree(ds.dbase);
@@ -1221,7 +1239,6 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
     fa.stream = s;
     fa.bn_hint = ctx->opts.gemm_bn;
     fa.pdl = ctx->opts.use_pdl != 0;
-    fa.fuse_ln = ctx->opts.fuse_ln != 0;
     // the host enqueues ~100 launches behind a ~1.5 ms spin, so e0..e1 is device time only
     const int64_t chain = timed([&] { run_forward(fa); }, true, 3000000);
     DP_CUDA(cudaStreamSynchronize(s));

@@ -657,7 +657,7 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
   }
   dim3 grid((seq + ATT_BQ - 1) / ATT_BQ, heads, batch);
   const float scale_log2 = 1.4426950408889634f / sqrtf((float)ATT_D);
-  static const int env_att = getenv("DP_ATT_GROUPS") ? atoi(getenv("DP_ATT_GROUPS")) : 0;  // experiments
+  static const int env_att = experiment_env("DP_ATT_GROUPS", 0);  // experiments
   // >= 3 key tiles: 2 or 4 key-tile groups per query tile (K5b).  At 2 tiles (BERT-Base
   // S = 128) the merge and the larger footprint cost more than the shorter chain saves (warm
   // forward 0.480 vs 0.472 ms); with 2 groups BERT-Large S = 384 1.78 -> 1.58 ms, GPT-2 Medium
@@ -672,7 +672,7 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
                                    smem));
     }
     const dim3 g2(heads, grid.x, batch);
-    static const int env_lpt = getenv("DP_ATT_LPT") ? atoi(getenv("DP_ATT_LPT")) : 1;  // experiments
+    static const int env_lpt = experiment_env("DP_ATT_LPT", 1);  // experiments
     const int cmode = causal ? (env_lpt ? 2 : 1) : 0;  // 2: causal, longest query tiles first
     if (dtype == DP_BF16)
       launch_kernel(attention2_kernel<__nv_bfloat16, G>, g2, dim3(128 * G), smem, s, (const __nv_bfloat16*)qkv,

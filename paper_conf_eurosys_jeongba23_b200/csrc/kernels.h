@@ -31,13 +31,6 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
 
 // K2: resident tcgen05/TMA GEMM -- a12.  W must be device memory.
 struct GemmPlan;  // cached tensor map for a weight
-// K2+K4 fused (gemm_ln.cu): out = LN(x . W^T + b + res) over complete rows of N <= 1024 via
-// a thread-block cluster along N; y (optional) receives the pre-LN sum (io bit 1: fp32),
-// out32 (optional) an fp32 copy of out.
-bool gemm_ln_supported(int N);
-void launch_gemm_ln(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
-                    void* y, int ldy, int M, int N, int K, int io, const void* gamma, const void* beta, float eps,
-                    void* out, int ldo, void* out32, cudaStream_t s);
 bool gemm_tc_supported(int N, int K);
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
                     void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);

@@ -53,7 +53,6 @@ struct Workspace {
   void* base = nullptr;
 };
 
-struct PersistProgram;  // K6 (persist.h)
 
 struct GraphEntry {
   cudaGraphExec_t exec = nullptr;
@@ -92,8 +91,6 @@ struct DevState {
   std::map<std::string, GraphEntry> graphs;  // captured cold / warm runs (opts.use_graph)
   UnitTrace trace;                           // last traced cold start
   cudaStream_t capture = nullptr;            // private stream the graphs are captured on
-  // K6 programs per (batch, seq, workspace): their tensor maps point into dbase and ws
-  std::map<std::string, std::shared_ptr<PersistProgram>> persist;
 };
 
 std::vector<ParamDesc> config_params(const dp_model_config& c);

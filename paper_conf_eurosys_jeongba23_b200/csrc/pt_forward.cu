@@ -168,10 +168,7 @@ void launch_pt_forward(const void* src, void* dst, int64_t bytes, cudaStream_t s
   DP_CUDA(cudaGetDevice(&dev));
   const long long per_cta = (long long)kFwdThreads * kFwdUnroll;
   const long long want = std::max<long long>(1, (n16 + per_cta - 1) / per_cta);
-  static const int cta_cap = [] {  // experiments: DP_PT_FWD_CTAS overrides the grid cap
-    const char* e = std::getenv("DP_PT_FWD_CTAS");
-    return e ? std::max(1, std::atoi(e)) : 0;
-  }();
+  static const int cta_cap = std::max(0, experiment_env("DP_PT_FWD_CTAS", 0));  // experiments: grid cap
   const int grid = (int)std::min<long long>(want, cta_cap ? cta_cap : 2LL * sm_count(dev));
   pt_forward_kernel<<<grid, kFwdThreads, 0, s>>>(static_cast<const uint4*>(src), static_cast<uint4*>(dst), n16,
                                                 static_cast<const uint8_t*>(src) + n16 * 16,

@@ -10,8 +10,8 @@
 //     lowest index), evicting LRU instances there until its resident bytes fit the budget;
 //   * start = max(arrival, GPU free time); finish = start + latency; the GPU's LRU list is
 //     touched.  PT borrows other GPUs' PCIe links, not their compute (Table 4).
-// dry_run = 1 replays with a latency table; the live mode executes the same decisions on
-// the GPUs with real cold/warm inferences (serve_live.cu).
+// dry_run = 1 replays with a latency table; the live mode (serve_live.cu) is an online
+// dispatcher on the GPUs' observed state with real cold / warm inferences and evictions.
 #include <algorithm>
 #include <list>
 #include <vector>
@@ -65,6 +65,7 @@ void serve_decide(const dp_serve_opts& o, const dp_trace_event* trace, int nreq,
     res.gpu = g;
     res.start_ns = std::max(trace[r].arrival_ns, busy[g]);
     res.finish_ns = res.start_ns + (res.cold ? o.cold_ns[model] : o.warm_ns[model]);
+    res.decide_ns = trace[r].arrival_ns;
     busy[g] = res.finish_ns;
   }
   (void)order_lat;
@@ -79,8 +80,10 @@ extern "C" dp_status dp_serve_run(dp_context* ctx, dp_model* const* models, int3
   return guard([&] {
     DP_CHECK(opts && (nreq == 0 || (trace && out)), DP_ERR_INVALID, "NULL argument");
     DP_CHECK(nreq >= 0, DP_ERR_INVALID, "nreq < 0");
-    serve_decide(*opts, trace, nreq, out, nullptr);
-    if (opts->dry_run) return;
+    if (opts->dry_run) {
+      serve_decide(*opts, trace, nreq, out, nullptr);
+      return;
+    }
     serve_live(ctx, models, nmodels, trace, nreq, *opts, out);
   });
 }

@@ -82,8 +82,7 @@ def test_attention_and_skinny_deterministic_under_contention(S, H, heads, causal
 
 
 @pytest.mark.parametrize("name,S,opts", [("bert_base", 128, {}), ("bert_large", 384, {}), ("gpt2", 256, {}),
-                                         ("bert_base", 128, {"fuse_ln": True}),
-                                         ("bert_base", 128, {"persistent": True})])
+                                         ("bert_base", 128, {"use_pdl": 0})])
 def test_warm_forward_deterministic_under_contention(name, S, opts, noise):
     """The whole warm forward (every kernel of the chain, PDL overlap included) beside the
     noise kernel: bit-identical to the quiet run, 40 times."""

@@ -56,14 +56,24 @@ def fake_cost(m, dtype, seed=0):
             "exe_dha_ns": np.maximum(dha, 0)}
 
 
-def tolerance(dtype, recipe, ref):
-    """DESIGN.md §6.  fp16, paper recipe: the north_star's max-abs 1e-2.  bf16 keeps 8
-    mantissa bits, so rounding the output ALONE errs by up to 2^-9 |ref| (0.008 at |ref| = 4):
-    an absolute 1e-2 is below its representation error; we allow 8 half-ulps, 2^-5 max(1,|ref|).
-    The "scaled" recipe (O(1) contributions from every sub-block) carries more rounding into
-    the residual stream: 3x those bounds."""
-    base = np.full_like(ref, 1e-2) if dtype == "fp16" else 2.0 ** -5 * np.maximum(1.0, np.abs(ref))
-    return base if recipe == "paper" else 3 * base
+def tolerance(dtype, recipe, ref, rep=0.0):
+    """DESIGN.md §6 / R15.  fp16, paper recipe: the north_star's max-abs 1e-2.  bf16: storing the
+    activations in bf16 (8 significand bits) errs by itself by more than 1e-2 on deep models, so
+    the north star's 1e-2 is granted on top of that representation error `rep` -- max |exact
+    oracle - oracle with bf16 activation roundings| (oracle.forward act_round), computed for the
+    same weights and ids.  The "scaled" recipe (O(1) contributions from every sub-block) carries
+    more rounding into the residual stream: 3x the 1e-2."""
+    base = 1e-2 if recipe == "paper" else 3e-2
+    return np.full_like(ref, base + (rep if dtype == "bf16" else 0.0))
+
+
+def rep_error(m, w, ids, dtype, ref, ref_pool):
+    """bf16 representation error of the activations (0 for fp16) for the output and the pooler."""
+    if dtype != "bf16":
+        return 0.0, 0.0
+    e, ep = F.forward(m, w, ids, dtype, act_round=dtype)
+    return float(np.abs(e.reshape(ref.shape) - ref).max()), \
+        (float(np.abs(ep - ref_pool).max()) if ref_pool is not None else 0.0)
 
 
 def run_cold(model, plan, ids_np, dtype, secondaries=(), pooled=True):
@@ -95,7 +105,8 @@ def test_all_modes_match_oracle(name, B, S, dtype, recipe):
     ref = ref.reshape(B * S, m.hidden)
     model = dp().Model(ctx(), m, w, dtype)
     cost = fake_cost(m, dtype)
-    tol = tolerance(dtype, recipe, ref)
+    rep, rep_pool = rep_error(m, w, ids, dtype, ref, ref_pool)
+    tol = tolerance(dtype, recipe, ref, rep)
     outs = {}
     for mode in ("BASELINE", "PIPESWITCH", "GREEDY", "DHA", "PT", "PT_DHA", "DHA_LINK", "PT_DHA_LINK", "PT_DHA_BAL",
                  "PT_DHA_LINK_BAL", "PT_DHA_STRIPE", "PT_DHA_LINK_STRIPE"):
@@ -106,7 +117,7 @@ def test_all_modes_match_oracle(name, B, S, dtype, recipe):
         err = np.abs(f64(out) - ref)
         assert np.all(err <= tol), (mode, err.max())
         if pool is not None:
-            assert np.all(np.abs(f64(pool) - ref_pool) <= tolerance(dtype, recipe, ref_pool))
+            assert np.all(np.abs(f64(pool) - ref_pool) <= tolerance(dtype, recipe, ref_pool, rep_pool))
         # transferred bytes per link = the oracle simulator's, bit-exactly
         om, osl, ser = OP.plan(cost, mode, k)
         assert list(plan.method) == om and list(plan.slot) == osl
@@ -260,42 +271,6 @@ def test_graph_replay_matches_eager(name, mode, k):
         torch.cuda.synchronize()
         assert torch.equal(w_out, eager)
         model.evict(0)
-    model.close()
-    c.close()
-
-
-@pytest.mark.parametrize("name,B,S", [("tiny_bert", 1, 77), ("tiny_gpt2", 1, 70), ("bert_base", 1, 128),
-                                      ("gpt2", 1, 200), ("tiny_roberta", 3, 50), ("bert_large", 1, 96)])
-@pytest.mark.parametrize("dtype", ["fp16", "bf16"])
-def test_fused_layernorm(name, B, S, dtype):
-    """A LayerNorm that follows a resident-weight linear runs in that GEMM's epilogue (K2+K4,
-    gemm_ln.cu: a cluster along N exchanges per-token statistics over DSMEM).  The fused forward
-    matches the oracle within the north_star tolerance, stays close to the unfused one (same
-    math, another summation order), is deterministic (eager == graph replay, bit for bit), and
-    launches 2 fewer kernels per layer."""
-    m = synth.SHAPES[name]
-    w = synth.make_weights(m, seed=21, dtype=dtype)
-    ids = synth.make_ids(m, B, S, seed=22)
-    ref, ref_pool = F.forward(m, w, ids, dtype)
-    ref = ref.reshape(B * S, -1)
-    c = dp().Context([0])
-    model = dp().Model(c, m, w, dtype)
-    plan = dp().plan_generate(fake_cost(m, dtype), "PIPESWITCH", 1)  # all loaded: every linear on the GEMM
-    outs, kern = [], []
-    for fuse, graph in ((False, 0), (True, 0), (True, 1)):
-        c.set_opts(fuse_ln=fuse, use_graph=graph)
-        o, p, st = run_cold(model, plan, ids, dtype)
-        outs.append((o.clone(), None if p is None else p.clone()))
-        kern.append(st["n_kernels"])
-        model.evict(0)
-    tol = tolerance(dtype, "paper", ref)
-    for o, p in outs:
-        assert np.all(np.abs(f64(o) - ref) <= tol)
-        if p is not None:
-            assert np.all(np.abs(f64(p) - ref_pool) <= tolerance(dtype, "paper", ref_pool))
-    assert np.abs(f64(outs[1][0]) - f64(outs[0][0])).max() <= tol.max()
-    assert torch.equal(outs[1][0], outs[2][0])  # deterministic
-    assert kern[1] == kern[0] - 2 * m.layers
     model.close()
     c.close()
 

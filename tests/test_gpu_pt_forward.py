@@ -255,12 +255,16 @@ def test_sm_transport_across_processes(name, mode, S, delay, transport, graph):
 @pytest.mark.parametrize("transport", ["sm", "ce"])
 def test_one_hop_transports_bf16_striped(name, S, transport):
     """bf16 storage, the striped plan (R22) over 4 loopback links: one-hop transports equal the
-    DMA path bit for bit and stay within the bf16 tolerance (R15) of the oracle."""
+    DMA path bit for bit and stay within the bf16 tolerance (R15) of the oracle: 1e-2 of
+    the oracle that stores activations in bf16 where the kernels must, 1e-2 + that representation
+    error of the exact oracle."""
     m = synth.SHAPES[name]
     dtype = "bf16"
     w = synth.make_weights(m, seed=61, dtype=dtype)
     ids = synth.make_ids(m, 1, S, seed=62)
     ref, _ = F.forward(m, w, ids, dtype)
+    emul, _ = F.forward(m, w, ids, dtype, act_round=dtype)  # bf16 representation error (R15)
+    rep = float(np.abs(emul - ref).max())
     c = dp().Context([0])
     model = dp().Model(c, m, w, dtype)
     plan = dp().plan_generate(fake_cost(m, dtype, seed=9), "PT_DHA_LINK_STRIPE", 4)
@@ -270,7 +274,8 @@ def test_one_hop_transports_bf16_striped(name, S, transport):
     b, _, sb = _run(model, plan, ids, dtype, 4)
     assert torch.equal(a, b)
     r = ref.reshape(S, -1)
-    assert np.all(np.abs(f64(b) - r) <= 2.0 ** -5 * np.maximum(1.0, np.abs(r)))
+    assert np.abs(f64(b) - emul.reshape(S, -1)).max() <= 1e-2
+    assert np.abs(f64(b) - r).max() <= 1e-2 + rep
     assert sa["h2d_bytes"] == sb["h2d_bytes"] and sa["nvlink_bytes"] == sb["nvlink_bytes"]
     model.close()
     c.close()

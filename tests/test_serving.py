@@ -95,3 +95,20 @@ def test_dry_run_matches_oracle_maf_like(seed):
     ref = OS.replay(arr, inst, **kw)
     for k in ref:
         assert np.array_equal(got[k], ref[k]), k
+
+
+def test_online_replay_hand_cases():
+    """R11-live on hand-checkable observations (the live dispatcher's decide / finish stamps)."""
+    # one GPU, budget for one instance: A cold; B arrives while A still runs -> A has work, so it
+    # cannot be evicted: B goes over budget; C arrives after both finished -> evicts A and B (LRU)
+    r = OS.replay_online([0, 1, 50], [0, 1, 2], ngpu=1, per_gpu_budget_bytes=10, resident_bytes=[10, 10, 10],
+                         decide_ns=[0, 1, 50], finish_ns=[20, 40, 60])
+    assert list(r["cold"]) == [1, 1, 1] and list(r["nevicted"]) == [0, 0, 2]
+    # two GPUs: the second cold request goes to the GPU with fewer outstanding requests
+    r = OS.replay_online([0, 1, 2, 100], [0, 1, 2, 0], ngpu=2, per_gpu_budget_bytes=100,
+                         resident_bytes=[10, 10, 10], decide_ns=[0, 1, 2, 100], finish_ns=[50, 2, 60, 110])
+    assert list(r["gpu"]) == [0, 1, 1, 0] and list(r["cold"]) == [1, 1, 1, 0]
+    # a completion observed exactly at the decision time counts as complete
+    r = OS.replay_online([0, 5], [0, 1], ngpu=2, per_gpu_budget_bytes=100, resident_bytes=[1, 1],
+                         decide_ns=[0, 5], finish_ns=[5, 9])
+    assert list(r["gpu"]) == [0, 0]

@@ -4,8 +4,10 @@ Instances are clones of registered base models (same shapes, shared pinned arena
 residency), mixed by ratio (BERT-Base : RoBERTa-Base : GPT-2 = 4:4:1).  Each plan mode
 (PIPESWITCH = all loaded, DHA = Algorithm 1, DHA_LINK, PT_DHA* with several GPUs) gets its
 measured cold / warm latency and resident bytes per model (DHA units stay in host memory,
-P:332); a seeded Poisson trace is replayed live through dp_serve_run with one request
-per GPU at a time and LRU eviction under a per-GPU budget.  Reports p99, goodput at the SLO,
+P:332); a seeded Poisson trace is served live through dp_serve_run -- the online
+dispatcher (one request per GPU at a time, real LRU evictions under a per-GPU budget, PT
+secondaries borrowed from idle GPUs) -- beside the dry-run replay with the measured latency
+table (tests/test_gpu_serving.py checks the live decisions against the oracle's re-derivation).  Reports p99, goodput at the SLO,
 the cold-start rate and throughput, beside the dry-run replay of the same decisions.
 
 python tools/serve_bench.py [--gpus 1] [--mix bert_base:128:1] [--instances 40] [--fit 8]
@@ -92,13 +94,14 @@ def main():
             warm.append(int(dev_ms(lambda: base.infer_warm(0, ids, out, pool)) * 1e6))
             base.evict(0)
             plans.append(plan)
-            resident.append(int(sum(b for b, mt in zip(base.unit_bytes(), plan.method) if mt == dp.LOAD)))
+            resident.append(dp.plan_resident_bytes(base, plan))  # the compact slot block (loaded units)
         kw = dict(ngpu=a.gpus, per_gpu_budget_bytes=budget, cold_ns=cold, warm_ns=warm, resident_bytes=resident,
                   model_of_instance=moi, slo_ns=int(a.slo_ms * 1e6), batch=1,
                   seq=max(s for _, s, _ in mix), seq_of_model=[s for _, s, _ in mix])
         dry = dp.serve_run(arr, inst, dry_run=True, **kw)
         live = dp.serve_run(arr, inst, dry_run=False, ctx=ctx, models=insts,
                             plans=[plans[moi[i]] for i in range(a.instances)], **kw)
+
         for i in insts + bases:
             for g in range(a.gpus):
                 if i.is_resident(g):
@@ -122,7 +125,8 @@ def main():
             "per_model": {mix[mi][0]: {"cold_ms": cold[mi] / 1e6, "warm_ms": warm[mi] / 1e6,
                                        "resident_mb": round(resident[mi] / 2 ** 20, 1),
                                        "dha_units": int(plans[mi].method.sum())} for mi in range(len(mix))},
-            "live": summarize(live, timeline=True), "replay": summarize(dry)}
+            "live": summarize(live, timeline=True), "replay": summarize(dry),
+            "pt_cold_starts_with_secondaries": int(np.sum((live["cold"] == 1) & (live["sec_mask"] != 0)))}
     print(json.dumps(report))
 
 

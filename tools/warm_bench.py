@@ -1,5 +1,4 @@
-"""Warm-forward latency (all units resident): per-kernel path, with the cluster-fused GEMM+LN, and
-the K6 persistent kernel, CUDA
+"""Warm-forward latency (all units resident) of the per-kernel PDL-chained path, CUDA
 graph replay, CUDA events on the launching stream, median of N after warm-up; L2 flushed
 between runs (256 MiB write) unless DP_NO_FLUSH=1.
 
@@ -36,8 +35,8 @@ for spec in specs:
     model.infer_cold(plan, 0, ids, out, pool)
     torch.cuda.synchronize()
     ref = out.clone()
-    for path, pers, fuse in (("per_kernel", False, False), ("fused_ln", False, True), ("persistent", True, False)):
-        ctx.set_opts(use_graph=True, persistent=pers, fuse_ln=fuse)
+    for path in ("per_kernel",):  # (the fused-LN and K6 persistent paths: tools/experiments)
+        ctx.set_opts(use_graph=True)
         s = torch.cuda.current_stream()
         ts = []
         for i in range(N + 5):
