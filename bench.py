@@ -373,6 +373,27 @@ def main():
     links_info = {"h2d_solo_gbs": [round(x, 2) for x in solo], "h2d_concurrent_gbs": [round(x, 2) for x in conc],
                   "h2d_aggregate_gbs": round(float(sum(conc)), 2), "nvlink_gbs": NVLINK_GBS if world > 1 else None,
                   "nvlink_source": "B200_PROFILING.md measured peer copy per direction" if world > 1 else None}
+    if dist_on:
+        # pairwise concurrency matrix (rank i's rate while rank j copies) -> which rank carries
+        # which PT slot (dp_select_secondaries, R25), instead of (primary + s) mod N
+        pair = np.array([[s_ for s_ in solo] for _ in range(world)], dtype=np.float64)
+        for i in range(world):
+            for j in range(i + 1, world):
+                torch.cuda.synchronize()
+                dist.barrier()
+                r_ = dp.measure_h2d(local, 64 << 20, 4) if rank in (i, j) else 0.0
+                got = [None] * world
+                dist.all_gather_object(got, r_)
+                pair[i][j], pair[j][i] = got[i], got[j]
+        numa = [None] * world
+        dist.all_gather_object(numa, dp.device_numa_node(local))
+        sec = dp.select_secondaries(solo, pair, 0, world, numa) if rank == 0 else None
+        box = [sec]
+        dist.broadcast_object_list(box, src=0)
+        sec = box[0]
+        ctx.set_slot_ranks(0, sec)
+        links_info.update({"pair_gbs": [[round(x, 2) for x in row] for row in pair], "numa_node": numa,
+                           "slot_ranks": sec})
 
     # profile on the primary, plan, share the plan (the plan never names GPUs)
     # default plan: Algorithm 1 on the link-aware model (R19); the paper's own

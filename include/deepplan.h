@@ -222,6 +222,34 @@ dp_status dp_peer_init(dp_context* ctx, const void* uid128, int32_t rank, int32_
  * primary.  DP_ERR_STATE if already initialised. */
 dp_status dp_peer_init_ipc(dp_context* ctx, int32_t rank, int32_t nranks);
 
+/* Which rank carries each PT slot when `primary` serves (after dp_peer_init[_ipc]; every rank
+ * must set the same map): rank_of_slot[s-1] for s = 1..k-1, distinct and != primary.  Without a
+ * map slot s is carried by rank (primary + s) mod nranks.  DP_ERR_INVALID on a bad map. */
+dp_status dp_peer_set_slot_ranks(dp_context* ctx, int32_t primary, const int32_t* rank_of_slot, int32_t k);
+
+/* ---------------------------------------------------------------------------------
+ * Host-link topology (P:148 PCIe-switch contention, P:186 / P:227-229 "GPUs
+ * attached to different PCIe switches")
+ * --------------------------------------------------------------------------------- */
+/* NUMA node of a device's PCI function (sysfs), -1 if unknown. */
+int32_t dp_device_numa_node(int32_t dev);
+/* NUMA node of the page holding host address p (move_pages), -1 if unknown. */
+int32_t dp_host_numa_node(const void* p);
+/* Pinned, mapped, portable host memory placed on NUMA node `node` (< 0: no placement): allocated
+ * and first-touched by a thread bound to the node's CPUs.  Free with dp_host_free. */
+dp_status dp_host_alloc_node(int64_t bytes, int32_t node, void** out);
+/* All n devices copy `bytes` host -> device at the same time (each from pinned memory on its own
+ * NUMA node), reps times after a warm-up; gbs[i] = device i's median GB/s.  n = 1: the solo rate;
+ * n = 2 over (i, j): one entry of the pairwise concurrency matrix. */
+dp_status dp_measure_h2d_concurrent(const int32_t* devs, int32_t n, int64_t bytes, int32_t reps, double* gbs);
+/* Secondaries for a PT cold start of `primary` over k links, from measured link rates: solo_gbs[n]
+ * and pair_gbs[n*n] (device i's rate while j copies concurrently), numa[n] nullable.  Greedy
+ * (R25): repeatedly add the GPU that keeps the slowest pairwise-concurrent link of the
+ * set fastest; ties -> the primary's NUMA node, then the faster solo link, then the lower index.
+ * out: k-1 device indices in slot order.  Pure host code. */
+dp_status dp_select_secondaries(const double* solo_gbs, const double* pair_gbs, const int32_t* numa, int32_t n,
+                                int32_t primary, int32_t k, int32_t* out);
+
 /* CUDA IPC exchange for the SM forwarder across processes.  dp_peer_ipc_export allocates
  * (once) this rank's HBM slots for `m` and its 16 KiB mailbox (a go word the primary
  * releases at the start of a cold start, and one done word per (slot, piece) the secondaries

@@ -413,3 +413,34 @@ def exhaustive(cost, k: int = 1, free=None, base_method=None, chunk: int = 1 << 
     for b, u in enumerate(free):
         method[u] = (best_idx >> (m - 1 - b)) & 1
     return best_lat, [int(x) for x in method], slot
+
+
+# ---------------------------------------------------------------------------------------
+# Secondary selection for PT (R25; "utilize GPUs attached to
+# different PCIe switches").  Not an algorithm of the paper -- the paper only says to prefer GPUs
+# on other switches; this is the greedy reading on measured link rates.
+# ---------------------------------------------------------------------------------------
+
+def select_secondaries(solo, pair, primary: int, k: int, numa=None) -> list:
+    """solo[i]: device i's H2D GB/s alone; pair[i][j]: device i's GB/s while j copies at the same
+    time.  Start from {primary}; k-1 times add the device c whose worst concurrent link with the
+    set, min over s in the set of min(pair[c][s], pair[s][c]) (capped by solo[c]), is largest.
+    Ties: same NUMA node as the primary first, then higher solo rate, then lower index."""
+    n = len(solo)
+    chosen = [primary]
+    out = []
+    for _ in range(k - 1):
+        best_key, best = None, None
+        for c in range(n):
+            if c in chosen:
+                continue
+            worst = solo[c]
+            for s in chosen:
+                worst = min(worst, pair[c][s], pair[s][c])
+            same_node = numa is not None and numa[c] == numa[primary]
+            key = (worst, same_node, solo[c], -c)  # larger is better
+            if best_key is None or key > best_key:
+                best_key, best = key, c
+        chosen.append(best)
+        out.append(best)
+    return out

@@ -120,6 +120,13 @@ _sig("dp_context_get_opts", [vp, C.POINTER(EngineOpts)])
 _sig("dp_peer_unique_id", [vp])
 _sig("dp_peer_init", [vp, vp, C.c_int32, C.c_int32])
 _sig("dp_peer_init_ipc", [vp, C.c_int32, C.c_int32])
+_sig("dp_peer_set_slot_ranks", [vp, C.c_int32, i32p, C.c_int32])
+_sig("dp_device_numa_node", [C.c_int32])
+_sig("dp_host_numa_node", [vp])
+_sig("dp_host_alloc_node", [C.c_int64, C.c_int32, C.POINTER(vp)])
+_sig("dp_measure_h2d_concurrent", [i32p, C.c_int32, C.c_int64, C.c_int32, C.POINTER(C.c_double)])
+_sig("dp_select_secondaries", [C.POINTER(C.c_double), C.POINTER(C.c_double), i32p, C.c_int32, C.c_int32,
+                               C.c_int32, i32p])
 _sig("dp_peer_ipc_export", [vp, vp, vp])
 _sig("dp_peer_ipc_import", [vp, vp, vp])
 _sig("dp_pt_forward", [vp, vp, C.c_int64, vp])
@@ -336,6 +343,11 @@ class Context:
         """Multi-process PT without NCCL (SM forwarder over CUDA IPC)."""
         _check(lib.dp_peer_init_ipc(self.h, int(rank), int(nranks)))
 
+    def set_slot_ranks(self, primary: int, ranks):
+        """PT slot s (1..k-1) of `primary`'s cold starts is carried by ranks[s-1]."""
+        arr = np.ascontiguousarray(list(ranks) or [0], dtype=np.int32)
+        _check(lib.dp_peer_set_slot_ranks(self.h, int(primary), _ptr(arr, i32p), len(ranks) + 1))
+
     def close(self):
         if self.h:
             _check(lib.dp_context_destroy(self.h))
@@ -530,6 +542,42 @@ def measure_h2d(dev: int, nbytes: int = 256 << 20, reps: int = 5) -> float:
     g = C.c_double()
     _check(lib.dp_measure_h2d(int(dev), int(nbytes), int(reps), C.byref(g)))
     return float(g.value)
+
+
+def device_numa_node(dev: int) -> int:
+    return int(lib.dp_device_numa_node(int(dev)))
+
+
+def host_numa_node(p) -> int:
+    return int(lib.dp_host_numa_node(_dptr(p)))
+
+
+def host_alloc_node(nbytes: int, node: int) -> int:
+    p = vp()
+    _check(lib.dp_host_alloc_node(int(nbytes), int(node), C.byref(p)))
+    return p.value
+
+
+def measure_h2d_concurrent(devs, nbytes: int = 256 << 20, reps: int = 5) -> list:
+    """Per-device GB/s when all `devs` copy host -> device at the same time."""
+    d = np.ascontiguousarray(devs, dtype=np.int32)
+    out = (C.c_double * len(d))()
+    _check(lib.dp_measure_h2d_concurrent(_ptr(d, i32p), len(d), int(nbytes), int(reps), out))
+    return [float(x) for x in out]
+
+
+def select_secondaries(solo_gbs, pair_gbs, primary: int, k: int, numa=None) -> list:
+    """dp_select_secondaries: k-1 secondaries for `primary` from measured link rates."""
+    solo = np.ascontiguousarray(solo_gbs, dtype=np.float64)
+    pair = np.ascontiguousarray(pair_gbs, dtype=np.float64)
+    n = len(solo)
+    nm = None if numa is None else np.ascontiguousarray(numa, dtype=np.int32)
+    out = np.zeros(max(1, k - 1), dtype=np.int32)
+    _check(lib.dp_select_secondaries(solo.ctypes.data_as(C.POINTER(C.c_double)),
+                                     pair.ctypes.data_as(C.POINTER(C.c_double)),
+                                     None if nm is None else _ptr(nm, i32p), n, int(primary), int(k),
+                                     _ptr(out, i32p)))
+    return [int(x) for x in out[:k - 1]]
 
 
 def pt_forward(src, dst, nbytes: int, stream=None):

@@ -21,6 +21,16 @@ extern "C" dp_status dp_host_free(void* p) {
   });
 }
 
+static bool is_host_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return true;  // unregistered host memory
+  }
+  return at.type == cudaMemoryTypeHost || at.type == cudaMemoryTypeUnregistered;
+}
+
 static void check_dtype(int32_t dtype) {
   DP_CHECK(dtype == DP_FP16 || dtype == DP_BF16 || dtype == DP_FP32, DP_ERR_UNSUPPORTED,
            "dtype must be DP_FP16, DP_BF16 or DP_FP32");
@@ -34,7 +44,7 @@ extern "C" dp_status dp_embed(const int32_t* d_ids, int32_t ntok, int32_t seq, i
     DP_CHECK(d_ids && word && pos && d_out, DP_ERR_INVALID, "NULL pointer");
     DP_CHECK((ln_g == nullptr) == (ln_b == nullptr), DP_ERR_INVALID, "ln_g and ln_b must both be set or NULL");
     launch_embed(dtype, d_ids, ntok, seq, pos_offset, word, pos, type, ln_g, ln_b, hidden, (float)eps, d_out,
-                 out_f32 != 0, (cudaStream_t)stream);
+                 out_f32 != 0, (cudaStream_t)stream, nullptr, 0, is_host_ptr(type) || is_host_ptr(ln_g));
   });
 }
 
@@ -66,7 +76,8 @@ extern "C" dp_status dp_layernorm(const void* x, const void* r, const void* g, c
   return guard([&] {
     check_dtype(dtype);
     DP_CHECK(x && g && b && y && rows >= 0, DP_ERR_INVALID, "bad arguments");
-    launch_layernorm(dtype, x, r, g, b, y, rows, n, (float)eps, x_f32 != 0, (cudaStream_t)stream);
+    launch_layernorm(dtype, x, r, g, b, y, rows, n, (float)eps, x_f32 != 0, (cudaStream_t)stream, nullptr,
+                     is_host_ptr(g));
   });
 }
 

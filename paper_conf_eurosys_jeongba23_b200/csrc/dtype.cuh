@@ -100,6 +100,36 @@ __device__ __forceinline__ void store1(void* base, size_t i, float v, int f32) {
     static_cast<T*>(base)[i] = Cvt<T>::from1(v);
 }
 
+// Thread-block clusters: this CTA's rank, and the broadcast of rank 0's shared-memory buffer to
+// every rank (DSMEM reads between two cluster barriers).  Used so that rows every CTA needs (LN
+// gamma / beta, the token-type row) cross the host link ONCE per cluster when they live in host
+// memory (DHA), instead of once per CTA.
+__device__ __forceinline__ uint32_t cta_cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+
+__device__ __forceinline__ void cluster_bcast_from_rank0(uint4* buf, int n16) {
+  // (1) rank 0's buffer is written and visible cluster-wide
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+  if (cta_cluster_rank() != 0) {
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(buf));
+    uint32_t remote;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(remote) : "r"(base));
+    for (int i = threadIdx.x; i < n16; i += blockDim.x) {
+      uint4 v;
+      asm volatile("ld.shared::cluster.v4.u32 {%0, %1, %2, %3}, [%4];"
+                   : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                   : "r"(remote + 16u * i)
+                   : "memory");
+      buf[i] = v;
+    }
+  }
+  // (2) every rank has its copy (rank 0 may exit; this CTA's copy is visible to its threads)
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 __device__ __forceinline__ float warp_sum(float v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);

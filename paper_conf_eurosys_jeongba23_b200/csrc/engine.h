@@ -104,6 +104,8 @@ struct dp_context {
   uint32_t* peer_mailbox[DP_MAX_DEVICES] = {};     // other ranks' (IPC-mapped), by rank
   uint32_t pt_epoch = 0;                          // cold starts run in SM/IPC mode so far
   uint64_t ring_gen = 0;  // bumped whenever a staging ring is reallocated (part of graph keys)
+  int slot_map_primary = -1;              // dp_peer_set_slot_ranks: the primary the map is for
+  int slot_rank[DP_MAX_DEVICES] = {-1, -1, -1, -1, -1, -1, -1, -1};  // slot s -> rank
   bool multiproc() const { return nranks > 0; }
   dp::DevCtx& on(int dev);
 };

@@ -7,7 +7,7 @@
 // and wide in N (768..4096), so the kernel is "swap-AB": the MMA's M axis (128 lanes of
 // TMEM) runs over W's rows (N) and the MMA's N axis over tokens (BN = 32..256 columns).
 //
-// Per CTA (128 threads, one 128 x BN output tile, a K range):
+// Per CTA (256 threads, one 128 x BN output tile, a K range):
 //   warp 0 / lane 0  : TMA producer -- W tile [128 x 64] and X tile [BN x 64] per stage,
 //                      both K-major with the 128-byte swizzle, into a STAGES-deep ring; the
 //                      first ring of W tiles is issued BEFORE the grid-dependency wait (PDL):
@@ -15,8 +15,10 @@
 //   warp 1 / lane 0  : MMA issuer  -- 4 x tcgen05.mma (K = 16 each) per stage, fp32
 //                      accumulator in TMEM; tcgen05.commit releases the smem stage;
 //   warp 1           : TMEM allocate / free (BN columns);
-//   all 4 warps      : epilogue -- tcgen05.ld 32 lanes x 16 columns into a shared-memory
-//                      fp32 tile, then + bias, activation, + residual and 16-byte stores.
+//   all 8 warps      : epilogue -- tcgen05.ld 32 lanes x 16 columns (warp w: lane quarter w%4,
+//                      column half w/4) into a shared-memory fp32 tile, then + bias,
+//                      activation, + residual and 16-byte stores (8 warps: the epilogue is
+//                      latency-bound, 39% of a 1024-token tile with 4 warps).
 // blockIdx.z selects one of up to 3 weight matrices sharing X (BERT q/k/v in one launch).
 // Explored and measured slower on B200 (profiles/r01_gemm_sweep_v1.txt): split-K over a
 // thread-block cluster with a DSMEM reduction (cluster-barrier waits dominated).
@@ -90,6 +92,7 @@ CUtensorMap make_plain_map(const void* base, CUtensorMapDataType dt, int rank, c
 namespace {
 
 constexpr int BM = 128;  // W rows per tile (MMA M)
+constexpr int NT = 256;  // threads per CTA: warp 0 TMA, warp 1 MMA + TMEM, all 8 warps the epilogue
 constexpr int BK = 64;   // K per stage: 64 x 2 B = one 128-byte swizzle row
 
 // Ring depth per tile width: as many stages as ~224 KB of shared memory holds (<= 12), so a
@@ -149,7 +152,7 @@ __device__ __forceinline__ float ld_cluster_f32(uint32_t addr) {
 // 128-token shapes a CTA's time is set by the bytes it ingests (~100 GB/s per SM measured,
 // profiles/r01_gemm_trace.jsonl), so spreading a weight tile over `splits` SMs pays.
 template <class T, int BN, int ACT>
-__global__ void __launch_bounds__(128, 1)
+__global__ void __launch_bounds__(NT, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
                    const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io, int splits,
                    int nst) {
@@ -159,7 +162,7 @@ __global__ void __launch_bounds__(128, 1)
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
   constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free TMEM->smem writes)
-  constexpr int RP = BN <= 64 ? BN / 8 : 0;  // residual rows prefetched per thread (single split)
+  constexpr int RP = BN <= 64 ? BN / (NT / 16) : 0;  // residual rows prefetched per thread (single split)
   // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
   constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
                              (uint32_t(BM >> 4) << 24);
@@ -223,19 +226,19 @@ __global__ void __launch_bounds__(128, 1)
   const int pre = num_kb < nst ? num_kb : nst;
   // the bias never depends on the previous kernel either (128 threads = 128 rows of the tile;
   // read after the W tiles are in flight, visible to the epilogue after its barrier)
-  sbias[threadIdx.x] = bias != nullptr ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
+  if (threadIdx.x < BM) sbias[threadIdx.x] = bias != nullptr ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
   if (threadIdx.x == 0) TRACE(2);
   pdl_wait();
   if (threadIdx.x == 0) TRACE(3);
 
   // epilogue thread mapping (single split): thread t owns 8 consecutive W rows
-  // nl = 8*(t%16) of tokens ml = t/16 + 8*j; their residual is fetched now, under the mainloop
+  // nl = 8*(t%16) of tokens ml = t/16 + (NT/16)*j; their residual is fetched now, under the mainloop
   const int nl_t = 8 * (threadIdx.x & 15);
   float rpre[RP > 0 ? RP : 1][8];
   if (RP > 0 && splits == 1 && res != nullptr) {
 #pragma unroll
     for (int j = 0; j < RP; ++j) {
-      const int ml = (threadIdx.x >> 4) + 8 * j;
+      const int ml = (threadIdx.x >> 4) + (NT / 16) * j;
       if (ml < mcount) load8<T>(res, (size_t)(m0 + ml) * ldr + n0 + nl_t, rpre[j], res32);
     }
   }
@@ -285,13 +288,15 @@ __global__ void __launch_bounds__(128, 1)
   // 1) TMEM -> shared memory (the ring is free once the MMAs are done): the fp32 tile,
   //    [128 W rows][BN tokens] with an odd row stride
   //    (split-K: unpadded [128][BN], so each owner's rows are one contiguous block to push)
-  const int row = warp * 32 + lane;  // TMEM lane = W row within the tile
+  // warp w reads TMEM lanes 32*(w%4).. (its lane quarter) for columns half w/4 of the tile
+  const int row = (warp & 3) * 32 + lane;  // TMEM lane = W row within the tile
   float* tile = reinterpret_cast<float*>(smem);
   const int rstride = splits == 1 ? PROW : BN;
+  const int chalf = (warp >> 2) * (BN / 2);
 #pragma unroll 1
-  for (int c0 = 0; c0 < BN; c0 += 16) {
+  for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
     uint32_t v[16];
-    tmem_ld16(tmem_d + (uint32_t(warp * 32) << 16) + c0, v);
+    tmem_ld16(tmem_d + (uint32_t((warp & 3) * 32) << 16) + c0, v);
     if (splits == 1) {
 #pragma unroll
       for (int j = 0; j < 16; ++j) tile[row * rstride + c0 + j] = __uint_as_float(v[j]);
@@ -332,30 +337,30 @@ __global__ void __launch_bounds__(128, 1)
     if constexpr (RP > 0) {
       // the prefetched residual goes to shared memory (after the fp32 tile) so the store loop
       // below can stay rolled: one small loop body, hot in the instruction cache
-      float* rs = tile + BM * PROW + threadIdx.x * 8;  // [RP][128 threads][8]
+      float* rs = tile + BM * PROW + threadIdx.x * 8;  // [RP][NT threads][8]
       if (res != nullptr) {
 #pragma unroll
         for (int j = 0; j < RP; ++j) {
-          float4* d = reinterpret_cast<float4*>(rs + j * 128 * 8);
+          float4* d = reinterpret_cast<float4*>(rs + j * NT * 8);
           d[0] = make_float4(rpre[j][0], rpre[j][1], rpre[j][2], rpre[j][3]);
           d[1] = make_float4(rpre[j][4], rpre[j][5], rpre[j][6], rpre[j][7]);
         }
       }
 #pragma unroll 1
       for (int j = 0; j < RP; ++j) {
-        const int ml = (threadIdx.x >> 4) + 8 * j;
+        const int ml = (threadIdx.x >> 4) + (NT / 16) * j;
         if (ml < mcount) {
           float acc[8];
 #pragma unroll
           for (int e = 0; e < 8; ++e) acc[e] = tile[(nl_t + e) * PROW + ml];
-          finish(nl_t, ml, acc, res != nullptr ? rs + j * 128 * 8 : nullptr);
+          finish(nl_t, ml, acc, res != nullptr ? rs + j * NT * 8 : nullptr);
         }
         if (threadIdx.x == 0 && j < 4) TRACE(9 + j);
       }
     } else {
       // wide tiles: a rolled loop (an unrolled 32-pass epilogue is instruction-fetch bound)
 #pragma unroll 1
-      for (int ml = threadIdx.x >> 4; ml < mcount; ml += 8) {
+      for (int ml = threadIdx.x >> 4; ml < mcount; ml += NT / 16) {
         float acc[8];
 #pragma unroll
         for (int e = 0; e < 8; ++e) acc[e] = tile[(nl_t + e) * PROW + ml];
@@ -397,7 +402,7 @@ __global__ void __launch_bounds__(128, 1)
     mbar_wait(&recv_bar, 0);
     if (threadIdx.x == 0) TRACE(7);
     const int units = (RPR / 8) * mcount;
-    for (int u = threadIdx.x; u < units; u += 128) {
+    for (int u = threadIdx.x; u < units; u += NT) {
       const int gi = u / mcount, ml = u - gi * mcount;  // 8-row group within the owned rows
       float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
       for (int p = 0; p < splits; ++p) {
@@ -434,7 +439,7 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   constexpr size_t STAGE_BYTES = BM * BK * 2 + BN * BK * 2;
   constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
   // the fp32 tile (+ the staged residual for BN <= 64) must fit the ring
-  constexpr size_t epi_bytes = size_t(BM) * (BN + 1) * 4 + (BN <= 64 ? size_t(BN / 8) * 128 * 8 * 4 : 0);
+  constexpr size_t epi_bytes = size_t(BM) * (BN + 1) * 4 + (BN <= 64 ? size_t(BN / (NT / 16)) * NT * 8 * 4 : 0);
   static_assert(epi_bytes + 1024 <= smem_max, "epilogue buffers must fit the ring");
   // split-K: unpadded send tile + receive slots, 2 x BM x BN fp32
   const size_t need = splits > 1 ? size_t(2) * BM * BN * 4 : epi_bytes;
@@ -460,7 +465,7 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   }
   CUtensorMap mx = make_kmajor_map(x, dtype, M, K, ldx, BN);
   const int mt = (M + BN - 1) / BN;
-  launch_kernel_cluster(gemm_tc_kernel<T, BN, ACT>, dim3(N / BM, mt, ngroups * splits), dim3(128), smem,
+  launch_kernel_cluster(gemm_tc_kernel<T, BN, ACT>, dim3(N / BM, mt, ngroups * splits), dim3(NT), smem,
                         dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, nst);
 }
 

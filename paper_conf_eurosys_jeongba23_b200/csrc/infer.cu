@@ -606,20 +606,32 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   // opts.trace_units: timing events for dp_run_timeline (eager only: graphs are off)
   const bool trace = ctx->opts.trace_units != 0;
   UnitTrace& tr = ds.trace;
+  auto stamp = [&](cudaStream_t on) {  // a globaltimer slot written when `on` reaches this point
+    DP_CHECK(tr.used < tr.cap, DP_ERR_STATE, "internal: trace buffer full");
+    launch_timestamp(tr.dbuf + tr.used, on);
+    return tr.used++;
+  };
   if (trace) {
+    const int cap = 3 * n + 2 * 1024 + 8;
+    if (tr.cap < cap) {
+      if (tr.dbuf) DP_CUDA(cudaFree(tr.dbuf));
+      tr.dbuf = nullptr;
+      DP_CUDA(cudaMalloc(&tr.dbuf, sizeof(uint64_t) * cap));
+      tr.cap = cap;
+    }
+    DP_CUDA(cudaMemsetAsync(tr.dbuf, 0, sizeof(uint64_t) * tr.cap, stream));
     tr.valid = false;
     tr.used = 0;
-    tr.ready.assign(n, nullptr);
-    tr.pre.assign(n, nullptr);
-    tr.start.assign(n, nullptr);
-    tr.t0 = tr.get();
-    DP_CUDA(cudaEventRecord(tr.t0, stream));
+    tr.ready.assign(n, -1);
+    tr.pre.assign(n, -1);
+    tr.start.assign(n, -1);
+    tr.t0 = stamp(stream);
+    tr.last_stream = stream;
   }
   auto trace_piece = [&](const Piece& p, cudaStream_t on) {  // the piece's bytes have landed
     if (!trace) return;
-    cudaEvent_t e = tr.get();
-    DP_CUDA(cudaEventRecord(e, on));
-    for (int u = p.first_unit; u <= p.last_unit; ++u) tr.ready[u] = e;
+    const int sl = stamp(on);
+    for (int u = p.first_unit; u <= p.last_unit; ++u) tr.ready[u] = sl;
   };
 
   // (1) slot-0 loads on the primary's link
@@ -828,17 +840,14 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
   if (trace) {  // an event on each side of the unit's dependency wait
     auto gate = a.before_unit;
     a.before_unit = [&, gate](int u) {
-      tr.pre[u] = tr.get();
-      DP_CUDA(cudaEventRecord(tr.pre[u], stream));
+      tr.pre[u] = stamp(stream);
       gate(u);
-      tr.start[u] = tr.get();
-      DP_CUDA(cudaEventRecord(tr.start[u], stream));
+      tr.start[u] = stamp(stream);
     };
   }
   run_forward(a);
   if (trace) {
-    tr.fin = tr.get();
-    DP_CUDA(cudaEventRecord(tr.fin, stream));
+    tr.fin = stamp(stream);
     tr.valid = true;
   }
   // join every side stream (units never read, e.g. an unused pooler, still finish loading)
@@ -903,22 +912,19 @@ extern "C" dp_status dp_run_timeline(dp_context* ctx, dp_model* m, int32_t dev, 
     DP_CHECK(tr.valid, DP_ERR_STATE, "no traced cold start (set opts.trace_units) of this model on this device");
     DP_CHECK(n == (int)m->units.size() && (int)tr.pre.size() == n, DP_ERR_INVALID, "n must be the unit count");
     DeviceGuard g(dev);
-    DP_CUDA(cudaEventSynchronize(tr.fin));
-    for (cudaEvent_t e : tr.ready)  // a piece on a side stream may land after the forward's end
-      if (e) DP_CUDA(cudaEventSynchronize(e));
-    auto ns = [&](cudaEvent_t e) -> int64_t {
-      if (!e) return -1;
-      float ms = 0.f;
-      DP_CUDA(cudaEventElapsedTime(&ms, tr.t0, e));
-      return (int64_t)llround(double(ms) * 1e6);
-    };
-    const int8_t* method = m->dev[dev].method.data();
+    DP_CUDA(cudaDeviceSynchronize());  // pieces on side streams may land after the forward's end
+    std::vector<uint64_t> h(tr.used);
+    DP_CUDA(cudaMemcpy(h.data(), tr.dbuf, sizeof(uint64_t) * tr.used, cudaMemcpyDeviceToHost));
+    auto ns = [&](int slot) -> int64_t {
+      if (slot < 0 || h[slot] == 0) return -1;
+      return (int64_t)h[slot] - (int64_t)h[tr.t0];
+    };    const int8_t* method = m->dev[dev].method.data();
     for (int u = 0; u < n; ++u) {
       const int64_t pre = ns(tr.pre[u]), start = ns(tr.start[u]);
       int64_t end = -1;
       if (start >= 0) {
         int v = u + 1;
-        while (v < n && !tr.pre[v]) ++v;
+        while (v < n && tr.pre[v] < 0) ++v;
         end = v < n ? ns(tr.pre[v]) : ns(tr.fin);
       }
       if (ready_ns) ready_ns[u] = method[u] == DP_DHA ? 0 : ns(tr.ready[u]);
@@ -1092,6 +1098,7 @@ extern "C" dp_status dp_model_destroy(dp_context* ctx, dp_model* m) {
         cudaDeviceSynchronize();
         for (auto& kv : ds.graphs) cudaGraphExecDestroy(kv.second.exec);
         ds.graphs.clear();
+        if (ds.trace.dbuf) cudaFree(ds.trace.dbuf);
         if (ds.capture) cudaStreamDestroy(ds.capture);
         if (ds.pinned_full) {
           cudaFree(ds.dbase);

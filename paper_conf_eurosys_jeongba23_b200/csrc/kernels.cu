@@ -29,9 +29,14 @@ PdlState& pdl_state() {
 }
 
 // -------------------------------------------------------------------------------------
-// K1: embedding gather + LayerNorm.  One warp per token; VPL 16-byte vectors per lane.
+// K1: embedding gather + LayerNorm.  One warp per token (TPW tokens per warp, all of their host
+// reads issued before any is used); VPL 16-byte vectors per lane.  The rows every token needs
+// (token type 0, LN gamma / beta) are staged in shared memory: by every CTA, or -- CL = true,
+// when they are host-mapped (DHA) -- by rank 0 of each cluster and broadcast over DSMEM, so they
+// cross the host link once per cluster (one cluster up to 512 tokens) instead of once per CTA.
+// The arithmetic per token is the same in every variant (bit-identical outputs).
 // -------------------------------------------------------------------------------------
-template <class T, int VPL>
+template <class T, int VPL, int TPW, bool CL>
 __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ ids, int ntok, int seq, int pos_off,
                                                     const T* word, const T* pos, const T* type, const T* g,
                                                     const T* b, int H, float eps, void* __restrict__ out_,
@@ -40,14 +45,15 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
   pdl_trigger();
   const int nv = H / 8;
   const bool has_type = type != nullptr, has_ln = g != nullptr;
-  // the shared rows (token type 0, gamma, beta) go into registers first; their host round
-  // trip overlaps the word/position gathers below (one PCIe latency per CTA, not two)
+  const bool stager = !CL || cta_cluster_rank() == 0;
+  // the shared rows go into registers first; their host round trip overlaps the word/position
+  // gathers below (one PCIe latency per CTA, not two)
   constexpr int SPT = 3;  // 3*nv <= 3*192 vectors over 256 threads
   uint4 stage[SPT];
 #pragma unroll
   for (int k = 0; k < SPT; ++k) {
     const int i = threadIdx.x + k * 256;
-    if (i < 3 * nv) {
+    if (stager && i < 3 * nv) {
       const int which = i / nv, c = i - which * nv;
       const T* src = which == 0 ? type : (which == 1 ? g : b);
       if (src) stage[k] = ldg16(src + 8 * c);
@@ -55,103 +61,151 @@ __global__ void __launch_bounds__(256) embed_kernel(const int32_t* __restrict__ 
   }
   pdl_wait();
   const int lane = threadIdx.x & 31;
-  const int t = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-  const bool live = t < ntok;
-  // ids outside [0, vocab) are clamped: a bad id must never make a DHA gather read past the
-  // table in the pinned arena (vocab <= 0: unchecked, the caller's tables)
-  int id = live ? ids[t] : 0;
-  if (vocab > 0) id = min(max(id, 0), vocab - 1);
-  const int p = pos_off + (live ? t % seq : 0);
-  uint4 wv[VPL], pv[VPL];
+  const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5), nw = gridDim.x * (blockDim.x >> 5);
+  uint4 wv[TPW][VPL], pv[TPW][VPL];
 #pragma unroll
-  for (int v = 0; v < VPL; ++v) {  // issue every host read of this row before using any
-    const int c = lane + 32 * v;
-    if (live && c < nv) {
-      wv[v] = ldg16(word + (size_t)id * H + 8 * c);
-      pv[v] = ldg16(pos + (size_t)p * H + 8 * c);
+  for (int j = 0; j < TPW; ++j) {  // issue every host read of this warp's rows before using any
+    const int t = gw + j * nw;
+    const bool live = t < ntok;
+    // ids outside [0, vocab) are clamped: a bad id must never make a DHA gather read past the
+    // table in the pinned arena (vocab <= 0: unchecked, the caller's tables)
+    int id = live ? ids[t] : 0;
+    if (vocab > 0) id = min(max(id, 0), vocab - 1);
+    const int p = pos_off + (live ? t % seq : 0);
+#pragma unroll
+    for (int v = 0; v < VPL; ++v) {
+      const int c = lane + 32 * v;
+      if (live && c < nv) {
+        wv[j][v] = ldg16(word + (size_t)id * H + 8 * c);
+        pv[j][v] = ldg16(pos + (size_t)p * H + 8 * c);
+      }
     }
   }
 #pragma unroll
   for (int k = 0; k < SPT; ++k) {
     const int i = threadIdx.x + k * 256;
-    if (i < 3 * nv) {
+    if (stager && i < 3 * nv) {
       const int which = i / nv;
       const T* src = which == 0 ? type : (which == 1 ? g : b);
       if (src) sm[i] = stage[k];
     }
   }
-  __syncthreads();
-  if (!live) return;
-  float x[VPL][8];
-  float sum = 0.f;
+  if (CL)
+    cluster_bcast_from_rank0(sm, 3 * nv);
+  else
+    __syncthreads();
 #pragma unroll
-  for (int v = 0; v < VPL; ++v) {
-    const int c = lane + 32 * v;
-    if (c < nv) {
-      float a[8], q[8];
-      unpack8<T>(wv[v], a);
-      unpack8<T>(pv[v], q);
-      if (has_type) {
-        float y[8];
-        unpack8<T>(sm[c], y);
-#pragma unroll
-        for (int e = 0; e < 8; ++e) x[v][e] = a[e] + q[e] + y[e];
-      } else {
-#pragma unroll
-        for (int e = 0; e < 8; ++e) x[v][e] = a[e] + q[e];
-      }
-#pragma unroll
-      for (int e = 0; e < 8; ++e) sum += x[v][e];
-    }
-  }
-  if (!has_ln) {
+  for (int j = 0; j < TPW; ++j) {
+    const int t = gw + j * nw;
+    if (t >= ntok) break;
+    float x[VPL][8];
+    float sum = 0.f;
 #pragma unroll
     for (int v = 0; v < VPL; ++v) {
       const int c = lane + 32 * v;
-      if (c < nv) store8<T>(out_, (size_t)t * H + 8 * c, x[v], out_f32);
+      if (c < nv) {
+        float a[8], q[8];
+        unpack8<T>(wv[j][v], a);
+        unpack8<T>(pv[j][v], q);
+        if (has_type) {
+          float y[8];
+          unpack8<T>(sm[c], y);
+#pragma unroll
+          for (int e = 0; e < 8; ++e) x[v][e] = a[e] + q[e] + y[e];
+        } else {
+#pragma unroll
+          for (int e = 0; e < 8; ++e) x[v][e] = a[e] + q[e];
+        }
+#pragma unroll
+        for (int e = 0; e < 8; ++e) sum += x[v][e];
+      }
     }
-    return;
-  }
-  const float mean = warp_sum(sum) / H;
-  float sq = 0.f;
+    if (!has_ln) {
 #pragma unroll
-  for (int v = 0; v < VPL; ++v) {
-    const int c = lane + 32 * v;
-    if (c < nv) {
+      for (int v = 0; v < VPL; ++v) {
+        const int c = lane + 32 * v;
+        if (c < nv) store8<T>(out_, (size_t)t * H + 8 * c, x[v], out_f32);
+      }
+      continue;
+    }
+    const float mean = warp_sum(sum) / H;
+    float sq = 0.f;
 #pragma unroll
-      for (int e = 0; e < 8; ++e) {
-        const float d = x[v][e] - mean;
-        sq += d * d;
+    for (int v = 0; v < VPL; ++v) {
+      const int c = lane + 32 * v;
+      if (c < nv) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          const float d = x[v][e] - mean;
+          sq += d * d;
+        }
+      }
+    }
+    const float rstd = rsqrtf(warp_sum(sq) / H + eps);
+#pragma unroll
+    for (int v = 0; v < VPL; ++v) {
+      const int c = lane + 32 * v;
+      if (c < nv) {
+        float gg[8], bb[8], y[8];
+        unpack8<T>(sm[nv + c], gg);
+        unpack8<T>(sm[2 * nv + c], bb);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) y[e] = (x[v][e] - mean) * rstd * gg[e] + bb[e];
+        store8<T>(out_, (size_t)t * H + 8 * c, y, out_f32);
+        if (out32 != nullptr) store8<T>(out32, (size_t)t * H + 8 * c, y, 1);  // fp32 residual-stream copy
       }
     }
   }
-  const float rstd = rsqrtf(warp_sum(sq) / H + eps);
-#pragma unroll
-  for (int v = 0; v < VPL; ++v) {
-    const int c = lane + 32 * v;
-    if (c < nv) {
-      float gg[8], bb[8], y[8];
-      unpack8<T>(sm[nv + c], gg);
-      unpack8<T>(sm[2 * nv + c], bb);
-#pragma unroll
-      for (int e = 0; e < 8; ++e) y[e] = (x[v][e] - mean) * rstd * gg[e] + bb[e];
-      store8<T>(out_, (size_t)t * H + 8 * c, y, out_f32);
-      if (out32 != nullptr) store8<T>(out32, (size_t)t * H + 8 * c, y, 1);  // fp32 residual-stream copy
-    }
+}
+
+template <class T, int V, int TPW, bool CL>
+static void embed_launch(int grid, int cluster, size_t sm, cudaStream_t s, const int32_t* ids, int ntok, int seq,
+                         int pos_off, const void* word, const void* pos, const void* type, const void* g,
+                         const void* b, int H, float eps, void* out, bool out_f32, float* out32, int vocab) {
+  if (CL) {
+    static std::atomic<unsigned> attr{0};
+    if (first_on_device(attr))
+      DP_CUDA(cudaFuncSetAttribute(embed_kernel<T, V, TPW, CL>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
   }
+  launch_kernel_cluster(embed_kernel<T, V, TPW, CL>, dim3(grid), dim3(256), sm, dim3(cluster), s, ids, ntok, seq,
+                        pos_off, (const T*)word, (const T*)pos, (const T*)type, (const T*)g, (const T*)b, H, eps, out,
+                        (int)out_f32, out32, vocab);
+}
+
+template <class T, int V>
+static void embed_v(bool shared_host, int ntok, int grid_one, size_t sm, cudaStream_t s, const int32_t* ids, int seq,
+                    int pos_off, const void* word, const void* pos, const void* type, const void* g, const void* b,
+                    int H, float eps, void* out, bool out_f32, float* out32, int vocab) {
+  if (!shared_host) {  // one token per warp, every CTA stages the shared rows (HBM / L2)
+    embed_launch<T, V, 1, false>(grid_one, 1, sm, s, ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out,
+                                 out_f32, out32, vocab);
+    return;
+  }
+  // host-mapped shared rows: clusters of 16 CTAs (128 warps), up to 4 tokens per warp
+  const int tpw = ntok <= 128 ? 1 : ntok <= 256 ? 2 : 4;
+  int grid = (ntok + 8 * tpw - 1) / (8 * tpw);
+  const int cluster = std::min(16, grid);
+  grid = (grid + cluster - 1) / cluster * cluster;
+#define DP_EMB_T(P) embed_launch<T, V, P, true>(grid, cluster, sm, s, ids, ntok, seq, pos_off, word, pos, type, g, b, H, \
+                                               eps, out, out_f32, out32, vocab)
+  if (tpw == 1) DP_EMB_T(1);
+  else if (tpw == 2) DP_EMB_T(2);
+  else DP_EMB_T(4);
+#undef DP_EMB_T
 }
 
 template <class T>
 static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                     const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
-                    float* out32, int vocab, cudaStream_t s) {
+                    float* out32, int vocab, bool shared_host, cudaStream_t s) {
   const int warps = 8;
-  dim3 grid((ntok + warps - 1) / warps);
+  const int grid = (ntok + warps - 1) / warps;
   const size_t sm = size_t(3) * (H / 8) * 16;
   const int vpl = (H / 8 + 31) / 32;
-#define DP_EMB(V)                                                                                      \
-  launch_kernel(embed_kernel<T, V>, grid, dim3(warps * 32), sm, s, ids, ntok, seq, pos_off, (const T*)word, \
-                (const T*)pos, (const T*)type, (const T*)g, (const T*)b, H, eps, out, (int)out_f32, out32, vocab)
+  shared_host = shared_host && (type != nullptr || g != nullptr);  // GPT-2 has no shared rows
+#define DP_EMB(V)                                                                                                   \
+  embed_v<T, V>(shared_host, ntok, grid, sm, s, ids, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, out32, \
+                vocab)
   switch (vpl) {
     case 1: DP_EMB(1); break;
     case 2: DP_EMB(2); break;
@@ -167,7 +221,7 @@ static void embed_t(const int32_t* ids, int ntok, int seq, int pos_off, const vo
 
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                   const void* type, const void* g, const void* b, int H, float eps, void* out, bool out_f32,
-                  cudaStream_t s, void* out32, int vocab) {
+                  cudaStream_t s, void* out32, int vocab, bool shared_host) {
   DP_CHECK(H % 8 == 0 && H > 0, DP_ERR_INVALID, "hidden must be a multiple of 8");
   DP_CHECK(seq > 0 && ntok >= 0, DP_ERR_INVALID, "bad token counts");
   if (ntok == 0) return;
@@ -177,45 +231,66 @@ void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off,
   }
   if (dtype == DP_BF16)
     embed_t<__nv_bfloat16>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32,
-                           static_cast<float*>(out32), vocab, s);
+                           static_cast<float*>(out32), vocab, shared_host, s);
   else
     embed_t<__half>(ids, ntok, seq, pos_off, word, pos, type, g, b, H, eps, out, out_f32, static_cast<float*>(out32),
-                    vocab, s);
+                    vocab, shared_host, s);
 }
 
 // -------------------------------------------------------------------------------------
-// K4: LayerNorm (+ residual).  gamma/beta staged once per CTA (they may be host-mapped).
+// K4: LayerNorm (+ residual).  gamma/beta staged in shared memory: by every CTA when they are in
+// HBM, or -- when they are host-mapped (DHA), CL = true -- by rank 0 of a single cluster of <= 16
+// CTAs and broadcast over DSMEM, so the host link carries them exactly once per launch.
 // -------------------------------------------------------------------------------------
-template <class T, int VPL>
+template <class T, int VPL, bool CL>
 __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__ x, const void* __restrict__ r,
                                                         const T* g, const T* b, T* __restrict__ y, int rows,
                                                         int n, float eps, int in_f32, float* __restrict__ y32) {
   extern __shared__ uint4 sm[];  // [gamma | beta]
   pdl_trigger();
   const int nv = n / 8;
-  for (int i = threadIdx.x; i < 2 * nv; i += blockDim.x) sm[i] = ldg16(i < nv ? g + 8 * i : b + 8 * (i - nv));
+  if (!CL || cta_cluster_rank() == 0)
+    for (int i = threadIdx.x; i < 2 * nv; i += blockDim.x) sm[i] = ldg16(i < nv ? g + 8 * i : b + 8 * (i - nv));
   pdl_wait();
-  __syncthreads();
+  if (CL)
+    cluster_bcast_from_rank0(sm, 2 * nv);
+  else
+    __syncthreads();
   const int lane = threadIdx.x & 31;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
   for (int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); row < rows; row += nwarps)
     ln_row_warp<T, VPL, 0>(x, r, (size_t)row * n, n, eps, in_f32, sm, y, (size_t)row * n, y32);
 }
 
+template <class T, int V, bool CL>
+static void layernorm_launch(int grid, size_t sm, cudaStream_t s, const void* x, const void* r, const void* g,
+                             const void* b, void* y, int rows, int n, float eps, bool in_f32, float* y32) {
+  if (CL) {
+    static std::atomic<unsigned> attr{0};
+    if (first_on_device(attr))
+      DP_CUDA(cudaFuncSetAttribute(layernorm_kernel<T, V, CL>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+  }
+  launch_kernel_cluster(layernorm_kernel<T, V, CL>, dim3(grid), dim3(256), sm, dim3(CL ? grid : 1), s, x, r,
+                        (const T*)g, (const T*)b, (T*)y, rows, n, eps, (int)in_f32, y32);
+}
+
 template <class T>
 static void layernorm_t(const void* x, const void* r, const void* g, const void* b, void* y, int rows, int n,
-                        float eps, bool in_f32, float* y32, cudaStream_t s) {
-  // one row per warp (latency: every row's loads in flight at once); gamma/beta are read
-  // once per CTA, so a DHA LayerNorm costs rows/8 x 4H bytes of host reads
+                        float eps, bool in_f32, float* y32, bool gb_host, cudaStream_t s) {
+  // one row per warp (latency: every row's loads in flight at once).  gamma/beta in HBM: every
+  // CTA stages them (L2 hits); host-mapped (DHA): ONE cluster of <= 16 CTAs (up to 128 warps,
+  // several rows each beyond 128 rows) reads them once and shares them over DSMEM, so the host
+  // link carries exactly 2 x n elements (the algorithmic bytes)
   const int warps = 8;
   int grid = (rows + warps - 1) / warps;
   if (grid > 148 * 8) grid = 148 * 8;
+  if (gb_host && grid > 16) grid = 16;
   if (grid < 1) grid = 1;
   const size_t sm = size_t(2) * (n / 8) * 16;
   const int vpl = (n / 8 + 31) / 32;
-#define DP_LN(V)                                                                                       \
-  launch_kernel(layernorm_kernel<T, V>, dim3(grid), dim3(warps * 32), sm, s, x, r, (const T*)g, (const T*)b, (T*)y, \
-                rows, n, eps, (int)in_f32, y32)
+#define DP_LN(V)                                                                                               \
+  (gb_host ? layernorm_launch<T, V, true>(grid, sm, s, x, r, g, b, y, rows, n, eps, in_f32, y32)               \
+           : layernorm_launch<T, V, false>(grid, sm, s, x, r, g, b, y, rows, n, eps, in_f32, y32))
   switch (vpl) {
     case 1: DP_LN(1); break;
     case 2: DP_LN(2); break;
@@ -230,7 +305,7 @@ static void layernorm_t(const void* x, const void* r, const void* g, const void*
 }
 
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
-                      int n, float eps, bool in_f32, cudaStream_t s, void* y32) {
+                      int n, float eps, bool in_f32, cudaStream_t s, void* y32, bool gb_host) {
   if (ablate_mask() & 2) return;
   DP_CHECK(n % 8 == 0 && n > 0, DP_ERR_INVALID, "LN width must be a multiple of 8");
   if (rows <= 0) return;
@@ -239,9 +314,9 @@ void launch_layernorm(int dtype, const void* x, const void* r, const void* g, co
     return;
   }
   if (dtype == DP_BF16)
-    layernorm_t<__nv_bfloat16>(x, r, g, b, y, rows, n, eps, in_f32, static_cast<float*>(y32), s);
+    layernorm_t<__nv_bfloat16>(x, r, g, b, y, rows, n, eps, in_f32, static_cast<float*>(y32), gb_host, s);
   else
-    layernorm_t<__half>(x, r, g, b, y, rows, n, eps, in_f32, static_cast<float*>(y32), s);
+    layernorm_t<__half>(x, r, g, b, y, rows, n, eps, in_f32, static_cast<float*>(y32), gb_host, s);
 }
 
 // -------------------------------------------------------------------------------------
@@ -907,6 +982,17 @@ __global__ void spin_kernel(long long cycles) {
   const long long t0 = clock64();
   while (clock64() - t0 < cycles) {
   }
+}
+
+__global__ void timestamp_kernel(uint64_t* slot) {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  *slot = t;
+}
+
+void launch_timestamp(uint64_t* slot, cudaStream_t s) {
+  timestamp_kernel<<<1, 1, 0, s>>>(slot);
+  DP_CUDA(cudaGetLastError());
 }
 
 void launch_spin(long long cycles, cudaStream_t s) {

@@ -15,11 +15,13 @@ enum Io { IO_RES_F32 = 1, IO_OUT_F32 = 2 };
 void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off, const void* word, const void* pos,
                   const void* type, const void* ln_g, const void* ln_b, int H, float eps, void* out, bool out_f32,
                   cudaStream_t s, void* out32 = nullptr,  // out32: optional fp32 copy of the LN output
-                  int vocab = 0);  // > 0: ids are clamped to [0, vocab) (engine path)
+                  int vocab = 0,                          // > 0: ids are clamped to [0, vocab) (engine path)
+                  bool shared_host = false);  // type / gamma / beta host-mapped: read once per cluster
 
 // K4: y = LN(x (+ r)) * g + b; g/b may be host-mapped.
 void launch_layernorm(int dtype, const void* x, const void* r, const void* g, const void* b, void* y, int rows,
-                      int n, float eps, bool in_f32, cudaStream_t s, void* y32 = nullptr);  // y32: optional fp32 copy
+                      int n, float eps, bool in_f32, cudaStream_t s, void* y32 = nullptr,  // y32: optional fp32 copy
+                      bool gb_host = false);  // gamma/beta host-mapped (DHA): read once per launch (cluster)
 
 // K3: skinny linear reading W exactly once (W may be host-mapped) -- a11.
 void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res,
@@ -54,5 +56,7 @@ void launch_attention_f32(const void* qkv, int ldqkv, void* ctx, int batch, int 
 // Scratch kernels
 void launch_l2_flush(void* buf, size_t bytes, cudaStream_t s);
 void launch_spin(long long cycles, cudaStream_t s);
+// Trace: one thread writes %globaltimer (ns) to *slot when the stream reaches it.
+void launch_timestamp(uint64_t* slot, cudaStream_t s);
 
 }  // namespace dp

@@ -3,7 +3,6 @@
 #include <cuda_runtime.h>
 
 #include <map>
-#include <stdexcept>
 #include <memory>
 #include <string>
 #include <vector>
@@ -59,21 +58,16 @@ struct GraphEntry {
   dp_run_stats stats{};
 };
 
-// Per-unit timestamps of a traced cold start (opts.trace_units; dp_run_timeline).
+// Per-unit timestamps of a traced cold start (opts.trace_units; dp_run_timeline): one-thread
+// kernels write %globaltimer into slots of a device buffer (timing events were measured to lag by
+// up to ~25 us on the execution stream while a DMA is in flight, which swamps per-unit stalls).
 struct UnitTrace {
   bool valid = false;
-  std::vector<cudaEvent_t> pool;  // timing-enabled events, recycled
-  size_t used = 0;
-  cudaEvent_t t0 = nullptr, fin = nullptr;
-  std::vector<cudaEvent_t> ready, pre, start;  // per unit (nullptr: not observed)
-  cudaEvent_t get() {
-    if (used == pool.size()) {
-      cudaEvent_t e;
-      if (cudaEventCreate(&e) != cudaSuccess) throw std::runtime_error("cudaEventCreate failed");
-      pool.push_back(e);
-    }
-    return pool[used++];
-  }
+  uint64_t* dbuf = nullptr;  // device slots
+  int cap = 0, used = 0;
+  int t0 = -1, fin = -1;
+  std::vector<int> ready, pre, start;  // per unit: slot index (-1: not observed)
+  cudaStream_t last_stream = nullptr;
 };
 
 struct DevState {

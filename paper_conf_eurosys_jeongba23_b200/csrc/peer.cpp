@@ -94,7 +94,13 @@ constexpr int kRing = 3;
 
 }  // namespace
 
-int peer_rank_of_slot(const dp_context* ctx, int primary, int slot) { return (primary + slot) % ctx->nranks; }
+int peer_rank_of_slot(const dp_context* ctx, int primary, int slot) {
+  // a map set by dp_peer_set_slot_ranks (e.g. from dp_select_secondaries on the measured link
+  // matrix) for this primary, else the fixed rotation
+  if (slot > 0 && ctx->slot_map_primary == primary && slot < DP_MAX_DEVICES && ctx->slot_rank[slot] >= 0)
+    return ctx->slot_rank[slot];
+  return (primary + slot) % ctx->nranks;
+}
 
 void peer_recv_all(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, int dev, cudaEvent_t fork,
                    std::vector<cudaEvent_t>& unit_ev, dp_run_stats& st) {
@@ -207,6 +213,24 @@ extern "C" dp_status dp_peer_unique_id(void* out128) {
     ncclUniqueId id;
     DP_NCCL(nccl().getUniqueId(&id));
     std::memcpy(out128, &id, sizeof(id));
+  });
+}
+
+extern "C" dp_status dp_peer_set_slot_ranks(dp_context* ctx, int32_t primary, const int32_t* rank_of_slot,
+                                            int32_t k) {
+  return guard([&] {
+    DP_CHECK(ctx && ctx->multiproc(), DP_ERR_STATE, "call dp_peer_init or dp_peer_init_ipc first");
+    DP_CHECK(primary >= 0 && primary < ctx->nranks && k >= 1 && k <= ctx->nranks && (k == 1 || rank_of_slot),
+             DP_ERR_INVALID, "bad primary / k");
+    std::vector<char> seen(ctx->nranks, 0);
+    seen[primary] = 1;
+    for (int s = 1; s < k; ++s) {
+      const int r = rank_of_slot[s - 1];
+      DP_CHECK(r >= 0 && r < ctx->nranks && !seen[r], DP_ERR_INVALID, "slot ranks must be distinct non-primary ranks");
+      seen[r] = 1;
+    }
+    ctx->slot_map_primary = primary;
+    for (int s = 0; s < DP_MAX_DEVICES; ++s) ctx->slot_rank[s] = (s >= 1 && s < k) ? rank_of_slot[s - 1] : -1;
   });
 }
 

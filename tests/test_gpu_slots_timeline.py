@@ -140,11 +140,12 @@ def test_timeline_gates_and_tracks_the_simulator(mode):
     r = ready[loaded]
     assert np.all(np.diff(r) >= 0)
     # the pipeline recurrence of P:162-170 holds on the hardware: a unit starts when
-    # the stream reached it or when its bytes landed, whichever is later (a dependency wait
-    # costs a few us), so its stall is max(0, ready - reached)
+    # the stream reached it or when its bytes landed, whichever is later, so its stall is
+    # max(0, ready - reached) -- up to the timestamp kernels' own launch (a few us) and the event
+    # wait's latency
     pre = start - stall
     want = np.where(loaded, np.maximum(0, ready - pre), 0)
-    assert np.all(np.abs(stall - want) <= 25_000), np.abs(stall - want).max()
+    assert np.all(np.abs(stall - want) <= 15_000), np.abs(stall - want).max()
     # against the simulator on the same live profile (R23 calibration).  Tracing puts two events
     # around every unit (no PDL overlap), which slows the compute chain and hides some stall, so
     # the comparison is loose; the paper-model DHA plan is known to under-predict (it ignores
@@ -154,7 +155,7 @@ def test_timeline_gates_and_tracks_the_simulator(mode):
         assert abs(end.max() - lat) <= 0.35 * lat, (end.max(), lat)
     if mode == "PIPESWITCH":  # load-bound: the stalls dominate and must match
         meas_total, sim_total = float(stall.sum()), float(sim_stall.sum())
-        assert abs(meas_total - sim_total) <= 0.3 * sim_total + 100_000, (meas_total, sim_total)
+        assert abs(meas_total - sim_total) <= 0.3 * sim_total + 300_000, (meas_total, sim_total)
     model.close()
     c.close()
 
