@@ -358,7 +358,8 @@ __global__ void __launch_bounds__(NT, 1)
         if (threadIdx.x == 0 && j < 4) TRACE(9 + j);
       }
     } else {
-      // wide tiles: a rolled loop (an unrolled 32-pass epilogue is instruction-fetch bound)
+      // wide tiles: a rolled loop (an unrolled 32-pass epilogue is instruction-fetch bound; 4x
+      // unrolled measured slower too, profiles/r02_gemm_trace.jsonl)
 #pragma unroll 1
       for (int ml = threadIdx.x >> 4; ml < mcount; ml += NT / 16) {
         float acc[8];

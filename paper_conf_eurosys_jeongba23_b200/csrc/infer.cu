@@ -125,10 +125,11 @@ static int64_t pool_trim(HbmPool& p, int dev) {
   return freed;
 }
 
-// A block of >= bytes: `prefer` if it is free and fits (a model re-acquiring its last block keeps
-// its captured graphs valid), else the best fit among the free blocks not more than 2x too large,
-// else a new cudaMalloc (trimming the free blocks and retrying once if HBM is exhausted).
-static void* pool_alloc(HbmPool& p, int dev, int64_t bytes, void* prefer) {
+// A block of >= bytes: the first of `prefer` that is free and fits (a model re-acquiring a block
+// it has captured graphs on keeps them valid: no re-capture), else the best fit among the free
+// blocks not more than 2x too large, else a new cudaMalloc (trimming the free blocks and retrying
+// once if HBM is exhausted).
+static void* pool_alloc(HbmPool& p, int dev, int64_t bytes, const std::vector<void*>& prefer) {
   bytes = (bytes + kPoolGrain - 1) / kPoolGrain * kPoolGrain;
   auto take = [&](std::multimap<int64_t, void*>::iterator it) {
     void* b = it->second;
@@ -136,9 +137,10 @@ static void* pool_alloc(HbmPool& p, int dev, int64_t bytes, void* prefer) {
     p.free_.erase(it);
     return b;
   };
-  if (prefer) {
+  for (void* want : prefer) {
+    if (!want) continue;
     for (auto it = p.free_.begin(); it != p.free_.end(); ++it)
-      if (it->second == prefer && it->first >= bytes && it->first <= 2 * bytes) return take(it);
+      if (it->second == want && it->first >= bytes && it->first <= 2 * bytes) return take(it);
   }
   auto it = p.free_.lower_bound(bytes);
   if (it != p.free_.end() && it->first <= 2 * bytes) return take(it);
@@ -199,7 +201,9 @@ void acquire_slots(dp_context* ctx, dp_model* m, int dev, const int8_t* method) 
   DP_CHECK(!ds.dbase, DP_ERR_STATE, "internal: HBM slots already held");
   std::vector<int64_t> doff;
   const int64_t bytes = std::max<int64_t>(compact_layout(m, method, doff), 256);
-  ds.dbase = pool_alloc(ctx->on(dev).pool, dev, bytes, ds.last_block);
+  std::vector<void*> prefer{ds.last_block};
+  prefer.insert(prefer.end(), ds.graph_blocks.begin(), ds.graph_blocks.end());
+  ds.dbase = pool_alloc(ctx->on(dev).pool, dev, bytes, prefer);
   ds.dbytes = bytes;
   ds.doff.swap(doff);
 }
@@ -510,6 +514,8 @@ static dp_run_stats run_graph(DevState& ds, const std::string& key, cudaStream_t
     cudaGraphDestroy(gph);
     DP_CUDA(e);
     it = ds.graphs.emplace(key, GraphEntry{ex, st}).first;
+    if (ds.dbase && std::find(ds.graph_blocks.begin(), ds.graph_blocks.end(), ds.dbase) == ds.graph_blocks.end())
+      ds.graph_blocks.push_back(ds.dbase);
   }
   DP_CUDA(cudaGraphLaunch(it->second.exec, stream));
   return it->second.stats;
@@ -727,7 +733,12 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       continue;
     }
     std::vector<cudaEvent_t> fwd_done(pcs.size(), nullptr);
-    {
+    // eager enqueue only: a captured graph's branches are ordered by the graph launches on the
+    // caller's stream, and a capture may not wait on work recorded outside it
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    DP_CUDA(cudaStreamIsCapturing(stream, &cap));
+    const bool eager = cap == cudaStreamCaptureStatusNone;
+    if (eager) {
       DeviceGuard gs(sdev);
       if (!r.tail) DP_CUDA(cudaEventCreateWithFlags(&r.tail, cudaEventDisableTiming));
       if (r.tail_set) DP_CUDA(cudaStreamWaitEvent(r.h2d, r.tail, 0));
@@ -760,7 +771,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
       add_wp(s, p, done);
       if (sdev == primary) trace_piece(p, r.mig);
     }
-    {
+    if (eager) {
       DeviceGuard gs(sdev);
       DP_CUDA(cudaEventRecord(r.tail, r.mig));
       r.tail_set = true;

@@ -79,6 +79,7 @@ struct DevState {
   std::vector<int64_t> doff;   // per unit: offset in the block, -1 for a DHA unit (read in place)
   bool pinned_full = false;    // IPC-exported slots: full arena layout, outside the pool, kept
   void* last_block = nullptr;  // the block released by the last eviction (reacquired if free)
+  std::vector<void*> graph_blocks;  // blocks this model has captured graphs on (preferred next)
   bool resident = false;
   std::vector<int8_t> method;  // per unit, fixed when the model became resident
   Workspace ws;

@@ -263,12 +263,13 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
         start_job(g, j);
       }
       if (done < nreq) {
+        // OS sleeps wake ~50-60 us late (timer slack): sleep only while nothing can happen for
+        // longer than that, otherwise spin (the dispatcher owns one host core)
         bool busy = false;
         for (auto& q : gpu) busy |= q.running >= 0;
-        if (!busy && next < nreq) {  // nothing to poll: sleep until the next arrival
-          std::this_thread::sleep_until(t0 + std::chrono::nanoseconds(trace[next].arrival_ns));
-        } else {
-          std::this_thread::sleep_for(std::chrono::microseconds(5));
+        if (!busy && next < nreq) {
+          const auto wake = t0 + std::chrono::nanoseconds(trace[next].arrival_ns) - std::chrono::microseconds(200);
+          if (wake > clk::now()) std::this_thread::sleep_until(wake);
         }
       }
     }

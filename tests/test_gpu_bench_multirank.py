@@ -37,3 +37,21 @@ def test_bench_two_ranks_one_gpu(transport):
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["config"]["pt_transport"] == transport
     assert d["e2e"]["value"] > 0
+    links = d["links"]
+    assert len(links["h2d_solo_gbs"]) == 2 and len(links["pair_gbs"]) == 2 and links["slot_ranks"] == [1]
+    assert [p["rank"] for p in d["pcie_rx"]] == [0, 1]
+
+
+def test_bench_spawns_its_own_ranks():
+    """`python bench.py --gpus 2` without a launcher (no WORLD_SIZE) re-launches itself under
+    torch.distributed.run; the line carries the output check against the oracle."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    env["DP_BENCH_ONE_GPU"] = "1"
+    cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "3", "--warmup", "3", "--model",
+           "tiny_bert", "--seq", "32", "--quick", "--profile-iters", "2", "--pt-transport", "ce"]
+    r = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["check"]["ok"] and d["cpu_baseline"]["kind"] == "oracle"

@@ -58,7 +58,7 @@ def test_live_decisions_equal_oracle_replay_and_evictions_free_hbm(name, seq):
     plans = plans_for(models, "DHA")
     rb = [dp().plan_resident_bytes(mm, p) for mm, p in zip(models, plans)]
     budget = int(3.5 * rb[0])
-    arr, inst = synth.make_poisson_trace(300, 3000.0, len(models), seed=5)
+    arr, inst = synth.make_poisson_trace(300, 1000.0, len(models), seed=5)
     res = run_live(c, models, plans, arr, inst, budget, seq=seq)
     ref = OS.replay_online(arr, inst, ngpu=1, per_gpu_budget_bytes=budget, resident_bytes=rb,
                            decide_ns=res["decide_ns"], finish_ns=res["finish_ns"])
@@ -101,7 +101,7 @@ def test_dha_fits_more_instances_than_pipeswitch():
     models = [base.clone() for _ in range(8)]
     full = dp().plan_resident_bytes(models[0], plans_for(models, "PIPESWITCH")[0])
     budget = int(3.3 * full)
-    arr, inst = synth.make_poisson_trace(400, 2000.0, len(models), seed=9)
+    arr, inst = synth.make_poisson_trace(400, 800.0, len(models), seed=9)
     cold = {}
     for mode in ("PIPESWITCH", "DHA"):
         plans = plans_for(models, mode)

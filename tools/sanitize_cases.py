@@ -25,7 +25,7 @@ def main():
         w = (torch.randn(N, K, device=dev) / math.sqrt(K)).half()
         b = torch.randn(N, device=dev).half()
         r = torch.randn(M, N, device=dev).half()
-        y = torch.empty(M, N, device=dev).half()
+        y = torch.zeros(M, N, device=dev).half()
         dp.linear(x, K, w, b, r, N, y, N, M, N, K, act="gelu_erf", path=0)
         # skinny (cluster split-K for K > 768), device and host-mapped weights
         dp.linear(x, K, w, b, r, N, y, N, M, N, K, path=1)
@@ -37,7 +37,7 @@ def main():
     for rows in (77, 384):
         n = 768
         x = torch.randn(rows, n, device=dev).half()
-        y = torch.empty_like(x)
+        y = torch.zeros_like(x)
         g = dp.host_alloc(n * 2)
         bb = dp.host_alloc(n * 2)
         dp.layernorm(x, None, g, bb, y, rows, n, 1e-12)
@@ -50,8 +50,8 @@ def main():
     ctx = dp.Context([0])
     model = dp.Model(ctx, m, w)
     ids = torch.from_numpy(synth.make_ids(m, 2, 40)).cuda()
-    out = torch.empty(80, m.hidden, dtype=torch.float16, device=dev)
-    pool = torch.empty(2, m.hidden, dtype=torch.float16, device=dev)
+    out = torch.zeros(80, m.hidden, dtype=torch.float16, device=dev)
+    pool = torch.zeros(2, m.hidden, dtype=torch.float16, device=dev)
     n = model.n
     kinds = [u["kind"] for u in model.units()]
     for meth in (np.zeros(n, np.int8), np.array([1 if k != "linear" else 0 for k in kinds], np.int8), np.ones(n, np.int8)):
@@ -73,14 +73,14 @@ def main():
     for S, causal in ((128, False), (384, False), (300, True)):
         H, heads = 256, 4
         qkv = torch.randn(S, 3 * H, device=dev).half()
-        o = torch.empty(S, H, device=dev).half()
+        o = torch.zeros(S, H, device=dev).half()
         dp.attention(qkv, 3 * H, o, 1, S, H, heads, causal)
-        o32 = torch.empty(S, H, device=dev)
+        o32 = torch.zeros(S, H, device=dev)
         dp.attention(qkv.float(), 3 * H, o32, 1, S, H, heads, causal, dtype="fp32")
     w32 = synth.make_weights(m, seed=0, dtype="fp32")
     model32 = dp.Model(ctx, m, w32, "fp32")
-    out32 = torch.empty(80, m.hidden, device=dev)
-    pool32 = torch.empty(2, m.hidden, device=dev)
+    out32 = torch.zeros(80, m.hidden, device=dev)
+    pool32 = torch.zeros(2, m.hidden, device=dev)
     model32.infer_cold(dp._lib.PlanArrays(n, np.zeros(n, np.int8), None, 1, 1), 0, ids, out32, pool32)
     torch.cuda.synchronize()
     model32.evict(0)
