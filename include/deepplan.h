@@ -199,7 +199,10 @@ typedef struct {
                              every unit's dependency wait on the execution stream.  Costs event
                              records between kernels (no PDL overlap) and forces eager enqueue (no
                              graph): a measurement mode [0] */
-  int32_t reserved[2];
+  int32_t attention_tc;   /* 1 = the attention core runs on tcgen05 (K5t: S and P.V in TMEM, the
+                             softmax row per thread); correct but measured slower than the mma.sync
+                             flash kernels K5 / K5b at the hot-path shapes [0] */
+  int32_t reserved[1];
 } dp_engine_opts;
 #define DP_PT_DMA 0
 #define DP_PT_SM 1
@@ -472,6 +475,11 @@ dp_status dp_layernorm(const void* x, const void* r, const void* g, const void* 
  * Sequences are contiguous blocks of `seq` tokens. */
 dp_status dp_attention(const void* qkv, int32_t ldqkv, void* ctx_out, int32_t batch, int32_t seq, int32_t hidden,
                        int32_t heads, int32_t causal, int32_t dtype, void* stream);
+/* The same on tcgen05 (K5t, the engine's opts.attention_tc): one CTA per (head, 128 queries);
+ * S = Q K^T and O_j = P V_j in TMEM, the online softmax per row in one thread, P rounded to the
+ * storage type before P.V.  fp16 / bf16, head dim 64, 16-byte aligned rows. */
+dp_status dp_attention_tc(const void* qkv, int32_t ldqkv, void* ctx_out, int32_t batch, int32_t seq, int32_t hidden,
+                          int32_t heads, int32_t causal, int32_t dtype, void* stream);
 
 /* ---------------------------------------------------------------------------------
  * Serving harness (§5.3): one inference per GPU at a time (Clockwork-like),

@@ -53,7 +53,7 @@ class EngineOpts(C.Structure):
                 ("gemm_bn", C.c_int32), ("debug_delay_us", C.c_int32), ("debug_poison", C.c_int32),
                 ("use_pdl", C.c_int32), ("fuse_ln", C.c_int32), ("tail_bytes", C.c_int64),
                 ("persistent", C.c_int32), ("pt_transport", C.c_int32), ("profile_chain", C.c_int32),
-                ("trace_units", C.c_int32), ("reserved", C.c_int32 * 2)]
+                ("trace_units", C.c_int32), ("attention_tc", C.c_int32), ("reserved", C.c_int32 * 1)]
 
 
 class ModelConfig(C.Structure):
@@ -161,6 +161,7 @@ _sig("dp_linear", [vp, C.c_int32, vp, vp, vp, C.c_int32, vp, C.c_int32, C.c_int3
                    C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
 _sig("dp_layernorm", [vp, vp, vp, vp, vp, C.c_int32, C.c_int32, C.c_double, C.c_int32, C.c_int32, vp])
 _sig("dp_attention", [vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
+_sig("dp_attention_tc", [vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
 _sig("dp_serve_run", [vp, C.POINTER(vp), C.c_int32, C.POINTER(TraceEvent), C.c_int32, C.POINTER(ServeOpts),
                       C.POINTER(ServeResult)])
 
@@ -293,7 +294,7 @@ class Context:
 
     def set_opts(self, chunk_bytes=None, n_h2d_streams=None, use_graph=None, gemm_bn=None, debug_delay_us=None,
                  debug_poison=None, use_pdl=None, tail_bytes=None, fuse_ln=None, persistent=None,
-                 pt_transport=None, profile_chain=None, trace_units=None):
+                 pt_transport=None, profile_chain=None, trace_units=None, attention_tc=None):
         o = EngineOpts()
         _check(lib.dp_context_get_opts(self.h, C.byref(o)))
         if chunk_bytes is not None:
@@ -320,6 +321,8 @@ class Context:
             o.profile_chain = 1 if profile_chain else 0
         if trace_units is not None:
             o.trace_units = 1 if trace_units else 0
+        if attention_tc is not None:
+            o.attention_tc = 1 if attention_tc else 0
         if pt_transport is not None:
             o.pt_transport = PT_TRANSPORTS[pt_transport] if isinstance(pt_transport, str) else int(pt_transport)
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))
@@ -617,6 +620,12 @@ def layernorm(x, r, g, b, y, rows, n, eps, dtype="fp16", x_f32=False, stream=Non
 def attention(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp16", stream=None):
     _check(lib.dp_attention(_dptr(qkv), int(ldqkv), _dptr(ctx_out), int(batch), int(seq), int(hidden), int(heads),
                             int(bool(causal)), DTYPES[dtype], _stream_ptr(stream)))
+
+
+def attention_tc(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp16", stream=None):
+    """The tcgen05 attention core (K5t, opts.attention_tc)."""
+    _check(lib.dp_attention_tc(_dptr(qkv), int(ldqkv), _dptr(ctx_out), int(batch), int(seq), int(hidden), int(heads),
+                               int(bool(causal)), DTYPES[dtype], _stream_ptr(stream)))
 
 
 # --------------------------------------------------------------------------------------

@@ -81,6 +81,17 @@ extern "C" dp_status dp_layernorm(const void* x, const void* r, const void* g, c
   });
 }
 
+extern "C" dp_status dp_attention_tc(const void* qkv, int32_t ldqkv, void* ctx_out, int32_t batch, int32_t seq,
+                                     int32_t hidden, int32_t heads, int32_t causal, int32_t dtype, void* stream) {
+  return guard([&] {
+    DP_CHECK(dtype == DP_FP16 || dtype == DP_BF16, DP_ERR_UNSUPPORTED, "tcgen05 attention: fp16 / bf16");
+    DP_CHECK(qkv && ctx_out && ldqkv >= 3 * hidden && attention_tc_supported(ldqkv, hidden, heads, qkv), DP_ERR_INVALID,
+             "bad arguments (head dim 64, 16-byte aligned rows)");
+    if (batch > 0 && seq > 0)
+      launch_attention_tc(dtype, qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal != 0, (cudaStream_t)stream);
+  });
+}
+
 extern "C" dp_status dp_attention(const void* qkv, int32_t ldqkv, void* ctx_out, int32_t batch, int32_t seq,
                                   int32_t hidden, int32_t heads, int32_t causal, int32_t dtype, void* stream) {
   return guard([&] {

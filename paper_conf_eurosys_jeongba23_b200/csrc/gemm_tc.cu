@@ -154,15 +154,14 @@ __device__ __forceinline__ float ld_cluster_f32(uint32_t addr) {
 template <class T, int BN, int ACT>
 __global__ void __launch_bounds__(NT, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
-                   const void* res, int ldr, void* Y, int ldy, int M, int N, int K, int act, int io, int splits,
-                   int nst) {
+                   const __grid_constant__ CUtensorMap tmY, const void* res, int ldr, void* Y, int ldy, int M, int N,
+                   int K, int act, int io, int splits, int nst) {
   constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
   constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free TMEM->smem writes)
-  constexpr int RP = BN <= 64 ? BN / (NT / 16) : 0;  // residual rows prefetched per thread (single split)
   // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
   constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
                              (uint32_t(BM >> 4) << 24);
@@ -231,18 +230,6 @@ __global__ void __launch_bounds__(NT, 1)
   pdl_wait();
   if (threadIdx.x == 0) TRACE(3);
 
-  // epilogue thread mapping (single split): thread t owns 8 consecutive W rows
-  // nl = 8*(t%16) of tokens ml = t/16 + (NT/16)*j; their residual is fetched now, under the mainloop
-  const int nl_t = 8 * (threadIdx.x & 15);
-  float rpre[RP > 0 ? RP : 1][8];
-  if (RP > 0 && splits == 1 && res != nullptr) {
-#pragma unroll
-    for (int j = 0; j < RP; ++j) {
-      const int ml = (threadIdx.x >> 4) + (NT / 16) * j;
-      if (ml < mcount) load8<T>(res, (size_t)(m0 + ml) * ldr + n0 + nl_t, rpre[j], res32);
-    }
-  }
-
   if (warp == 0 && lane == 0) {
     // TMA producer
     for (int kb = 0; kb < num_kb; ++kb) {
@@ -275,7 +262,11 @@ __global__ void __launch_bounds__(NT, 1)
   }
   __syncwarp();
 
-  mbar_wait(&done_bar, 0);
+  // one thread spins on the MMAs' completion and releases the CTA through its barrier (every
+  // warp waiting on the mbarrier itself woke ~1 us late: try_wait suspends the waiter)
+  if (threadIdx.x == 32) mbar_wait_spin(&done_bar, 0);
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
   if (threadIdx.x == 0) TRACE(5);
   // split-K: announce that this CTA's MMAs are done, i.e. its TMA ring -- which the receive
   // slots below overlap -- is free.  Peers push into our receive slots only after the
@@ -285,90 +276,80 @@ __global__ void __launch_bounds__(NT, 1)
   // the peers' async-proxy writes into it.
   if (splits > 1) asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
   asm volatile("tcgen05.fence::after_thread_sync;");
-  // 1) TMEM -> shared memory (the ring is free once the MMAs are done): the fp32 tile,
-  //    [128 W rows][BN tokens] with an odd row stride
-  //    (split-K: unpadded [128][BN], so each owner's rows are one contiguous block to push)
-  // warp w reads TMEM lanes 32*(w%4).. (its lane quarter) for columns half w/4 of the tile
-  const int row = (warp & 3) * 32 + lane;  // TMEM lane = W row within the tile
-  float* tile = reinterpret_cast<float*>(smem);
-  const int rstride = splits == 1 ? PROW : BN;
+  // TMEM lane = W row within the tile; warp w reads its lane quarter (w % 4) for the column
+  // half w / 4 of the tile
+  const int row = (warp & 3) * 32 + lane;
   const int chalf = (warp >> 2) * (BN / 2);
-#pragma unroll 1
-  for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
-    uint32_t v[16];
-    tmem_ld16(tmem_d + (uint32_t((warp & 3) * 32) << 16) + c0, v);
-    if (splits == 1) {
-#pragma unroll
-      for (int j = 0; j < 16; ++j) tile[row * rstride + c0 + j] = __uint_as_float(v[j]);
-    } else {
-#pragma unroll
-      for (int j = 0; j < 16; j += 4)
-        *reinterpret_cast<float4*>(&tile[row * rstride + c0 + j]) =
-            make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
-                        __uint_as_float(v[j + 3]));
-    }
-  }
-  // 2) + bias, activation, + residual; one 16-byte store per 8 outputs (8 W rows of a token)
-  // rs: the residual already staged in shared memory (8 floats), or nullptr to load it now
-  auto finish = [&](int nl, int ml, float* acc, const float* rs) {
-    const size_t m = (size_t)(m0 + ml);
-    const int n = n0 + nl;
-#pragma unroll
-    for (int e = 0; e < 8; ++e) acc[e] = apply_act_c<ACT>(acc[e] + sbias[nl + e]);
-    if (res) {
-      float r8[8];
-      if (rs != nullptr) {
-        const float4 a = reinterpret_cast<const float4*>(rs)[0], b = reinterpret_cast<const float4*>(rs)[1];
-        r8[0] = a.x, r8[1] = a.y, r8[2] = a.z, r8[3] = a.w, r8[4] = b.x, r8[5] = b.y, r8[6] = b.z, r8[7] = b.w;
-      } else {
-        load8<T>(res, m * ldr + n, r8, res32);
-      }
-#pragma unroll
-      for (int e = 0; e < 8; ++e) acc[e] += r8[e];
-    }
-    store8<T>(Y, m * ldy + n + ycol, acc, out32);
-  };
+  float* tile = reinterpret_cast<float*>(smem);
   if (splits == 1) {
+    // Single split: straight from TMEM to the output.  Each thread owns one W row (feature n) and
+    // walks the token columns 16 at a time: + bias, activation, + residual (a warp's 32 lanes read
+    // 32 consecutive features of a token: coalesced), and writes the value into an output tile in
+    // shared memory laid out like Y ([BN tokens][128 features], the output dtype) -- a warp writes
+    // 32 consecutive elements per token, conflict-free.  One TMA bulk tensor store then writes the
+    // tile (rows past M are clipped by the tensor map), replacing the fp32 round trip through
+    // shared memory and the per-thread 16-byte stores of round 1.
+    uint8_t* otile = smem;  // the ring is free once the MMAs are done
+    const int n = n0 + row;
+    const float bsv = sbias[row];
+#pragma unroll 1
+    for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
+      float rv[16];
+      if (res != nullptr) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const int ml = c0 + j;
+          rv[j] = ml < mcount ? load1<T>(res, (size_t)(m0 + ml) * ldr + n, res32) : 0.f;
+        }
+      }
+      uint32_t v[16];
+      tmem_ld16(tmem_d + (uint32_t((warp & 3) * 32) << 16) + c0, v);
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        float a = apply_act_c<ACT>(__uint_as_float(v[j]) + bsv);
+        if (res != nullptr) a += rv[j];
+        if (out32)
+          reinterpret_cast<float*>(otile)[(c0 + j) * BM + row] = a;
+        else
+          reinterpret_cast<T*>(otile)[(c0 + j) * BM + row] = Cvt<T>::from1(a);
+      }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
     __syncthreads();
     if (threadIdx.x == 0) {
       TRACE(6);
       TRACE(7);
-    }
-    if constexpr (RP > 0) {
-      // the prefetched residual goes to shared memory (after the fp32 tile) so the store loop
-      // below can stay rolled: one small loop body, hot in the instruction cache
-      float* rs = tile + BM * PROW + threadIdx.x * 8;  // [RP][NT threads][8]
-      if (res != nullptr) {
-#pragma unroll
-        for (int j = 0; j < RP; ++j) {
-          float4* d = reinterpret_cast<float4*>(rs + j * NT * 8);
-          d[0] = make_float4(rpre[j][0], rpre[j][1], rpre[j][2], rpre[j][3]);
-          d[1] = make_float4(rpre[j][4], rpre[j][5], rpre[j][6], rpre[j][7]);
-        }
-      }
-#pragma unroll 1
-      for (int j = 0; j < RP; ++j) {
-        const int ml = (threadIdx.x >> 4) + (NT / 16) * j;
-        if (ml < mcount) {
-          float acc[8];
-#pragma unroll
-          for (int e = 0; e < 8; ++e) acc[e] = tile[(nl_t + e) * PROW + ml];
-          finish(nl_t, ml, acc, res != nullptr ? rs + j * NT * 8 : nullptr);
-        }
-        if (threadIdx.x == 0 && j < 4) TRACE(9 + j);
-      }
-    } else {
-      // wide tiles: a rolled loop (an unrolled 32-pass epilogue is instruction-fetch bound; 4x
-      // unrolled measured slower too, profiles/r02_gemm_trace.jsonl)
-#pragma unroll 1
-      for (int ml = threadIdx.x >> 4; ml < mcount; ml += NT / 16) {
-        float acc[8];
-#pragma unroll
-        for (int e = 0; e < 8; ++e) acc[e] = tile[(nl_t + e) * PROW + ml];
-        finish(nl_t, ml, acc, nullptr);
-      }
+      tma_store_2d(&tmY, otile, n0 + (int)ycol, m0);
+      bulk_commit();
+      bulk_wait0();  // the tile is written (and its shared memory read) before the CTA exits
     }
   } else {
+    // 1) TMEM -> shared memory: this split's fp32 partial tile [128 W rows][BN tokens], unpadded,
+    //    so each owner's rows are one contiguous block to push
+#pragma unroll 1
+    for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
+      uint32_t v[16];
+      tmem_ld16(tmem_d + (uint32_t((warp & 3) * 32) << 16) + c0, v);
+#pragma unroll
+      for (int j = 0; j < 16; j += 4)
+        *reinterpret_cast<float4*>(&tile[row * BN + c0 + j]) =
+            make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
+                        __uint_as_float(v[j + 3]));
+    }
+    // 2) + bias, activation, + residual; one 16-byte store per 8 outputs (8 W rows of a token)
+    auto finish = [&](int nl, int ml, float* acc) {
+      const size_t m = (size_t)(m0 + ml);
+      const int nn = n0 + nl;
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] = apply_act_c<ACT>(acc[e] + sbias[nl + e]);
+      if (res) {
+        float r8[8];
+        load8<T>(res, m * ldr + nn, r8, res32);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) acc[e] += r8[e];
+      }
+      store8<T>(Y, m * ldy + nn + ycol, acc, out32);
+    };
     // 1b) cluster split-K reduction: rank r owns tile rows [r*RPR, (r+1)*RPR).  Every CTA pushes
     //     the rows each peer owns from its send buffer into that peer's receive slot with a
     //     bulk async copy (cp.async.bulk shared::cta -> shared::cluster) that completes on the
@@ -411,7 +392,7 @@ __global__ void __launch_bounds__(NT, 1)
 #pragma unroll
         for (int e = 0; e < 8; ++e) acc[e] += sl[(8 * gi + e) * BN + ml];
       }
-      finish(sp * RPR + 8 * gi, ml, acc, nullptr);
+      finish(sp * RPR + 8 * gi, ml, acc);
     }
     // the pushes must have read this CTA's send buffer before it exits
     if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
@@ -439,8 +420,8 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   constexpr int STAGES = stages_for<BN>();
   constexpr size_t STAGE_BYTES = BM * BK * 2 + BN * BK * 2;
   constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
-  // the fp32 tile (+ the staged residual for BN <= 64) must fit the ring
-  constexpr size_t epi_bytes = size_t(BM) * (BN + 1) * 4 + (BN <= 64 ? size_t(BN / (NT / 16)) * NT * 8 * 4 : 0);
+  // the output tile (at most fp32) must fit the ring
+  constexpr size_t epi_bytes = size_t(BM) * BN * 4;
   static_assert(epi_bytes + 1024 <= smem_max, "epilogue buffers must fit the ring");
   // split-K: unpadded send tile + receive slots, 2 x BM x BN fp32
   const size_t need = splits > 1 ? size_t(2) * BM * BN * 4 : epi_bytes;
@@ -465,9 +446,19 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
     g.ycol[i] = ycol ? ycol[i] : 0;
   }
   CUtensorMap mx = make_kmajor_map(x, dtype, M, K, ldx, BN);
+  // the output tile store (single split): Y as [M rows][ldy columns] in the output dtype, box
+  // [BN tokens][128 features]
+  const bool o32 = (io & IO_OUT_F32) != 0;
+  const uint64_t ydims[2] = {(uint64_t)ldy, (uint64_t)M};
+  const uint64_t ystr[1] = {(uint64_t)ldy * (o32 ? 4 : 2)};
+  const uint32_t ybox[2] = {(uint32_t)BM, (uint32_t)BN};
+  CUtensorMap my = make_plain_map(y, o32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                         : (dtype == DP_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                                             : CU_TENSOR_MAP_DATA_TYPE_FLOAT16),
+                                  2, ydims, ystr, ybox);
   const int mt = (M + BN - 1) / BN;
   launch_kernel_cluster(gemm_tc_kernel<T, BN, ACT>, dim3(N / BM, mt, ngroups * splits), dim3(NT), smem,
-                        dim3(1, 1, splits), s, g, mx, res, ldr, y, ldy, M, N, K, act, io, splits, nst);
+                        dim3(1, 1, splits), s, g, mx, my, res, ldr, y, ldy, M, N, K, act, io, splits, nst);
 }
 
 template <class T>

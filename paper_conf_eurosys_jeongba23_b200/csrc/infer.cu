@@ -482,7 +482,7 @@ static std::string graph_key(const dp_context* ctx, const DevState& ds, const dp
        std::to_string((uintptr_t)pooled) + "|" + std::to_string(batch) + "x" + std::to_string(seq) + "|" +
        std::to_string(ctx->opts.chunk_bytes) + "," + std::to_string(ctx->opts.n_h2d_streams) + "," +
        std::to_string(ctx->opts.gemm_bn) + "," + std::to_string(ctx->opts.debug_delay_us) + "," +
-       std::to_string(ctx->opts.use_pdl) + "," +
+       std::to_string(ctx->opts.use_pdl) + "," + std::to_string(ctx->opts.attention_tc) + "," +
        std::to_string(ctx->opts.pt_transport);
   return k;
 }
@@ -848,6 +848,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     pdl_state().block_next = true;  // the next kernel must see the landed weights: no PDL overlap
   };
   a.pdl = ctx->opts.use_pdl != 0;
+  a.attention_tc = ctx->opts.attention_tc != 0;
   if (trace) {  // an event on each side of the unit's dependency wait
     auto gate = a.before_unit;
     a.before_unit = [&, gate](int u) {
@@ -968,6 +969,7 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.stream = (cudaStream_t)stream;
     a.bn_hint = ctx->opts.gemm_bn;
     a.pdl = ctx->opts.use_pdl != 0;
+  a.attention_tc = ctx->opts.attention_tc != 0;
     // Experiment (tools/wait_cost.py): the cost of a dependency wait before every unit on the
     // execution stream, all already satisfied -- 1: event wait, 2: one-thread acquire-spin
     // kernel on a device word, 3: cuStreamWaitValue32 (stream memory op)
@@ -1257,6 +1259,7 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
     fa.stream = s;
     fa.bn_hint = ctx->opts.gemm_bn;
     fa.pdl = ctx->opts.use_pdl != 0;
+    fa.attention_tc = ctx->opts.attention_tc != 0;
     // the host enqueues ~100 launches behind a ~1.5 ms spin, so e0..e1 is device time only
     const int64_t chain = timed([&] { run_forward(fa); }, true, 3000000);
     DP_CUDA(cudaStreamSynchronize(s));

@@ -721,13 +721,19 @@ __global__ void __launch_bounds__(128 * G) attention2_kernel(const T* __restrict
 }
 
 void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
-                      bool causal, cudaStream_t s) {
+                      bool causal, cudaStream_t s, bool use_tc) {
   if (ablate_mask() & 1) return;
   DP_CHECK(heads > 0 && H % heads == 0 && H / heads == ATT_D, DP_ERR_UNSUPPORTED, "attention needs head dim 64");
   DP_CHECK(ldqkv % 8 == 0, DP_ERR_INVALID, "ldqkv must be a multiple of 8");
   if (batch <= 0 || seq <= 0) return;
   if (dtype == DP_FP32) {
     launch_attention_f32(qkv, ldqkv, ctx, batch, seq, H, heads, causal, s);
+    return;
+  }
+  // K5t (tcgen05, attn_tc.cu) when the engine option asks for it (opts.attention_tc; measured
+  // slower than K5 / K5b below at every hot-path shape)
+  if (use_tc && attention_tc_supported(ldqkv, H, heads, qkv)) {
+    launch_attention_tc(dtype, qkv, ldqkv, ctx, batch, seq, H, heads, causal, s);
     return;
   }
   dim3 grid((seq + ATT_BQ - 1) / ATT_BQ, heads, batch);

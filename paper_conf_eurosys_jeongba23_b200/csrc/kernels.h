@@ -29,7 +29,12 @@ void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, cons
 
 // K5: attention core (mma.sync flash attention, d = 64).
 void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
-                      bool causal, cudaStream_t s);
+                      bool causal, cudaStream_t s, bool use_tc = false);  // use_tc: K5t (attn_tc.cu)
+
+// K5t: attention on tcgen05 (attn_tc.cu): S and O in TMEM, the softmax row per thread.
+bool attention_tc_supported(int ldqkv, int H, int heads, const void* qkv);
+void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
+                         bool causal, cudaStream_t s);
 
 // K2: resident tcgen05/TMA GEMM -- a12.  W must be device memory.
 struct GemmPlan;  // cached tensor map for a weight

@@ -7,6 +7,7 @@
 // place by a DHA kernel, portable so every GPU of the context can DMA from it, packed in
 // forward order with 256-byte aligned units so a run of adjacent loaded units is one
 // contiguous DMA.  Planning units follow SURVEY G1 (one weight-bearing leaf module).
+#include "engine.h"
 #include "model.h"
 
 #include <cstring>
@@ -193,11 +194,12 @@ extern "C" dp_status dp_model_create(dp_context* ctx, const dp_model_config* cfg
     DP_CHECK(nparams == (int32_t)m->params.size(), DP_ERR_INVALID,
              "expected " + std::to_string(m->params.size()) + " parameters, got " + std::to_string(nparams));
     build_units(m);
-    cudaError_t e = cudaHostAlloc(&m->arena, m->arena_bytes, cudaHostAllocPortable | cudaHostAllocMapped);
-    if (e != cudaSuccess) {
-      m->arena = nullptr;
-      fail(DP_ERR_OOM, std::string("cudaHostAlloc of the weight arena failed: ") + cudaGetErrorString(e));
-    }
+    // the arena lives on the NUMA node of the context's first (serving) device: its loads and
+    // DHA reads cross no socket interconnect (topo.cpp)
+    const int node = (ctx && !ctx->devs.empty()) ? device_numa_node(ctx->devs[0]) : -1;
+    m->arena = host_alloc_on_node(m->arena_bytes, node);
+    if (!m->arena) fail(DP_ERR_OOM, "cudaHostAlloc of the weight arena failed");
+    m->arena_node = node;
     m->arena_owner = std::shared_ptr<void>(m->arena, [](void* p) { cudaFreeHost(p); });
     std::memset(m->arena, 0, m->arena_bytes);
     uint8_t* base = static_cast<uint8_t*>(m->arena);

@@ -89,6 +89,9 @@ struct DevState {
 };
 
 std::vector<ParamDesc> config_params(const dp_model_config& c);
+// topo.cpp
+int device_numa_node(int dev);
+void* host_alloc_on_node(int64_t bytes, int node);
 void validate_config(const dp_model_config& c);
 
 }  // namespace dp
@@ -103,7 +106,8 @@ struct dp_model {
   dp_model_config cfg{};
   std::vector<dp::ParamDesc> params;
   std::vector<dp::UnitDesc> units;
-  void* arena = nullptr;  // cudaHostAlloc(Portable | Mapped)
+  void* arena = nullptr;  // cudaHostAlloc(Portable | Mapped), on NUMA node arena_node
+  int arena_node = -1;
   std::shared_ptr<void> arena_owner;  // shared by dp_model_clone instances
   int64_t arena_bytes = 0;
   dp::DevState dev[DP_MAX_DEVICES];

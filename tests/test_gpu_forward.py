@@ -349,3 +349,22 @@ def test_graph_replay_after_workspace_regrowth():
         model.evict(0)
     model.close()
     c.close()
+
+
+@pytest.mark.parametrize("name,S", [("bert_large", 384), ("gpt2", 256), ("tiny_roberta", 77)])
+def test_attention_tc_engine_option(name, S):
+    """opts.attention_tc runs every layer's attention on K5t: the whole cold start stays within the
+    north star's tolerance of the oracle."""
+    m = synth.SHAPES[name]
+    w = synth.make_weights(m, seed=41, dtype="fp16")
+    ids = synth.make_ids(m, 1, S, seed=42)
+    ref, ref_pool = F.forward(m, w, ids, "fp16")
+    c = dp().Context([0])
+    c.set_opts(attention_tc=1)
+    model = dp().Model(c, m, w, "fp16")
+    plan = dp().plan_generate(fake_cost(m, "fp16"), "DHA", 1)
+    out, pool, _ = run_cold(model, plan, ids, "fp16")
+    model.evict(0)
+    assert np.abs(f64(out) - ref.reshape(S, -1)).max() <= 1e-2
+    model.close()
+    c.close()

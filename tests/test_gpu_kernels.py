@@ -243,6 +243,26 @@ def test_attention_parity(B, S, H, heads, causal, dtype):
     assert np.all(err <= tol), err.max()
 
 
+@pytest.mark.parametrize("B,S,H,heads", [(1, 32, 128, 2), (2, 77, 256, 4), (1, 128, 768, 12), (1, 384, 1024, 16),
+                                         (1, 1024, 1024, 16), (3, 200, 256, 4)])
+@pytest.mark.parametrize("causal", [False, True])
+@pytest.mark.parametrize("dtype", ["fp16", "bf16"])
+def test_attention_tc_parity(B, S, H, heads, causal, dtype):
+    """K5t (tcgen05: S and P.V in TMEM, one softmax row per thread) against the oracle, same bound as
+    K5 (P is rounded to the storage type before P.V)."""
+    rng = np.random.default_rng(B * 1000 + S + H + 7)
+    qkv = synth.round_to((1.5 * rng.standard_normal((B * S, 3 * H))).astype(np.float32), dtype)
+    Q = to_t(qkv, dtype)
+    O = torch.empty(B * S, H, dtype=DT[dtype], device="cuda")
+    dp().attention_tc(Q, 3 * H, O, B, S, H, heads, causal, dtype)
+    torch.cuda.synchronize()
+    q64 = synth.storage_to_f64(qkv, dtype).reshape(B, S, 3 * H)
+    ref = F.attention(q64[..., :H], q64[..., H:2 * H], q64[..., 2 * H:], heads, causal).reshape(B * S, H)
+    tol = (4 if dtype == "fp16" else 8) * EPS_OUT[dtype] * (np.abs(ref) + np.abs(q64).max())
+    err = np.abs(f64(O) - ref)
+    assert np.all(err <= tol), err.max()
+
+
 def test_fp32_residual_stream_io():
     """GPT-2's pre-LN residual stream stays fp32: linear with fp32 residual+output (io=3),
     LayerNorm reading fp32, embedding writing fp32."""

@@ -77,3 +77,21 @@ def test_numa_queries_on_this_host():
         assert dp.host_numa_node(p) in (0, -1)
     finally:
         dp.host_free(p)
+
+
+@pytest.mark.gpu
+def test_weight_arena_is_on_the_serving_gpus_numa_node():
+    import synth
+    m = synth.SHAPES["tiny_bert"]
+    ctx = dp.Context([0])
+    model = dp.Model(ctx, m, synth.make_weights(m, seed=0))
+    node = dp.device_numa_node(0)
+    page = model.arena().ctypes.data
+    got = dp.host_numa_node(page)
+    if node >= 0 and got >= 0:
+        assert got == node
+    model.close()
+    ctx.close()
+    # the concurrent probe on one device equals a solo measurement in kind (GB/s of a PCIe link)
+    gbs = dp.measure_h2d_concurrent([0], 64 << 20, 3)
+    assert 5.0 < gbs[0] < 200.0

@@ -100,6 +100,35 @@ if which in ("all", "embed"):
     us = timeit(lambda: dp.embed(ids, S, word, pos, typ, g, bb, H, 1e-12, out), n=20)
     res["embed DHA S128 H768"] = {"us": round(us, 2), "pcie_gbs": round((2 * S + 3) * H * 2 / us / 1e3, 1)}
 
+if which in ("all", "lnhost"):
+    # DHA LayerNorm: gamma / beta host-mapped, read once per launch (one cluster, DSMEM broadcast)
+    for rows, n in [(128, 768), (384, 1024)]:
+        x = torch.randn(rows, n, device="cuda").half()
+        g = dp.host_alloc(n * 2)
+        bb = dp.host_alloc(n * 2)
+        y = torch.empty_like(x)
+        us = timeit(lambda: dp.layernorm(x, None, g, bb, y, rows, n, 1e-5), n=20)
+        res[f"layernorm DHA {rows}x{n}"] = {"us": round(us, 2), "host_bytes": 4 * n}
+        dp.host_free(g)
+        dp.host_free(bb)
+if which in ("all", "fp32"):
+    # fp32 storage (DP_FP32): the CUDA-core linear with weights from host (DHA) and HBM, attention
+    for (M, N, K) in [(128, 768, 768), (128, 3072, 768)]:
+        x = torch.randn(M, K, device="cuda")
+        wh = dp.host_alloc(N * K * 4)
+        wd = torch.randn(N, K, device="cuda")
+        y = torch.empty(M, N, device="cuda")
+        us_h = timeit(lambda: dp.linear(x, K, wh, None, None, 0, y, N, M, N, K, path=1, dtype="fp32"), n=10)
+        us_d = timeit(lambda: dp.linear(x, K, wd, None, None, 0, y, N, M, N, K, path=1, dtype="fp32"), n=20)
+        res[f"fp32 linear M{M} N{N} K{K}"] = {"us_host": round(us_h, 2), "pcie_gbs": round(N * K * 4 / us_h / 1e3, 1),
+                                             "us_hbm": round(us_d, 2), "tflops_hbm": round(2 * M * N * K / us_d / 1e6, 2)}
+        dp.host_free(wh)
+    for S, causal in ((128, 0), (1024, 1)):
+        H, heads = 768, 12
+        qkv = torch.randn(S, 3 * H, device="cuda")
+        o = torch.empty(S, H, device="cuda")
+        us = timeit(lambda: dp.attention(qkv, 3 * H, o, 1, S, H, heads, causal, dtype="fp32"), n=10)
+        res[f"fp32 attention S{S} causal{causal}"] = {"us": round(us, 2)}
 if which in ("all", "ptfwd"):
     # SM-driven PT forwarder vs the copy engine, host -> this GPU's HBM (on one GPU
     # the NVLink hop of the multi-GPU case is a local store): the per-link read side of PT.
