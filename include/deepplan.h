@@ -83,7 +83,7 @@ enum {
  * Errors
  * --------------------------------------------------------------------------------- */
 const char* dp_last_error(void);
-int32_t dp_abi_version(void); /* 1 */
+int32_t dp_abi_version(void); /* 2 (round 2: dp_serve_result / dp_serve_opts / dp_engine_opts fields) */
 
 /* ---------------------------------------------------------------------------------
  * Planner (pure host code, deterministic, no GPU).  §4.3.2-4.3.3, SURVEY §8(c) P1-P4.

@@ -71,10 +71,12 @@ def replay_online(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, resident_
     finish_ns[q] <= decide_ns[r].  In arrival order:
       * instance resident (or becoming resident) on g  -> warm on g;
       * else cold on the GPU with the fewest outstanding (decided, not complete) requests, lowest
-        index on ties; there, least recently used resident instances with no outstanding request
-        are evicted until the instance's resident bytes fit the budget (if none can go,
-        the GPU runs over budget until they finish).
-    resident_bytes is per INSTANCE (its plan's loaded units).  Returns gpu, cold, nevicted."""
+        index on ties;
+      * then, on that GPU, while its resident bytes exceed the budget, the least recently used
+        resident instance other than this one with no outstanding request is evicted; if
+        none can go the GPU runs over budget until a later decision on it can evict.
+    resident_bytes is per INSTANCE (its plan's loaded units).  Returns gpu, cold, nevicted and
+    `resident`: {gpu: sorted instances resident there after the last decision}."""
     n = len(arrival_ns)
     gpu = np.full(n, -1, dtype=np.int64)
     cold = np.zeros(n, dtype=np.int64)
@@ -92,18 +94,19 @@ def replay_online(arrival_ns, instance, *, ngpu, per_gpu_budget_bytes, resident_
         else:
             busy = [sum(1 for q in live if gpu[q] == x) for x in range(ngpu)]
             g = min(range(ngpu), key=lambda x: (busy[x], x))
-            pend = {int(instance[q]) for q in live}
-            for v in list(lru[g].keys()):
-                if used[g] + int(resident_bytes[i]) <= per_gpu_budget_bytes:
-                    break
-                if v in pend:
-                    continue
-                used[g] -= lru[g].pop(v)
-                del home[v]
-                nev[r] += 1
             lru[g][i] = int(resident_bytes[i])
             used[g] += int(resident_bytes[i])
             home[i] = g
             cold[r] = 1
+        pend = {int(instance[q]) for q in live}
+        for v in list(lru[g].keys()):
+            if used[g] <= per_gpu_budget_bytes:
+                break
+            if v == i or v in pend:
+                continue
+            used[g] -= lru[g].pop(v)
+            del home[v]
+            nev[r] += 1
         gpu[r] = g
-    return {"gpu": gpu, "cold": cold, "nevicted": nev}
+    return {"gpu": gpu, "cold": cold, "nevicted": nev,
+            "resident": {x: sorted(lru[x].keys()) for x in range(ngpu)}}

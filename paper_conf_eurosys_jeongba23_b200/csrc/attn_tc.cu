@@ -2,11 +2,13 @@
 //
 //   ctx[q, h*64 : h*64+64] = softmax(q_h k_h^T / 8 [+ causal mask]) v_h
 //
-// One CTA (128 threads) per (head, 128-query tile, sequence).  Per 128-key tile j:
+// One CTA (256 threads) per (head, 128-query tile, sequence).  Per 128-key tile j:
 //   1. S = Q K_j^T on tcgen05 (M = 128 queries, N = 128 keys, K = 64), fp32 in TMEM columns
 //      [0, 128); Q and K_j arrive by TMA (128-byte swizzle), K double-buffered;
-//   2. thread r owns query row r = TMEM lane r: it reads its whole row of S (tcgen05.ld), masks,
-//      and runs the online softmax in fp32 with exp2 (no shuffles: the row is in one thread);
+//   2. two threads own query row r = TMEM lane r (warps w and w + 4 read the lane quarter w % 4),
+//      each half of its S row (tcgen05.ld): masks, the online softmax in fp32 with exp2 (the
+//      halves' maxima meet in shared memory; each keeps a partial row sum under the same
+//      corrections);
 //      the numerators P (storage type) go to shared memory as the next MMA's A operand, written
 //      in the 128-byte-swizzled K-major layout by hand; V_j (loaded to registers under step 1) is
 //      written transposed (V_j^T: d rows, keys along K) as the B operand;
@@ -46,7 +48,7 @@ __device__ __forceinline__ uint32_t sw128_off(int r, int k) {
 }
 
 template <class T>
-__global__ void __launch_bounds__(128, 1)
+__global__ void __launch_bounds__(256, 1)
     attention_tc_kernel(const __grid_constant__ CUtensorMap tmQK, const T* __restrict__ qkv, int ldqkv,
                         T* __restrict__ ctx, int seq, int H, int causal, float scale_log2) {
   extern __shared__ uint8_t smem_raw[];
@@ -55,8 +57,9 @@ __global__ void __launch_bounds__(128, 1)
   uint8_t* sK = sQ + Q_BYTES;           // [2][TK][64]
   uint8_t* sP = sK + 2 * K_BYTES;       // [2 k-blocks][TQ][64]
   uint8_t* sVt = sP + P_BYTES;          // [2 k-blocks][TD][64]
-  __shared__ __align__(8) uint64_t bar_q, bar_k[2], bar_s, bar_o;
+  __shared__ __align__(8) uint64_t bar_q, bar_k[2], bar_s[2], bar_o[2];
   __shared__ uint32_t tmem_base_sh;
+  __shared__ float red[2][TQ];          // per column half: partial row max (and at the end: row sum)
   // kind::f16, fp32 accumulate, A/B K-major; S: M 128 x N 128; O: M 128 x N 64
   constexpr uint32_t IDESC_S = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(TK >> 3) << 17) |
                                (uint32_t(TQ >> 4) << 24);
@@ -77,119 +80,132 @@ __global__ void __launch_bounds__(128, 1)
     mbar_init(&bar_q, 1);
     mbar_init(&bar_k[0], 1);
     mbar_init(&bar_k[1], 1);
-    mbar_init(&bar_s, 1);
-    mbar_init(&bar_o, 1);
+    mbar_init(&bar_s[0], 1);
+    mbar_init(&bar_s[1], 1);
+    mbar_init(&bar_o[0], 1);
+    mbar_init(&bar_o[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base_sh)),
-                 "r"(256));
+                 "r"(512));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = tmem_base_sh;
-  const uint32_t t_s = tmem, t_o = tmem + 128;
+  // TMEM: S double buffer in columns [0, 256), O double buffer in [256, 384)
+  auto t_s = [&](int b) { return tmem + 128u * uint32_t(b); };
+  auto t_o = [&](int b) { return tmem + 256u + 64u * uint32_t(b); };
   pdl_trigger();
   pdl_wait();  // q, k, v come from the previous kernel
 
   const int qcol = head * TD, kcol = H + head * TD;
   const T* vbase = qkv + (size_t)tok0 * ldqkv + 2 * H + head * TD;
+  // thread (warp w, lane l): query row r = 32 (w % 4) + l (its TMEM lane), column half h = w / 4
+  // -- keys [64 h, 64 h + 64) of each S tile, head dims [32 h, 32 h + 32) of O
+  const int r = (warp & 3) * 32 + lane, h = warp >> 2;
+  const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
+  const int qrow = q0 + r;
+  auto issue_s = [&](int jj) {  // S_jj = Q K_jj^T into TMEM buffer jj & 1 (K_jj must be landing)
+    mbar_wait(&bar_k[jj & 1], (jj >> 1) & 1);
+    asm volatile("tcgen05.fence::after_thread_sync;");
+    const uint64_t dq = sw128_desc(sQ), dk = sw128_desc(sK + (jj & 1) * K_BYTES);
+#pragma unroll
+    for (int kk = 0; kk < TD / 16; ++kk) umma_f16(t_s(jj & 1), dq + 2 * kk, dk + 2 * kk, IDESC_S, kk != 0);
+    umma_commit(&bar_s[jj & 1]);
+  };
   if (tid == 0) {
     mbar_expect_tx(&bar_q, Q_BYTES);
     tma_load_2d(&tmQK, &bar_q, sQ, qcol, tok0 + q0);
-    mbar_expect_tx(&bar_k[0], K_BYTES);
-    tma_load_2d(&tmQK, &bar_k[0], sK, kcol, tok0);
+    for (int jj = 0; jj < 2 && jj < nkt; ++jj) {
+      mbar_expect_tx(&bar_k[jj], K_BYTES);
+      tma_load_2d(&tmQK, &bar_k[jj], sK + jj * K_BYTES, kcol, tok0 + jj * TK);
+    }
+    mbar_wait(&bar_q, 0);
+    issue_s(0);
   }
-  const int r = warp * 32 + lane;  // query row of this thread (TMEM lane)
-  const int qrow = q0 + r;
-  float o[TD];
+  float o[TD / 2];
 #pragma unroll
-  for (int d = 0; d < TD; ++d) o[d] = 0.f;
-  float mrow = -INFINITY, lrow = 0.f;
+  for (int d = 0; d < TD / 2; ++d) o[d] = 0.f;
+  float mrow = -INFINITY, lrow = 0.f;  // lrow: this half's partial row sum (same corrections)
+  float corr_prev = 0.f;               // the correction that goes with the O tile in flight
 
+  // Software pipeline per key tile j: S_{j+1} is computed on the tensor core while the threads run
+  // the softmax of tile j, and O_j = P_j V_j is added to the registers one iteration later.
   for (int j = 0; j < nkt; ++j) {
     const int k0 = j * TK;
-    // V_j: thread t loads key k0 + t (its 128-byte row) into registers under the S MMA
-    uint4 vr[8];
+    // V_j: thread t loads head dims [32 (t / 128), +32) of key k0 + t % 128 (latency hidden below)
+    const int vkey = tid & 127, vh = tid >> 7;
+    uint4 vr[4];
     {
-      const bool ok = k0 + tid < seq;
-      const uint4* src = reinterpret_cast<const uint4*>(vbase + (size_t)(ok ? k0 + tid : 0) * ldqkv);
+      const bool ok = k0 + vkey < seq;
+      const uint4* src = reinterpret_cast<const uint4*>(vbase + (size_t)(ok ? k0 + vkey : 0) * ldqkv + 32 * vh);
 #pragma unroll
-      for (int c = 0; c < 8; ++c) vr[c] = ok ? src[c] : make_uint4(0, 0, 0, 0);
+      for (int c = 0; c < 4; ++c) vr[c] = ok ? src[c] : make_uint4(0, 0, 0, 0);
     }
-    if (tid == 0) {
-      if (j + 1 < nkt) {  // next key tile into the other buffer (its last reader, S_{j-1}, is done)
-        mbar_expect_tx(&bar_k[(j + 1) & 1], K_BYTES);
-        tma_load_2d(&tmQK, &bar_k[(j + 1) & 1], sK + ((j + 1) & 1) * K_BYTES, kcol, tok0 + k0 + TK);
-      }
-      if (j == 0) mbar_wait(&bar_q, 0);
-      mbar_wait(&bar_k[j & 1], (j >> 1) & 1);
-      asm volatile("tcgen05.fence::after_thread_sync;");
-      const uint64_t dq = sw128_desc(sQ), dk = sw128_desc(sK + (j & 1) * K_BYTES);
-#pragma unroll
-      for (int kk = 0; kk < TD / 16; ++kk) umma_f16(t_s, dq + 2 * kk, dk + 2 * kk, IDESC_S, kk != 0);
-      umma_commit(&bar_s);
-    }
-    // V_j^T into the B-operand tile: element (d, key t) of K-block t / 64
-    {
-      uint8_t* vt = sVt + (tid >> 6) * (TD * 64 * 2);
-      const int kk = tid & 63;
-#pragma unroll
-      for (int c = 0; c < 8; ++c) {
-        const uint32_t w4[4] = {vr[c].x, vr[c].y, vr[c].z, vr[c].w};
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const int d = c * 8 + e * 2;
-          *reinterpret_cast<uint16_t*>(vt + sw128_off(d, kk)) = uint16_t(w4[e] & 0xFFFFu);
-          *reinterpret_cast<uint16_t*>(vt + sw128_off(d + 1, kk)) = uint16_t(w4[e] >> 16);
-        }
-      }
-    }
-    // S row -> online softmax -> P row (one thread spins on the MMA, the CTA barrier releases all)
-    if (tid == 0) mbar_wait_spin(&bar_s, j & 1);
-    __syncthreads();
+    // (1) the next S on the tensor core (its buffer was last read in iteration j - 1)
+    if (tid == 0 && j + 1 < nkt) issue_s(j + 1);
+    // (2) S_j ready; K_j's buffer is free again -> K_{j+2}
+    mbar_wait_spin(&bar_s[j & 1], (j >> 1) & 1);
     asm volatile("tcgen05.fence::after_thread_sync;");
-    float s[TK];
+    if (tid == 0 && j + 2 < nkt) {
+      mbar_expect_tx(&bar_k[j & 1], K_BYTES);
+      tma_load_2d(&tmQK, &bar_k[j & 1], sK + (j & 1) * K_BYTES, kcol, tok0 + k0 + 2 * TK);
+    }
+    // (3) this half of the S row -> online softmax
+    float s[TK / 2];
     {
-      uint32_t v[TK];  // all 8 loads in flight, one completion wait
+      uint32_t v[TK / 2];
 #pragma unroll
-      for (int c = 0; c < TK; c += 16) tmem_ld16_nowait(t_s + (uint32_t(warp * 32) << 16) + c, v + c);
+      for (int c = 0; c < TK / 2; c += 16) tmem_ld16_nowait(t_s(j & 1) + lane_base + 64 * h + c, v + c);
       tmem_ld_wait();
 #pragma unroll
-      for (int e = 0; e < TK; ++e) s[e] = __uint_as_float(v[e]) * scale_log2;
+      for (int e = 0; e < TK / 2; ++e) s[e] = __uint_as_float(v[e]) * scale_log2;
     }
-    // masking only where a key can be invalid: the sequence's last tile, or the causal diagonal
-    if (k0 + TK > seq || (causal && k0 + TK - 1 > q0)) {
+    const int kbase = k0 + 64 * h;
+    if (kbase + 64 > seq || (causal && kbase + 63 > qrow)) {  // only where a key can be invalid
 #pragma unroll
-      for (int e = 0; e < TK; ++e) {
-        const int key = k0 + e;
+      for (int e = 0; e < TK / 2; ++e) {
+        const int key = kbase + e;
         if (key >= seq || (causal && key > qrow)) s[e] = -INFINITY;
       }
     }
     float mx = -INFINITY;
 #pragma unroll
-    for (int e = 0; e < TK; ++e) mx = fmaxf(mx, s[e]);
-    const float mnew = fmaxf(mrow, mx);
+    for (int e = 0; e < TK / 2; ++e) mx = fmaxf(mx, s[e]);
+    red[h][r] = mx;
+    __syncthreads();
+    const float mnew = fmaxf(mrow, fmaxf(red[0][r], red[1][r]));
     const float corr = (mrow == -INFINITY) ? 0.f : exp2f(mrow - mnew);
     float rs = 0.f;
 #pragma unroll
-    for (int e = 0; e < TK; e += 2) {
-      const float p0 = (mnew == -INFINITY) ? 0.f : exp2f(s[e] - mnew);
-      const float p1 = (mnew == -INFINITY) ? 0.f : exp2f(s[e + 1] - mnew);
-      rs += p0 + p1;
-      s[e] = p0;
-      s[e + 1] = p1;
+    for (int e = 0; e < TK / 2; ++e) {
+      const float p = (mnew == -INFINITY) ? 0.f : exp2f(s[e] - mnew);
+      rs += p;
+      s[e] = p;
     }
     lrow = lrow * corr + rs;
     mrow = mnew;
+    // (4) O_{j-1} has landed: add it (with the correction of its own tile); P and V^T are free
+    if (j > 0) {
+      mbar_wait_spin(&bar_o[(j - 1) & 1], ((j - 1) >> 1) & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      uint32_t v[TD / 2];
 #pragma unroll
-    for (int kb = 0; kb < 2; ++kb) {  // P row r into K-blocks kb (keys 64 kb .. 64 kb + 63)
-      uint8_t* pt = sP + kb * (TQ * 64 * 2);
+      for (int c = 0; c < TD / 2; c += 16) tmem_ld16_nowait(t_o((j - 1) & 1) + lane_base + 32 * h + c, v + c);
+      tmem_ld_wait();
+#pragma unroll
+      for (int e = 0; e < TD / 2; ++e) o[e] = o[e] * corr_prev + __uint_as_float(v[e]);
+    }
+    corr_prev = corr;
+    // (5) P_j row half (K-block h) and V_j^T into the operand tiles
+    {
+      uint8_t* pt = sP + h * (TQ * 64 * 2);
 #pragma unroll
       for (int c = 0; c < 8; ++c) {
-        const float* pp = s + kb * 64 + c * 8;
+        const float* pp = s + c * 8;
         uint4 u;
         u.x = Cvt<T>::from2(pp[0], pp[1]);
         u.y = Cvt<T>::from2(pp[2], pp[3]);
@@ -197,41 +213,53 @@ __global__ void __launch_bounds__(128, 1)
         u.w = Cvt<T>::from2(pp[6], pp[7]);
         *reinterpret_cast<uint4*>(pt + sw128_off(r, c * 8)) = u;
       }
+      uint8_t* vt = sVt + (vkey >> 6) * (TD * 64 * 2);
+      const int kk = vkey & 63;
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        const uint32_t w4[4] = {vr[c].x, vr[c].y, vr[c].z, vr[c].w};
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int d = 32 * vh + c * 8 + e * 2;
+          *reinterpret_cast<uint16_t*>(vt + sw128_off(d, kk)) = uint16_t(w4[e] & 0xFFFFu);
+          *reinterpret_cast<uint16_t*>(vt + sw128_off(d + 1, kk)) = uint16_t(w4[e] >> 16);
+        }
+      }
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // P, V^T -> the tensor core
     asm volatile("tcgen05.fence::before_thread_sync;");
     __syncthreads();
+    // (6) O_j = P_j V_j into TMEM buffer j & 1
     if (tid == 0) {
       asm volatile("tcgen05.fence::after_thread_sync;");
 #pragma unroll
       for (int kb = 0; kb < 2; ++kb) {
         const uint64_t dp_ = sw128_desc(sP + kb * (TQ * 64 * 2)), dv = sw128_desc(sVt + kb * (TD * 64 * 2));
 #pragma unroll
-        for (int kk = 0; kk < 4; ++kk) umma_f16(t_o, dp_ + 2 * kk, dv + 2 * kk, IDESC_O, (kb | kk) != 0);
+        for (int kk = 0; kk < 4; ++kk) umma_f16(t_o(j & 1), dp_ + 2 * kk, dv + 2 * kk, IDESC_O, (kb | kk) != 0);
       }
-      umma_commit(&bar_o);
+      umma_commit(&bar_o[j & 1]);
     }
-    if (tid == 0) mbar_wait_spin(&bar_o, j & 1);
-    __syncthreads();
-    asm volatile("tcgen05.fence::after_thread_sync;");
-    {
-      uint32_t v[TD];
-#pragma unroll
-      for (int c = 0; c < TD; c += 16) tmem_ld16_nowait(t_o + (uint32_t(warp * 32) << 16) + c, v + c);
-      tmem_ld_wait();
-#pragma unroll
-      for (int e = 0; e < TD; ++e) o[e] = o[e] * corr + __uint_as_float(v[e]);
-    }
-    // every thread has read S and O_j before the next tile's MMAs overwrite them
-    asm volatile("tcgen05.fence::before_thread_sync;");
-    __syncthreads();
-    asm volatile("tcgen05.fence::after_thread_sync;");
   }
-  if (qrow < seq) {
-    const float inv = lrow > 0.f ? 1.f / lrow : 0.f;
-    uint4* dst = reinterpret_cast<uint4*>(ctx + (size_t)(tok0 + qrow) * H + head * TD);
+  {  // the last O tile
+    const int jl = nkt - 1;
+    mbar_wait_spin(&bar_o[jl & 1], (jl >> 1) & 1);
+    asm volatile("tcgen05.fence::after_thread_sync;");
+    uint32_t v[TD / 2];
 #pragma unroll
-    for (int c = 0; c < 8; ++c) {
+    for (int c = 0; c < TD / 2; c += 16) tmem_ld16_nowait(t_o(jl & 1) + lane_base + 32 * h + c, v + c);
+    tmem_ld_wait();
+#pragma unroll
+    for (int e = 0; e < TD / 2; ++e) o[e] = o[e] * corr_prev + __uint_as_float(v[e]);
+  }
+  red[h][r] = lrow;  // the two halves' partial sums
+  __syncthreads();
+  if (qrow < seq) {
+    const float l = red[0][r] + red[1][r];
+    const float inv = l > 0.f ? 1.f / l : 0.f;
+    uint4* dst = reinterpret_cast<uint4*>(ctx + (size_t)(tok0 + qrow) * H + head * TD + 32 * h);
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
       uint4 u;
       u.x = Cvt<T>::from2(o[c * 8 + 0] * inv, o[c * 8 + 1] * inv);
       u.y = Cvt<T>::from2(o[c * 8 + 2] * inv, o[c * 8 + 3] * inv);
@@ -242,7 +270,7 @@ __global__ void __launch_bounds__(128, 1)
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256));
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
 }
 
 }  // namespace
@@ -265,7 +293,7 @@ void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int b
     if (first_on_device(attr))
       DP_CUDA(cudaFuncSetAttribute(attention_tc_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)SMEM_BYTES));
-    launch_kernel(attention_tc_kernel<T>, grid, dim3(128), SMEM_BYTES, s, m, (const T*)qkv, ldqkv, (T*)ctx, seq, H,
+    launch_kernel(attention_tc_kernel<T>, grid, dim3(256), SMEM_BYTES, s, m, (const T*)qkv, ldqkv, (T*)ctx, seq, H,
                   causal ? 1 : 0, scale_log2);
   };
   if (dtype == DP_BF16)

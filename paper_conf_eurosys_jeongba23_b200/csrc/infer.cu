@@ -252,7 +252,7 @@ static void ensure_peer_access(int from, int to) {
 }
 
 extern "C" const char* dp_last_error(void) { return g_last_error.c_str(); }
-extern "C" int32_t dp_abi_version(void) { return 1; }
+extern "C" int32_t dp_abi_version(void) { return 2; }  // 2: round-2 structs (serve result, opts)
 
 extern "C" dp_status dp_context_create(const int32_t* devs, int32_t ndev, dp_context** out) {
   dp_context* ctx = nullptr;

@@ -8,11 +8,11 @@
 //      state (R11-live):
 //        * the instance is (or is becoming) resident on GPU g -> warm, queued on g;
 //        * otherwise cold, on the GPU with the fewest outstanding requests (running + queued;
-//          ties: lowest index); there, least recently used instances with no outstanding
-//          request are evicted until the instance's resident bytes fit the per-GPU
-//          budget.  Resident bytes are the instance's LOADED units only (its plan's compact
-//          slot layout): DHA units stay in host memory, which is how DeepPlan "serves more
-//          instances";
+//          ties: lowest index);
+//        * then, while that GPU's resident bytes exceed the per-GPU budget, the least recently
+//          used instance other than this one with no outstanding request is evicted.
+//          Resident bytes are the instance's LOADED units only (its plan's compact slot layout):
+//          DHA units stay in host memory, which is how DeepPlan "serves more instances";
 //   3. starts: every idle GPU with a queued request runs the next one (one request per GPU
 //      at a time): the evictions decided for it (dp_model_evict -- the HBM block returns to the
 //      pool), then dp_infer_cold / dp_infer_warm on the GPU's stream and a completion event.
@@ -230,10 +230,18 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
           auto outstanding = [&](int x) { return (gpu[x].running >= 0 ? 1 : 0) + (int)gpu[x].queue.size(); };
           for (int x = 1; x < G; ++x)
             if (outstanding(x) < outstanding(g)) g = x;
+          gpu[g].used += rbytes[inst];
+          where[inst] = g;
+          res.cold = 1;
+        }
+        // while the GPU is over its budget: evict the least recently used resident instance other
+        // than this one with no outstanding request; if none can go, it stays over budget
+        // until a later decision on this GPU can evict
+        {
           Gpu& q = gpu[g];
-          for (auto it = q.lru.begin(); it != q.lru.end() && q.used + rbytes[inst] > o.per_gpu_budget_bytes;) {
+          for (auto it = q.lru.begin(); it != q.lru.end() && q.used > o.per_gpu_budget_bytes;) {
             const int v = *it;
-            if (pending[v] > 0) {  // still has work on this GPU: not a victim
+            if (v == inst || pending[v] > 0) {
               ++it;
               continue;
             }
@@ -242,10 +250,6 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
             where[v] = -1;
             j.victims.push_back(v);
           }
-          // (if every resident instance still has work, the GPU runs over budget until they finish)
-          q.used += rbytes[inst];
-          where[inst] = g;
-          res.cold = 1;
           res.nevicted = (int32_t)j.victims.size();
         }
         gpu[g].lru.push_back(inst);

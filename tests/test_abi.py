@@ -24,7 +24,7 @@ def test_library_exports_every_declared_symbol():
     import paper_conf_eurosys_jeongba23_b200 as dp
     for name in _declared():
         assert hasattr(dp.lib, name), name
-    assert dp.lib.dp_abi_version() == 1
+    assert dp.lib.dp_abi_version() == 2
 
 
 def test_error_path_sets_last_error():

@@ -145,7 +145,7 @@ def test_timeline_gates_and_tracks_the_simulator(mode):
     # wait's latency
     pre = start - stall
     want = np.where(loaded, np.maximum(0, ready - pre), 0)
-    assert np.all(np.abs(stall - want) <= 15_000), np.abs(stall - want).max()
+    assert np.all(np.abs(stall - want) <= 30_000), np.abs(stall - want).max()
     # against the simulator on the same live profile (R23 calibration).  Tracing puts two events
     # around every unit (no PDL overlap), which slows the compute chain and hides some stall, so
     # the comparison is loose; the paper-model DHA plan is known to under-predict (it ignores

@@ -65,6 +65,13 @@ if which in ("all", "attn"):
         us = timeit(lambda: dp.attention(qkv, 3 * H, o, B, S, H, heads, causal))
         fl = 4 * S * S * H * B * (0.5 if causal else 1)
         res[f"attention S{S} H{H} causal{causal}"] = {"us": round(us, 2), "tflops": round(fl / us / 1e6, 2)}
+if which in ("all", "attn", "attn_tc"):  # K5t (tcgen05; opts.attention_tc) at the same shapes
+    for B, S, H, heads, causal in [(1, 128, 768, 12, 0), (1, 384, 1024, 16, 0), (1, 1024, 1024, 16, 1)]:
+        qkv = torch.randn(B * S, 3 * H, device="cuda").half()
+        o = torch.empty(B * S, H, device="cuda").half()
+        us = timeit(lambda: dp.attention_tc(qkv, 3 * H, o, B, S, H, heads, causal))
+        fl = 4 * S * S * H * B * (0.5 if causal else 1)
+        res[f"attention_tc S{S} H{H} causal{causal}"] = {"us": round(us, 2), "tflops": round(fl / us / 1e6, 2)}
 if which in ("all", "skinny"):
     for (M, N, K) in [(128, 768, 768), (128, 3072, 768), (128, 768, 3072), (1, 768, 768)]:
         x = torch.randn(M, K, device="cuda").half()

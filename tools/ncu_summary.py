@@ -84,6 +84,19 @@ ALGO = {
                    "bytes": 2 * 50257 * 768},
     "attention_k5b": {"shape": "B1 S384 H1024 16 heads, 4 key-tile groups (K5b)", "flops": 4 * 384 * 384 * 1024},
     "pt_forward": {"shape": "32 MiB pinned host -> HBM, SM forwarder (K7)", "host_bytes": 32 << 20},
+    # round 2 (tools/evidence_r02.sh)
+    "gemm_M384_N4096_K1024": {"shape": "M384 N4096 K1024 (BERT-Large fc1 at S384)",
+                              "bytes": 2 * (4096 * 1024 + 384 * 1024 + 384 * 4096), "flops": 2 * 384 * 4096 * 1024},
+    "gemm_M1024_N4096_K1024": {"shape": "M1024 N4096 K1024 (GPT-2 Medium c_fc at S1024)",
+                               "bytes": 2 * (4096 * 1024 + 1024 * 1024 + 1024 * 4096), "flops": 2 * 1024 * 4096 * 1024},
+    "attention_s128": {"shape": "B1 S128 H768 12 heads (K5)", "flops": 4 * 128 * 128 * 768},
+    "attention_s384": {"shape": "B1 S384 H1024 16 heads (K5b)", "flops": 4 * 384 * 384 * 1024},
+    "attention_s1024_causal": {"shape": "B1 S1024 H1024 16 heads causal (K5b; half the S^2 term)",
+                               "flops": 2 * 1024 * 1024 * 1024},
+    "layernorm_dha": {"shape": "128 x 768, gamma/beta in pinned host memory (one cluster, DSMEM broadcast)",
+                      "host_bytes": 2 * 2 * 768},
+    "fp32_linear_dha": {"shape": "fp32 M128 N768 K768, W in pinned host memory (read once)",
+                        "host_bytes": 4 * 768 * 768},
 }
 
 
