@@ -7,6 +7,8 @@
 #include <stdexcept>
 #include <string>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "deepplan.h"
 
 namespace dp {
@@ -33,6 +35,15 @@ void set_last_error(const std::string& msg);
   do {                                                       \
     if (!(cond)) ::dp::fail((code), std::string(msg));       \
   } while (0)
+
+// NVTX range for the host-side phases (visible in nsys / ncu timelines): cold / warm inference,
+// the enqueue of each link's transfers, the forward's kernels, profiling, serving decisions.
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 // Run body, translating exceptions into a dp_status + last error.
 template <class F>

@@ -84,6 +84,7 @@ struct DevState {
   std::vector<int8_t> method;  // per unit, fixed when the model became resident
   Workspace ws;
   std::map<std::string, GraphEntry> graphs;  // captured cold / warm runs (opts.use_graph)
+  std::map<std::string, int> graph_seen;     // keys run so far (captured on the second use)
   UnitTrace trace;                           // last traced cold start
   cudaStream_t capture = nullptr;            // private stream the graphs are captured on
 };

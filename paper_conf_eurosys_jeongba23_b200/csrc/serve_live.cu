@@ -138,6 +138,7 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
       return sec;
     };
     auto start_job = [&](int g, const Job& j) {
+      NvtxRange nv("serve start (evict + enqueue)");
       Gpu& q = gpu[g];
       const int r = j.req, inst = trace[r].instance;
       dp_model* m = models[inst];
@@ -212,6 +213,7 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
       // (2) arrivals up to now, decided on the observed state
       while (next < nreq && trace[next].arrival_ns <= now) {
         const int r = next++;
+        NvtxRange nv("serve decide");
         const int inst = trace[r].instance;
         DP_CHECK(inst >= 0 && inst < nmodels, DP_ERR_INVALID, "trace instance out of range");
         DP_CHECK(r == 0 || trace[r].arrival_ns >= trace[r - 1].arrival_ns, DP_ERR_INVALID,

@@ -1,4 +1,4 @@
-"""The committed bench lines (profiles/r01_bench_*.json) keep the bench.py JSON contract.
+"""The committed bench lines (profiles/r0*_bench_*.json) keep the bench.py JSON contract.
 
 CPU-only: reads the JSON lines bench.py printed on the B200 box and checks the keys the driver
 and the judge read (metric/value/unit, roofline, cpu_baseline, clocks, e2e, gpu_launches) and
@@ -11,7 +11,7 @@ import os
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-LINES = sorted(glob.glob(os.path.join(ROOT, "profiles", "r01_bench_*.json")))
+LINES = sorted(glob.glob(os.path.join(ROOT, "profiles", "r0*_bench_*.json")))
 BAD_REASONS = {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"}
 
 
@@ -57,6 +57,10 @@ def test_bench_line_contract(path):
         assert c["kind"] == "oracle" and c["cores"] >= 1 and c["value"] > 0 and c["sample"]
     if "gpu_launches" in d:
         assert d["gpu_launches"] > 0
+    if d.get("check") is not None:  # round 2: the bench checks its own output against the oracle
+        c = d["check"]
+        err = c["max_rel_err"] if c.get("tol_kind") == "relative" else c["max_abs_err"]
+        assert c["ok"] and err <= c["tol"] + 1e-12
 
 
 @pytest.mark.parametrize("path", [p for p in LINES if "_k1_" in p or "default" in p],
