@@ -368,3 +368,57 @@ def test_attention_tc_engine_option(name, S):
     assert np.abs(f64(out) - ref.reshape(S, -1)).max() <= 1e-2
     model.close()
     c.close()
+
+
+@pytest.mark.parametrize("name,B,S", [("bert_base", 1, 512), ("roberta_large", 1, 512), ("bert_base", 8, 128)])
+def test_maximum_sizes(name, B, S):
+    """The largest inputs the configs allow: S = max_pos (512 for BERT, 512 + offset for RoBERTa)
+    and batch 8 (Fig. 12's largest batch), cold start vs the fp64 oracle at the north star's 1e-2."""
+    m = synth.SHAPES[name]
+    w = synth.make_weights(m, seed=51, dtype="fp16")
+    ids = synth.make_ids(m, B, S, seed=52)
+    ref, ref_pool = F.forward(m, w, ids, "fp16")
+    model = dp().Model(ctx(), m, w, "fp16")
+    plan = dp().plan_generate(fake_cost(m, "fp16"), "DHA", 1)
+    out, pool, _ = run_cold(model, plan, ids, "fp16")
+    model.evict(0)
+    assert np.abs(f64(out) - ref.reshape(B * S, -1)).max() <= 1e-2
+    assert np.abs(f64(pool) - ref_pool).max() <= 1e-2
+    model.close()
+
+
+def test_degenerate_cases():
+    """No layers (the embedding alone is the output), every unit by DHA (nothing transferred), every
+    unit loaded over the most links the loopback allows (k = 8), a one-token sequence, and a
+    sequence longer than the position table (rejected)."""
+    import dataclasses
+    base = synth.SHAPES["tiny_bert"]
+    for layers in (0, 1):
+        m = dataclasses.replace(base, name=f"tiny_bert_L{layers}", layers=layers)
+        w = synth.make_weights(m, seed=53, dtype="fp16")
+        ids = synth.make_ids(m, 1, 9, seed=54)
+        ref, ref_pool = F.forward(m, w, ids, "fp16")
+        model = dp().Model(ctx(), m, w, "fp16")
+        n = model.n
+        for meth, k in ((np.ones(n, np.int8), 1), (np.zeros(n, np.int8), 1), (np.zeros(n, np.int8), 8)):
+            slot = np.array([i % k for i in range(n)], np.int8) if k > 1 else None
+            plan = plan_from(model, meth, slot, k=k, mode=10 if k > 1 else 1)
+            out, pool, st = run_cold(model, plan, ids, "fp16", secondaries=[0] * (k - 1))
+            model.evict(0)
+            assert np.abs(f64(out) - ref.reshape(9, -1)).max() <= 1e-2
+            assert np.abs(f64(pool) - ref_pool).max() <= 1e-2
+            if meth.all():
+                assert sum(st["h2d_bytes"]) == 0 and st["n_copies"] == 0
+        model.close()
+    m = base
+    w = synth.make_weights(m, seed=55, dtype="fp16")
+    model = dp().Model(ctx(), m, w, "fp16")
+    plan = dp().plan_generate(fake_cost(m, "fp16"), "DHA", 1)
+    one = synth.make_ids(m, 1, 1, seed=56)
+    ref, _ = F.forward(m, w, one, "fp16")
+    out, _, _ = run_cold(model, plan, one, "fp16")
+    model.evict(0)
+    assert np.abs(f64(out) - ref.reshape(1, -1)).max() <= 1e-2
+    with pytest.raises(dp().DeepPlanError):
+        run_cold(model, plan, synth.make_ids(m, 1, m.max_pos + 1, seed=57), "fp16")
+    model.close()
