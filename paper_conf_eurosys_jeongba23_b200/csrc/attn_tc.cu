@@ -10,8 +10,8 @@
 //      halves' maxima meet in shared memory; each keeps a partial row sum under the same
 //      corrections);
 //      the numerators P (storage type) go to shared memory as the next MMA's A operand, written
-//      in the 128-byte-swizzled K-major layout by hand; V_j (loaded to registers under step 1) is
-//      written transposed (V_j^T: d rows, keys along K) as the B operand;
+//      in the 128-byte-swizzled K-major layout by hand; V_j arrives by TMA as [keys][head dims]
+//      and is the MN-major B operand as it lands (no transpose);
 //   3. O_j = P V_j on tcgen05 (M = 128, N = 64, K = 128 keys) into TMEM columns [128, 192);
 //   4. thread r accumulates o_r = o_r * corr + O_j[r] in registers.
 // After the last key tile o_r / l_r is stored (128 bytes per row).  Arithmetic contract: S and
@@ -39,8 +39,8 @@ constexpr int TD = 64;   // head dim
 constexpr uint32_t Q_BYTES = TQ * TD * 2;      // 16 KB
 constexpr uint32_t K_BYTES = TK * TD * 2;      // 16 KB
 constexpr uint32_t P_BYTES = TQ * TK * 2;      // 32 KB: two [128][64] swizzled K-blocks
-constexpr uint32_t VT_BYTES = TD * TK * 2;     // 16 KB: two [64][64] swizzled K-blocks
-constexpr uint32_t SMEM_BYTES = Q_BYTES + 2 * K_BYTES + P_BYTES + VT_BYTES + 1024;
+constexpr uint32_t V_BYTES = TK * TD * 2;      // 16 KB: [128 keys][64] swizzled (MN-major B operand)
+constexpr uint32_t SMEM_BYTES = Q_BYTES + 2 * K_BYTES + P_BYTES + 2 * V_BYTES + 1024;
 
 // byte offset of element (r, k) of a K-major [rows][64] tile with the 128-byte swizzle
 __device__ __forceinline__ uint32_t sw128_off(int r, int k) {
@@ -56,15 +56,16 @@ __global__ void __launch_bounds__(256, 1)
   uint8_t* sQ = smem;
   uint8_t* sK = sQ + Q_BYTES;           // [2][TK][64]
   uint8_t* sP = sK + 2 * K_BYTES;       // [2 k-blocks][TQ][64]
-  uint8_t* sVt = sP + P_BYTES;          // [2 k-blocks][TD][64]
-  __shared__ __align__(8) uint64_t bar_q, bar_k[2], bar_s[2], bar_o[2];
+  uint8_t* sV = sP + P_BYTES;           // [2][TK][64]: V tiles as TMA lands them (keys x head dims)
+  __shared__ __align__(8) uint64_t bar_q, bar_k[2], bar_v[2], bar_s[2], bar_o[2];
   __shared__ uint32_t tmem_base_sh;
   __shared__ float red[2][TQ];          // per column half: partial row max (and at the end: row sum)
   // kind::f16, fp32 accumulate, A/B K-major; S: M 128 x N 128; O: M 128 x N 64
   constexpr uint32_t IDESC_S = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(TK >> 3) << 17) |
                                (uint32_t(TQ >> 4) << 24);
-  constexpr uint32_t IDESC_O = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(TD >> 3) << 17) |
-                               (uint32_t(TQ >> 4) << 24);
+  // O: B = V_j is MN-major (head dims contiguous, keys along K): the transpose-B bit (16)
+  constexpr uint32_t IDESC_O = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (1u << 16) |
+                               (uint32_t(TD >> 3) << 17) | (uint32_t(TQ >> 4) << 24);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   // grid (heads, query tiles, batch); causal query tiles longest first
@@ -80,6 +81,8 @@ __global__ void __launch_bounds__(256, 1)
     mbar_init(&bar_q, 1);
     mbar_init(&bar_k[0], 1);
     mbar_init(&bar_k[1], 1);
+    mbar_init(&bar_v[0], 1);
+    mbar_init(&bar_v[1], 1);
     mbar_init(&bar_s[0], 1);
     mbar_init(&bar_s[1], 1);
     mbar_init(&bar_o[0], 1);
@@ -102,14 +105,14 @@ __global__ void __launch_bounds__(256, 1)
   pdl_wait();  // q, k, v come from the previous kernel
 
   const int qcol = head * TD, kcol = H + head * TD;
-  const T* vbase = qkv + (size_t)tok0 * ldqkv + 2 * H + head * TD;
+  const int vcol = 2 * H + head * TD;
   // thread (warp w, lane l): query row r = 32 (w % 4) + l (its TMEM lane), column half h = w / 4
   // -- keys [64 h, 64 h + 64) of each S tile, head dims [32 h, 32 h + 32) of O
   const int r = (warp & 3) * 32 + lane, h = warp >> 2;
   const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
   const int qrow = q0 + r;
   auto issue_s = [&](int jj) {  // S_jj = Q K_jj^T into TMEM buffer jj & 1 (K_jj must be landing)
-    mbar_wait(&bar_k[jj & 1], (jj >> 1) & 1);
+    mbar_wait_spin(&bar_k[jj & 1], (jj >> 1) & 1);
     asm volatile("tcgen05.fence::after_thread_sync;");
     const uint64_t dq = sw128_desc(sQ), dk = sw128_desc(sK + (jj & 1) * K_BYTES);
 #pragma unroll
@@ -122,8 +125,10 @@ __global__ void __launch_bounds__(256, 1)
     for (int jj = 0; jj < 2 && jj < nkt; ++jj) {
       mbar_expect_tx(&bar_k[jj], K_BYTES);
       tma_load_2d(&tmQK, &bar_k[jj], sK + jj * K_BYTES, kcol, tok0 + jj * TK);
+      mbar_expect_tx(&bar_v[jj], V_BYTES);
+      tma_load_2d(&tmQK, &bar_v[jj], sV + jj * V_BYTES, vcol, tok0 + jj * TK);
     }
-    mbar_wait(&bar_q, 0);
+    mbar_wait_spin(&bar_q, 0);
     issue_s(0);
   }
   float o[TD / 2];
@@ -136,15 +141,6 @@ __global__ void __launch_bounds__(256, 1)
   // the softmax of tile j, and O_j = P_j V_j is added to the registers one iteration later.
   for (int j = 0; j < nkt; ++j) {
     const int k0 = j * TK;
-    // V_j: thread t loads head dims [32 (t / 128), +32) of key k0 + t % 128 (latency hidden below)
-    const int vkey = tid & 127, vh = tid >> 7;
-    uint4 vr[4];
-    {
-      const bool ok = k0 + vkey < seq;
-      const uint4* src = reinterpret_cast<const uint4*>(vbase + (size_t)(ok ? k0 + vkey : 0) * ldqkv + 32 * vh);
-#pragma unroll
-      for (int c = 0; c < 4; ++c) vr[c] = ok ? src[c] : make_uint4(0, 0, 0, 0);
-    }
     // (1) the next S on the tensor core (its buffer was last read in iteration j - 1)
     if (tid == 0 && j + 1 < nkt) issue_s(j + 1);
     // (2) S_j ready; K_j's buffer is free again -> K_{j+2}
@@ -198,9 +194,14 @@ __global__ void __launch_bounds__(256, 1)
       tmem_ld_wait();
 #pragma unroll
       for (int e = 0; e < TD / 2; ++e) o[e] = o[e] * corr_prev + __uint_as_float(v[e]);
+      // V_{j-1}'s buffer is free (O_{j-1} done): V_{j+1} into it
+      if (tid == 0 && j + 1 < nkt) {
+        mbar_expect_tx(&bar_v[(j + 1) & 1], V_BYTES);
+        tma_load_2d(&tmQK, &bar_v[(j + 1) & 1], sV + ((j + 1) & 1) * V_BYTES, vcol, tok0 + k0 + TK);
+      }
     }
     corr_prev = corr;
-    // (5) P_j row half (K-block h) and V_j^T into the operand tiles
+    // (5) P_j row half (K-block h) into the A-operand tile
     {
       uint8_t* pt = sP + h * (TQ * 64 * 2);
 #pragma unroll
@@ -213,30 +214,23 @@ __global__ void __launch_bounds__(256, 1)
         u.w = Cvt<T>::from2(pp[6], pp[7]);
         *reinterpret_cast<uint4*>(pt + sw128_off(r, c * 8)) = u;
       }
-      uint8_t* vt = sVt + (vkey >> 6) * (TD * 64 * 2);
-      const int kk = vkey & 63;
-#pragma unroll
-      for (int c = 0; c < 4; ++c) {
-        const uint32_t w4[4] = {vr[c].x, vr[c].y, vr[c].z, vr[c].w};
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const int d = 32 * vh + c * 8 + e * 2;
-          *reinterpret_cast<uint16_t*>(vt + sw128_off(d, kk)) = uint16_t(w4[e] & 0xFFFFu);
-          *reinterpret_cast<uint16_t*>(vt + sw128_off(d + 1, kk)) = uint16_t(w4[e] >> 16);
-        }
-      }
     }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // P, V^T -> the tensor core
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // P -> the tensor core
     asm volatile("tcgen05.fence::before_thread_sync;");
     __syncthreads();
     // (6) O_j = P_j V_j into TMEM buffer j & 1
     if (tid == 0) {
+      mbar_wait_spin(&bar_v[j & 1], (j >> 1) & 1);
       asm volatile("tcgen05.fence::after_thread_sync;");
+      // V_j as the MN-major B operand: 128-byte swizzle atoms of 8 keys x 64 head dims, 1024 B apart
+      // along K (SBO); a 16-key step advances 2048 B (128 in descriptor units)
+      const uint64_t dv = sw128_desc(sV + (j & 1) * V_BYTES);
 #pragma unroll
       for (int kb = 0; kb < 2; ++kb) {
-        const uint64_t dp_ = sw128_desc(sP + kb * (TQ * 64 * 2)), dv = sw128_desc(sVt + kb * (TD * 64 * 2));
+        const uint64_t dp_ = sw128_desc(sP + kb * (TQ * 64 * 2));
 #pragma unroll
-        for (int kk = 0; kk < 4; ++kk) umma_f16(t_o(j & 1), dp_ + 2 * kk, dv + 2 * kk, IDESC_O, (kb | kk) != 0);
+        for (int kk = 0; kk < 4; ++kk)
+          umma_f16(t_o(j & 1), dp_ + 2 * kk, dv + 128 * (kb * 4 + kk), IDESC_O, (kb | kk) != 0);
       }
       umma_commit(&bar_o[j & 1]);
     }
