@@ -541,6 +541,21 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
            "sequence longer than the position table");
   DeviceGuard g(primary);
   acquire_slots(ctx, m, primary, plan->method);
+  // a failure before the model became resident hands the block back (the model stays usable)
+  struct ReleaseOnError {
+    dp_context* c;
+    dp_model* mm;
+    int d;
+    bool armed = true;
+    ~ReleaseOnError() {
+      if (!armed) return;
+      try {
+        cudaDeviceSynchronize();  // transfers already enqueued into the block must finish first
+        release_slots(c, mm, d);
+      } catch (...) {
+      }
+    }
+  } release_on_error{ctx, m, primary};
   ensure_h2d_streams(ctx, primary);
   ensure_workspace(m, primary, int64_t(batch) * seq);
   // across processes: the IPC transports capture (the epoch lives in a device word); the NCCL
@@ -576,6 +591,7 @@ void infer_cold(dp_context* ctx, dp_model* m, const dp_plan* plan, int primary, 
     st = enqueue_cold(ctx, m, plan, primary, prim_rank, secondaries, ids, batch, seq, out, pooled, stream);
   }
   ds.resident = true;
+  release_on_error.armed = false;
   ds.method.assign(plan->method, plan->method + plan->n);
   st.wall_enqueue_us =
       std::chrono::duration<float, std::micro>(std::chrono::steady_clock::now() - t0).count();

@@ -165,8 +165,14 @@ void serve_live(dp_context* ctx, dp_model* const* models, int nmodels, const dp_
       q.running = r;
       q.running_cold = out[r].cold != 0;
     };
-    // pre-warm: every instance once on every GPU (HBM slot block, workspace, captured graphs),
-    // then evicted -- the trace measures serving, not first-touch allocation
+    // live serving starts from every instance non-resident on the served GPUs
+    for (int g = 0; g < G; ++g)
+      for (int i = 0; i < nmodels; ++i)
+        if (models[i]->dev[gpu[g].dev].resident)
+          DP_CHECK(dp_model_evict(ctx, models[i], gpu[g].dev) == DP_OK, DP_ERR_CUDA, "eviction failed");
+    // pre-warm: every instance once on every GPU (workspace, first-use host costs), then evicted
+    // -- the trace measures serving, not first-touch allocation (graphs are captured on a key's
+    // second use, so instances that keep a pool block capture during the trace)
     if (!o.no_prewarm) {
       for (int g = 0; g < G; ++g) {
         for (int i = 0; i < nmodels; ++i) {

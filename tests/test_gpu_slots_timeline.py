@@ -169,3 +169,25 @@ def test_timeline_needs_a_traced_run():
         model.timeline(0)
     model.close()
     c.close()
+
+
+def test_failed_cold_start_returns_the_block():
+    """A cold start that fails after taking its HBM block (here: a PT secondary outside the context)
+    hands the block back: nothing is held and the next cold start works."""
+    m = synth.SHAPES["tiny_bert"]
+    w = synth.make_weights(m, seed=9, dtype="fp16")
+    ids = synth.make_ids(m, 1, 32, seed=10)
+    c = dp().Context([0])
+    model = dp().Model(c, m, w, "fp16")
+    n = model.n
+    pt = dp()._lib.PlanArrays(n, np.zeros(n, np.int8), np.array([i % 2 for i in range(n)], np.int8), 4, 2)
+    out = torch.empty(32, m.hidden, dtype=torch.float16, device="cuda")
+    with pytest.raises(dp().DeepPlanError):
+        model.infer_cold(pt, 0, torch.from_numpy(ids).cuda(), out, secondaries=[5])
+    assert not model.is_resident(0) and c.pool_stats(0)[1] == 0
+    ok = dp()._lib.PlanArrays(n, np.zeros(n, np.int8), None, 1, 1)
+    run_cold(model, ok, ids)
+    assert model.is_resident(0)
+    model.evict(0)
+    model.close()
+    c.close()
