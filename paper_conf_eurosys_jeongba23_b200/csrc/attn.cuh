@@ -90,28 +90,37 @@ __device__ __forceinline__ void attention_key_tile(const T* skt, const T* svt, c
         MmaOp<T>::mma(s[nb + 1], qa[kk], bfr + 2);
       }
     }
-    // mask + online softmax (rows qrow0, qrow0+8; each row spread over 4 lanes)
+    // mask + online softmax (rows qrow0, qrow0+8; each row spread over 4 lanes).  Scores stay
+    // unscaled until the exponent: p = exp2(s * scale_log2 - m) is one FFMA + MUFU per element.
+    // Only the sequence's last key tile and the causal diagonal need the mask (the warp's rows
+    // start at qrow0 - lane / 4); the running max is kept in scaled units.
+    const bool need_mask = k0 + 64 > seq || (causal && k0 + 63 > qrow0 - (lane >> 2));
+    if (need_mask) {
+#pragma unroll
+      for (int nb = 0; nb < 8; ++nb) {
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int key = k0 + nb * 8 + (lane & 3) * 2 + (e & 1);
+          const int qr = qrow0 + (e >> 1) * 8;
+          if (key >= seq || (causal && key > qr)) s[nb][e] = -INFINITY;
+        }
+      }
+    }
     float mx[2] = {-INFINITY, -INFINITY};
 #pragma unroll
     for (int nb = 0; nb < 8; ++nb) {
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int key = k0 + nb * 8 + (lane & 3) * 2 + (e & 1);
-        const int qr = qrow0 + (e >> 1) * 8;
-        float v = s[nb][e] * scale_log2;
-        if (key >= seq || (causal && key > qr)) v = -INFINITY;
-        s[nb][e] = v;
-        mx[e >> 1] = fmaxf(mx[e >> 1], v);
-      }
+      mx[0] = fmaxf(mx[0], fmaxf(s[nb][0], s[nb][1]));
+      mx[1] = fmaxf(mx[1], fmaxf(s[nb][2], s[nb][3]));
     }
-    float corr[2];
+    float corr[2], mref[2];
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
       mx[h] = fmaxf(mx[h], __shfl_xor_sync(0xffffffffu, mx[h], 1));
       mx[h] = fmaxf(mx[h], __shfl_xor_sync(0xffffffffu, mx[h], 2));
-      const float mnew = fmaxf(mrow[h], mx[h]);
+      const float mnew = fmaxf(mrow[h], mx[h] * scale_log2);
       corr[h] = (mrow[h] == -INFINITY) ? 0.f : exp2f(mrow[h] - mnew);
       mrow[h] = mnew;
+      mref[h] = (mnew == -INFINITY) ? 0.f : mnew;  // a fully masked row: every p is exp2(-inf) = 0
     }
     float rs[2] = {0.f, 0.f};
 #pragma unroll
@@ -119,7 +128,7 @@ __device__ __forceinline__ void attention_key_tile(const T* skt, const T* svt, c
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
         const int h = e >> 1;
-        const float p = (mrow[h] == -INFINITY) ? 0.f : exp2f(s[nb][e] - mrow[h]);
+        const float p = exp2f(fmaf(s[nb][e], scale_log2, -mref[h]));
         s[nb][e] = p;
         rs[h] += p;
       }
