@@ -118,7 +118,7 @@ __device__ __forceinline__ void attention_key_tile(const T* skt, const T* svt, c
       mx[h] = fmaxf(mx[h], __shfl_xor_sync(0xffffffffu, mx[h], 1));
       mx[h] = fmaxf(mx[h], __shfl_xor_sync(0xffffffffu, mx[h], 2));
       const float mnew = fmaxf(mrow[h], mx[h] * scale_log2);
-      corr[h] = (mrow[h] == -INFINITY) ? 0.f : exp2f(mrow[h] - mnew);
+      corr[h] = (mrow[h] == -INFINITY) ? 0.f : fast_exp2(mrow[h] - mnew);
       mrow[h] = mnew;
       mref[h] = (mnew == -INFINITY) ? 0.f : mnew;  // a fully masked row: every p is exp2(-inf) = 0
     }
@@ -128,7 +128,7 @@ __device__ __forceinline__ void attention_key_tile(const T* skt, const T* svt, c
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
         const int h = e >> 1;
-        const float p = exp2f(fmaf(s[nb][e], scale_log2, -mref[h]));
+        const float p = fast_exp2(fmaf(s[nb][e], scale_log2, -mref[h]));
         s[nb][e] = p;
         rs[h] += p;
       }

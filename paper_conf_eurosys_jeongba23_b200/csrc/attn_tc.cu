@@ -158,7 +158,7 @@ __global__ void __launch_bounds__(256, 1)
       for (int c = 0; c < TK / 2; c += 16) tmem_ld16_nowait(t_s(j & 1) + lane_base + 64 * h + c, v + c);
       tmem_ld_wait();
 #pragma unroll
-      for (int e = 0; e < TK / 2; ++e) s[e] = __uint_as_float(v[e]) * scale_log2;
+      for (int e = 0; e < TK / 2; ++e) s[e] = __uint_as_float(v[e]);  // scaled inside the exponent
     }
     const int kbase = k0 + 64 * h;
     if (kbase + 64 > seq || (causal && kbase + 63 > qrow)) {  // only where a key can be invalid
@@ -173,12 +173,13 @@ __global__ void __launch_bounds__(256, 1)
     for (int e = 0; e < TK / 2; ++e) mx = fmaxf(mx, s[e]);
     red[h][r] = mx;
     __syncthreads();
-    const float mnew = fmaxf(mrow, fmaxf(red[0][r], red[1][r]));
-    const float corr = (mrow == -INFINITY) ? 0.f : exp2f(mrow - mnew);
+    const float mnew = fmaxf(mrow, fmaxf(red[0][r], red[1][r]) * scale_log2);
+    const float corr = (mrow == -INFINITY) ? 0.f : fast_exp2(mrow - mnew);
+    const float mref = (mnew == -INFINITY) ? 0.f : mnew;  // a fully masked row: every p = 2^-inf = 0
     float rs = 0.f;
 #pragma unroll
     for (int e = 0; e < TK / 2; ++e) {
-      const float p = (mnew == -INFINITY) ? 0.f : exp2f(s[e] - mnew);
+      const float p = fast_exp2(fmaf(s[e], scale_log2, -mref));
       rs += p;
       s[e] = p;
     }

@@ -130,6 +130,15 @@ __device__ __forceinline__ void cluster_bcast_from_rank0(uint4* buf, int n16) {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+// 2^x on the MUFU, flushing subnormal results to zero (exp2f adds the subnormal-range fix-up --
+// two FMULs and a select per call -- which the softmax numerators never need: p < 2^-126 is
+// irrelevant next to the row maximum's 1).  2^-inf = +0.
+__device__ __forceinline__ float fast_exp2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
 __device__ __forceinline__ float warp_sum(float v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
