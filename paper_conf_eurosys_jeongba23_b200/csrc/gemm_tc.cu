@@ -160,7 +160,7 @@ __global__ void __launch_bounds__(NT, 1)
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
-  constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
+  constexpr uint32_t TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;  // a power of 2
   constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free TMEM->smem writes)
   // kind::f16, fp32 accumulate, A/B K-major, M = 128, N = BN
   constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
@@ -477,9 +477,10 @@ void dispatch(int bn, const void* x, int ldx, int ngroups, const void* const* w,
   switch (bn) {
     case 32: DP_ACTS(32); break;
     case 64: DP_ACTS(64); break;
+    case 96: DP_ACTS(96); break;
     case 128: DP_ACTS(128); break;
     case 256: DP_ACTS(256); break;
-    default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/128/256");
+    default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/96/128/256");
   }
 #undef DP_ACTS
 #undef DP_RUN

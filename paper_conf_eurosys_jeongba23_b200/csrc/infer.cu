@@ -315,8 +315,9 @@ extern "C" dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* 
     DP_CHECK(ctx && o, DP_ERR_INVALID, "NULL argument");
     DP_CHECK(o->chunk_bytes >= 4096, DP_ERR_INVALID, "chunk_bytes must be >= 4096");
     DP_CHECK(o->n_h2d_streams >= 1 && o->n_h2d_streams <= 8, DP_ERR_INVALID, "n_h2d_streams must be 1..8");
-    DP_CHECK(o->gemm_bn == 0 || o->gemm_bn == 32 || o->gemm_bn == 64 || o->gemm_bn == 128 || o->gemm_bn == 256,
-             DP_ERR_INVALID, "gemm_bn must be 0/32/64/128/256");
+    DP_CHECK(o->gemm_bn == 0 || o->gemm_bn == 32 || o->gemm_bn == 64 || o->gemm_bn == 96 || o->gemm_bn == 128 ||
+                 o->gemm_bn == 256,
+             DP_ERR_INVALID, "gemm_bn must be 0/32/64/96/128/256");
     DP_CHECK(o->pt_transport == DP_PT_DMA || o->pt_transport == DP_PT_SM || o->pt_transport == DP_PT_CE,
              DP_ERR_INVALID, "pt_transport must be DP_PT_DMA, DP_PT_SM or DP_PT_CE");
     // measured slower and moved out of the library (tools/experiments)
