@@ -158,7 +158,7 @@ typedef struct {
   int64_t chunk_bytes;
   int32_t n_h2d_streams;
   int32_t use_graph;
-  int32_t gemm_bn;        /* 0 = auto */
+  int32_t gemm_bn;        /* 0 = auto; 32..256 one CTA per tile; -64..-256 CTA pairs (dp_gemm_tc) */
   int32_t debug_delay_us; /* fault injection: stall every load/migration stream this long
                              before each transfer (tests event gating) [0] */
   int32_t debug_poison;   /* 1 = fill HBM slots with 0xFF (NaN) on eviction [0] */
@@ -199,9 +199,10 @@ typedef struct {
                              every unit's dependency wait on the execution stream.  Costs event
                              records between kernels (no PDL overlap) and forces eager enqueue (no
                              graph): a measurement mode [0] */
-  int32_t attention_tc;   /* 1 = the attention core runs on tcgen05 (K5t: S and P.V in TMEM, the
-                             softmax row per thread); correct but measured slower than the mma.sync
-                             flash kernels K5 / K5b at the hot-path shapes [0] */
+  int32_t attention_tc;   /* attention core: 0 = by sequence length (K5t, tcgen05 with S and O in
+                             TMEM, from 768 tokens -- GPT-2 Medium S1024 warm 2.02 -> 1.88 ms --
+                             else the mma.sync flash kernels K5 / K5b, faster at S <= 384), 1 =
+                             always K5t, 2 = never [0] */
   int32_t reserved[1];
 } dp_engine_opts;
 #define DP_PT_DMA 0
@@ -464,6 +465,17 @@ dp_status dp_embed(const int32_t* d_ids, int32_t ntok, int32_t seq, int32_t pos_
 dp_status dp_linear(const void* x, int32_t ldx, const void* w, const void* b, const void* residual, int32_t ldr,
                     void* y, int32_t ldy, int32_t M, int32_t N, int32_t K, int32_t act, int32_t path, int32_t dtype,
                     int32_t io, void* stream);
+
+/* The resident tcgen05 GEMM of dp_linear(path 0) with its tile configuration forced (tests,
+ * sweeps): bn = 0 the cost model's choice; 32/64/96/128/256 one CTA per 128 x bn output tile
+ * (K2); -64/-128/-192/-256 a CTA pair per 256 x |bn| tile (K2p: cta_group::2 MMAs issued by
+ * the even CTA, each CTA staging its 128 W rows and |bn|/2 tokens; needs N % 256 == 0).
+ * split = 0 the model's K split, 1 none, 2/4/8 (<= K/64, with a single-CTA bn <= 128) that many
+ * K ranges reduced over a thread-block cluster.  Same arguments, layout and errors as
+ * dp_linear otherwise; w must be device memory. */
+dp_status dp_gemm_tc(const void* x, int32_t ldx, const void* w, const void* b, const void* residual, int32_t ldr,
+                     void* y, int32_t ldy, int32_t M, int32_t N, int32_t K, int32_t act, int32_t dtype, int32_t io,
+                     int32_t bn, int32_t split, void* stream);
 
 /* LayerNorm over rows of width n: y = LN(x (+ r)) * g + b.  g/b may be host-mapped.
  * x_f32 = 1: x and r are fp32; y is always the storage dtype. */

@@ -10,7 +10,7 @@ from ._lib import (  # noqa: F401
     DHA, LOAD, MODES, UNIT_KINDS, Context, DeepPlanError, Model, attention, embed, host_alloc, host_free,
     layernorm, lib, linear, plan_exhaustive, plan_generate, plan_partition, plan_simulate, serve_run,
     peer_unique_id, measure_h2d, transfer_schedule, config_units, pt_forward, plan_resident_bytes,
-    device_numa_node, host_numa_node, host_alloc_node, measure_h2d_concurrent, select_secondaries, attention_tc,
+    device_numa_node, host_numa_node, host_alloc_node, measure_h2d_concurrent, select_secondaries, attention_tc, gemm_tc,
 )
 
 __all__ = [
@@ -18,5 +18,5 @@ __all__ = [
     "host_alloc", "host_free", "layernorm", "lib", "linear", "plan_exhaustive", "plan_generate",
     "plan_partition", "plan_simulate", "serve_run", "peer_unique_id", "measure_h2d", "transfer_schedule",
     "config_units", "pt_forward", "plan_resident_bytes", "device_numa_node", "host_numa_node", "host_alloc_node",
-    "measure_h2d_concurrent", "select_secondaries", "attention_tc",
+    "measure_h2d_concurrent", "select_secondaries", "attention_tc", "gemm_tc",
 ]

@@ -159,6 +159,8 @@ _sig("dp_embed", [vp, C.c_int32, C.c_int32, C.c_int32, vp, vp, vp, vp, vp, C.c_i
                   C.c_int32, vp, vp])
 _sig("dp_linear", [vp, C.c_int32, vp, vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
                    C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
+_sig("dp_gemm_tc", [vp, C.c_int32, vp, vp, vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
+                    C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
 _sig("dp_layernorm", [vp, vp, vp, vp, vp, C.c_int32, C.c_int32, C.c_double, C.c_int32, C.c_int32, vp])
 _sig("dp_attention", [vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
 _sig("dp_attention_tc", [vp, C.c_int32, vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32, vp])
@@ -321,8 +323,8 @@ class Context:
             o.profile_chain = 1 if profile_chain else 0
         if trace_units is not None:
             o.trace_units = 1 if trace_units else 0
-        if attention_tc is not None:
-            o.attention_tc = 1 if attention_tc else 0
+        if attention_tc is not None:  # 0 by sequence length, 1 always K5t, 2 never (True / False: 1 / 2)
+            o.attention_tc = (1 if attention_tc else 2) if isinstance(attention_tc, bool) else int(attention_tc)
         if pt_transport is not None:
             o.pt_transport = PT_TRANSPORTS[pt_transport] if isinstance(pt_transport, str) else int(pt_transport)
         _check(lib.dp_context_set_opts(self.h, C.byref(o)))
@@ -612,6 +614,15 @@ def linear(x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act="none", path=0, dty
                          DTYPES[dtype], int(io), _stream_ptr(stream)))
 
 
+def gemm_tc(x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act="none", bn=0, split=0, dtype="fp16", io=0,
+            stream=None):
+    """The resident tcgen05 GEMM with its tile forced: bn 0 = the cost model's choice, > 0 one CTA
+    per 128 x bn tile, < 0 a CTA pair per 256 x |bn| tile (K2p); split > 0 forces the K split."""
+    _check(lib.dp_gemm_tc(_dptr(x), int(ldx), _dptr(w), _dptr(b), _dptr(residual), int(ldr), _dptr(y), int(ldy),
+                          int(M), int(N), int(K), ACTS[act] if isinstance(act, str) else int(act), DTYPES[dtype],
+                          int(io), int(bn), int(split), _stream_ptr(stream)))
+
+
 def layernorm(x, r, g, b, y, rows, n, eps, dtype="fp16", x_f32=False, stream=None):
     _check(lib.dp_layernorm(_dptr(x), _dptr(r), _dptr(g), _dptr(b), _dptr(y), int(rows), int(n), float(eps),
                             DTYPES[dtype], int(bool(x_f32)), _stream_ptr(stream)))
@@ -623,7 +634,7 @@ def attention(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp1
 
 
 def attention_tc(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp16", stream=None):
-    """The tcgen05 attention core (K5t, opts.attention_tc)."""
+    """The tcgen05 attention core (K5t; the engine uses it from 768 tokens, opts.attention_tc)."""
     _check(lib.dp_attention_tc(_dptr(qkv), int(ldqkv), _dptr(ctx_out), int(batch), int(seq), int(hidden), int(heads),
                                int(bool(causal)), DTYPES[dtype], _stream_ptr(stream)))
 

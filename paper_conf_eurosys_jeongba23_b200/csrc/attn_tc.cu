@@ -2,20 +2,25 @@
 //
 //   ctx[q, h*64 : h*64+64] = softmax(q_h k_h^T / 8 [+ causal mask]) v_h
 //
-// One CTA (256 threads) per (head, 128-query tile, sequence).  Per 128-key tile j:
-//   1. S = Q K_j^T on tcgen05 (M = 128 queries, N = 128 keys, K = 64), fp32 in TMEM columns
-//      [0, 128); Q and K_j arrive by TMA (128-byte swizzle), K double-buffered;
-//   2. two threads own query row r = TMEM lane r (warps w and w + 4 read the lane quarter w % 4),
-//      each half of its S row (tcgen05.ld): masks, the online softmax in fp32 with exp2 (the
-//      halves' maxima meet in shared memory; each keeps a partial row sum under the same
-//      corrections);
-//      the numerators P (storage type) go to shared memory as the next MMA's A operand, written
-//      in the 128-byte-swizzled K-major layout by hand; V_j arrives by TMA as [keys][head dims]
-//      and is the MN-major B operand as it lands (no transpose);
-//   3. O_j = P V_j on tcgen05 (M = 128, N = 64, K = 128 keys) into TMEM columns [128, 192);
-//   4. thread r accumulates o_r = o_r * corr + O_j[r] in registers.
-// After the last key tile o_r / l_r is stored (128 bytes per row).  Arithmetic contract: S and
-// O_j in fp32, P rounded to the storage type before P V (as the mma.sync K5), row sums in fp32.
+// One CTA (320 threads, warp-specialised) per (head, 128-query tile, sequence); keys in tiles of
+// 64.  The key tiles alternate between two softmax warpgroups, each with its own running row
+// max / sum / output (merged once at the end, like K5b's key-tile groups), so two independent
+// softmax chains share the SM while the tensor core serves both:
+//   warp 8 (one lane)  : TMA -- Q once, then K_j / V_j into a 4-stage ring;
+//   warp 9 (one lane)  : tcgen05.mma -- S_j = Q K_j^T (M 128, N 64, K 64) into the owning
+//                        group's TMEM S buffer (two per group: S_{j+2} is computed while the
+//                        group works on S_j), and O_g += P_j V_j (M 128, N 64, K 64 keys) into
+//                        the group's TMEM accumulator once the group has published P_j;
+//   warps 0-3 / 4-7    : group g = even / odd key tiles; thread r owns query row r (TMEM lane
+//                        r): it reads its 64 scores (tcgen05.ld), masks, runs the online
+//                        softmax in fp32 with exp2 and writes the numerators P (storage type)
+//                        into the 128-byte-swizzled K-major A tile.
+// The softmax reference max of a row moves only when the row max grows by more than 2^8 (then
+// the thread rescales its O row in TMEM, tcgen05.ld / st, and its row sum): between moves the
+// numerators stay <= 2^8, so the O accumulator never leaves TMEM (no per-tile correction pass).
+// V_j lands as [keys][head dims] and is the MN-major B operand as is (no transpose).  TMEM: three S
+// buffers per group in columns [0, 384), the two O accumulators in [384, 512).  Arithmetic contract: S and
+// O in fp32, P rounded to the storage type before P V (as the mma.sync K5), row sums in fp32.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -33,41 +38,78 @@ namespace dp {
 
 namespace {
 
+#ifdef DP_ATT_TRACE
+// per-CTA globaltimer stamps (tools/att_trace.py): 0 entry, 1 after setup + PDL wait, 2 / 3 group
+// 0 / 1 first scores read, 4 / 5 group 0 / 1 last P published, 6 / 7 group 0 / 1 accumulator
+// read, 8 stored, 9 MMA warp done issuing, 10 loader done issuing; [15] = key tiles
+__device__ unsigned long long g_att_trace[2048][64];
+#define ATRACE(i)                                                                                \
+  do {                                                                                           \
+    unsigned long long t_;                                                                       \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                                       \
+    const int b_ = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;               \
+    if (b_ < 2048 && (i) < 64) g_att_trace[b_][i] = t_;                                          \
+  } while (0)
+#else
+#define ATRACE(i) \
+  do {            \
+  } while (0)
+#endif
+
 constexpr int TQ = 128;  // queries per CTA (MMA M, TMEM lanes)
-constexpr int TK = 128;  // keys per tile (MMA N of S, K of P V)
+constexpr int TK = 64;   // keys per tile (MMA N of S, K of P V)
 constexpr int TD = 64;   // head dim
-constexpr uint32_t Q_BYTES = TQ * TD * 2;      // 16 KB
-constexpr uint32_t K_BYTES = TK * TD * 2;      // 16 KB
-constexpr uint32_t P_BYTES = TQ * TK * 2;      // 32 KB: two [128][64] swizzled K-blocks
-constexpr uint32_t V_BYTES = TK * TD * 2;      // 16 KB: [128 keys][64] swizzled (MN-major B operand)
-constexpr uint32_t SMEM_BYTES = Q_BYTES + 2 * K_BYTES + P_BYTES + 2 * V_BYTES + 1024;
+constexpr int NS = 6;    // stages of the K ring and of the V ring
+constexpr int SB = 3;    // TMEM S buffers per softmax group
+constexpr uint32_t Q_BYTES = TQ * TD * 2;   // 16 KB
+constexpr uint32_t KV_BYTES = TK * TD * 2;  // 8 KB each for K_j and V_j
+constexpr uint32_t P_BYTES = TQ * TK * 2;   // 16 KB: one [128][64] swizzled K-block
+constexpr uint32_t MERGE_BYTES = TQ * 68 * 4;  // group 1's (o[64], m, l) per row
+constexpr uint32_t SMEM_BYTES = Q_BYTES + 2 * NS * KV_BYTES + 4 * P_BYTES + MERGE_BYTES + 1024;
+constexpr int NTHR = 352;  // 8 softmax warps, the TMA warp, two MMA warps
 
 // byte offset of element (r, k) of a K-major [rows][64] tile with the 128-byte swizzle
 __device__ __forceinline__ uint32_t sw128_off(int r, int k) {
   return uint32_t(r) * 128u + ((uint32_t((k >> 3) ^ (r & 7))) << 4) + uint32_t(k & 7) * 2u;
 }
 
+// One lane polls the barrier and releases its warp: 256 softmax threads polling the same
+// barriers flooded the shared-memory barrier unit and delayed the MMA warp's own polls.
+__device__ __forceinline__ void warp_wait(uint64_t* bar, uint32_t phase) {
+  if ((threadIdx.x & 31) == 0) mbar_wait(bar, phase);
+  __syncwarp();
+}
+
+__device__ __forceinline__ void named_sync(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void named_arrive(int id, int n) {
+  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
 template <class T>
-__global__ void __launch_bounds__(256, 1)
-    attention_tc_kernel(const __grid_constant__ CUtensorMap tmQK, const T* __restrict__ qkv, int ldqkv,
+__global__ void __launch_bounds__(NTHR, 1)
+    attention_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
                         T* __restrict__ ctx, int seq, int H, int causal, float scale_log2) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sQ = smem;
-  uint8_t* sK = sQ + Q_BYTES;           // [2][TK][64]
-  uint8_t* sP = sK + 2 * K_BYTES;       // [2 k-blocks][TQ][64]
-  uint8_t* sV = sP + P_BYTES;           // [2][TK][64]: V tiles as TMA lands them (keys x head dims)
-  __shared__ __align__(8) uint64_t bar_q, bar_k[2], bar_v[2], bar_s[2], bar_o[2];
+  uint8_t* sK = sQ + Q_BYTES;               // [NS][64 keys][64]: freed by S_j
+  uint8_t* sV = sK + NS * KV_BYTES;         // [NS][64 keys][64]: freed by P_j V_j
+  uint8_t* sP = sV + NS * KV_BYTES;         // [group][buffer][128][64]
+  float* xs = reinterpret_cast<float*>(sP + 4 * P_BYTES);  // [128][68]
+  __shared__ __align__(8) uint64_t bar_q, k_full[NS], k_empty[NS], v_full[NS], v_empty[NS], s_full[2][SB], s_free[2][SB], p_full[2][2],
+      o_full[2][2];
   __shared__ uint32_t tmem_base_sh;
-  __shared__ float red[2][TQ];          // per column half: partial row max (and at the end: row sum)
-  // kind::f16, fp32 accumulate, A/B K-major; S: M 128 x N 128; O: M 128 x N 64
+  // kind::f16, fp32 accumulate; S: A = Q, B = K_j both K-major, M 128 x N 64
   constexpr uint32_t IDESC_S = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(TK >> 3) << 17) |
                                (uint32_t(TQ >> 4) << 24);
-  // O: B = V_j is MN-major (head dims contiguous, keys along K): the transpose-B bit (16)
+  // O: A = P K-major, B = V_j MN-major (head dims contiguous, keys along K): transpose-B bit 16
   constexpr uint32_t IDESC_O = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (1u << 16) |
                                (uint32_t(TD >> 3) << 17) | (uint32_t(TQ >> 4) << 24);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (tid == 0) ATRACE(0);
   // grid (heads, query tiles, batch); causal query tiles longest first
   const int head = blockIdx.x, bidx = blockIdx.z;
   const int qt = causal ? (int)gridDim.y - 1 - (int)blockIdx.y : (int)blockIdx.y;
@@ -77,19 +119,28 @@ __global__ void __launch_bounds__(256, 1)
   if (causal) nkt = min(nkt, (q0 + TQ - 1) / TK + 1);
 
   if (tid == 0) {
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmQK)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmQ)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmKV)) : "memory");
     mbar_init(&bar_q, 1);
-    mbar_init(&bar_k[0], 1);
-    mbar_init(&bar_k[1], 1);
-    mbar_init(&bar_v[0], 1);
-    mbar_init(&bar_v[1], 1);
-    mbar_init(&bar_s[0], 1);
-    mbar_init(&bar_s[1], 1);
-    mbar_init(&bar_o[0], 1);
-    mbar_init(&bar_o[1], 1);
+    for (int i = 0; i < NS; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_empty[i], 1);
+      mbar_init(&v_full[i], 1);
+      mbar_init(&v_empty[i], 1);
+    }
+    for (int g = 0; g < 2; ++g) {
+      for (int b = 0; b < 2; ++b) {
+        mbar_init(&o_full[g][b], 1);
+        mbar_init(&p_full[g][b], 4);  // one arrival per warp of the group
+      }
+      for (int b = 0; b < SB; ++b) {
+        mbar_init(&s_full[g][b], 1);
+        mbar_init(&s_free[g][b], 4);
+      }
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 0) {
+  if (warp == 9) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base_sh)),
                  "r"(512));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -98,115 +149,166 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = tmem_base_sh;
-  // TMEM: S double buffer in columns [0, 256), O double buffer in [256, 384)
-  auto t_s = [&](int b) { return tmem + 128u * uint32_t(b); };
-  auto t_o = [&](int b) { return tmem + 256u + 64u * uint32_t(b); };
+  auto t_s = [&](int g, int b) { return tmem + 64u * uint32_t(SB * g + b); };
+  auto t_o = [&](int g) { return tmem + 64u * uint32_t(2 * SB + g); };
   pdl_trigger();
   pdl_wait();  // q, k, v come from the previous kernel
-
-  const int qcol = head * TD, kcol = H + head * TD;
-  const int vcol = 2 * H + head * TD;
-  // thread (warp w, lane l): query row r = 32 (w % 4) + l (its TMEM lane), column half h = w / 4
-  // -- keys [64 h, 64 h + 64) of each S tile, head dims [32 h, 32 h + 32) of O
-  const int r = (warp & 3) * 32 + lane, h = warp >> 2;
-  const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
-  const int qrow = q0 + r;
-  auto issue_s = [&](int jj) {  // S_jj = Q K_jj^T into TMEM buffer jj & 1 (K_jj must be landing)
-    mbar_wait_spin(&bar_k[jj & 1], (jj >> 1) & 1);
-    asm volatile("tcgen05.fence::after_thread_sync;");
-    const uint64_t dq = sw128_desc(sQ), dk = sw128_desc(sK + (jj & 1) * K_BYTES);
-#pragma unroll
-    for (int kk = 0; kk < TD / 16; ++kk) umma_f16(t_s(jj & 1), dq + 2 * kk, dk + 2 * kk, IDESC_S, kk != 0);
-    umma_commit(&bar_s[jj & 1]);
-  };
+  if (tid == 0) ATRACE(1);
+#ifdef DP_ATT_TRACE
   if (tid == 0) {
-    mbar_expect_tx(&bar_q, Q_BYTES);
-    tma_load_2d(&tmQK, &bar_q, sQ, qcol, tok0 + q0);
-    for (int jj = 0; jj < 2 && jj < nkt; ++jj) {
-      mbar_expect_tx(&bar_k[jj], K_BYTES);
-      tma_load_2d(&tmQK, &bar_k[jj], sK + jj * K_BYTES, kcol, tok0 + jj * TK);
-      mbar_expect_tx(&bar_v[jj], V_BYTES);
-      tma_load_2d(&tmQK, &bar_v[jj], sV + jj * V_BYTES, vcol, tok0 + jj * TK);
-    }
-    mbar_wait_spin(&bar_q, 0);
-    issue_s(0);
+    const int b_ = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
+    if (b_ < 2048) g_att_trace[b_][15] = (unsigned long long)nkt;
   }
-  float o[TD / 2];
-#pragma unroll
-  for (int d = 0; d < TD / 2; ++d) o[d] = 0.f;
-  float mrow = -INFINITY, lrow = 0.f;  // lrow: this half's partial row sum (same corrections)
-  float corr_prev = 0.f;               // the correction that goes with the O tile in flight
+#endif
 
-  // Software pipeline per key tile j: S_{j+1} is computed on the tensor core while the threads run
-  // the softmax of tile j, and O_j = P_j V_j is added to the registers one iteration later.
-  for (int j = 0; j < nkt; ++j) {
-    const int k0 = j * TK;
-    // (1) the next S on the tensor core (its buffer was last read in iteration j - 1)
-    if (tid == 0 && j + 1 < nkt) issue_s(j + 1);
-    // (2) S_j ready; K_j's buffer is free again -> K_{j+2}
-    mbar_wait_spin(&bar_s[j & 1], (j >> 1) & 1);
-    asm volatile("tcgen05.fence::after_thread_sync;");
-    if (tid == 0 && j + 2 < nkt) {
-      mbar_expect_tx(&bar_k[j & 1], K_BYTES);
-      tma_load_2d(&tmQK, &bar_k[j & 1], sK + (j & 1) * K_BYTES, kcol, tok0 + k0 + 2 * TK);
-    }
-    // (3) this half of the S row -> online softmax
-    float s[TK / 2];
-    {
-      uint32_t v[TK / 2];
-#pragma unroll
-      for (int c = 0; c < TK / 2; c += 16) tmem_ld16_nowait(t_s(j & 1) + lane_base + 64 * h + c, v + c);
-      tmem_ld_wait();
-#pragma unroll
-      for (int e = 0; e < TK / 2; ++e) s[e] = __uint_as_float(v[e]);  // scaled inside the exponent
-    }
-    const int kbase = k0 + 64 * h;
-    if (kbase + 64 > seq || (causal && kbase + 63 > qrow)) {  // only where a key can be invalid
-#pragma unroll
-      for (int e = 0; e < TK / 2; ++e) {
-        const int key = kbase + e;
-        if (key >= seq || (causal && key > qrow)) s[e] = -INFINITY;
+  const int qcol = head * TD, kcol = H + head * TD, vcol = 2 * H + head * TD;
+  if (warp == 8) {
+    // TMA producer: Q, then K_j and V_j in key order into their rings (a K stage is free once
+    // S_j is done, a V stage once P_j V_j is done)
+    if (lane == 0) {
+      mbar_expect_tx(&bar_q, Q_BYTES);
+      tma_load_2d(&tmQ, &bar_q, sQ, qcol, tok0 + q0);
+      for (int j = 0; j < nkt; ++j) {
+        const int st = j % NS;
+        if (j >= NS) mbar_wait(&k_empty[st], ((j / NS) - 1) & 1);
+        mbar_expect_tx(&k_full[st], KV_BYTES);
+        tma_load_2d(&tmKV, &k_full[st], sK + st * KV_BYTES, kcol, tok0 + j * TK);
+        if (j >= NS) mbar_wait(&v_empty[st], ((j / NS) - 1) & 1);
+        mbar_expect_tx(&v_full[st], KV_BYTES);
+        tma_load_2d(&tmKV, &v_full[st], sV + st * KV_BYTES, vcol, tok0 + j * TK);
       }
+      ATRACE(10);
     }
-    float mx = -INFINITY;
+  } else if (warp >= 9) {
+    // MMA issuers, one thread per softmax group (warp 9: group 0, warp 10: group 1), each in its
+    // group's order: S_0, S_1, then P_i V_i and S_{i+2} as P_i is published and S_i's buffer is
+    // read.  One issuer alternating between the groups could not keep up: a tcgen05.mma issue costs
+    // ~80 cycles and a commit ~50 (profiles/r02_attn_tc_trace.jsonl), against ~0.5 us of softmax
+    // per 64-key tile.
+    if (lane == 0) {
+      const int g = warp - 9;
+      mbar_wait(&bar_q, 0);
+      const uint64_t dq = sw128_desc(sQ);
+      const int nl = (nkt - g + 1) / 2;
+      auto issue_s = [&](int i) {
+        const int j = 2 * i + g, b = i % SB, st = j % NS;
+        if (j < 8) ATRACE(56 + j);
+        mbar_wait(&k_full[st], (j / NS) & 1);
+        if (i >= SB) mbar_wait(&s_free[g][b], ((i / SB) - 1) & 1);  // the group has read S of tile i - SB
+        asm volatile("tcgen05.fence::after_thread_sync;");
+        const uint64_t dk = sw128_desc(sK + st * KV_BYTES);
 #pragma unroll
-    for (int e = 0; e < TK / 2; ++e) mx = fmaxf(mx, s[e]);
-    red[h][r] = mx;
-    __syncthreads();
-    const float mnew = fmaxf(mrow, fmaxf(red[0][r], red[1][r]) * scale_log2);
-    const float corr = (mrow == -INFINITY) ? 0.f : fast_exp2(mrow - mnew);
-    const float mref = (mnew == -INFINITY) ? 0.f : mnew;  // a fully masked row: every p = 2^-inf = 0
-    float rs = 0.f;
+        for (int kk = 0; kk < TD / 16; ++kk) umma_f16(t_s(g, b), dq + 2 * kk, dk + 2 * kk, IDESC_S, kk != 0);
+        umma_commit(&s_full[g][b]);
+        umma_commit(&k_empty[st]);  // K_j consumed
+      };
+      auto issue_pv = [&](int i) {
+        const int j = 2 * i + g, b = i & 1, st = j % NS;
+        mbar_wait(&p_full[g][b], (i >> 1) & 1);
+        mbar_wait(&v_full[st], (j / NS) & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;");
+        // V_j as the MN-major B operand: 128-byte swizzle atoms of 8 keys x 64 head dims, 1024 B
+        // apart along K (SBO); a 16-key step advances 2048 B (128 in descriptor units)
+        const uint64_t dpp = sw128_desc(sP + (2 * g + b) * P_BYTES), dv = sw128_desc(sV + st * KV_BYTES);
 #pragma unroll
-    for (int e = 0; e < TK / 2; ++e) {
-      const float p = fast_exp2(fmaf(s[e], scale_log2, -mref));
-      rs += p;
-      s[e] = p;
+        for (int kk = 0; kk < TK / 16; ++kk) umma_f16(t_o(g), dpp + 2 * kk, dv + 128 * kk, IDESC_O, (i | kk) != 0);
+        umma_commit(&o_full[g][b]);  // P_j's buffer is free again, O holds tiles <= j
+        umma_commit(&v_empty[st]);   // V_j consumed
+      };
+      for (int i = 0; i < nl && i < SB; ++i) issue_s(i);
+      for (int i = 0; i < nl; ++i) {
+        issue_pv(i);
+        if (i + SB < nl) issue_s(i + SB);
+      }
+      if (g == 0) ATRACE(9);
     }
-    lrow = lrow * corr + rs;
-    mrow = mnew;
-    // (4) O_{j-1} has landed: add it (with the correction of its own tile); P and V^T are free
-    if (j > 0) {
-      mbar_wait_spin(&bar_o[(j - 1) & 1], ((j - 1) >> 1) & 1);
+  } else {
+    // softmax group g = warp / 4: key tiles g, g + 2, g + 4, ...; thread r = query row r
+    const int g = warp >> 2, r = (warp & 3) * 32 + lane;
+    const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
+    const int qrow = q0 + r;
+    float mref = -INFINITY, lrow = 0.f;  // the row's softmax reference max (scaled units) and sum
+    const int nloc = (nkt - g + 1) / 2, nl0 = (nkt + 1) / 2, nl1 = nkt / 2;
+    if (g == 1 && nl0 > 0) named_arrive(2, 256);  // group 0 takes the first turn
+    for (int i = 0; i < nloc; ++i) {
+      const int j = 2 * i + g, b = i & 1, sb = i % SB, k0 = j * TK;
+      warp_wait(&s_full[g][sb], (i / SB) & 1);
+      if (tid == 0 && i < 8) ATRACE(16 + 4 * i);
       asm volatile("tcgen05.fence::after_thread_sync;");
-      uint32_t v[TD / 2];
+      float s[TK];
+      {
+        uint32_t v[TK];
 #pragma unroll
-      for (int c = 0; c < TD / 2; c += 16) tmem_ld16_nowait(t_o((j - 1) & 1) + lane_base + 32 * h + c, v + c);
-      tmem_ld_wait();
+        for (int c = 0; c < TK; c += 16) tmem_ld16_nowait(t_s(g, sb) + lane_base + c, v + c);
+        tmem_ld_wait();
 #pragma unroll
-      for (int e = 0; e < TD / 2; ++e) o[e] = o[e] * corr_prev + __uint_as_float(v[e]);
-      // V_{j-1}'s buffer is free (O_{j-1} done): V_{j+1} into it
-      if (tid == 0 && j + 1 < nkt) {
-        mbar_expect_tx(&bar_v[(j + 1) & 1], V_BYTES);
-        tma_load_2d(&tmQK, &bar_v[(j + 1) & 1], sV + ((j + 1) & 1) * V_BYTES, vcol, tok0 + k0 + TK);
+        for (int e = 0; e < TK; ++e) s[e] = __uint_as_float(v[e]);  // scaled inside the exponent
       }
-    }
-    corr_prev = corr;
-    // (5) P_j row half (K-block h) into the A-operand tile
-    {
-      uint8_t* pt = sP + h * (TQ * 64 * 2);
+      if (tid == 0 && i < 8) ATRACE(17 + 4 * i);
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&s_free[g][sb]);  // this warp's lanes of S_j are read
+      if (i == 0 && r == 0) ATRACE(2 + g);
+      if (r == 0 && j < 8) ATRACE(48 + j);
+      if (k0 + TK > seq || (causal && k0 + TK - 1 > qrow)) {  // only where a key can be invalid
 #pragma unroll
-      for (int c = 0; c < 8; ++c) {
+        for (int e = 0; e < TK; ++e) {
+          const int key = k0 + e;
+          if (key >= seq || (causal && key > qrow)) s[e] = -INFINITY;
+        }
+      }
+      float mx;
+      {  // 8 independent chains, not one 64-long dependency chain
+        float m8[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) m8[q] = s[q];
+#pragma unroll
+        for (int e = 8; e < TK; ++e) m8[e & 7] = fmaxf(m8[e & 7], s[e]);
+        mx = fmaxf(fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])), fmaxf(fmaxf(m8[4], m8[5]), fmaxf(m8[6], m8[7])));
+      }
+      mx *= scale_log2;
+      // move the reference only when the row max outgrows it by > 2^8 (or on the first finite max);
+      // O and the row sum then scale by f = 2^(old - new)
+      float f = 1.f;
+      const bool move = mx > mref + 8.f;
+      if (move) {
+        f = (mref == -INFINITY) ? 0.f : fast_exp2(mref - mx);
+        lrow *= f;
+        mref = mx;
+      }
+      if (i > 0 && __any_sync(0xffffffffu, move)) {  // collective: a lane that keeps its reference scales by 1
+        // the group's previous P V (into the O rows being rescaled) has completed
+        warp_wait(&o_full[g][(i - 1) & 1], ((i - 1) >> 1) & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;");
+#pragma unroll
+        for (int c = 0; c < TD; c += 16) {
+          uint32_t v[16];
+          tmem_ld16(t_o(g) + lane_base + c, v);
+#pragma unroll
+          for (int e = 0; e < 16; ++e) v[e] = __float_as_uint(__uint_as_float(v[e]) * f);
+          tmem_st16(t_o(g) + lane_base + c, v);
+        }
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      }
+      const float mr = (mref == -INFINITY) ? 0.f : mref;  // a fully masked row: every p = 2^-inf = 0
+      float r8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+      // the exponentials (MUFU, 16 per clock per SM: the softmax's bound) alternate between the
+      // groups, so one group's exponentials overlap the other's loads, P stores and waits
+      named_sync(2 + g, 256);
+#pragma unroll
+      for (int e = 0; e < TK; ++e) {
+        const float pv = fast_exp2(fmaf(s[e], scale_log2, -mr));
+        r8[e & 7] += pv;
+        s[e] = pv;
+      }
+      if (g == 0 ? i < nl1 : i + 1 < nl0) named_arrive(3 - g, 256);  // the other group's turn
+      lrow += ((r8[0] + r8[1]) + (r8[2] + r8[3])) + ((r8[4] + r8[5]) + (r8[6] + r8[7]));
+      if (tid == 0 && i < 8) ATRACE(18 + 4 * i);
+      // P_j (row r) into the group's A-operand buffer b, once P_{j-4} there has been consumed
+      if (i >= 2) warp_wait(&o_full[g][b], ((i - 2) >> 1) & 1);
+      uint8_t* pt = sP + (2 * g + b) * P_BYTES;
+#pragma unroll
+      for (int c = 0; c < TK / 8; ++c) {
         const float* pp = s + c * 8;
         uint4 u;
         u.x = Cvt<T>::from2(pp[0], pp[1]);
@@ -215,57 +317,66 @@ __global__ void __launch_bounds__(256, 1)
         u.w = Cvt<T>::from2(pp[6], pp[7]);
         *reinterpret_cast<uint4*>(pt + sw128_off(r, c * 8)) = u;
       }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // P -> the tensor core
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&p_full[g][b]);
+      if (tid == 0 && i < 8) ATRACE(19 + 4 * i);
     }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // P -> the tensor core
-    asm volatile("tcgen05.fence::before_thread_sync;");
-    __syncthreads();
-    // (6) O_j = P_j V_j into TMEM buffer j & 1
-    if (tid == 0) {
-      mbar_wait_spin(&bar_v[j & 1], (j >> 1) & 1);
+    if (r == 0) ATRACE(4 + g);
+    float o[TD];
+    if (nloc > 0) {
+      warp_wait(&o_full[g][(nloc - 1) & 1], ((nloc - 1) >> 1) & 1);
       asm volatile("tcgen05.fence::after_thread_sync;");
-      // V_j as the MN-major B operand: 128-byte swizzle atoms of 8 keys x 64 head dims, 1024 B apart
-      // along K (SBO); a 16-key step advances 2048 B (128 in descriptor units)
-      const uint64_t dv = sw128_desc(sV + (j & 1) * V_BYTES);
+      uint32_t v[TD];
 #pragma unroll
-      for (int kb = 0; kb < 2; ++kb) {
-        const uint64_t dp_ = sw128_desc(sP + kb * (TQ * 64 * 2));
+      for (int c = 0; c < TD; c += 16) tmem_ld16_nowait(t_o(g) + lane_base + c, v + c);
+      tmem_ld_wait();
 #pragma unroll
-        for (int kk = 0; kk < 4; ++kk)
-          umma_f16(t_o(j & 1), dp_ + 2 * kk, dv + 128 * (kb * 4 + kk), IDESC_O, (kb | kk) != 0);
+      for (int e = 0; e < TD; ++e) o[e] = __uint_as_float(v[e]);
+    } else {
+#pragma unroll
+      for (int e = 0; e < TD; ++e) o[e] = 0.f;
+    }
+    const float mrow = mref;
+    if (r == 0) ATRACE(6 + g);
+    // merge the two groups (group 1 publishes, group 0 combines in a fixed order) and store
+    if (g == 1) {
+      float* mine = xs + r * 68;
+#pragma unroll
+      for (int e = 0; e < TD; e += 4) *reinterpret_cast<float4*>(mine + e) = make_float4(o[e], o[e + 1], o[e + 2], o[e + 3]);
+      mine[64] = mrow;
+      mine[65] = lrow;
+    }
+    named_sync(1, 256);
+    if (g == 0 && qrow < seq) {
+      const float* ot = xs + r * 68;
+      const float m1 = ot[64], l1 = ot[65];
+      const float m = fmaxf(mrow, m1);
+      const float a0 = (mrow == -INFINITY) ? 0.f : fast_exp2(mrow - m);
+      const float a1 = (m1 == -INFINITY) ? 0.f : fast_exp2(m1 - m);
+      const float l = lrow * a0 + l1 * a1;
+      const float inv = l > 0.f ? 1.f / l : 0.f;
+      const float c0 = a0 * inv, c1 = a1 * inv;
+      uint4* dst = reinterpret_cast<uint4*>(ctx + (size_t)(tok0 + qrow) * H + head * TD);
+#pragma unroll
+      for (int c = 0; c < TD / 8; ++c) {
+        float v[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[e] = o[c * 8 + e] * c0 + ot[c * 8 + e] * c1;
+        uint4 u;
+        u.x = Cvt<T>::from2(v[0], v[1]);
+        u.y = Cvt<T>::from2(v[2], v[3]);
+        u.z = Cvt<T>::from2(v[4], v[5]);
+        u.w = Cvt<T>::from2(v[6], v[7]);
+        dst[c] = u;
       }
-      umma_commit(&bar_o[j & 1]);
     }
-  }
-  {  // the last O tile
-    const int jl = nkt - 1;
-    mbar_wait_spin(&bar_o[jl & 1], (jl >> 1) & 1);
-    asm volatile("tcgen05.fence::after_thread_sync;");
-    uint32_t v[TD / 2];
-#pragma unroll
-    for (int c = 0; c < TD / 2; c += 16) tmem_ld16_nowait(t_o(jl & 1) + lane_base + 32 * h + c, v + c);
-    tmem_ld_wait();
-#pragma unroll
-    for (int e = 0; e < TD / 2; ++e) o[e] = o[e] * corr_prev + __uint_as_float(v[e]);
-  }
-  red[h][r] = lrow;  // the two halves' partial sums
-  __syncthreads();
-  if (qrow < seq) {
-    const float l = red[0][r] + red[1][r];
-    const float inv = l > 0.f ? 1.f / l : 0.f;
-    uint4* dst = reinterpret_cast<uint4*>(ctx + (size_t)(tok0 + qrow) * H + head * TD + 32 * h);
-#pragma unroll
-    for (int c = 0; c < 4; ++c) {
-      uint4 u;
-      u.x = Cvt<T>::from2(o[c * 8 + 0] * inv, o[c * 8 + 1] * inv);
-      u.y = Cvt<T>::from2(o[c * 8 + 2] * inv, o[c * 8 + 3] * inv);
-      u.z = Cvt<T>::from2(o[c * 8 + 4] * inv, o[c * 8 + 5] * inv);
-      u.w = Cvt<T>::from2(o[c * 8 + 6] * inv, o[c * 8 + 7] * inv);
-      dst[c] = u;
-    }
+    if (tid == 0) ATRACE(8);
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
+  if (warp == 9) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
 }
 
 }  // namespace
@@ -277,9 +388,11 @@ bool attention_tc_supported(int ldqkv, int H, int heads, const void* qkv) {
 void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
                          bool causal, cudaStream_t s) {
   const int T = batch * seq;
-  // one map over the whole qkv matrix: box [128 rows][64 columns] with the 128-byte swizzle, for
-  // the Q tile (columns h*64) and the K tiles (columns H + h*64); rows past T read as zeros
-  const CUtensorMap m = make_kmajor_map(qkv, dtype, T, 3 * H, ldqkv, 128);
+  // maps over the whole qkv matrix with the 128-byte swizzle: box [128 rows][64 columns] for the Q
+  // tile (columns h*64), [64 rows][64 columns] for the K / V tiles (columns H + h*64, 2H + h*64);
+  // rows past T read as zeros
+  const CUtensorMap mq = make_kmajor_map(qkv, dtype, T, 3 * H, ldqkv, TQ);
+  const CUtensorMap mkv = make_kmajor_map(qkv, dtype, T, 3 * H, ldqkv, TK);
   const float scale_log2 = 1.4426950408889634f / 8.0f;  // log2(e) / sqrt(64)
   const dim3 grid(heads, (seq + TQ - 1) / TQ, batch);
   auto go = [&](auto tag) {
@@ -288,8 +401,8 @@ void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int b
     if (first_on_device(attr))
       DP_CUDA(cudaFuncSetAttribute(attention_tc_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)SMEM_BYTES));
-    launch_kernel(attention_tc_kernel<T>, grid, dim3(256), SMEM_BYTES, s, m, (const T*)qkv, ldqkv, (T*)ctx, seq, H,
-                  causal ? 1 : 0, scale_log2);
+    launch_kernel(attention_tc_kernel<T>, grid, dim3(NTHR), SMEM_BYTES, s, mq, mkv, (T*)ctx, seq, H, causal ? 1 : 0,
+                  scale_log2);
   };
   if (dtype == DP_BF16)
     go(__nv_bfloat16{});
@@ -299,3 +412,10 @@ void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int b
 }
 
 }  // namespace dp
+
+#ifdef DP_ATT_TRACE
+extern "C" __attribute__((visibility("default"))) int dp_debug_att_trace(void* host, int nblocks) {
+  if (nblocks > 2048) nblocks = 2048;
+  return (int)cudaMemcpyFromSymbol(host, dp::g_att_trace, size_t(nblocks) * 64 * sizeof(unsigned long long));
+}
+#endif

@@ -71,6 +71,30 @@ extern "C" dp_status dp_linear(const void* x, int32_t ldx, const void* w, const 
   });
 }
 
+extern "C" dp_status dp_gemm_tc(const void* x, int32_t ldx, const void* w, const void* b, const void* residual,
+                                int32_t ldr, void* y, int32_t ldy, int32_t M, int32_t N, int32_t K, int32_t act,
+                                int32_t dtype, int32_t io, int32_t bn, int32_t split, void* stream) {
+  return guard([&] {
+    check_dtype(dtype);
+    DP_CHECK(dtype != DP_FP32, DP_ERR_UNSUPPORTED, "the tcgen05 path has no fp32 kind");
+    DP_CHECK(x && w && y, DP_ERR_INVALID, "NULL pointer");
+    DP_CHECK(M >= 0 && N > 0 && K > 0 && ldx >= K && ldy >= N && (!residual || ldr >= N), DP_ERR_INVALID,
+             "bad shapes / strides");
+    DP_CHECK(act >= 0 && act <= 3, DP_ERR_INVALID, "act must be 0..3");
+    DP_CHECK(bn == 0 || bn == 32 || bn == 64 || bn == 96 || bn == 128 || bn == 256 || bn == -64 || bn == -128 ||
+                 bn == -192 || bn == -256,
+             DP_ERR_INVALID, "bn must be 0, 32/64/96/128/256 or -64/-128/-192/-256");
+    DP_CHECK(bn >= 0 || N % 256 == 0, DP_ERR_INVALID, "a CTA pair needs N % 256 == 0");
+    DP_CHECK(split == 0 || split == 1 ||
+                 ((split & (split - 1)) == 0 && split <= 8 && bn > 0 && bn <= 128 && split <= K / 64),
+             DP_ERR_INVALID, "split must be 0, 1, or 2/4/8 <= K/64 with a single-CTA bn <= 128");
+    cudaPointerAttributes at;
+    DP_CUDA(cudaPointerGetAttributes(&at, w));
+    DP_CHECK(at.type == cudaMemoryTypeDevice, DP_ERR_INVALID, "the tcgen05 path needs W in device memory");
+    launch_gemm_tc(dtype, x, ldx, w, b, residual, ldr, y, ldy, M, N, K, act, io, bn, (cudaStream_t)stream, split);
+  });
+}
+
 extern "C" dp_status dp_layernorm(const void* x, const void* r, const void* g, const void* b, void* y, int32_t rows,
                                   int32_t n, double eps, int32_t dtype, int32_t x_f32, void* stream) {
   return guard([&] {

@@ -73,7 +73,7 @@ struct ForwardArgs {
   int kernels = 0;
   int bn_hint = 0;
   bool pdl = false;  // chain kernels with programmatic dependent launch (opts.use_pdl)
-  bool attention_tc = false;  // K5t tcgen05 attention (opts.attention_tc)
+  int attention_tc = 0;  // attention core choice (opts.attention_tc: 0 by length, 1 K5t, 2 K5 / K5b)
 };
 
 void ensure_workspace(dp_model* m, int dev, int64_t tokens);

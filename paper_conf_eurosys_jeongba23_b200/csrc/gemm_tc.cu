@@ -144,6 +144,74 @@ __device__ __forceinline__ float ld_cluster_f32(uint32_t addr) {
   return v;
 }
 
+// The epilogue's kernel parameters, copied to shared memory in the prologue: read from the
+// constant bank only after the mainloop, each cold parameter line cost a constant-cache miss on
+// the critical path (the compiler rematerialises a register copy from the bank, so the copy has
+// to be opaque to it).
+struct EpiParams {
+  const void* res;
+  int ldr, ycol, io, mcount;
+};
+
+// Single-split epilogue, shared by K2 and its CTA-pair variant: straight from TMEM to the
+// output.  Each thread owns one W row (feature n) and walks the token columns 16 at a time:
+// + bias, activation, + residual (a warp's 32 lanes read 32 consecutive features of a token:
+// coalesced), and writes the value into an output tile in shared memory laid out like Y
+// ([BN tokens][128 features], the output dtype) -- a warp writes 32 consecutive elements per
+// token, conflict-free.  One TMA bulk tensor store then writes the tile (rows past M are
+// clipped by the tensor map), replacing the fp32 round trip through shared memory and the
+// per-thread 16-byte stores of round 1.  `otile` is the ring, free once the MMAs are done.
+template <class T, int BN, int ACT>
+__device__ __forceinline__ void store_tile(uint8_t* otile, uint32_t tmem_d, const float* sbias,
+                                           const CUtensorMap* tmY, int n0, int m0, const EpiParams& ep) {
+  if (threadIdx.x == 64) TRACE(14);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const void* res = ep.res;
+  const int ldr = ep.ldr, ycol = ep.ycol, mcount = ep.mcount;
+  const bool res32 = ep.io & IO_RES_F32, out32 = ep.io & IO_OUT_F32;
+  // TMEM lane = W row within the tile; warp w reads its lane quarter (w % 4) for the column
+  // half w / 4 of the tile
+  const int row = (warp & 3) * 32 + lane;
+  const int chalf = (warp >> 2) * (BN / 2);
+  const int n = n0 + row;
+  const float bsv = sbias[row];
+#pragma unroll 1
+  for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
+    float rv[16];
+    if (res != nullptr) {
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        const int ml = c0 + j;
+        rv[j] = ml < mcount ? load1<T>(res, (size_t)(m0 + ml) * ldr + n, res32) : 0.f;
+      }
+    }
+    uint32_t v[16];
+    if (threadIdx.x == 0 && c0 == 0) TRACE(9);
+    tmem_ld16(tmem_d + (uint32_t((warp & 3) * 32) << 16) + c0, v);
+    if (threadIdx.x == 0 && c0 == 0) TRACE(10);
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+      float a = apply_act_c<ACT>(__uint_as_float(v[j]) + bsv);
+      if (res != nullptr) a += rv[j];
+      if (out32)
+        reinterpret_cast<float*>(otile)[(c0 + j) * BM + row] = a;
+      else
+        reinterpret_cast<T*>(otile)[(c0 + j) * BM + row] = Cvt<T>::from1(a);
+    }
+  }
+  if (threadIdx.x == 0) TRACE(11);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
+  if (threadIdx.x == 0) TRACE(12);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    TRACE(6);
+    TRACE(7);
+    tma_store_2d(tmY, otile, n0 + ycol, m0);
+    bulk_commit();
+    bulk_wait0();  // the tile is written (and its shared memory read) before the CTA exits
+  }
+}
+
 // Split-K over a thread-block cluster: blockIdx.z = group * splits + split, and the `splits`
 // CTAs of one output tile form a cluster (1 x 1 x splits).  Each accumulates its K range in
 // TMEM and stages its fp32 tile in its own shared memory; after one cluster barrier rank r
@@ -174,6 +242,7 @@ __global__ void __launch_bounds__(NT, 1)
   __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], done_bar, recv_bar;
   __shared__ uint32_t tmem_base_sh;
   __shared__ float sbias[BM];
+  __shared__ EpiParams ep;
 
   TRACE(0);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -191,6 +260,8 @@ __global__ void __launch_bounds__(NT, 1)
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmW)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
+    ep = EpiParams{res, ldr, (int)ycol, io, mcount};
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full_bar[s], 1);
       mbar_init(&empty_bar[s], 1);
@@ -268,6 +339,7 @@ __global__ void __launch_bounds__(NT, 1)
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (threadIdx.x == 0) TRACE(5);
+  if (threadIdx.x == 64) TRACE(13);
   // split-K: announce that this CTA's MMAs are done, i.e. its TMA ring -- which the receive
   // slots below overlap -- is free.  Peers push into our receive slots only after the
   // matching wait.  (An arrive right after setup let a fast peer push while a slow CTA was
@@ -282,47 +354,7 @@ __global__ void __launch_bounds__(NT, 1)
   const int chalf = (warp >> 2) * (BN / 2);
   float* tile = reinterpret_cast<float*>(smem);
   if (splits == 1) {
-    // Single split: straight from TMEM to the output.  Each thread owns one W row (feature n) and
-    // walks the token columns 16 at a time: + bias, activation, + residual (a warp's 32 lanes read
-    // 32 consecutive features of a token: coalesced), and writes the value into an output tile in
-    // shared memory laid out like Y ([BN tokens][128 features], the output dtype) -- a warp writes
-    // 32 consecutive elements per token, conflict-free.  One TMA bulk tensor store then writes the
-    // tile (rows past M are clipped by the tensor map), replacing the fp32 round trip through
-    // shared memory and the per-thread 16-byte stores of round 1.
-    uint8_t* otile = smem;  // the ring is free once the MMAs are done
-    const int n = n0 + row;
-    const float bsv = sbias[row];
-#pragma unroll 1
-    for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
-      float rv[16];
-      if (res != nullptr) {
-#pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const int ml = c0 + j;
-          rv[j] = ml < mcount ? load1<T>(res, (size_t)(m0 + ml) * ldr + n, res32) : 0.f;
-        }
-      }
-      uint32_t v[16];
-      tmem_ld16(tmem_d + (uint32_t((warp & 3) * 32) << 16) + c0, v);
-#pragma unroll
-      for (int j = 0; j < 16; ++j) {
-        float a = apply_act_c<ACT>(__uint_as_float(v[j]) + bsv);
-        if (res != nullptr) a += rv[j];
-        if (out32)
-          reinterpret_cast<float*>(otile)[(c0 + j) * BM + row] = a;
-        else
-          reinterpret_cast<T*>(otile)[(c0 + j) * BM + row] = Cvt<T>::from1(a);
-      }
-    }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      TRACE(6);
-      TRACE(7);
-      tma_store_2d(&tmY, otile, n0 + (int)ycol, m0);
-      bulk_commit();
-      bulk_wait0();  // the tile is written (and its shared memory read) before the CTA exits
-    }
+    store_tile<T, BN, ACT>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
   } else {
     // 1) TMEM -> shared memory: this split's fp32 partial tile [128 W rows][BN tokens], unpadded,
     //    so each owner's rows are one contiguous block to push
@@ -413,6 +445,183 @@ __global__ void __launch_bounds__(NT, 1)
   }
 }
 
+// ---------------------------------------------------------------------------------------------
+// K2p: the CTA-pair variant (tcgen05 cta_group::2).  Two CTAs of a (2 x 1 x 1) cluster -- one
+// TPC -- compute a 256 x BN output tile with M = 256 MMAs issued by the even CTA (the leader):
+// each CTA stages its own 128 W rows (the MMA's A halves) and HALF of the tile's BN tokens
+// (the B halves), and the tensor cores read the peer's B half over the pair's shared-memory
+// path.  Per CTA the ingest drops from 128 + BN to 128 + BN / 2 rows per k-block at the same
+// MMA work; at the large models' shapes (M = 384 / 1024 tokens) the single-CTA mainloop was
+// bound by what an SM can pull from L2 (~110 GB/s per SM, profiles/r02_gemm_trace.jsonl), not
+// by the tensor pipe.  Each CTA's TMEM holds its own 128 W rows x all BN tokens, so the
+// epilogue is K2's, per CTA.
+//   * both CTAs' TMA loads complete on the LEADER's full barrier (the leader arms it with the
+//     pair's bytes); the leader's MMA commits multicast to both CTAs' empty / done barriers;
+//   * TMEM is allocated / freed by warp 1 of both CTAs (cta_group::2), and a cluster barrier
+//     separates barrier init / allocation from the first TMA and the epilogue from the free.
+template <int BN>
+__host__ __device__ constexpr int stages_for_pair() {
+  constexpr int bytes = BM * BK * 2 + (BN / 2) * BK * 2;
+  constexpr int s = (224 * 1024) / bytes;
+  return s > 12 ? 12 : s;
+}
+
+__device__ __forceinline__ void tma_load_2d_pair(const CUtensorMap* map, uint32_t bar_cluster, void* dst, int c0,
+                                                 int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, "
+      "%3}], [%4];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(bar_cluster)
+      : "memory");
+}
+__device__ __forceinline__ void umma_f16_pair(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+// arrive on the barrier at this shared::cta offset in both CTAs of the pair when the MMAs
+// issued so far complete
+__device__ __forceinline__ void umma_commit_pair(uint64_t* bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          smem_u32(bar)),
+      "h"((unsigned short)3)
+      : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <class T, int BN, int ACT>
+__global__ void __launch_bounds__(NT, 1)
+    gemm_tc_pair_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
+                        const __grid_constant__ CUtensorMap tmY, const void* res, int ldr, int M, int K, int io,
+                        int nst) {
+  constexpr int HB = BN / 2;                 // tokens staged by each CTA
+  constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
+  constexpr uint32_t B_BYTES = HB * BK * 2;
+  constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
+  constexpr int STAGES = stages_for_pair<BN>();
+  constexpr uint32_t TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  // kind::f16, fp32 accumulate, A/B K-major, M = 256 (the pair), N = BN
+  constexpr uint32_t IDESC = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(BN >> 3) << 17) |
+                             (uint32_t((2 * BM) >> 4) << 24);
+  static_assert(BN % 32 == 0 && BN >= 64 && BN <= 256, "pair tile: BN in 64..256, a multiple of 32");
+
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  __shared__ __align__(8) uint64_t full_bar[STAGES], empty_bar[STAGES], done_bar;
+  __shared__ uint32_t tmem_base_sh;
+  __shared__ float sbias[BM];
+  __shared__ EpiParams ep;
+
+  TRACE(0);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cta_cluster_rank();  // = blockIdx.x & 1
+  const int n0 = blockIdx.x * BM, m0 = blockIdx.y * BN;
+  const int xrow = m0 + int(rank) * HB;
+  const CUtensorMap* tmW = &grp.w[blockIdx.z];
+  const T* bias = static_cast<const T*>(grp.bias[blockIdx.z]);
+  const int ycol = (int)grp.ycol[blockIdx.z];
+  const int num_kb = K / BK;
+  const int mcount = min(BN, M - m0);
+  const bool res32 = io & IO_RES_F32, out32 = io & IO_OUT_F32;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmW)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
+    ep = EpiParams{res, ldr, ycol, io, mcount};
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full_bar[s], 1);
+      mbar_init(&empty_bar[s], 1);
+    }
+    mbar_init(&done_bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base_sh)),
+                 "r"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  // the leader's barriers are initialised (the peer's loads complete on them) and both CTAs'
+  // TMEM is allocated before anything is issued
+  cluster_sync_all();
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  const uint32_t tmem_d = tmem_base_sh;
+  const bool leader = rank == 0;
+  // the leader's full barrier of stage s, as a shared::cluster address
+  const uint32_t full0 = mapa_u32(smem_u32(&full_bar[0]), 0);
+  const int pre = num_kb < nst ? num_kb : nst;
+  if (warp == 0 && lane == 0) {
+    // weights never depend on the previous kernel: the first ring of W tiles before the PDL wait
+    for (int kb = 0; kb < pre; ++kb) {
+      if (leader) mbar_expect_tx(&full_bar[kb], 2 * STAGE_BYTES);
+      tma_load_2d_pair(tmW, full0 + kb * 8, smem + kb * STAGE_BYTES, kb * BK, n0);
+    }
+    TRACE(1);
+  }
+  pdl_trigger();
+  if (threadIdx.x < BM) sbias[threadIdx.x] = bias != nullptr ? Cvt<T>::to1(bias[n0 + threadIdx.x]) : 0.f;
+  if (threadIdx.x == 0) TRACE(2);
+  pdl_wait();
+  if (threadIdx.x == 0) TRACE(3);
+
+  if (warp == 0 && lane == 0) {
+    // TMA producer (both CTAs: own W rows, own half of the tokens)
+    for (int kb = 0; kb < num_kb; ++kb) {
+      const int s = kb % nst;
+      uint8_t* a = smem + s * STAGE_BYTES;
+      if (kb >= pre) {
+        mbar_wait(&empty_bar[s], ((kb / nst) - 1) & 1);
+        if (leader) mbar_expect_tx(&full_bar[s], 2 * STAGE_BYTES);
+        tma_load_2d_pair(tmW, full0 + s * 8, a, kb * BK, n0);
+      }
+      tma_load_2d_pair(&tmX, full0 + s * 8, a + A_BYTES, kb * BK, xrow);
+    }
+  } else if (warp == 1 && lane == 0 && leader) {
+    // MMA issuer (the leader only): the descriptors address the same offsets in both CTAs
+    for (int kb = 0; kb < num_kb; ++kb) {
+      const int s = kb % nst;
+      mbar_wait(&full_bar[s], (kb / nst) & 1);
+      if (kb == 0) TRACE(4);
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      const uint8_t* a = smem + s * STAGE_BYTES;
+      const uint64_t da = sw128_desc(a), db = sw128_desc(a + A_BYTES);
+#pragma unroll
+      for (int kk = 0; kk < BK / 16; ++kk) umma_f16_pair(tmem_d, da + 2 * kk, db + 2 * kk, IDESC, (kb | kk) != 0);
+      umma_commit_pair(&empty_bar[s]);
+    }
+    umma_commit_pair(&done_bar);
+  }
+  __syncwarp();
+  if (threadIdx.x == 32) mbar_wait_spin(&done_bar, 0);
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  if (threadIdx.x == 0) TRACE(5);
+  asm volatile("tcgen05.fence::after_thread_sync;");
+  store_tile<T, BN, ACT>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
+#ifdef DP_GEMM_TRACE
+  if (threadIdx.x == 0) {
+    TRACE(8);
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    const int b_ = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
+    if (b_ < 4096) g_gemm_trace[b_][15] = smid;
+  }
+#endif
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  cluster_sync_all();  // both CTAs are done with the pair's TMEM before it is freed
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_d), "r"(TMEM_COLS));
+  }
+}
+
 template <class T, int BN, int ACT>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
@@ -461,10 +670,71 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
                         dim3(1, 1, splits), s, g, mx, my, res, ldr, y, ldy, M, N, K, act, io, splits, nst);
 }
 
+// K2p host side: grid (N / 128, ceil(M / BN), groups), clusters of 2 along x (the pair's two
+// 128-row W halves), one wave of BN-token tiles.
+template <class T, int BN, int ACT>
+void run_pair(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
+              const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int io,
+              cudaStream_t s) {
+  constexpr int STAGES = stages_for_pair<BN>();
+  constexpr size_t STAGE_BYTES = BM * BK * 2 + (BN / 2) * BK * 2;
+  constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
+  constexpr size_t epi_bytes = size_t(BM) * BN * 4;
+  static_assert(epi_bytes + 1024 <= smem_max, "the output tile must fit the ring");
+  static const int env_st = experiment_env("DP_GEMM_STAGES", 0);
+  int nst = env_st > 0 ? std::min(env_st, STAGES) : STAGES;
+  nst = std::max(nst, int((epi_bytes + STAGE_BYTES - 1) / STAGE_BYTES));
+  const size_t smem = size_t(nst) * STAGE_BYTES + 1024;
+  static std::atomic<unsigned> attr{0};
+  if (first_on_device(attr))
+    DP_CUDA(cudaFuncSetAttribute(gemm_tc_pair_kernel<T, BN, ACT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smem_max));
+  const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
+  GemmGroup g;
+  std::memset(&g, 0, sizeof(g));
+  for (int i = 0; i < ngroups; ++i) {
+    g.w[i] = make_kmajor_map(w[i], dtype, N, K, K, BM);
+    g.bias[i] = bias ? bias[i] : nullptr;
+    g.ycol[i] = ycol ? ycol[i] : 0;
+  }
+  CUtensorMap mx = make_kmajor_map(x, dtype, M, K, ldx, BN / 2);
+  const bool o32 = (io & IO_OUT_F32) != 0;
+  const uint64_t ydims[2] = {(uint64_t)ldy, (uint64_t)M};
+  const uint64_t ystr[1] = {(uint64_t)ldy * (o32 ? 4 : 2)};
+  const uint32_t ybox[2] = {(uint32_t)BM, (uint32_t)BN};
+  CUtensorMap my = make_plain_map(y, o32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                         : (dtype == DP_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                                             : CU_TENSOR_MAP_DATA_TYPE_FLOAT16),
+                                  2, ydims, ystr, ybox);
+  launch_kernel_cluster(gemm_tc_pair_kernel<T, BN, ACT>, dim3(N / BM, (M + BN - 1) / BN, ngroups), dim3(NT), smem,
+                        dim3(2, 1, 1), s, g, mx, my, res, ldr, M, K, io, nst);
+}
+
 template <class T>
-void dispatch(int bn, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
+void dispatch(int bn, bool pair, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
               const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io,
               int sp, cudaStream_t s) {
+  if (pair) {
+#define DP_RUNP(B, A) run_pair<T, B, A>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, io, s)
+#define DP_ACTSP(B)                                            \
+  switch (act) {                                               \
+    case ACT_NONE: DP_RUNP(B, ACT_NONE); break;                \
+    case ACT_GELU_ERF: DP_RUNP(B, ACT_GELU_ERF); break;        \
+    case ACT_GELU_TANH: DP_RUNP(B, ACT_GELU_TANH); break;      \
+    case ACT_TANH: DP_RUNP(B, ACT_TANH); break;                \
+    default: fail(DP_ERR_INVALID, "gemm: unknown activation"); \
+  }
+    switch (bn) {
+      case 64: DP_ACTSP(64); break;
+      case 128: DP_ACTSP(128); break;
+      case 192: DP_ACTSP(192); break;
+      case 256: DP_ACTSP(256); break;
+      default: fail(DP_ERR_INVALID, "gemm: CTA-pair BN must be 64/128/192/256");
+    }
+#undef DP_ACTSP
+#undef DP_RUNP
+    return;
+  }
 #define DP_RUN(B, A) run<T, B, A>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s)
 #define DP_ACTS(B)                                 \
   switch (act) {                                   \
@@ -509,10 +779,11 @@ static int pick_bn(int M, int N) {
 // Picks the best measured configuration at every swept shape.
 struct GemmCfg {
   int bn, sp;
+  bool pair;
 };
 static GemmCfg pick_cfg(int M, int N, int K) {
   const int ntile = N / BM, kb = K / BK;
-  GemmCfg best{pick_bn(M, N), 1};
+  GemmCfg best{pick_bn(M, N), 1, false};
   double best_t = 1e30;
   for (int bn : {32, 64, 128, 256}) {
     if (bn > 32 && M < bn) continue;
@@ -524,7 +795,7 @@ static GemmCfg pick_cfg(int M, int N, int K) {
       const double t = std::max(waves * per / 1e5, ctas * per / 8e6) + (sp > 1 ? 1.2 : 0.0);
       if (t < best_t - 1e-9) {
         best_t = t;
-        best = {bn, sp};
+        best = {bn, sp, false};
       }
     }
   }
@@ -533,7 +804,7 @@ static GemmCfg pick_cfg(int M, int N, int K) {
 
 static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias,
                       const long long* ycol, const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act,
-                      int io, int bn_hint, cudaStream_t s) {
+                      int io, int bn_hint, int sp_hint, cudaStream_t s) {
   DP_CHECK(gemm_tc_supported(N, K), DP_ERR_UNSUPPORTED, "tcgen05 GEMM needs N % 128 == 0 and K % 64 == 0");
   DP_CHECK(ngroups >= 1 && ngroups <= 3, DP_ERR_INVALID, "gemm: 1..3 weight groups");
   DP_CHECK(ldx % 8 == 0 && ((uintptr_t)x % 16) == 0, DP_ERR_INVALID, "GEMM activations must be 16-byte aligned");
@@ -546,28 +817,43 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
   static const int env_bn = experiment_env("DP_GEMM_BN", 0);
   static const int env_sp = experiment_env("DP_GEMM_SPLIT", 0);
   const GemmCfg cfg = pick_cfg(M, N * ngroups, K);
+  // bn_hint: 0 = the model's configuration, > 0 = a single-CTA tile of that width, < 0 = a
+  // CTA pair (K2p) of width -bn_hint
+  const bool hint_pair = bn_hint < 0;
+  if (hint_pair) bn_hint = -bn_hint;
   const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : cfg.bn);
-  int sp = env_sp > 0 ? env_sp : (bn_hint > 0 || env_bn > 0 ? 1 : cfg.sp);
+  int sp = sp_hint > 0 ? sp_hint : env_sp > 0 ? env_sp : (bn_hint > 0 || env_bn > 0 ? 1 : cfg.sp);
   sp = std::max(1, std::min(std::min(sp, 8), K / BK));
   while (sp & (sp - 1)) --sp;  // a power of two: every rank owns BM / sp rows
   if (bn >= 256) sp = 1;       // the send + receive buffers (2 x 128 x BN fp32) must fit the ring
+  // CTA pair (K2p): the model's choice unless a tile width is forced; DP_GEMM_PAIR=1 forces it
+  // (with DP_GEMM_BN as the pair's tile width) for experiments
+  static const int env_pair = experiment_env("DP_GEMM_PAIR", -1);
+  bool pair = bn_hint > 0 || env_bn > 0 ? hint_pair : cfg.pair;
+  if (env_pair >= 0) pair = env_pair > 0;
+  if (pair) {
+    DP_CHECK((N / BM) % 2 == 0, DP_ERR_INVALID, "gemm: a CTA pair needs N % 256 == 0");
+    sp = 1;
+  }
   if (dtype == DP_BF16)
-    dispatch<__nv_bfloat16>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
+    dispatch<__nv_bfloat16>(bn, pair, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
   else
-    dispatch<__half>(bn, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
+    dispatch<__half>(bn, pair, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);
 }
 
 void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
                           const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
-                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
+                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s, int sp_hint) {
   if (ablate_mask() & 4) return;
-  gemm_impl(dtype, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, bn_hint, s);
+  gemm_impl(dtype, x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, bn_hint, sp_hint, s);
 }
 
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
-                    void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s) {
+                    void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s,
+                    int sp_hint) {
   if (ablate_mask() & 4) return;
-  launch_gemm_tc_group(dtype, x, ldx, 1, &w, &bias, nullptr, res, ldr, y, ldy, M, N, K, act, io, bn_hint, s);
+  launch_gemm_tc_group(dtype, x, ldx, 1, &w, &bias, nullptr, res, ldr, y, ldy, M, N, K, act, io, bn_hint, s,
+                       sp_hint);
 }
 
 }  // namespace dp

@@ -316,11 +316,13 @@ extern "C" dp_status dp_context_set_opts(dp_context* ctx, const dp_engine_opts* 
     DP_CHECK(o->chunk_bytes >= 4096, DP_ERR_INVALID, "chunk_bytes must be >= 4096");
     DP_CHECK(o->n_h2d_streams >= 1 && o->n_h2d_streams <= 8, DP_ERR_INVALID, "n_h2d_streams must be 1..8");
     DP_CHECK(o->gemm_bn == 0 || o->gemm_bn == 32 || o->gemm_bn == 64 || o->gemm_bn == 96 || o->gemm_bn == 128 ||
-                 o->gemm_bn == 256,
-             DP_ERR_INVALID, "gemm_bn must be 0/32/64/96/128/256");
+                 o->gemm_bn == 256 || o->gemm_bn == -64 || o->gemm_bn == -128 || o->gemm_bn == -192 ||
+                 o->gemm_bn == -256,
+             DP_ERR_INVALID, "gemm_bn must be 0/32/64/96/128/256 (one CTA) or -64/-128/-192/-256 (a CTA pair)");
     DP_CHECK(o->pt_transport == DP_PT_DMA || o->pt_transport == DP_PT_SM || o->pt_transport == DP_PT_CE,
              DP_ERR_INVALID, "pt_transport must be DP_PT_DMA, DP_PT_SM or DP_PT_CE");
     // measured slower and moved out of the library (tools/experiments)
+    DP_CHECK(o->attention_tc >= 0 && o->attention_tc <= 2, DP_ERR_INVALID, "attention_tc must be 0, 1 or 2");
     DP_CHECK(!o->fuse_ln && !o->persistent, DP_ERR_UNSUPPORTED,
              "fuse_ln / persistent: experiments kept in tools/experiments, not built into the library");
     ctx->opts = *o;
@@ -873,7 +875,7 @@ static dp_run_stats enqueue_cold(dp_context* ctx, dp_model* m, const dp_plan* pl
     pdl_state().block_next = true;  // the next kernel must see the landed weights: no PDL overlap
   };
   a.pdl = ctx->opts.use_pdl != 0;
-  a.attention_tc = ctx->opts.attention_tc != 0;
+  a.attention_tc = ctx->opts.attention_tc;
   if (trace) {  // an event on each side of the unit's dependency wait
     auto gate = a.before_unit;
     a.before_unit = [&, gate](int u) {
@@ -995,7 +997,7 @@ extern "C" dp_status dp_infer_warm(dp_context* ctx, dp_model* m, int32_t dev, co
     a.stream = (cudaStream_t)stream;
     a.bn_hint = ctx->opts.gemm_bn;
     a.pdl = ctx->opts.use_pdl != 0;
-  a.attention_tc = ctx->opts.attention_tc != 0;
+  a.attention_tc = ctx->opts.attention_tc;
     // Experiment (tools/wait_cost.py): the cost of a dependency wait before every unit on the
     // execution stream, all already satisfied -- 1: event wait, 2: one-thread acquire-spin
     // kernel on a device word, 3: cuStreamWaitValue32 (stream memory op)
@@ -1286,7 +1288,7 @@ void profile(dp_context* ctx, dp_model* m, int dev, int batch, int seq, int iter
     fa.stream = s;
     fa.bn_hint = ctx->opts.gemm_bn;
     fa.pdl = ctx->opts.use_pdl != 0;
-    fa.attention_tc = ctx->opts.attention_tc != 0;
+    fa.attention_tc = ctx->opts.attention_tc;
     // the host enqueues ~100 launches behind a ~1.5 ms spin, so e0..e1 is device time only
     const int64_t chain = timed([&] { run_forward(fa); }, true, 3000000);
     DP_CUDA(cudaStreamSynchronize(s));

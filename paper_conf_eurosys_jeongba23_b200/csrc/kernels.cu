@@ -721,7 +721,7 @@ __global__ void __launch_bounds__(128 * G) attention2_kernel(const T* __restrict
 }
 
 void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
-                      bool causal, cudaStream_t s, bool use_tc) {
+                      bool causal, cudaStream_t s, int tc_mode) {
   if (ablate_mask() & 1) return;
   DP_CHECK(heads > 0 && H % heads == 0 && H / heads == ATT_D, DP_ERR_UNSUPPORTED, "attention needs head dim 64");
   DP_CHECK(ldqkv % 8 == 0, DP_ERR_INVALID, "ldqkv must be a multiple of 8");
@@ -730,8 +730,10 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
     launch_attention_f32(qkv, ldqkv, ctx, batch, seq, H, heads, causal, s);
     return;
   }
-  // K5t (tcgen05, attn_tc.cu) when the engine option asks for it (opts.attention_tc; measured
-  // slower than K5 / K5b below at every hot-path shape)
+  // K5t (tcgen05, attn_tc.cu) from 768 tokens (tc_mode 0) or when forced (1): GPT-2 Medium S1024
+  // warm forward 2.02 -> 1.88 ms; at S <= 384 the mma.sync kernels below are as fast or faster
+  // (BERT-Large S384 1.364 vs 1.372 ms, GPT-2 S256 0.508 vs 0.560; profiles/r02_warm_attention_tc.jsonl)
+  const bool use_tc = tc_mode == 1 || (tc_mode == 0 && seq >= 768);
   if (use_tc && attention_tc_supported(ldqkv, H, heads, qkv)) {
     launch_attention_tc(dtype, qkv, ldqkv, ctx, batch, seq, H, heads, causal, s);
     return;

@@ -29,7 +29,7 @@ void launch_skinny_linear(int dtype, const void* x, int ldx, const void* w, cons
 
 // K5: attention core (mma.sync flash attention, d = 64).
 void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batch, int seq, int H, int heads,
-                      bool causal, cudaStream_t s, bool use_tc = false);  // use_tc: K5t (attn_tc.cu)
+                      bool causal, cudaStream_t s, int tc_mode = 0);  // tc_mode: opts.attention_tc
 
 // K5t: attention on tcgen05 (attn_tc.cu): S and O in TMEM, the softmax row per thread.
 bool attention_tc_supported(int ldqkv, int H, int heads, const void* qkv);
@@ -40,11 +40,14 @@ void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int b
 struct GemmPlan;  // cached tensor map for a weight
 bool gemm_tc_supported(int N, int K);
 void launch_gemm_tc(int dtype, const void* x, int ldx, const void* w, const void* bias, const void* res, int ldr,
-                    void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);
+                    void* y, int ldy, int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s,
+                    int sp_hint = 0);
+// bn_hint: 0 = the cost model's tile, > 0 one CTA per 128 x bn_hint tile, < 0 a CTA pair per
+// 256 x -bn_hint tile; sp_hint > 0 forces that many K splits (single-CTA tiles only).
 // ngroups (1..3) weights sharing X; group i writes y at column offset ycol[i].
 void launch_gemm_tc_group(int dtype, const void* x, int ldx, int ngroups, const void* const* w,
                           const void* const* bias, const long long* ycol, const void* res, int ldr, void* y, int ldy,
-                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s);
+                          int M, int N, int K, int act, int io, int bn_hint, cudaStream_t s, int sp_hint = 0);
 
 // fp32 storage (DP_FP32, kernels_f32.cu): CUDA-core kernels with the same contracts; the
 // launchers above dispatch to them when dtype == DP_FP32 (all activations are then fp32).

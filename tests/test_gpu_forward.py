@@ -351,16 +351,18 @@ def test_graph_replay_after_workspace_regrowth():
     c.close()
 
 
-@pytest.mark.parametrize("name,S", [("bert_large", 384), ("gpt2", 256), ("tiny_roberta", 77)])
-def test_attention_tc_engine_option(name, S):
-    """opts.attention_tc runs every layer's attention on K5t: the whole cold start stays within the
-    north star's tolerance of the oracle."""
+@pytest.mark.parametrize("name,S,mode", [("bert_large", 384, 1), ("gpt2", 256, 1), ("tiny_roberta", 77, 1),
+                                         ("gpt2", 1024, 0), ("gpt2", 1024, 2), ("bert_base", 512, 1)])
+def test_attention_tc_engine_option(name, S, mode):
+    """opts.attention_tc: 1 runs every layer's attention on K5t, 2 on the mma.sync kernels, 0 picks
+    K5t from 768 tokens: the whole cold start stays within the north star's tolerance of the
+    oracle in every mode."""
     m = synth.SHAPES[name]
     w = synth.make_weights(m, seed=41, dtype="fp16")
     ids = synth.make_ids(m, 1, S, seed=42)
     ref, ref_pool = F.forward(m, w, ids, "fp16")
     c = dp().Context([0])
-    c.set_opts(attention_tc=1)
+    c.set_opts(attention_tc=mode)
     model = dp().Model(c, m, w, "fp16")
     plan = dp().plan_generate(fake_cost(m, "fp16"), "DHA", 1)
     out, pool, _ = run_cold(model, plan, ids, "fp16")

@@ -243,8 +243,9 @@ def test_attention_parity(B, S, H, heads, causal, dtype):
     assert np.all(err <= tol), err.max()
 
 
-@pytest.mark.parametrize("B,S,H,heads", [(1, 32, 128, 2), (2, 77, 256, 4), (1, 128, 768, 12), (1, 384, 1024, 16),
-                                         (1, 1024, 1024, 16), (3, 200, 256, 4)])
+@pytest.mark.parametrize("B,S,H,heads", [(1, 1, 128, 2), (2, 5, 128, 2), (1, 32, 128, 2), (1, 64, 768, 12),
+                                         (1, 65, 128, 2), (2, 77, 256, 4), (1, 128, 768, 12), (1, 192, 256, 4),
+                                         (1, 384, 1024, 16), (1, 1024, 1024, 16), (3, 200, 256, 4)])
 @pytest.mark.parametrize("causal", [False, True])
 @pytest.mark.parametrize("dtype", ["fp16", "bf16"])
 def test_attention_tc_parity(B, S, H, heads, causal, dtype):
@@ -289,45 +290,57 @@ def test_fp32_residual_stream_io():
     close(f64(Y), ref, "fp16", K=N, scale=8)
 
 
-_SPLIT_SCRIPT = r"""
-import math, sys, numpy as np, torch
-sys.path.insert(0, '.')
-import synth
-from oracle import forward as F
-import paper_conf_eurosys_jeongba23_b200 as dp
-M, N, K = (int(v) for v in sys.argv[1:4])
-rng = np.random.default_rng(M + N + K)
-x = synth.round_to(rng.standard_normal((M, K)).astype(np.float32), 'fp16')
-w = synth.round_to((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32), 'fp16')
-b = synth.round_to((0.1 * rng.standard_normal(N)).astype(np.float32), 'fp16')
-r = synth.round_to(rng.standard_normal((M, N)).astype(np.float32), 'fp16')
-X, W, B, R = (torch.from_numpy(a).cuda() for a in (x, w, b, r))
-Y = torch.empty(M, N, dtype=torch.float16, device='cuda')
-Y2 = torch.empty_like(Y)
-dp.linear(X, K, W, B, R, N, Y, N, M, N, K, act='gelu_erf', path=0)
-dp.linear(X, K, W, B, R, N, Y2, N, M, N, K, act='gelu_erf', path=0)
-torch.cuda.synchronize()
-assert torch.equal(Y, Y2), 'split-K GEMM not deterministic'
-ref = F.linear(*(synth.storage_to_f64(a, 'fp16') for a in (x, w, b)), 'gelu_erf', synth.storage_to_f64(r, 'fp16'))
-err = np.abs(Y.double().cpu().numpy() - ref)
-tol = 2.0 ** -10 * np.abs(ref) + K * 2.0 ** -22 * 4 * np.abs(x).max() * np.abs(w).max() + 1e-6
-assert np.all(err <= tol), err.max()
-print('ok')
-"""
+def _gemm_forced_case(bn, split, M, N, K, act, res, dtype, seed):
+    """One forced tile configuration through dp_gemm_tc: parity with the oracle (the module's
+    fp32-accumulation bound) and run-to-run bit equality (every reduction order is fixed)."""
+    rng = np.random.default_rng(seed)
+    x = synth.round_to(rng.standard_normal((M, K)).astype(np.float32), dtype)
+    w = synth.round_to((rng.standard_normal((N, K)) / math.sqrt(K)).astype(np.float32), dtype)
+    b = synth.round_to((0.1 * rng.standard_normal(N)).astype(np.float32), dtype)
+    r = synth.round_to(rng.standard_normal((M, N)).astype(np.float32), dtype)
+    X, W, B, R = (to_t(a, dtype) for a in (x, w, b, r))
+    Y = torch.empty(M, N, dtype=DT[dtype], device="cuda")
+    Y2 = torch.empty_like(Y)
+    for out in (Y, Y2):
+        dp().gemm_tc(X, K, W, B, R if res else None, N, out, N, M, N, K, act=act, bn=bn, split=split, dtype=dtype)
+    torch.cuda.synchronize()
+    assert torch.equal(Y, Y2), "forced GEMM configuration not deterministic"
+    x64, w64, b64, r64 = (synth.storage_to_f64(a, dtype) for a in (x, w, b, r))
+    ref = F.linear(x64, w64, b64, act, r64 if res else None)
+    close(f64(Y), ref, dtype, K=K, scale=np.abs(x64).max() * np.abs(w64).max() * 4)
 
 
 @pytest.mark.parametrize("bn,split,M,N,K", [(32, 2, 128, 768, 768), (32, 4, 128, 768, 3072), (32, 8, 100, 256, 1024),
                                              (64, 4, 200, 512, 2048), (128, 2, 384, 1024, 1024),
                                              (128, 4, 333, 768, 4096), (64, 8, 64, 128, 4096)])
 def test_gemm_split_k_cluster_configs(bn, split, M, N, K):
-    """Every (BN, split) the cluster split-K path can take, forced through DP_GEMM_BN /
-    DP_GEMM_SPLIT in a fresh process (they are read once): parity with the oracle and
-    run-to-run bit equality (the reduction order is fixed)."""
-    import os
-    import subprocess
-    import sys
-    env = dict(os.environ, DP_GEMM_BN=str(bn), DP_GEMM_SPLIT=str(split))
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", _SPLIT_SCRIPT, str(M), str(N), str(K)], env=env, cwd=root,
-                       capture_output=True, text=True, timeout=120)
-    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stderr[-2000:]
+    """Every (BN, split) the cluster split-K path can take, forced through dp_gemm_tc."""
+    _gemm_forced_case(bn, split, M, N, K, "gelu_erf", True, "fp16", M + N + K)
+
+
+@pytest.mark.parametrize("bn", [32, 64, 96, 128, 256])
+@pytest.mark.parametrize("M,N,K", [(100, 256, 512), (384, 1024, 1024), (1024, 512, 128)])
+def test_gemm_single_cta_tile_widths(bn, M, N, K):
+    """Every single-CTA tile width (K2) forced, ragged token tails included."""
+    _gemm_forced_case(bn, 1, M, N, K, "gelu_tanh", True, "bf16", bn + M + N + K)
+
+
+@pytest.mark.parametrize("bn", [-64, -128, -192, -256])
+@pytest.mark.parametrize("M,N,K,dtype", [(1024, 4096, 1024, "fp16"), (384, 1024, 4096, "bf16"), (333, 2304, 768, "fp16"),
+                                         (1, 256, 64, "fp16"), (100, 512, 64, "bf16"), (1000, 768, 3072, "fp16")])
+def test_gemm_cta_pair_parity(bn, M, N, K, dtype):
+    """K2p (tcgen05 cta_group::2, one 256 x |bn| tile per CTA pair): parity at the large models'
+    shapes and ragged cases -- a token tile where only the leader's half holds rows (M = 1,
+    M = 100 < |bn| / 2 for some widths), K = 64 (one k-block), a tail past M."""
+    for act, res in (("none", False), ("gelu_erf", True)):
+        _gemm_forced_case(bn, 0, M, N, K, act, res, dtype, -bn + M + N + K)
+
+
+def test_gemm_cta_pair_rejects_odd_tile_count():
+    X = torch.zeros(128, 64, dtype=torch.float16, device="cuda")
+    W = torch.zeros(384, 64, dtype=torch.float16, device="cuda")
+    Y = torch.empty(128, 384, dtype=torch.float16, device="cuda")
+    with pytest.raises(dp().DeepPlanError, match="N % 256"):
+        dp().gemm_tc(X, 64, W, None, None, 0, Y, 384, 128, 384, 64, bn=-128)
+    with pytest.raises(dp().DeepPlanError, match="bn must be"):
+        dp().gemm_tc(X, 64, W, None, None, 0, Y, 384, 128, 384, 64, bn=48)
