@@ -199,9 +199,9 @@ typedef struct {
                              every unit's dependency wait on the execution stream.  Costs event
                              records between kernels (no PDL overlap) and forces eager enqueue (no
                              graph): a measurement mode [0] */
-  int32_t attention_tc;   /* attention core: 0 = by sequence length (K5t, tcgen05 with S and O in
-                             TMEM, from 768 tokens -- GPT-2 Medium S1024 warm 2.02 -> 1.88 ms --
-                             else the mma.sync flash kernels K5 / K5b, faster at S <= 384), 1 =
+  int32_t attention_tc;   /* attention core: 0 = by sequence length (K5t, tcgen05 with S, P and O
+                             in TMEM, from 384 tokens -- GPT-2 Medium S1024 warm 2.01 -> 1.82 ms --
+                             else the mma.sync flash kernels K5 / K5b, faster below 384), 1 =
                              always K5t, 2 = never [0] */
   int32_t reserved[1];
 } dp_engine_opts;

@@ -634,7 +634,7 @@ def attention(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp1
 
 
 def attention_tc(qkv, ldqkv, ctx_out, batch, seq, hidden, heads, causal, dtype="fp16", stream=None):
-    """The tcgen05 attention core (K5t; the engine uses it from 768 tokens, opts.attention_tc)."""
+    """The tcgen05 attention core (K5t; the engine uses it from 384 tokens, opts.attention_tc)."""
     _check(lib.dp_attention_tc(_dptr(qkv), int(ldqkv), _dptr(ctx_out), int(batch), int(seq), int(hidden), int(heads),
                                int(bool(causal)), DTYPES[dtype], _stream_ptr(stream)))
 

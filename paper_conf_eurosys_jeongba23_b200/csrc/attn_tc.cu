@@ -13,8 +13,12 @@
 //                        the group's TMEM accumulator once the group has published P_j;
 //   warps 0-3 / 4-7    : group g = even / odd key tiles; thread r owns query row r (TMEM lane
 //                        r): it reads its 64 scores (tcgen05.ld), masks, runs the online
-//                        softmax in fp32 with exp2 and writes the numerators P (storage type)
-//                        into the 128-byte-swizzled K-major A tile.
+//                        softmax in fp32 with exp2 and writes the numerators P (storage type, two
+//                        per column) back over its S row (tcgen05.st): P V takes A from TMEM.
+// MUFU (16 exponentials per clock per SM, profiles/r02_mufu_probe.txt) bounds the softmax: the
+// two groups' exponentials run at ~12 per clock per SM (profiles/r02_attn_tc_trace.jsonl).
+// Measured and dropped: the groups taking strict turns on the exponentials (named barriers), and
+// a quarter / half of the exponentials as a degree-3 polynomial on the FMA pipe (both slower).
 // The softmax reference max of a row moves only when the row max grows by more than 2^8 (then
 // the thread rescales its O row in TMEM, tcgen05.ld / st, and its row sum): between moves the
 // numerators stay <= 2^8, so the O accumulator never leaves TMEM (no per-tile correction pass).
@@ -63,15 +67,10 @@ constexpr int NS = 6;    // stages of the K ring and of the V ring
 constexpr int SB = 3;    // TMEM S buffers per softmax group
 constexpr uint32_t Q_BYTES = TQ * TD * 2;   // 16 KB
 constexpr uint32_t KV_BYTES = TK * TD * 2;  // 8 KB each for K_j and V_j
-constexpr uint32_t P_BYTES = TQ * TK * 2;   // 16 KB: one [128][64] swizzled K-block
 constexpr uint32_t MERGE_BYTES = TQ * 68 * 4;  // group 1's (o[64], m, l) per row
-constexpr uint32_t SMEM_BYTES = Q_BYTES + 2 * NS * KV_BYTES + 4 * P_BYTES + MERGE_BYTES + 1024;
+constexpr uint32_t SMEM_BYTES = Q_BYTES + 2 * NS * KV_BYTES + MERGE_BYTES + 1024;
 constexpr int NTHR = 352;  // 8 softmax warps, the TMA warp, two MMA warps
 
-// byte offset of element (r, k) of a K-major [rows][64] tile with the 128-byte swizzle
-__device__ __forceinline__ uint32_t sw128_off(int r, int k) {
-  return uint32_t(r) * 128u + ((uint32_t((k >> 3) ^ (r & 7))) << 4) + uint32_t(k & 7) * 2u;
-}
 
 // One lane polls the barrier and releases its warp: 256 softmax threads polling the same
 // barriers flooded the shared-memory barrier unit and delayed the MMA warp's own polls.
@@ -83,9 +82,7 @@ __device__ __forceinline__ void warp_wait(uint64_t* bar, uint32_t phase) {
 __device__ __forceinline__ void named_sync(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
-__device__ __forceinline__ void named_arrive(int id, int n) {
-  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
-}
+
 
 template <class T>
 __global__ void __launch_bounds__(NTHR, 1)
@@ -96,9 +93,8 @@ __global__ void __launch_bounds__(NTHR, 1)
   uint8_t* sQ = smem;
   uint8_t* sK = sQ + Q_BYTES;               // [NS][64 keys][64]: freed by S_j
   uint8_t* sV = sK + NS * KV_BYTES;         // [NS][64 keys][64]: freed by P_j V_j
-  uint8_t* sP = sV + NS * KV_BYTES;         // [group][buffer][128][64]
-  float* xs = reinterpret_cast<float*>(sP + 4 * P_BYTES);  // [128][68]
-  __shared__ __align__(8) uint64_t bar_q, k_full[NS], k_empty[NS], v_full[NS], v_empty[NS], s_full[2][SB], s_free[2][SB], p_full[2][2],
+  float* xs = reinterpret_cast<float*>(sV + NS * KV_BYTES);  // [128][68]
+  __shared__ __align__(8) uint64_t bar_q, k_full[NS], k_empty[NS], v_full[NS], v_empty[NS], s_full[2][SB], p_full[2][SB],
       o_full[2][2];
   __shared__ uint32_t tmem_base_sh;
   // kind::f16, fp32 accumulate; S: A = Q, B = K_j both K-major, M 128 x N 64
@@ -129,13 +125,10 @@ __global__ void __launch_bounds__(NTHR, 1)
       mbar_init(&v_empty[i], 1);
     }
     for (int g = 0; g < 2; ++g) {
-      for (int b = 0; b < 2; ++b) {
-        mbar_init(&o_full[g][b], 1);
-        mbar_init(&p_full[g][b], 4);  // one arrival per warp of the group
-      }
+      for (int b = 0; b < 2; ++b) mbar_init(&o_full[g][b], 1);
       for (int b = 0; b < SB; ++b) {
         mbar_init(&s_full[g][b], 1);
-        mbar_init(&s_free[g][b], 4);
+        mbar_init(&p_full[g][b], 4);  // one arrival per warp of the group
       }
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -194,7 +187,7 @@ __global__ void __launch_bounds__(NTHR, 1)
         const int j = 2 * i + g, b = i % SB, st = j % NS;
         if (j < 8) ATRACE(56 + j);
         mbar_wait(&k_full[st], (j / NS) & 1);
-        if (i >= SB) mbar_wait(&s_free[g][b], ((i / SB) - 1) & 1);  // the group has read S of tile i - SB
+        // (S buffer b held P_{i-SB}: this MMA executes after that tile's P V, issued before it)
         asm volatile("tcgen05.fence::after_thread_sync;");
         const uint64_t dk = sw128_desc(sK + st * KV_BYTES);
 #pragma unroll
@@ -203,16 +196,18 @@ __global__ void __launch_bounds__(NTHR, 1)
         umma_commit(&k_empty[st]);  // K_j consumed
       };
       auto issue_pv = [&](int i) {
-        const int j = 2 * i + g, b = i & 1, st = j % NS;
-        mbar_wait(&p_full[g][b], (i >> 1) & 1);
+        const int j = 2 * i + g, b = i & 1, sb = i % SB, st = j % NS;
+        mbar_wait(&p_full[g][sb], (i / SB) & 1);
         mbar_wait(&v_full[st], (j / NS) & 1);
         asm volatile("tcgen05.fence::after_thread_sync;");
-        // V_j as the MN-major B operand: 128-byte swizzle atoms of 8 keys x 64 head dims, 1024 B
-        // apart along K (SBO); a 16-key step advances 2048 B (128 in descriptor units)
-        const uint64_t dpp = sw128_desc(sP + (2 * g + b) * P_BYTES), dv = sw128_desc(sV + st * KV_BYTES);
+        // A = P_j from TMEM (the S buffer's first 32 columns: 2 numerators per column, a 16-key
+        // step = 8 columns); B = V_j as the MN-major operand: 128-byte swizzle atoms of 8 keys x 64
+        // head dims, 1024 B apart along K (SBO), a 16-key step = 2048 B (128 in descriptor units)
+        const uint64_t dv = sw128_desc(sV + st * KV_BYTES);
 #pragma unroll
-        for (int kk = 0; kk < TK / 16; ++kk) umma_f16(t_o(g), dpp + 2 * kk, dv + 128 * kk, IDESC_O, (i | kk) != 0);
-        umma_commit(&o_full[g][b]);  // P_j's buffer is free again, O holds tiles <= j
+        for (int kk = 0; kk < TK / 16; ++kk)
+          umma_f16_ts(t_o(g), t_s(g, sb) + 8 * kk, dv + 128 * kk, IDESC_O, (i | kk) != 0);
+        umma_commit(&o_full[g][b]);  // O holds tiles <= j
         umma_commit(&v_empty[st]);   // V_j consumed
       };
       for (int i = 0; i < nl && i < SB; ++i) issue_s(i);
@@ -228,8 +223,7 @@ __global__ void __launch_bounds__(NTHR, 1)
     const uint32_t lane_base = uint32_t((warp & 3) * 32) << 16;
     const int qrow = q0 + r;
     float mref = -INFINITY, lrow = 0.f;  // the row's softmax reference max (scaled units) and sum
-    const int nloc = (nkt - g + 1) / 2, nl0 = (nkt + 1) / 2, nl1 = nkt / 2;
-    if (g == 1 && nl0 > 0) named_arrive(2, 256);  // group 0 takes the first turn
+    const int nloc = (nkt - g + 1) / 2;
     for (int i = 0; i < nloc; ++i) {
       const int j = 2 * i + g, b = i & 1, sb = i % SB, k0 = j * TK;
       warp_wait(&s_full[g][sb], (i / SB) & 1);
@@ -245,9 +239,6 @@ __global__ void __launch_bounds__(NTHR, 1)
         for (int e = 0; e < TK; ++e) s[e] = __uint_as_float(v[e]);  // scaled inside the exponent
       }
       if (tid == 0 && i < 8) ATRACE(17 + 4 * i);
-      asm volatile("tcgen05.fence::before_thread_sync;");
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&s_free[g][sb]);  // this warp's lanes of S_j are read
       if (i == 0 && r == 0) ATRACE(2 + g);
       if (r == 0 && j < 8) ATRACE(48 + j);
       if (k0 + TK > seq || (causal && k0 + TK - 1 > qrow)) {  // only where a key can be invalid
@@ -267,6 +258,9 @@ __global__ void __launch_bounds__(NTHR, 1)
         mx = fmaxf(fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])), fmaxf(fmaxf(m8[4], m8[5]), fmaxf(m8[6], m8[7])));
       }
       mx *= scale_log2;
+      // P V of tile i - 2 has completed: each O barrier is then at most one phase behind, so the
+      // parity wait for tile i - 1 below (and the next iteration's) is unambiguous
+      if (i >= 2) warp_wait(&o_full[g][i & 1], ((i - 2) >> 1) & 1);
       // move the reference only when the row max outgrows it by > 2^8 (or on the first finite max);
       // O and the row sum then scale by f = 2^(old - new)
       float f = 1.f;
@@ -292,35 +286,26 @@ __global__ void __launch_bounds__(NTHR, 1)
       }
       const float mr = (mref == -INFINITY) ? 0.f : mref;  // a fully masked row: every p = 2^-inf = 0
       float r8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-      // the exponentials (MUFU, 16 per clock per SM: the softmax's bound) alternate between the
-      // groups, so one group's exponentials overlap the other's loads, P stores and waits
-      named_sync(2 + g, 256);
 #pragma unroll
       for (int e = 0; e < TK; ++e) {
         const float pv = fast_exp2(fmaf(s[e], scale_log2, -mr));
         r8[e & 7] += pv;
         s[e] = pv;
       }
-      if (g == 0 ? i < nl1 : i + 1 < nl0) named_arrive(3 - g, 256);  // the other group's turn
       lrow += ((r8[0] + r8[1]) + (r8[2] + r8[3])) + ((r8[4] + r8[5]) + (r8[6] + r8[7]));
       if (tid == 0 && i < 8) ATRACE(18 + 4 * i);
-      // P_j (row r) into the group's A-operand buffer b, once P_{j-4} there has been consumed
-      if (i >= 2) warp_wait(&o_full[g][b], ((i - 2) >> 1) & 1);
-      uint8_t* pt = sP + (2 * g + b) * P_BYTES;
+      // P_j (row r, storage type, 2 per column) over the S row it came from: the A operand of P V
+      {
+        uint32_t pk[TK / 2];
 #pragma unroll
-      for (int c = 0; c < TK / 8; ++c) {
-        const float* pp = s + c * 8;
-        uint4 u;
-        u.x = Cvt<T>::from2(pp[0], pp[1]);
-        u.y = Cvt<T>::from2(pp[2], pp[3]);
-        u.z = Cvt<T>::from2(pp[4], pp[5]);
-        u.w = Cvt<T>::from2(pp[6], pp[7]);
-        *reinterpret_cast<uint4*>(pt + sw128_off(r, c * 8)) = u;
+        for (int c = 0; c < TK / 2; ++c) pk[c] = Cvt<T>::from2(s[2 * c], s[2 * c + 1]);
+        tmem_st16(t_s(g, sb) + lane_base, pk);
+        tmem_st16(t_s(g, sb) + lane_base + 16, pk + 16);
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // P -> the tensor core
       asm volatile("tcgen05.fence::before_thread_sync;");
       __syncwarp();
-      if (lane == 0) mbar_arrive(&p_full[g][b]);
+      if (lane == 0) mbar_arrive(&p_full[g][sb]);
       if (tid == 0 && i < 8) ATRACE(19 + 4 * i);
     }
     if (r == 0) ATRACE(4 + g);

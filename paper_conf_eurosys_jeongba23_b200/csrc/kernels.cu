@@ -730,10 +730,11 @@ void launch_attention(int dtype, const void* qkv, int ldqkv, void* ctx, int batc
     launch_attention_f32(qkv, ldqkv, ctx, batch, seq, H, heads, causal, s);
     return;
   }
-  // K5t (tcgen05, attn_tc.cu) from 768 tokens (tc_mode 0) or when forced (1): GPT-2 Medium S1024
-  // warm forward 2.02 -> 1.88 ms; at S <= 384 the mma.sync kernels below are as fast or faster
-  // (BERT-Large S384 1.364 vs 1.372 ms, GPT-2 S256 0.508 vs 0.560; profiles/r02_warm_attention_tc.jsonl)
-  const bool use_tc = tc_mode == 1 || (tc_mode == 0 && seq >= 768);
+  // K5t (tcgen05, attn_tc.cu) from 384 tokens (tc_mode 0) or when forced (1).  Warm forwards, K5t
+  // vs K5 / K5b: GPT-2 Medium S1024 1.82 vs 2.01 ms, BERT-Large S384 1.347 vs 1.362, GPT-2 S512
+  // 0.631 vs 0.652; below 384 tokens the mma.sync kernels win (GPT-2 S256 0.550 vs 0.505, BERT-Base
+  // S128 0.475 vs 0.465; profiles/r02_warm_attention_tc.jsonl)
+  const bool use_tc = tc_mode == 1 || (tc_mode == 0 && seq >= 384);
   if (use_tc && attention_tc_supported(ldqkv, H, heads, qkv)) {
     launch_attention_tc(dtype, qkv, ldqkv, ctx, batch, seq, H, heads, causal, s);
     return;

@@ -355,7 +355,7 @@ def test_graph_replay_after_workspace_regrowth():
                                          ("gpt2", 1024, 0), ("gpt2", 1024, 2), ("bert_base", 512, 1)])
 def test_attention_tc_engine_option(name, S, mode):
     """opts.attention_tc: 1 runs every layer's attention on K5t, 2 on the mma.sync kernels, 0 picks
-    K5t from 768 tokens: the whole cold start stays within the north star's tolerance of the
+    K5t from 384 tokens: the whole cold start stays within the north star's tolerance of the
     oracle in every mode."""
     m = synth.SHAPES[name]
     w = synth.make_weights(m, seed=41, dtype="fp16")
