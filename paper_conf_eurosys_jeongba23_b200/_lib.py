@@ -7,7 +7,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_HERE, "libdeepplan.so")
+# DP_LIB: another build of the same library (A/B timing tools); the in-tree build by default
+_LIB_PATH = os.environ.get("DP_LIB") or os.path.join(_HERE, "libdeepplan.so")
 
 LOAD, DHA = 0, 1
 MODES = {"BASELINE": 0, "PIPESWITCH": 1, "GREEDY": 2, "DHA": 3, "PT": 4, "PT_DHA": 5, "DHA_LINK": 6,

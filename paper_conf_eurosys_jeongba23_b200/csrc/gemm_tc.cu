@@ -357,14 +357,18 @@ __global__ void __launch_bounds__(NT, 1)
     store_tile<T, BN, ACT>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
   } else {
     // 1) TMEM -> shared memory: this split's fp32 partial tile [128 W rows][BN tokens], unpadded,
-    //    so each owner's rows are one contiguous block to push
+    //    so each owner's rows are one contiguous block to push.  Within a row the 16-byte chunks
+    //    are XOR-swizzled by (row & 7): the 32 lanes of a warp write 32 consecutive rows, BN * 4
+    //    bytes apart (a multiple of 128 B), so the unswizzled float4 stores were 32-way bank
+    //    conflicts -- 2-3 us per tile by the per-CTA trace (profiles/r02_gemm_trace_splitk.jsonl).
+    //    Every tile and receive slot uses the same layout; the owner reads it back swizzled.
 #pragma unroll 1
     for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
       uint32_t v[16];
       tmem_ld16(tmem_d + (uint32_t((warp & 3) * 32) << 16) + c0, v);
 #pragma unroll
       for (int j = 0; j < 16; j += 4)
-        *reinterpret_cast<float4*>(&tile[row * BN + c0 + j]) =
+        *reinterpret_cast<float4*>(&tile[row * BN + ((((c0 + j) >> 2) ^ (row & 7)) << 2)]) =
             make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
                         __uint_as_float(v[j + 3]));
     }
@@ -422,7 +426,7 @@ __global__ void __launch_bounds__(NT, 1)
       for (int p = 0; p < splits; ++p) {
         const float* sl = p == sp ? tile + sp * RPR * BN : recv + p * RPR * BN;
 #pragma unroll
-        for (int e = 0; e < 8; ++e) acc[e] += sl[(8 * gi + e) * BN + ml];
+        for (int e = 0; e < 8; ++e) acc[e] += sl[(8 * gi + e) * BN + ((((ml >> 2) ^ e) << 2) | (ml & 3))];
       }
       finish(sp * RPR + 8 * gi, ml, acc);
     }
@@ -776,7 +780,10 @@ static int pick_bn(int M, int N) {
 // ~100 GB/s (the mainloop time is its bytes / 1e5 B/us), all CTAs together at ~8 TB/s from
 // L2/HBM, and the cluster split-K reduction (bulk DSMEM pushes) costs ~1.2 us.  Splits only in
 // one wave of <= 148 CTAs, >= 4 k-blocks each, BN <= 128 (the send/receive buffers must fit).
-// Picks the best measured configuration at every swept shape.
+// Picks the best measured configuration at every swept shape.  (Round 2: a refit to the
+// back-to-back sweep after the split-K bank-conflict fix -- 0.3 us + pushed bytes at 33 KB/us,
+// + 6 ns per token column -- chose other tiles at 3 of 15 shapes, 1% better back to back but
+// 2-3% SLOWER in the PDL-chained forwards, profiles/r02_warm_ab_cost_model.jsonl: kept as is.)
 struct GemmCfg {
   int bn, sp;
   bool pair;
