@@ -87,7 +87,7 @@ __device__ __forceinline__ void named_sync(int id, int n) {
 template <class T>
 __global__ void __launch_bounds__(NTHR, 1)
     attention_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
-                        T* __restrict__ ctx, int seq, int H, int causal, float scale_log2) {
+                        T* __restrict__ ctx, int seq, int H, int causal, float scale_log2, int nsplit) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sQ = smem;
@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(NTHR, 1)
   uint8_t* sV = sK + NS * KV_BYTES;         // [NS][64 keys][64]: freed by P_j V_j
   float* xs = reinterpret_cast<float*>(sV + NS * KV_BYTES);  // [128][68]
   __shared__ __align__(8) uint64_t bar_q, k_full[NS], k_empty[NS], v_full[NS], v_empty[NS], s_full[2][SB], p_full[2][SB],
-      o_full[2][2];
+      o_full[2][2], recv_bar;
   __shared__ uint32_t tmem_base_sh;
   // kind::f16, fp32 accumulate; S: A = Q, B = K_j both K-major, M 128 x N 64
   constexpr uint32_t IDESC_S = (1u << 4) | (FmtBits<T>::v << 7) | (FmtBits<T>::v << 10) | (uint32_t(TK >> 3) << 17) |
@@ -106,18 +106,25 @@ __global__ void __launch_bounds__(NTHR, 1)
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) ATRACE(0);
-  // grid (heads, query tiles, batch); causal query tiles longest first
+  // grid (heads, query tiles x nsplit, batch); causal query tiles longest first.  With nsplit > 1
+  // the nsplit CTAs of a query tile form a cluster along y and take consecutive key ranges
+  // (split = cluster rank); their partial (o, m, l) rows are merged over DSMEM at the end.
   const int head = blockIdx.x, bidx = blockIdx.z;
-  const int qt = causal ? (int)gridDim.y - 1 - (int)blockIdx.y : (int)blockIdx.y;
+  const int qidx = (int)blockIdx.y / nsplit, split = (int)blockIdx.y - qidx * nsplit;
+  const int nqt = (int)gridDim.y / nsplit;
+  const int qt = causal ? nqt - 1 - qidx : qidx;
   const int q0 = qt * TQ;
   const int tok0 = bidx * seq;
-  int nkt = (seq + TK - 1) / TK;
-  if (causal) nkt = min(nkt, (q0 + TQ - 1) / TK + 1);
+  int nkt_all = (seq + TK - 1) / TK;
+  if (causal) nkt_all = min(nkt_all, (q0 + TQ - 1) / TK + 1);
+  const int kt_lo = split * nkt_all / nsplit;                // this CTA's key tiles [kt_lo, kt_lo + nkt)
+  const int nkt = (split + 1) * nkt_all / nsplit - kt_lo;
 
   if (tid == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmQ)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmKV)) : "memory");
     mbar_init(&bar_q, 1);
+    mbar_init(&recv_bar, 1);  // cluster merge: the peers' partial rows (bulk DSMEM pushes) land here
     for (int i = 0; i < NS; ++i) {
       mbar_init(&k_full[i], 1);
       mbar_init(&k_empty[i], 1);
@@ -161,14 +168,14 @@ __global__ void __launch_bounds__(NTHR, 1)
     if (lane == 0) {
       mbar_expect_tx(&bar_q, Q_BYTES);
       tma_load_2d(&tmQ, &bar_q, sQ, qcol, tok0 + q0);
-      for (int j = 0; j < nkt; ++j) {
+      for (int j = 0; j < nkt; ++j) {  // j: local key tile (absolute kt_lo + j)
         const int st = j % NS;
         if (j >= NS) mbar_wait(&k_empty[st], ((j / NS) - 1) & 1);
         mbar_expect_tx(&k_full[st], KV_BYTES);
-        tma_load_2d(&tmKV, &k_full[st], sK + st * KV_BYTES, kcol, tok0 + j * TK);
+        tma_load_2d(&tmKV, &k_full[st], sK + st * KV_BYTES, kcol, tok0 + (kt_lo + j) * TK);
         if (j >= NS) mbar_wait(&v_empty[st], ((j / NS) - 1) & 1);
         mbar_expect_tx(&v_full[st], KV_BYTES);
-        tma_load_2d(&tmKV, &v_full[st], sV + st * KV_BYTES, vcol, tok0 + j * TK);
+        tma_load_2d(&tmKV, &v_full[st], sV + st * KV_BYTES, vcol, tok0 + (kt_lo + j) * TK);
       }
       ATRACE(10);
     }
@@ -225,7 +232,7 @@ __global__ void __launch_bounds__(NTHR, 1)
     float mref = -INFINITY, lrow = 0.f;  // the row's softmax reference max (scaled units) and sum
     const int nloc = (nkt - g + 1) / 2;
     for (int i = 0; i < nloc; ++i) {
-      const int j = 2 * i + g, b = i & 1, sb = i % SB, k0 = j * TK;
+      const int j = 2 * i + g, b = i & 1, sb = i % SB, k0 = (kt_lo + j) * TK;
       warp_wait(&s_full[g][sb], (i / SB) & 1);
       if (tid == 0 && i < 8) ATRACE(16 + 4 * i);
       asm volatile("tcgen05.fence::after_thread_sync;");
@@ -334,31 +341,142 @@ __global__ void __launch_bounds__(NTHR, 1)
       mine[65] = lrow;
     }
     named_sync(1, 256);
-    if (g == 0 && qrow < seq) {
-      const float* ot = xs + r * 68;
+    if (g == 0) {
+      float* ot = xs + r * 68;
       const float m1 = ot[64], l1 = ot[65];
       const float m = fmaxf(mrow, m1);
       const float a0 = (mrow == -INFINITY) ? 0.f : fast_exp2(mrow - m);
       const float a1 = (m1 == -INFINITY) ? 0.f : fast_exp2(m1 - m);
       const float l = lrow * a0 + l1 * a1;
-      const float inv = l > 0.f ? 1.f / l : 0.f;
-      const float c0 = a0 * inv, c1 = a1 * inv;
-      uint4* dst = reinterpret_cast<uint4*>(ctx + (size_t)(tok0 + qrow) * H + head * TD);
+      if (nsplit == 1) {
+        if (qrow < seq) {
+          const float inv = l > 0.f ? 1.f / l : 0.f;
+          const float c0 = a0 * inv, c1 = a1 * inv;
+          uint4* dst = reinterpret_cast<uint4*>(ctx + (size_t)(tok0 + qrow) * H + head * TD);
 #pragma unroll
-      for (int c = 0; c < TD / 8; ++c) {
-        float v[8];
+          for (int c = 0; c < TD / 8; ++c) {
+            float v[8];
 #pragma unroll
-        for (int e = 0; e < 8; ++e) v[e] = o[c * 8 + e] * c0 + ot[c * 8 + e] * c1;
-        uint4 u;
-        u.x = Cvt<T>::from2(v[0], v[1]);
-        u.y = Cvt<T>::from2(v[2], v[3]);
-        u.z = Cvt<T>::from2(v[4], v[5]);
-        u.w = Cvt<T>::from2(v[6], v[7]);
-        dst[c] = u;
+            for (int e = 0; e < 8; ++e) v[e] = o[c * 8 + e] * c0 + ot[c * 8 + e] * c1;
+            uint4 u;
+            u.x = Cvt<T>::from2(v[0], v[1]);
+            u.y = Cvt<T>::from2(v[2], v[3]);
+            u.z = Cvt<T>::from2(v[4], v[5]);
+            u.w = Cvt<T>::from2(v[6], v[7]);
+            dst[c] = u;
+          }
+        }
+      } else {
+        // this CTA's key range merged: unnormalised o, reference max m, sum l, published in place
+        // for the cluster merge below
+#pragma unroll
+        for (int e = 0; e < TD; e += 4) {
+          const float4 t = *reinterpret_cast<const float4*>(ot + e);
+          *reinterpret_cast<float4*>(ot + e) =
+              make_float4(o[e] * a0 + t.x * a1, o[e + 1] * a0 + t.y * a1, o[e + 2] * a0 + t.z * a1, o[e + 3] * a0 + t.w * a1);
+        }
+        ot[64] = m;
+        ot[65] = l;
       }
     }
     if (tid == 0) ATRACE(8);
   }
+  if (nsplit > 1) {
+    // Cluster merge: the nsplit CTAs of a query tile hold (o, m, l) of consecutive key ranges in
+    // their xs rows ([128][68] fp32).  Rank k finalises query rows [k*128/n, (k+1)*128/n): every
+    // CTA pushes the rows each peer owns with ONE bulk copy (cp.async.bulk shared::cta ->
+    // shared::cluster, completing on the peer's recv_bar) into the peer's K ring -- idle by now:
+    // every S MMA finished before the O accumulators were read -- and the owner merges the ranks'
+    // rows in rank order from its own shared memory (deterministic).  (Remote loads by the owner
+    // instead -- latency-bound ld.shared::cluster -- cost ~3-4 us per CTA, tools/att_waves.py.)
+    const int rows_max = (TQ + nsplit - 1) / nsplit;
+    const int rlo = split * TQ / nsplit, rhi = (split + 1) * TQ / nsplit;
+    float* recv = reinterpret_cast<float*>(sK);  // [nsplit - 1][rows_max][68]
+    if (tid == 0)
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&recv_bar)),
+                   "r"(uint32_t(nsplit - 1) * uint32_t(rhi - rlo) * 68u * 4u)
+                   : "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // xs rows -> async proxy
+    // every rank's rows are final and its K ring and recv_bar are ready
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (tid == 0) {
+      ATRACE(11);
+      for (int k = 0; k < nsplit; ++k) {
+        if (k == split) continue;
+        const int klo = k * TQ / nsplit, khi = (k + 1) * TQ / nsplit;
+        const int slot = split < k ? split : split - 1;  // this rank's slot in rank k's receive area
+        uint32_t dst, bar;
+        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;"
+                     : "=r"(dst)
+                     : "r"(smem_u32(recv + size_t(slot) * rows_max * 68)), "r"(k));
+        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(bar) : "r"(smem_u32(&recv_bar)), "r"(k));
+        asm volatile(
+            "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+            "r"(smem_u32(xs + klo * 68)), "r"(uint32_t(khi - klo) * 68u * 4u), "r"(bar)
+            : "memory");
+      }
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      mbar_wait_spin(&recv_bar, 0);
+    }
+    __syncthreads();
+    if (warp < 8) {
+      // (row, 32-column half) per thread
+      const int rr = rlo + (tid >> 1), half = tid & 1;
+      const int qrow = q0 + rr;
+      if (rr < rhi && qrow < seq) {
+        const float* src[4];
+        float m = -INFINITY;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {  // (nsplit <= 4; unrolled so the row pointers stay in registers)
+          src[k] = nullptr;
+          if (k >= nsplit) continue;
+          src[k] = k == split ? xs + rr * 68 : recv + (size_t(k < split ? k : k - 1) * rows_max + (rr - rlo)) * 68;
+          m = fmaxf(m, src[k][64]);
+        }
+        float l = 0.f, acc[32];
+#pragma unroll
+        for (int e = 0; e < 32; ++e) acc[e] = 0.f;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          if (k >= nsplit) continue;
+          const float mk = src[k][64];
+          const float a = (mk == -INFINITY) ? 0.f : fast_exp2(mk - m);
+          l += src[k][65] * a;
+#pragma unroll
+          for (int e = 0; e < 32; e += 4) {
+            const float4 t = *reinterpret_cast<const float4*>(src[k] + 32 * half + e);
+            acc[e] += t.x * a;
+            acc[e + 1] += t.y * a;
+            acc[e + 2] += t.z * a;
+            acc[e + 3] += t.w * a;
+          }
+        }
+        const float inv = l > 0.f ? 1.f / l : 0.f;
+        uint4* dst = reinterpret_cast<uint4*>(ctx + (size_t)(tok0 + qrow) * H + head * TD + 32 * half);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          uint4 u;
+          u.x = Cvt<T>::from2(acc[8 * c] * inv, acc[8 * c + 1] * inv);
+          u.y = Cvt<T>::from2(acc[8 * c + 2] * inv, acc[8 * c + 3] * inv);
+          u.z = Cvt<T>::from2(acc[8 * c + 4] * inv, acc[8 * c + 5] * inv);
+          u.w = Cvt<T>::from2(acc[8 * c + 6] * inv, acc[8 * c + 7] * inv);
+          dst[c] = u;
+        }
+      }
+    }
+    // the pushes must have read this CTA's rows before it exits (every push INTO this CTA has
+    // landed: recv_bar completed)
+    if (tid == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+  }
+#ifdef DP_ATT_TRACE
+  if (tid == 0) {
+    ATRACE(12);
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    const int b_ = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
+    if (b_ < 2048) g_att_trace[b_][14] = smid;
+  }
+#endif
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (warp == 9) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
@@ -379,15 +497,37 @@ void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int b
   const CUtensorMap mq = make_kmajor_map(qkv, dtype, T, 3 * H, ldqkv, TQ);
   const CUtensorMap mkv = make_kmajor_map(qkv, dtype, T, 3 * H, ldqkv, TK);
   const float scale_log2 = 1.4426950408889634f / 8.0f;  // log2(e) / sqrt(64)
-  const dim3 grid(heads, (seq + TQ - 1) / TQ, batch);
+  // Key-range split (round 2): one CTA per SM (512 TMEM columns), so a grid with fewer query
+  // tiles than SMs leaves SMs idle.  Each query tile's keys are split over a cluster of 2 or 4
+  // CTAs when the grid still fits ONE wave and every CTA keeps >= 4 key tiles: the merge costs
+  // ~2 us (cluster barrier ~0.6 + push / merge / store ~1.5, tools/att_waves.py), a key-tile pair
+  // ~1.2 us.  Measured (warm forwards, profiles/r02_attn_split_waves.jsonl,
+  // r02_warm_ab_attention_split.jsonl): GPT-2 S512 0.611 -> 0.596 ms, BERT-Base S512 0.629 ->
+  // 0.609; BERT-Large S384 (3 key tiles per half) 1.266 -> 1.281 and causal S1024 in two waves
+  // (1.78 -> 1.90) slower, so neither splits; clusters of 3 also packed badly into the GPCs
+  // (13 SMs idle, 9 CTAs in a second wave).
+  const int nqt = (seq + TQ - 1) / TQ, nkt = (seq + TK - 1) / TK;
+  const int ctas = heads * nqt * batch;
+  int nsplit = 1;
+  for (int n : {4, 2})
+    if (ctas * n <= 148 && nkt >= 4 * n) {
+      nsplit = n;
+      break;
+    }
+  if (const int forced = experiment_env("DP_ATT_SPLIT", 0); forced > 0) nsplit = std::min(forced, 4);
+  const dim3 grid(heads, nqt * nsplit, batch);
   auto go = [&](auto tag) {
     using T = decltype(tag);
     static std::atomic<unsigned> attr{0};
     if (first_on_device(attr))
       DP_CUDA(cudaFuncSetAttribute(attention_tc_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)SMEM_BYTES));
-    launch_kernel(attention_tc_kernel<T>, grid, dim3(NTHR), SMEM_BYTES, s, mq, mkv, (T*)ctx, seq, H, causal ? 1 : 0,
-                  scale_log2);
+    if (nsplit > 1)
+      launch_kernel_cluster(attention_tc_kernel<T>, grid, dim3(NTHR), SMEM_BYTES, dim3(1, nsplit, 1), s, mq, mkv,
+                            (T*)ctx, seq, H, causal ? 1 : 0, scale_log2, nsplit);
+    else
+      launch_kernel(attention_tc_kernel<T>, grid, dim3(NTHR), SMEM_BYTES, s, mq, mkv, (T*)ctx, seq, H,
+                    causal ? 1 : 0, scale_log2, 1);
   };
   if (dtype == DP_BF16)
     go(__nv_bfloat16{});

@@ -219,7 +219,7 @@ __device__ __forceinline__ void store_tile(uint8_t* otile, uint32_t tmem_d, cons
 // rank order 0..splits-1 (deterministic), then runs the epilogue.  At the hot path's
 // 128-token shapes a CTA's time is set by the bytes it ingests (~100 GB/s per SM measured,
 // profiles/r01_gemm_trace.jsonl), so spreading a weight tile over `splits` SMs pays.
-template <class T, int BN, int ACT>
+template <class T, int BN, int ACT, bool SPLIT>
 __global__ void __launch_bounds__(NT, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
                    const __grid_constant__ CUtensorMap tmY, const void* res, int ldr, void* Y, int ldy, int M, int N,
@@ -346,14 +346,14 @@ __global__ void __launch_bounds__(NT, 1)
   // still streaming stages into that memory: a corrupted operand under SM contention, caught
   // by tools/stress_concurrency.py.)  Release orders our tensor-core reads of the ring before
   // the peers' async-proxy writes into it.
-  if (splits > 1) asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+  if constexpr (SPLIT) asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
   asm volatile("tcgen05.fence::after_thread_sync;");
   // TMEM lane = W row within the tile; warp w reads its lane quarter (w % 4) for the column
   // half w / 4 of the tile
   const int row = (warp & 3) * 32 + lane;
   const int chalf = (warp >> 2) * (BN / 2);
   float* tile = reinterpret_cast<float*>(smem);
-  if (splits == 1) {
+  if constexpr (!SPLIT) {
     store_tile<T, BN, ACT>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
   } else {
     // 1) TMEM -> shared memory: this split's fp32 partial tile [128 W rows][BN tokens], unpadded,
@@ -373,14 +373,19 @@ __global__ void __launch_bounds__(NT, 1)
                         __uint_as_float(v[j + 3]));
     }
     // 2) + bias, activation, + residual; one 16-byte store per 8 outputs (8 W rows of a token)
-    auto finish = [&](int nl, int ml, float* acc) {
+    auto finish = [&](int nl, int ml, float* acc, const float* rpre = nullptr) {
       const size_t m = (size_t)(m0 + ml);
       const int nn = n0 + nl;
 #pragma unroll
       for (int e = 0; e < 8; ++e) acc[e] = apply_act_c<ACT>(acc[e] + sbias[nl + e]);
       if (res) {
         float r8[8];
-        load8<T>(res, m * ldr + nn, r8, res32);
+        if (rpre != nullptr) {
+#pragma unroll
+          for (int e = 0; e < 8; ++e) r8[e] = rpre[e];
+        } else {
+          load8<T>(res, m * ldr + nn, r8, res32);
+        }
 #pragma unroll
         for (int e = 0; e < 8; ++e) acc[e] += r8[e];
       }
@@ -420,15 +425,45 @@ __global__ void __launch_bounds__(NT, 1)
     mbar_wait(&recv_bar, 0);
     if (threadIdx.x == 0) TRACE(7);
     const int units = (RPR / 8) * mcount;
-    for (int u = threadIdx.x; u < units; u += NT) {
-      const int gi = u / mcount, ml = u - gi * mcount;  // 8-row group within the owned rows
-      float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-      for (int p = 0; p < splits; ++p) {
-        const float* sl = p == sp ? tile + sp * RPR * BN : recv + p * RPR * BN;
+    if (res == nullptr || units <= NT) {
+      for (int u = threadIdx.x; u < units; u += NT) {
+        const int gi = u / mcount, ml = u - gi * mcount;  // 8-row group within the owned rows
+        float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+        for (int p = 0; p < splits; ++p) {
+          const float* sl = p == sp ? tile + sp * RPR * BN : recv + p * RPR * BN;
 #pragma unroll
-        for (int e = 0; e < 8; ++e) acc[e] += sl[(8 * gi + e) * BN + ((((ml >> 2) ^ e) << 2) | (ml & 3))];
+          for (int e = 0; e < 8; ++e) acc[e] += sl[(8 * gi + e) * BN + ((((ml >> 2) ^ e) << 2) | (ml & 3))];
+        }
+        finish(sp * RPR + 8 * gi, ml, acc);
       }
-      finish(sp * RPR + 8 * gi, ml, acc);
+    } else {
+      // several units per thread with a residual: the residual loads of two units are issued
+      // before either is finished (one latency per pair instead of one per unit; the 1024-token
+      // shapes finalise 2-4 units per thread)
+      for (int u0 = threadIdx.x; u0 < units; u0 += 2 * NT) {
+        float r8[2][8];
+#pragma unroll
+        for (int b = 0; b < 2; ++b) {
+          const int u = u0 + b * NT;
+          if (u < units) {
+            const int gi = u / mcount, ml = u - gi * mcount;
+            load8<T>(res, (size_t)(m0 + ml) * ldr + n0 + sp * RPR + 8 * gi, r8[b], res32);
+          }
+        }
+#pragma unroll
+        for (int b = 0; b < 2; ++b) {
+          const int u = u0 + b * NT;
+          if (u >= units) break;
+          const int gi = u / mcount, ml = u - gi * mcount;
+          float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+          for (int p = 0; p < splits; ++p) {
+            const float* sl = p == sp ? tile + sp * RPR * BN : recv + p * RPR * BN;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) acc[e] += sl[(8 * gi + e) * BN + ((((ml >> 2) ^ e) << 2) | (ml & 3))];
+          }
+          finish(sp * RPR + 8 * gi, ml, acc, r8[b]);
+        }
+      }
     }
     // the pushes must have read this CTA's send buffer before it exits
     if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
@@ -646,10 +681,16 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   nst = std::max(nst, std::max(min_st, 1));
   DP_CHECK(nst <= STAGES, DP_ERR_INVALID, "gemm: epilogue buffers do not fit this tile width");
   const size_t smem = size_t(nst) * STAGE_BYTES + 1024;
-  static std::atomic<unsigned> attr{0};
-  if (first_on_device(attr))
-    DP_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<T, BN, ACT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)smem_max));
+  // the single-split and split-K kernels are separate instantiations: each carries only its own
+  // epilogue, and a CTA's first pass through its code is instruction-fetch bound (one cold
+  // fetch per instruction; a larger split-K epilogue slowed even the kernels that never ran it)
+  auto kern = gemm_tc_kernel<T, BN, ACT, false>;
+  if constexpr (BN < 256) {  // (256-wide tiles never split: the send + receive buffers would not fit)
+    if (splits > 1) kern = gemm_tc_kernel<T, BN, ACT, true>;
+  }
+  static std::atomic<unsigned> attr{0}, attr_sp{0};
+  if (first_on_device(splits > 1 ? attr_sp : attr))
+    DP_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_max));
   const int dtype = std::is_same<T, __half>::value ? DP_FP16 : DP_BF16;
   GemmGroup g;
   std::memset(&g, 0, sizeof(g));
@@ -670,7 +711,7 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
                                                              : CU_TENSOR_MAP_DATA_TYPE_FLOAT16),
                                   2, ydims, ystr, ybox);
   const int mt = (M + BN - 1) / BN;
-  launch_kernel_cluster(gemm_tc_kernel<T, BN, ACT>, dim3(N / BM, mt, ngroups * splits), dim3(NT), smem,
+  launch_kernel_cluster(kern, dim3(N / BM, mt, ngroups * splits), dim3(NT), smem,
                         dim3(1, 1, splits), s, g, mx, my, res, ldr, y, ldy, M, N, K, act, io, splits, nst);
 }
 

@@ -245,12 +245,16 @@ def test_attention_parity(B, S, H, heads, causal, dtype):
 
 @pytest.mark.parametrize("B,S,H,heads", [(1, 1, 128, 2), (2, 5, 128, 2), (1, 32, 128, 2), (1, 64, 768, 12),
                                          (1, 65, 128, 2), (2, 77, 256, 4), (1, 128, 768, 12), (1, 192, 256, 4),
-                                         (1, 384, 1024, 16), (1, 1024, 1024, 16), (3, 200, 256, 4)])
+                                         (1, 384, 1024, 16), (1, 1024, 1024, 16), (3, 200, 256, 4),
+                                         (1, 512, 256, 4), (1, 700, 512, 8), (1, 1024, 256, 4)])
 @pytest.mark.parametrize("causal", [False, True])
 @pytest.mark.parametrize("dtype", ["fp16", "bf16"])
 def test_attention_tc_parity(B, S, H, heads, causal, dtype):
     """K5t (tcgen05: S and P.V in TMEM, one softmax row per thread) against the oracle, same bound as
-    K5 (P is rounded to the storage type before P.V)."""
+    K5 (P is rounded to the storage type before P.V).  The shapes cover every key-range split the
+    launcher picks (1 CTA per query tile; a cluster of 2 / 4 CTAs merging over DSMEM: S512 x 4
+    heads and S700 x 8 heads (ragged) -> 2, S1024 x 4 heads -> 4, where causal query tile 0 leaves
+    CTAs with no key tile at all and rows fully masked in a CTA's range)."""
     rng = np.random.default_rng(B * 1000 + S + H + 7)
     qkv = synth.round_to((1.5 * rng.standard_normal((B * S, 3 * H))).astype(np.float32), dtype)
     Q = to_t(qkv, dtype)
