@@ -161,14 +161,28 @@ struct EpiParams {
 // token, conflict-free.  One TMA bulk tensor store then writes the tile (rows past M are
 // clipped by the tensor map), replacing the fp32 round trip through shared memory and the
 // per-thread 16-byte stores of round 1.  `otile` is the ring, free once the MMAs are done.
-template <class T, int BN, int ACT>
+// IOT: the epilogue's I/O as a compile-time constant where the forward pass fixes it -- 1 = no
+// residual, output in the storage type (q/k/v, fc1); 2 = fp32 residual, fp32 output (attn-out,
+// fc2, GPT-2's projections into the fp32 residual stream); 0 = any (read from io / res at run
+// time: the kernel test hooks).  Each variant carries only its own epilogue code: a CTA runs
+// its code once, and cold instruction fetch is on its critical path.
+template <int IOT>
+struct EpiIO {
+  __device__ __forceinline__ static const void* res(const void* r) { return IOT == 1 ? nullptr : r; }
+  __device__ __forceinline__ static bool has_res(const void* r) { return IOT == 2 ? true : IOT == 1 ? false : r != nullptr; }
+  __device__ __forceinline__ static bool res32(int io) { return IOT == 2 ? true : IOT == 1 ? false : (io & IO_RES_F32); }
+  __device__ __forceinline__ static bool out32(int io) { return IOT == 2 ? true : IOT == 1 ? false : (io & IO_OUT_F32); }
+};
+
+template <class T, int BN, int ACT, int IOT>
 __device__ __forceinline__ void store_tile(uint8_t* otile, uint32_t tmem_d, const float* sbias,
                                            const CUtensorMap* tmY, int n0, int m0, const EpiParams& ep) {
   if (threadIdx.x == 64) TRACE(14);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const void* res = ep.res;
+  const void* res = EpiIO<IOT>::res(ep.res);
+  const bool has_res = EpiIO<IOT>::has_res(res);
   const int ldr = ep.ldr, ycol = ep.ycol, mcount = ep.mcount;
-  const bool res32 = ep.io & IO_RES_F32, out32 = ep.io & IO_OUT_F32;
+  const bool res32 = EpiIO<IOT>::res32(ep.io), out32 = EpiIO<IOT>::out32(ep.io);
   // TMEM lane = W row within the tile; warp w reads its lane quarter (w % 4) for the column
   // half w / 4 of the tile
   const int row = (warp & 3) * 32 + lane;
@@ -178,7 +192,7 @@ __device__ __forceinline__ void store_tile(uint8_t* otile, uint32_t tmem_d, cons
 #pragma unroll 1
   for (int c0 = chalf; c0 < chalf + BN / 2; c0 += 16) {
     float rv[16];
-    if (res != nullptr) {
+    if (has_res) {
 #pragma unroll
       for (int j = 0; j < 16; ++j) {
         const int ml = c0 + j;
@@ -192,7 +206,7 @@ __device__ __forceinline__ void store_tile(uint8_t* otile, uint32_t tmem_d, cons
 #pragma unroll
     for (int j = 0; j < 16; ++j) {
       float a = apply_act_c<ACT>(__uint_as_float(v[j]) + bsv);
-      if (res != nullptr) a += rv[j];
+      if (has_res) a += rv[j];
       if (out32)
         reinterpret_cast<float*>(otile)[(c0 + j) * BM + row] = a;
       else
@@ -219,11 +233,13 @@ __device__ __forceinline__ void store_tile(uint8_t* otile, uint32_t tmem_d, cons
 // rank order 0..splits-1 (deterministic), then runs the epilogue.  At the hot path's
 // 128-token shapes a CTA's time is set by the bytes it ingests (~100 GB/s per SM measured,
 // profiles/r01_gemm_trace.jsonl), so spreading a weight tile over `splits` SMs pays.
-template <class T, int BN, int ACT, bool SPLIT>
+template <class T, int BN, int ACT, bool SPLIT, int IOT>
 __global__ void __launch_bounds__(NT, 1)
     gemm_tc_kernel(const __grid_constant__ GemmGroup grp, const __grid_constant__ CUtensorMap tmX,
-                   const __grid_constant__ CUtensorMap tmY, const void* res, int ldr, void* Y, int ldy, int M, int N,
+                   const __grid_constant__ CUtensorMap tmY, const void* res_, int ldr, void* Y, int ldy, int M, int N,
                    int K, int act, int io, int splits, int nst) {
+  const void* res = EpiIO<IOT>::res(res_);
+  const bool has_res = EpiIO<IOT>::has_res(res);
   constexpr int STAGES = stages_for<BN>();
   constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
   constexpr uint32_t B_BYTES = BN * BK * 2;
@@ -255,7 +271,7 @@ __global__ void __launch_bounds__(NT, 1)
   const int kb_lo = sp * kb_all / splits;
   const int num_kb = (sp + 1) * kb_all / splits - kb_lo;  // >= 1 (splits <= kb_all)
   const int mcount = min(BN, M - m0);
-  const bool res32 = io & IO_RES_F32, out32 = io & IO_OUT_F32;
+  const bool res32 = EpiIO<IOT>::res32(io), out32 = EpiIO<IOT>::out32(io);
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(tmW)) : "memory");
@@ -354,7 +370,7 @@ __global__ void __launch_bounds__(NT, 1)
   const int chalf = (warp >> 2) * (BN / 2);
   float* tile = reinterpret_cast<float*>(smem);
   if constexpr (!SPLIT) {
-    store_tile<T, BN, ACT>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
+    store_tile<T, BN, ACT, IOT>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
   } else {
     // 1) TMEM -> shared memory: this split's fp32 partial tile [128 W rows][BN tokens], unpadded,
     //    so each owner's rows are one contiguous block to push.  Within a row the 16-byte chunks
@@ -378,7 +394,7 @@ __global__ void __launch_bounds__(NT, 1)
       const int nn = n0 + nl;
 #pragma unroll
       for (int e = 0; e < 8; ++e) acc[e] = apply_act_c<ACT>(acc[e] + sbias[nl + e]);
-      if (res) {
+      if (has_res) {
         float r8[8];
         if (rpre != nullptr) {
 #pragma unroll
@@ -425,7 +441,7 @@ __global__ void __launch_bounds__(NT, 1)
     mbar_wait(&recv_bar, 0);
     if (threadIdx.x == 0) TRACE(7);
     const int units = (RPR / 8) * mcount;
-    if (res == nullptr || units <= NT) {
+    if (!has_res) {
       for (int u = threadIdx.x; u < units; u += NT) {
         const int gi = u / mcount, ml = u - gi * mcount;  // 8-row group within the owned rows
         float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
@@ -437,9 +453,9 @@ __global__ void __launch_bounds__(NT, 1)
         finish(sp * RPR + 8 * gi, ml, acc);
       }
     } else {
-      // several units per thread with a residual: the residual loads of two units are issued
-      // before either is finished (one latency per pair instead of one per unit; the 1024-token
-      // shapes finalise 2-4 units per thread)
+      // with a residual: the residual loads of two units are issued before either is finished
+      // (one latency per pair instead of one per unit; the 1024-token shapes finalise 2-4 units
+      // per thread, the 128-token ones 1)
       for (int u0 = threadIdx.x; u0 < units; u0 += 2 * NT) {
         float r8[2][8];
 #pragma unroll
@@ -644,7 +660,7 @@ __global__ void __launch_bounds__(NT, 1)
   __syncthreads();
   if (threadIdx.x == 0) TRACE(5);
   asm volatile("tcgen05.fence::after_thread_sync;");
-  store_tile<T, BN, ACT>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
+  store_tile<T, BN, ACT, 0>(smem, tmem_d, sbias, &tmY, n0, m0, ep);
 #ifdef DP_GEMM_TRACE
   if (threadIdx.x == 0) {
     TRACE(8);
@@ -661,7 +677,7 @@ __global__ void __launch_bounds__(NT, 1)
   }
 }
 
-template <class T, int BN, int ACT>
+template <class T, int BN, int ACT, int IOT>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
          cudaStream_t s) {
@@ -684,9 +700,9 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   // the single-split and split-K kernels are separate instantiations: each carries only its own
   // epilogue, and a CTA's first pass through its code is instruction-fetch bound (one cold
   // fetch per instruction; a larger split-K epilogue slowed even the kernels that never ran it)
-  auto kern = gemm_tc_kernel<T, BN, ACT, false>;
+  auto kern = gemm_tc_kernel<T, BN, ACT, false, IOT>;
   if constexpr (BN < 256) {  // (256-wide tiles never split: the send + receive buffers would not fit)
-    if (splits > 1) kern = gemm_tc_kernel<T, BN, ACT, true>;
+    if (splits > 1) kern = gemm_tc_kernel<T, BN, ACT, true, IOT>;
   }
   static std::atomic<unsigned> attr{0}, attr_sp{0};
   if (first_on_device(splits > 1 ? attr_sp : attr))
@@ -780,7 +796,17 @@ void dispatch(int bn, bool pair, const void* x, int ldx, int ngroups, const void
 #undef DP_RUNP
     return;
   }
-#define DP_RUN(B, A) run<T, B, A>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s)
+  // the epilogue I/O variant (EpiIO): the forward pass's two fixed combinations, else generic
+  const int iot = (res == nullptr && io == 0) ? 1 : (res != nullptr && io == (IO_RES_F32 | IO_OUT_F32)) ? 2 : 0;
+#define DP_RUN(B, A)                                                                                 \
+  do {                                                                                               \
+    if (iot == 1)                                                                                    \
+      run<T, B, A, 1>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);    \
+    else if (iot == 2 && A == ACT_NONE)                                                              \
+      run<T, B, A, (A == ACT_NONE ? 2 : 0)>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s); \
+    else                                                                                             \
+      run<T, B, A, 0>(x, ldx, ngroups, w, bias, ycol, res, ldr, y, ldy, M, N, K, act, io, sp, s);    \
+  } while (0)
 #define DP_ACTS(B)                                 \
   switch (act) {                                   \
     case ACT_NONE: DP_RUN(B, ACT_NONE); break;           \
