@@ -31,6 +31,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstring>
+#include <type_traits>
 
 #include "common.h"
 #include "dtype.cuh"
@@ -84,10 +85,14 @@ __device__ __forceinline__ void named_sync(int id, int n) {
 }
 
 
-template <class T>
+// CAUSAL and SPLIT (nsplit > 1) are compile-time: each variant carries only its masking and
+// merge code (a CTA runs its code once; cold instruction fetch is on its critical path).
+template <class T, bool CAUSAL, bool SPLIT>
 __global__ void __launch_bounds__(NTHR, 1)
     attention_tc_kernel(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmKV,
-                        T* __restrict__ ctx, int seq, int H, int causal, float scale_log2, int nsplit) {
+                        T* __restrict__ ctx, int seq, int H, float scale_log2, int nsplit_rt) {
+  constexpr bool causal = CAUSAL;
+  const int nsplit = SPLIT ? nsplit_rt : 1;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sQ = smem;
@@ -348,7 +353,7 @@ __global__ void __launch_bounds__(NTHR, 1)
       const float a0 = (mrow == -INFINITY) ? 0.f : fast_exp2(mrow - m);
       const float a1 = (m1 == -INFINITY) ? 0.f : fast_exp2(m1 - m);
       const float l = lrow * a0 + l1 * a1;
-      if (nsplit == 1) {
+      if constexpr (!SPLIT) {
         if (qrow < seq) {
           const float inv = l > 0.f ? 1.f / l : 0.f;
           const float c0 = a0 * inv, c1 = a1 * inv;
@@ -381,7 +386,7 @@ __global__ void __launch_bounds__(NTHR, 1)
     }
     if (tid == 0) ATRACE(8);
   }
-  if (nsplit > 1) {
+  if constexpr (SPLIT) {
     // Cluster merge: the nsplit CTAs of a query tile hold (o, m, l) of consecutive key ranges in
     // their xs rows ([128][68] fp32).  Rank k finalises query rows [k*128/n, (k+1)*128/n): every
     // CTA pushes the rows each peer owns with ONE bulk copy (cp.async.bulk shared::cta ->
@@ -516,18 +521,26 @@ void launch_attention_tc(int dtype, const void* qkv, int ldqkv, void* ctx, int b
     }
   if (const int forced = experiment_env("DP_ATT_SPLIT", 0); forced > 0) nsplit = std::min(forced, 4);
   const dim3 grid(heads, nqt * nsplit, batch);
-  auto go = [&](auto tag) {
+  auto go2 = [&](auto tag, auto ctag, auto stag) {
     using T = decltype(tag);
+    constexpr bool C = decltype(ctag)::value, SP = decltype(stag)::value;
+    auto kern = attention_tc_kernel<T, C, SP>;
     static std::atomic<unsigned> attr{0};
     if (first_on_device(attr))
-      DP_CUDA(cudaFuncSetAttribute(attention_tc_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)SMEM_BYTES));
-    if (nsplit > 1)
-      launch_kernel_cluster(attention_tc_kernel<T>, grid, dim3(NTHR), SMEM_BYTES, dim3(1, nsplit, 1), s, mq, mkv,
-                            (T*)ctx, seq, H, causal ? 1 : 0, scale_log2, nsplit);
+      DP_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES));
+    if (SP)
+      launch_kernel_cluster(kern, grid, dim3(NTHR), SMEM_BYTES, dim3(1, nsplit, 1), s, mq, mkv, (T*)ctx, seq, H,
+                            scale_log2, nsplit);
     else
-      launch_kernel(attention_tc_kernel<T>, grid, dim3(NTHR), SMEM_BYTES, s, mq, mkv, (T*)ctx, seq, H,
-                    causal ? 1 : 0, scale_log2, 1);
+      launch_kernel(kern, grid, dim3(NTHR), SMEM_BYTES, s, mq, mkv, (T*)ctx, seq, H, scale_log2, 1);
+  };
+  auto go = [&](auto tag) {
+    using B = std::bool_constant<true>;
+    using F = std::bool_constant<false>;
+    if (causal)
+      nsplit > 1 ? go2(tag, B{}, B{}) : go2(tag, B{}, F{});
+    else
+      nsplit > 1 ? go2(tag, F{}, B{}) : go2(tag, F{}, F{});
   };
   if (dtype == DP_BF16)
     go(__nv_bfloat16{});

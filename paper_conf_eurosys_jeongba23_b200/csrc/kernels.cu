@@ -242,7 +242,11 @@ void launch_embed(int dtype, const int32_t* ids, int ntok, int seq, int pos_off,
 // HBM, or -- when they are host-mapped (DHA), CL = true -- by rank 0 of a single cluster of <= 16
 // CTAs and broadcast over DSMEM, so the host link carries them exactly once per launch.
 // -------------------------------------------------------------------------------------
-template <class T, int VPL, bool CL>
+// MODE: the forward's two LayerNorm forms as compile-time variants (fp32 input, no residual;
+// 1 = with the fp32 copy of the output -- BERT's residual stream --, 2 = without -- GPT-2), 0 =
+// any (the test hooks, DHA gamma / beta).  A variant carries only its own load / store code: a
+// CTA runs its code once and cold instruction fetch is on its critical path (K2 round 2).
+template <class T, int VPL, bool CL, int MODE>
 __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__ x, const void* __restrict__ r,
                                                         const T* g, const T* b, T* __restrict__ y, int rows,
                                                         int n, float eps, int in_f32, float* __restrict__ y32) {
@@ -259,19 +263,40 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__
   const int lane = threadIdx.x & 31;
   const int nwarps = gridDim.x * (blockDim.x >> 5);
   for (int row = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); row < rows; row += nwarps)
-    ln_row_warp<T, VPL, 0>(x, r, (size_t)row * n, n, eps, in_f32, sm, y, (size_t)row * n, y32);
+    if constexpr (MODE == 1)
+      ln_row_warp<T, VPL, 0>(x, nullptr, (size_t)row * n, n, eps, 1, sm, y, (size_t)row * n, y32);
+    else if constexpr (MODE == 2)
+      ln_row_warp<T, VPL, 0>(x, nullptr, (size_t)row * n, n, eps, 1, sm, y, (size_t)row * n, nullptr);
+    else
+      ln_row_warp<T, VPL, 0>(x, r, (size_t)row * n, n, eps, in_f32, sm, y, (size_t)row * n, y32);
+}
+
+template <class T, int V, bool CL, int MODE>
+static void layernorm_launch_m(int grid, size_t sm, cudaStream_t s, const void* x, const void* r, const void* g,
+                               const void* b, void* y, int rows, int n, float eps, bool in_f32, float* y32) {
+  if (CL) {
+    static std::atomic<unsigned> attr{0};
+    if (first_on_device(attr))
+      DP_CUDA(cudaFuncSetAttribute(layernorm_kernel<T, V, CL, MODE>, cudaFuncAttributeNonPortableClusterSizeAllowed,
+                                   1));
+  }
+  launch_kernel_cluster(layernorm_kernel<T, V, CL, MODE>, dim3(grid), dim3(256), sm, dim3(CL ? grid : 1), s, x, r,
+                        (const T*)g, (const T*)b, (T*)y, rows, n, eps, (int)in_f32, y32);
 }
 
 template <class T, int V, bool CL>
 static void layernorm_launch(int grid, size_t sm, cudaStream_t s, const void* x, const void* r, const void* g,
                              const void* b, void* y, int rows, int n, float eps, bool in_f32, float* y32) {
-  if (CL) {
-    static std::atomic<unsigned> attr{0};
-    if (first_on_device(attr))
-      DP_CUDA(cudaFuncSetAttribute(layernorm_kernel<T, V, CL>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+  if constexpr (!CL) {
+    if (in_f32 && r == nullptr) {
+      if (y32 != nullptr)
+        layernorm_launch_m<T, V, CL, 1>(grid, sm, s, x, r, g, b, y, rows, n, eps, in_f32, y32);
+      else
+        layernorm_launch_m<T, V, CL, 2>(grid, sm, s, x, r, g, b, y, rows, n, eps, in_f32, y32);
+      return;
+    }
   }
-  launch_kernel_cluster(layernorm_kernel<T, V, CL>, dim3(grid), dim3(256), sm, dim3(CL ? grid : 1), s, x, r,
-                        (const T*)g, (const T*)b, (T*)y, rows, n, eps, (int)in_f32, y32);
+  layernorm_launch_m<T, V, CL, 0>(grid, sm, s, x, r, g, b, y, rows, n, eps, in_f32, y32);
 }
 
 template <class T>
