@@ -278,6 +278,9 @@ __global__ void __launch_bounds__(NT, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
     ep = EpiParams{res, ldr, (int)ycol, io, mcount};
+    // (rolled loops here and below: this thread runs them once, so unrolling only adds cold
+    // instruction fetch in front of the first TMA)
+#pragma unroll 1
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full_bar[s], 1);
       mbar_init(&empty_bar[s], 1);
@@ -290,6 +293,7 @@ __global__ void __launch_bounds__(NT, 1)
     // grid-dependency wait (PDL) -- so its HBM latency overlaps the setup and the
     // predecessor's tail.  Activations (X, residual) and every store come after the wait.
     const int pre0 = num_kb < nst ? num_kb : nst;
+#pragma unroll 1
     for (int kb = 0; kb < pre0; ++kb) {
       mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
       tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb_lo + kb) * BK, n0);
@@ -318,23 +322,28 @@ __global__ void __launch_bounds__(NT, 1)
   if (threadIdx.x == 0) TRACE(3);
 
   if (warp == 0 && lane == 0) {
-    // TMA producer
+    // TMA producer (stage s and its phase bit ph as running counters: no integer division)
+    int s = 0;
+    uint32_t ph = 0;
+#pragma unroll 1
     for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % nst;
       uint8_t* a = smem + s * STAGE_BYTES;
       uint8_t* b = a + A_BYTES;
       if (kb >= pre) {
-        mbar_wait(&empty_bar[s], ((kb / nst) - 1) & 1);
+        mbar_wait(&empty_bar[s], ph ^ 1u);
         mbar_expect_tx(&full_bar[s], STAGE_BYTES);
         tma_load_2d(tmW, &full_bar[s], a, (kb_lo + kb) * BK, n0);
       }
       tma_load_2d(&tmX, &full_bar[s], b, (kb_lo + kb) * BK, m0);
+      if (++s == nst) s = 0, ph ^= 1u;
     }
   } else if (warp == 1 && lane == 0) {
     // MMA issuer
+    int s = 0;
+    uint32_t ph = 0;
+#pragma unroll 1
     for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % nst;
-      mbar_wait(&full_bar[s], (kb / nst) & 1);
+      mbar_wait(&full_bar[s], ph);
       if (kb == 0) TRACE(4);
       asm volatile("tcgen05.fence::after_thread_sync;");
       const uint8_t* a = smem + s * STAGE_BYTES;
@@ -344,6 +353,7 @@ __global__ void __launch_bounds__(NT, 1)
       for (int kk = 0; kk < BK / 16; ++kk)  // advance 16 elements = 32 B = 2 in descriptor units
         umma_f16(tmem_d, da + 2 * kk, db + 2 * kk, IDESC, (kb | kk) != 0);
       umma_commit(&empty_bar[s]);
+      if (++s == nst) s = 0, ph ^= 1u;
     }
     umma_commit(&done_bar);
   }
