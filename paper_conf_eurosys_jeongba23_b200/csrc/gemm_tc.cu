@@ -8,7 +8,8 @@
 // TMEM) runs over W's rows (N) and the MMA's N axis over tokens (BN = 32..256 columns).
 //
 // Per CTA (256 threads, one 128 x BN output tile, a K range):
-//   warp 0 / lane 0  : TMA producer -- W tile [128 x 64] and X tile [BN x 64] per stage,
+//   warp 0 / lane 0  : TMA producer -- W tile [128 x 64 KS] and X tile [BN x 64 KS] per stage
+//                      (KS = ks_for<BN>() 64-deep chunks, one 3D box each when KS > 1),
 //                      both K-major with the 128-byte swizzle, into a STAGES-deep ring; the
 //                      first ring of W tiles is issued BEFORE the grid-dependency wait (PDL):
 //                      weights never depend on the previous kernel;
@@ -72,6 +73,24 @@ CUtensorMap make_kmajor_map(const void* base, int dtype, int rows, int K, int ld
   return m;
 }
 
+// K-major tile map whose box spans `kch` consecutive 64-element K chunks: dims {64, rows, K/64}
+// (the chunk dimension strides 128 B), box {64, box_rows, kch} -> shared memory [kch][box_rows]
+// [128 B], i.e. kch swizzled K-major sub-tiles back to back, in ONE TMA operation.
+CUtensorMap make_kmajor_map3(const void* base, int dtype, int rows, int K, int ld, int box_rows, int kch) {
+  CUtensorMap m;
+  std::memset(&m, 0, sizeof(m));
+  cuuint64_t dims[3] = {64, (cuuint64_t)rows, (cuuint64_t)(K / 64)};
+  cuuint64_t strides[2] = {(cuuint64_t)ld * 2, 128};
+  cuuint32_t box[3] = {64u, (cuuint32_t)box_rows, (cuuint32_t)kch};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = get_encode()(&m, dtype == DP_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16,
+                            3, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  DP_CHECK(r == CUDA_SUCCESS, DP_ERR_CUDA, "cuTensorMapEncodeTiled (3d) failed (" + std::to_string((int)r) + ")");
+  return m;
+}
+
 // Generic tiled map (no swizzle): rank 1..3, dims/strides in elements / bytes (strides of
 // dims 1.., as cuTensorMapEncodeTiled takes them).  Used for K6's TMA stores.
 CUtensorMap make_plain_map(const void* base, CUtensorMapDataType dt, int rank, const uint64_t* dims,
@@ -93,15 +112,52 @@ namespace {
 
 constexpr int BM = 128;  // W rows per tile (MMA M)
 constexpr int NT = 256;  // threads per CTA: warp 0 TMA, warp 1 MMA + TMEM, all 8 warps the epilogue
-constexpr int BK = 64;   // K per stage: 64 x 2 B = one 128-byte swizzle row
+constexpr int BK = 64;   // K per 128-byte swizzle row (64 x 2 B)
+// 64-deep K chunks per ring stage of the single-CTA kernel: > 1 makes one 3D TMA box per
+// operand span them.  The per-CTA traces put the 128-token mainloop at ~0.26 us per TMA
+// box pair whatever its bytes (BN 32..128 alike; W in 64- / 32-row boxes was slower), so fewer,
+// deeper boxes stream faster.  Measured in the warm forwards (profiles/r02_warm_ab_kchunks.jsonl,
+// A/B of 1..4 chunks per tile width): 3 for BN <= 64, 2 for BN 96 / 128, 1 for BN 256 (deeper
+// 256-wide stages leave only 2 ring stages).  BERT-Base 0.424 -> 0.365 ms, BERT-Large 1.199 ->
+// 1.109, GPT-2 Medium 1.671 -> 1.577.  (Experiment overrides: -DDP_GEMM_KS_{SMALL,MID,BIG}.)
+#ifndef DP_GEMM_KS_SMALL
+#define DP_GEMM_KS_SMALL 3
+#endif
+#ifndef DP_GEMM_KS_MID
+#define DP_GEMM_KS_MID 2
+#endif
+#ifndef DP_GEMM_KS_BIG
+#define DP_GEMM_KS_BIG 1
+#endif
+template <int BN>
+__host__ __device__ constexpr int ks_for() {
+  return BN <= 64 ? DP_GEMM_KS_SMALL : BN <= 128 ? DP_GEMM_KS_MID : DP_GEMM_KS_BIG;
+}
+
+__device__ __forceinline__ void tma_load_3d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1, int c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
+      : "memory");
+}
+// one stage's tile (rows x KS*64 K) from a KS-chunk map (KS == 1: the 2D map)
+template <int KS>
+__device__ __forceinline__ void tma_load_stage(const CUtensorMap* map, uint64_t* bar, void* dst, int kblk, int row) {
+  if constexpr (KS == 1)
+    tma_load_2d(map, bar, dst, kblk * BK, row);
+  else
+    tma_load_3d(map, bar, dst, 0, row, kblk * KS);
+}
 
 // Ring depth per tile width: as many stages as ~224 KB of shared memory holds (<= 12), so a
 // K = 768 layer (12 k-blocks) has its whole weight slice in flight at once.
 template <int BN>
 __host__ __device__ constexpr int stages_for() {
-  constexpr int bytes = BM * BK * 2 + BN * BK * 2;
+  constexpr int KS = ks_for<BN>();
+  constexpr int bytes = KS * (BM * BK * 2 + BN * BK * 2);
   constexpr int s = (224 * 1024) / bytes;
-  return s > 12 ? 12 : s;
+  return s > 12 / KS ? 12 / KS : s;
 }
 
 // Up to 3 independent weight matrices sharing X, M, N, K (BERT's q/k/v): blockIdx.z selects
@@ -240,9 +296,10 @@ __global__ void __launch_bounds__(NT, 1)
                    int K, int act, int io, int splits, int nst) {
   const void* res = EpiIO<IOT>::res(res_);
   const bool has_res = EpiIO<IOT>::has_res(res);
+  constexpr int KS = ks_for<BN>();
   constexpr int STAGES = stages_for<BN>();
-  constexpr uint32_t A_BYTES = BM * BK * 2;  // 16 KB
-  constexpr uint32_t B_BYTES = BN * BK * 2;
+  constexpr uint32_t A_BYTES = KS * BM * BK * 2;  // KS x 16 KB
+  constexpr uint32_t B_BYTES = KS * BN * BK * 2;
   constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   constexpr uint32_t TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;  // a power of 2
   constexpr int PROW = BN + 1;  // fp32 tile row stride (odd: conflict-free TMEM->smem writes)
@@ -267,7 +324,7 @@ __global__ void __launch_bounds__(NT, 1)
   const CUtensorMap* tmW = &grp.w[grp_i];
   const T* bias = static_cast<const T*>(grp.bias[grp_i]);
   const long long ycol = grp.ycol[grp_i];
-  const int kb_all = K / BK;
+  const int kb_all = (K / BK + KS - 1) / KS;  // ring stages over the whole K (a last odd chunk: TMA zero fill)
   const int kb_lo = sp * kb_all / splits;
   const int num_kb = (sp + 1) * kb_all / splits - kb_lo;  // >= 1 (splits <= kb_all)
   const int mcount = min(BN, M - m0);
@@ -296,7 +353,7 @@ __global__ void __launch_bounds__(NT, 1)
 #pragma unroll 1
     for (int kb = 0; kb < pre0; ++kb) {
       mbar_expect_tx(&full_bar[kb], STAGE_BYTES);
-      tma_load_2d(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, (kb_lo + kb) * BK, n0);
+      tma_load_stage<KS>(tmW, &full_bar[kb], smem + kb * STAGE_BYTES, kb_lo + kb, n0);
     }
     TRACE(1);
   }
@@ -332,9 +389,9 @@ __global__ void __launch_bounds__(NT, 1)
       if (kb >= pre) {
         mbar_wait(&empty_bar[s], ph ^ 1u);
         mbar_expect_tx(&full_bar[s], STAGE_BYTES);
-        tma_load_2d(tmW, &full_bar[s], a, (kb_lo + kb) * BK, n0);
+        tma_load_stage<KS>(tmW, &full_bar[s], a, kb_lo + kb, n0);
       }
-      tma_load_2d(&tmX, &full_bar[s], b, (kb_lo + kb) * BK, m0);
+      tma_load_stage<KS>(&tmX, &full_bar[s], b, kb_lo + kb, m0);
       if (++s == nst) s = 0, ph ^= 1u;
     }
   } else if (warp == 1 && lane == 0) {
@@ -350,8 +407,11 @@ __global__ void __launch_bounds__(NT, 1)
       const uint8_t* b = a + A_BYTES;
       const uint64_t da = sw128_desc(a), db = sw128_desc(b);
 #pragma unroll
-      for (int kk = 0; kk < BK / 16; ++kk)  // advance 16 elements = 32 B = 2 in descriptor units
-        umma_f16(tmem_d, da + 2 * kk, db + 2 * kk, IDESC, (kb | kk) != 0);
+      for (int kc = 0; kc < KS; ++kc)  // K chunk kc: sub-tiles BM x 128 B / BN x 128 B further on
+#pragma unroll
+        for (int kk = 0; kk < BK / 16; ++kk)  // advance 16 elements = 32 B = 2 in descriptor units
+          umma_f16(tmem_d, da + (kc * BM * 128 >> 4) + 2 * kk, db + (kc * BN * 128 >> 4) + 2 * kk, IDESC,
+                   (kb | kc | kk) != 0);
       umma_commit(&empty_bar[s]);
       if (++s == nst) s = 0, ph ^= 1u;
     }
@@ -691,8 +751,9 @@ template <class T, int BN, int ACT, int IOT>
 void run(const void* x, int ldx, int ngroups, const void* const* w, const void* const* bias, const long long* ycol,
          const void* res, int ldr, void* y, int ldy, int M, int N, int K, int act, int io, int splits,
          cudaStream_t s) {
+  constexpr int KS = ks_for<BN>();
   constexpr int STAGES = stages_for<BN>();
-  constexpr size_t STAGE_BYTES = BM * BK * 2 + BN * BK * 2;
+  constexpr size_t STAGE_BYTES = KS * (BM * BK * 2 + BN * BK * 2);
   constexpr size_t smem_max = size_t(STAGES) * STAGE_BYTES + 1024;
   // the output tile (at most fp32) must fit the ring
   constexpr size_t epi_bytes = size_t(BM) * BN * 4;
@@ -721,11 +782,11 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   GemmGroup g;
   std::memset(&g, 0, sizeof(g));
   for (int i = 0; i < ngroups; ++i) {
-    g.w[i] = make_kmajor_map(w[i], dtype, N, K, K, BM);
+    g.w[i] = KS == 1 ? make_kmajor_map(w[i], dtype, N, K, K, BM) : make_kmajor_map3(w[i], dtype, N, K, K, BM, KS);
     g.bias[i] = bias ? bias[i] : nullptr;
     g.ycol[i] = ycol ? ycol[i] : 0;
   }
-  CUtensorMap mx = make_kmajor_map(x, dtype, M, K, ldx, BN);
+  CUtensorMap mx = KS == 1 ? make_kmajor_map(x, dtype, M, K, ldx, BN) : make_kmajor_map3(x, dtype, M, K, ldx, BN, KS);
   // the output tile store (single split): Y as [M rows][ldy columns] in the output dtype, box
   // [BN tokens][128 features]
   const bool o32 = (io & IO_OUT_F32) != 0;
@@ -907,7 +968,9 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
   if (hint_pair) bn_hint = -bn_hint;
   const int bn = bn_hint > 0 ? bn_hint : (env_bn > 0 ? env_bn : cfg.bn);
   int sp = sp_hint > 0 ? sp_hint : env_sp > 0 ? env_sp : (bn_hint > 0 || env_bn > 0 ? 1 : cfg.sp);
-  sp = std::max(1, std::min(std::min(sp, 8), K / BK));
+  // every split needs >= 1 ring stage of ks_for<bn>() 64-deep K chunks
+  const int ks = bn <= 64 ? ks_for<64>() : bn <= 128 ? ks_for<128>() : ks_for<256>();
+  sp = std::max(1, std::min(std::min(sp, 8), (K / BK + ks - 1) / ks));
   while (sp & (sp - 1)) --sp;  // a power of two: every rank owns BM / sp rows
   if (bn >= 256) sp = 1;       // the send + receive buffers (2 x 128 x BN fp32) must fit the ring
   // CTA pair (K2p): the model's choice unless a tile width is forced; DP_GEMM_PAIR=1 forces it
