@@ -467,7 +467,7 @@ dp_status dp_linear(const void* x, int32_t ldx, const void* w, const void* b, co
                     int32_t io, void* stream);
 
 /* The resident tcgen05 GEMM of dp_linear(path 0) with its tile configuration forced (tests,
- * sweeps): bn = 0 the cost model's choice; 32/64/96/128/256 one CTA per 128 x bn output tile
+ * sweeps): bn = 0 the cost model's choice; 32/64/96/128/192/256 one CTA per 128 x bn output tile
  * (K2); -64/-128/-192/-256 a CTA pair per 256 x |bn| tile (K2p: cta_group::2 MMAs issued by
  * the even CTA, each CTA staging its 128 W rows and |bn|/2 tokens; needs N % 256 == 0).
  * split = 0 the model's K split, 1 none, 2/4/8 (<= K/64, with a single-CTA bn <= 128) that many

@@ -81,9 +81,9 @@ extern "C" dp_status dp_gemm_tc(const void* x, int32_t ldx, const void* w, const
     DP_CHECK(M >= 0 && N > 0 && K > 0 && ldx >= K && ldy >= N && (!residual || ldr >= N), DP_ERR_INVALID,
              "bad shapes / strides");
     DP_CHECK(act >= 0 && act <= 3, DP_ERR_INVALID, "act must be 0..3");
-    DP_CHECK(bn == 0 || bn == 32 || bn == 64 || bn == 96 || bn == 128 || bn == 256 || bn == -64 || bn == -128 ||
-                 bn == -192 || bn == -256,
-             DP_ERR_INVALID, "bn must be 0, 32/64/96/128/256 or -64/-128/-192/-256");
+    DP_CHECK(bn == 0 || bn == 32 || bn == 64 || bn == 96 || bn == 128 || bn == 192 || bn == 256 || bn == -64 ||
+                 bn == -128 || bn == -192 || bn == -256,
+             DP_ERR_INVALID, "bn must be 0, 32/64/96/128/192/256 or -64/-128/-192/-256");
     DP_CHECK(bn >= 0 || N % 256 == 0, DP_ERR_INVALID, "a CTA pair needs N % 256 == 0");
     DP_CHECK(split == 0 || split == 1 ||
                  ((split & (split - 1)) == 0 && split <= 8 && bn > 0 && bn <= 128 && split <= K / 64),

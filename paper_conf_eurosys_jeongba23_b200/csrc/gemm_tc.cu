@@ -773,7 +773,7 @@ void run(const void* x, int ldx, int ngroups, const void* const* w, const void* 
   // epilogue, and a CTA's first pass through its code is instruction-fetch bound (one cold
   // fetch per instruction; a larger split-K epilogue slowed even the kernels that never ran it)
   auto kern = gemm_tc_kernel<T, BN, ACT, false, IOT>;
-  if constexpr (BN < 256) {  // (256-wide tiles never split: the send + receive buffers would not fit)
+  if constexpr (BN <= 128) {  // (wider tiles never split: the send + receive buffers would not fit)
     if (splits > 1) kern = gemm_tc_kernel<T, BN, ACT, true, IOT>;
   }
   static std::atomic<unsigned> attr{0}, attr_sp{0};
@@ -892,8 +892,9 @@ void dispatch(int bn, bool pair, const void* x, int ldx, int ngroups, const void
     case 64: DP_ACTS(64); break;
     case 96: DP_ACTS(96); break;
     case 128: DP_ACTS(128); break;
+    case 192: DP_ACTS(192); break;
     case 256: DP_ACTS(256); break;
-    default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/96/128/256");
+    default: fail(DP_ERR_INVALID, "gemm: BN must be 32/64/96/128/192/256");
   }
 #undef DP_ACTS
 #undef DP_RUN
@@ -941,6 +942,7 @@ constexpr MeasuredCfg kMeasured[] = {
     {384, 1024, 1024, 64, 2},   // BERT-Large / RoBERTa-Large attn-out (S384)
     {384, 3072, 1024, 64, 1},   // BERT-Large / RoBERTa-Large q/k/v (S384)
     {1024, 1024, 1024, 64, 1},  // GPT-2 Medium c_proj (S1024)
+    {1024, 3072, 1024, 192, 1}, // GPT-2 Medium c_attn (S1024): 144 CTAs in one wave (256-wide: 96)
 };
 
 static GemmCfg pick_cfg(int M, int N, int K) {
@@ -1004,7 +1006,7 @@ static void gemm_impl(int dtype, const void* x, int ldx, int ngroups, const void
   const int ks = bn <= 64 ? ks_for<64>() : bn <= 128 ? ks_for<128>() : ks_for<256>();
   sp = std::max(1, std::min(std::min(sp, 8), (K / BK + ks - 1) / ks));
   while (sp & (sp - 1)) --sp;  // a power of two: every rank owns BM / sp rows
-  if (bn >= 256) sp = 1;       // the send + receive buffers (2 x 128 x BN fp32) must fit the ring
+  if (bn > 128) sp = 1;        // the send + receive buffers (2 x 128 x BN fp32) must fit the ring
   // CTA pair (K2p): the model's choice unless a tile width is forced; DP_GEMM_PAIR=1 forces it
   // (with DP_GEMM_BN as the pair's tile width) for experiments
   static const int env_pair = experiment_env("DP_GEMM_PAIR", -1);

@@ -322,7 +322,7 @@ def test_gemm_split_k_cluster_configs(bn, split, M, N, K):
     _gemm_forced_case(bn, split, M, N, K, "gelu_erf", True, "fp16", M + N + K)
 
 
-@pytest.mark.parametrize("bn", [32, 64, 96, 128, 256])
+@pytest.mark.parametrize("bn", [32, 64, 96, 128, 192, 256])
 @pytest.mark.parametrize("M,N,K", [(100, 256, 512), (384, 1024, 1024), (1024, 512, 128)])
 def test_gemm_single_cta_tile_widths(bn, M, N, K):
     """Every single-CTA tile width (K2) forced, ragged token tails included."""
