@@ -932,8 +932,9 @@ struct GemmCfg {
 // forced at a time against the model's choice, instrumented build, DP_GEMM_CFG;
 // profiles/r02_warm_ab_gemm_cfg.jsonl) where the model's pick lost: attn-out of BERT-Base
 // (0.364 -> 0.347 ms), attn-out and q/k/v of BERT-Large (1.105 -> 1.074), GPT-2 Medium's c_proj
-// (1.580 -> 1.516).  Every other forward shape kept the model's pick (the alternatives tried
-// were slower).  N is the total over the grouped weights (q/k/v: 3 x hidden).
+// (1.580 -> 1.516), BERT-Large fc1 on 96-token tiles (1.077 -> 1.065), GPT-2 Medium c_attn on
+// 192-token tiles (1.493 -> 1.477).  Every other forward shape kept the model's pick (the
+// alternatives tried were slower).  N is the total over the grouped weights (q/k/v: 3 x hidden).
 struct MeasuredCfg {
   int M, N, K, bn, sp;
 };
@@ -941,6 +942,7 @@ constexpr MeasuredCfg kMeasured[] = {
     {128, 768, 768, 32, 4},     // BERT-Base attn-out (S128)
     {384, 1024, 1024, 64, 2},   // BERT-Large / RoBERTa-Large attn-out (S384)
     {384, 3072, 1024, 64, 1},   // BERT-Large / RoBERTa-Large q/k/v (S384)
+    {384, 4096, 1024, 96, 1},   // BERT-Large / RoBERTa-Large fc1 (S384): 4 exact 96-token tiles, 128 CTAs
     {1024, 1024, 1024, 64, 1},  // GPT-2 Medium c_proj (S1024)
     {1024, 3072, 1024, 192, 1}, // GPT-2 Medium c_attn (S1024): 144 CTAs in one wave (256-wide: 96)
 };
