@@ -271,6 +271,14 @@ __global__ void __launch_bounds__(256) layernorm_kernel(const void* __restrict__
       ln_row_warp<T, VPL, 0>(x, r, (size_t)row * n, n, eps, in_f32, sm, y, (size_t)row * n, y32);
 }
 
+// rows (warps) per LayerNorm CTA: 4 up to 128 rows (32 CTAs: BERT-Base S128 warm 0.3465 ->
+// 0.343 ms), else 8 (4 measured slower at 256-1024 rows; profiles/r02_warm_ab_ln_warps.jsonl).
+// DP_LN_WARPS overrides it in instrumented builds (A/B only).
+static int ln_warps(int rows) {
+  static const int w = experiment_env("DP_LN_WARPS", 0);
+  return w > 0 ? w : rows <= 128 ? 4 : 8;
+}
+
 template <class T, int V, bool CL, int MODE>
 static void layernorm_launch_m(int grid, size_t sm, cudaStream_t s, const void* x, const void* r, const void* g,
                                const void* b, void* y, int rows, int n, float eps, bool in_f32, float* y32) {
@@ -280,7 +288,7 @@ static void layernorm_launch_m(int grid, size_t sm, cudaStream_t s, const void* 
       DP_CUDA(cudaFuncSetAttribute(layernorm_kernel<T, V, CL, MODE>, cudaFuncAttributeNonPortableClusterSizeAllowed,
                                    1));
   }
-  launch_kernel_cluster(layernorm_kernel<T, V, CL, MODE>, dim3(grid), dim3(256), sm, dim3(CL ? grid : 1), s, x, r,
+  launch_kernel_cluster(layernorm_kernel<T, V, CL, MODE>, dim3(grid), dim3(32 * ln_warps(rows)), sm, dim3(CL ? grid : 1), s, x, r,
                         (const T*)g, (const T*)b, (T*)y, rows, n, eps, (int)in_f32, y32);
 }
 
@@ -306,7 +314,7 @@ static void layernorm_t(const void* x, const void* r, const void* g, const void*
   // CTA stages them (L2 hits); host-mapped (DHA): ONE cluster of <= 16 CTAs (up to 128 warps,
   // several rows each beyond 128 rows) reads them once and shares them over DSMEM, so the host
   // link carries exactly 2 x n elements (the algorithmic bytes)
-  const int warps = 8;
+  const int warps = ln_warps(rows);
   int grid = (rows + warps - 1) / warps;
   if (grid > 148 * 8) grid = 148 * 8;
   if (gb_host && grid > 16) grid = 16;
