@@ -104,7 +104,11 @@ def test_embed_parity_and_dha_bit_identity(name, B, S, dtype):
 # ---------------------------------------------------------------------------------------
 
 SHAPES_LIN = [(1, 128, 64), (7, 256, 128), (32, 768, 768), (100, 384, 128), (128, 768, 768), (128, 3072, 768),
-              (128, 768, 3072), (200, 1024, 1024), (384, 4096, 1024), (1024, 1024, 4096), (333, 2304, 768)]
+              (128, 768, 3072), (200, 1024, 1024), (384, 4096, 1024), (1024, 1024, 4096), (333, 2304, 768),
+              # K ranges that are not a multiple of a ring stage's 3 / 2 chunks of 64 (the last 3D TMA
+              # box zero-fills past K), a single chunk, and the 96 / 192-token tiles of the measured table
+              (64, 256, 64), (48, 384, 192), (300, 512, 320), (200, 256, 64), (384, 4096, 1024),
+              (1024, 3072, 1024)]
 
 
 @pytest.mark.parametrize("M,N,K", SHAPES_LIN)
