@@ -33,6 +33,23 @@ def main():
         dp.linear(x, K, hw, None, None, 0, y, N, M, N, K, path=1)
         torch.cuda.synchronize()
         dp.host_free(hw)
+    # round 2: forced tile widths incl. 96 / 192 and K ranges ending in a partial 3D-box stage
+    for M, N, K, bn, sp in ((384, 512, 1024, 96, 1), (300, 512, 320, 192, 1), (128, 768, 768, 32, 4),
+                            (100, 256, 192, 64, 2)):
+        x = torch.randn(M, K, device=dev).half()
+        w = (torch.randn(N, K, device=dev) / math.sqrt(K)).half()
+        b = torch.randn(N, device=dev).half()
+        r = torch.randn(M, N, device=dev).half()
+        y = torch.zeros(M, N, device=dev).half()
+        dp.gemm_tc(x, K, w, b, r, N, y, N, M, N, K, act="gelu_tanh", bn=bn, split=sp)
+        torch.cuda.synchronize()
+    # K5t: no split, key split over clusters of 2 and 4 (bulk DSMEM push + merge), causal and not
+    for S, H, heads in ((384, 1024, 16), (512, 256, 4), (1024, 256, 4)):
+        qkv = torch.randn(S, 3 * H, device=dev).half()
+        o = torch.zeros(S, H, device=dev).half()
+        for causal in (False, True):
+            dp.attention_tc(qkv, 3 * H, o, 1, S, H, heads, causal)
+        torch.cuda.synchronize()
     # LayerNorm / embedding with host-mapped gamma / beta (cluster DSMEM broadcast) and device ones
     for rows in (77, 384):
         n = 768
